@@ -1,0 +1,363 @@
+"""Pins of the CPU oracle against what the paper and mathematics fix.
+
+None of these compare the oracle with itself: each checks a closed form, an invariant of the
+paper's checksum relations, a textbook/library special case, brute force on tiny inputs, or
+injection ground truth derived from the schedule (tests/_predict.py).
+"""
+import math
+import os
+
+import numpy as np
+import pytest
+import scipy.linalg
+
+import oracle
+import synthetic as syn
+from tests._predict import predict, V, KIND
+
+EPS = 2.0 ** -52
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def lucas_L(n):
+    i = np.arange(n)
+    return ((i[:, None] & i[None, :]) == i[None, :]).astype(np.float64)
+
+
+def floor_rel(L, Lref, A):
+    """|dL_ij| / max(|L_ij|, 1e-3 sqrt(A_ii))  (reading A18)."""
+    s = np.sqrt(np.diag(A))[:, None]
+    return np.max(np.abs(np.tril(L) - np.tril(Lref)) / np.maximum(np.abs(np.tril(Lref)), 1e-3 * s))
+
+
+# ---- P1: true Pascal, L_ij = C(i, j) exactly (closed form) --------------------------------
+@pytest.mark.parametrize("n,nb", [(8, 8), (16, 8), (24, 8), (29, 29)])
+def test_p1_pascal_binomial_factor(n, nb):
+    A = syn.pascal(n)
+    # At n = 29 (cond ~ 1e25) Alg. 2's triangular solve amplifies the rounding of the
+    # (> 2^53) checksums far beyond the Cauchy-Schwarz threshold of reading A4, so V3 raises
+    # false CHK2 alarms there: the factor arithmetic is pinned with the checks off, and the
+    # checked path on the n <= 24 cases (A4 limitation).
+    r = oracle.potrf(A, nb, abft=(n <= 24))
+    assert r.status == 0 and len(r.events) == 0
+    Lx = np.array([[float(math.comb(i, j)) if i >= j else 0.0 for j in range(n)] for i in range(n)])
+    assert np.array_equal(np.tril(r.L), Lx)
+    assert np.array_equal(np.triu(r.L, 1), np.triu(A, 1)), "strict upper triangle must be untouched"
+
+
+# ---- P2: Pascal mod 2 (config C1), L = Lucas, with the C1 injections (golden) -------------
+def _golden_c1():
+    rows = []
+    for line in open(os.path.join(GOLDEN, "c1_events.txt")):
+        line = line.strip()
+        if line and not line.startswith("#"):
+            k, v, ti, tj, row, col, kind, rank = map(int, line.split())
+            rows.append((k, v, tj, ti, col, row, kind, rank))
+    return sorted(rows)
+
+
+def test_p2_pascal_mod2_fault_free():
+    A = syn.pascal_mod2(256)
+    r = oracle.potrf(A, 32)
+    assert r.status == 0 and len(r.events) == 0
+    assert np.array_equal(np.tril(r.L), lucas_L(256))
+
+
+def test_p2_c1_injections_golden_events_and_exact_factor():
+    A = syn.pascal_mod2(256)
+    r = oracle.potrf(A, 32, inj=syn.inj_array(syn.c1_injections()))
+    assert r.status == 0
+    assert r.event_tuples() == _golden_c1()
+    assert np.array_equal(np.tril(r.L), lucas_L(256))      # P7: bit-exact after correction
+    # the schedule predictor agrees with the hand-derived golden file
+    assert sorted(predict(s, 256, 32) for s in syn.c1_injections()) == _golden_c1()
+
+
+def test_p2_four_injections_bits_51_52_55_63():
+    A = syn.pascal_mod2(256)
+    specs = [dict(k=1, hook="REST", row=100, col=70, bit=52),
+             dict(k=3, hook="UPDATE_OUT", row=250, col=140, bit=51),
+             dict(k=2, hook="TRSM_OUT", row=200, col=72, bit=55),
+             dict(k=5, hook="POTRF_OUT", row=170, col=165, bit=63)]
+    r = oracle.potrf(A, 32, inj=syn.inj_array(specs))
+    # an exact-zero element flipped in its sign bit (bit 63) is masked: -0.0 == 0.0
+    live = [s for s in specs if not (s["bit"] == 63 and lucas_L(256)[s["row"], s["col"]] == 0)]
+    assert r.status == 0
+    assert r.event_tuples() == sorted(predict(s, 256, 32) for s in live)
+    assert np.array_equal(np.tril(r.L), lucas_L(256))
+
+
+# ---- P3: brute force vs textbook unblocked Cholesky-Banachiewicz (separate code) ---------
+def banachiewicz(A):
+    n = A.shape[0]
+    L = [[0.0] * n for _ in range(n)]
+    for i in range(n):
+        for j in range(i + 1):
+            s = sum(L[i][p] * L[j][p] for p in range(j))
+            L[i][j] = math.sqrt(A[i, i] - s) if i == j else (A[i, j] - s) / L[j][j]
+    return np.array(L)
+
+
+@pytest.mark.parametrize("n,nb,seed", [(8, 4, 1), (24, 8, 2), (32, 8, 3), (48, 16, 4), (64, 16, 5),
+                                       (64, 32, 6), (60, 12, 7), (9, 3, 8)])
+def test_p3_blocked_vs_unblocked_textbook(n, nb, seed):
+    A = syn.spd_matrix(n, seed=seed)
+    r = oracle.potrf(A, nb)
+    assert r.status == 0 and len(r.events) == 0
+    Lt = banachiewicz(A)
+    s = np.sqrt(np.diag(A))[:, None]
+    assert np.max(np.abs(np.tril(r.L) - Lt) / s) <= 8 * EPS
+
+
+# ---- P4: LAPACK dpotrf at scale; backward error --------------------------------------------
+@pytest.mark.parametrize("n,nb", [(512, 64), (1024, 128), (1536, 256)])
+def test_p4_lapack_and_backward_error(n, nb):
+    A = syn.spd_matrix(n)
+    r = oracle.potrf(A, nb)
+    assert r.status == 0 and len(r.events) == 0
+    Lref = scipy.linalg.cholesky(A, lower=True)
+    assert floor_rel(r.L, Lref, A) <= 1e-11
+    L = np.tril(r.L)
+    be = np.linalg.norm(A - L @ L.T) / np.linalg.norm(A)
+    assert be <= 10 * n * EPS
+
+
+def test_p4_not_spd_info_matches_lapack():
+    n, nb = 96, 16
+    A = syn.spd_matrix(n, seed=3)
+    A[70, 70] = -5.0                       # leading minor of order 71 is not positive
+    r = oracle.potrf(A, nb)
+    _, info = scipy.linalg.lapack.dpotrf(A, lower=1)
+    assert r.status == 2 and r.info == info == 71
+
+
+# ---- P5: checksum maintenance invariants ---------------------
+@pytest.mark.parametrize("n,nb", [(512, 64), (1024, 256)])
+def test_p5_checksums_carried_to_v_tril_L(n, nb):
+    A = syn.spd_matrix(n)
+    r = oracle.potrf(A, nb)
+    N = n // nb
+    L = np.tril(r.L)
+    w = np.arange(1, nb + 1, dtype=np.float64)
+    S1 = r.scales[n:n + N]
+    for I in range(N):
+        for J in range(I + 1):
+            T = L[I * nb:(I + 1) * nb, J * nb:(J + 1) * nb]
+            c1 = r.chk[2 * I, J * nb:(J + 1) * nb]
+            c2 = r.chk[2 * I + 1, J * nb:(J + 1) * nb]
+            tau = 64 * EPS * S1[I]
+            assert np.max(np.abs(T.sum(0) - c1)) <= tau / 64
+            assert np.max(np.abs(w @ T - c2)) <= tau * nb / 64
+    # and every check in the run passed with a wide margin
+    assert r.counts["max_ratio"] <= 2.0 ** -6
+
+
+def test_p5_encode_is_column_sums_of_symmetric_tiles():
+    n, nb = 96, 32
+    A = syn.spd_matrix(n, seed=9)
+    Al = np.tril(A)
+    Asym = Al + np.tril(Al, -1).T
+    chk, scl = oracle.encode(np.asfortranarray(Al + np.triu(np.full((n, n), 7.0), 1)), nb)  # upper is junk
+    w = np.arange(1, nb + 1)
+    for I in range(n // nb):
+        for J in range(I + 1):
+            T = Asym[I * nb:(I + 1) * nb, J * nb:(J + 1) * nb]
+            assert np.allclose(chk[2 * I, J * nb:(J + 1) * nb], T.sum(0), rtol=0, atol=1e-12 * n)
+            assert np.allclose(chk[2 * I + 1, J * nb:(J + 1) * nb], w @ T, rtol=0, atol=1e-12 * n * nb)
+    s = np.sqrt(np.diag(A))
+    assert np.array_equal(scl[:n], s)
+    assert np.allclose(scl[n:n + 3], s.reshape(3, nb).sum(1), rtol=1e-15)
+    assert np.allclose(scl[n + 3:], (s.reshape(3, nb) * w).sum(1), rtol=1e-15)
+
+
+# ---- P6/P7: injection ground truth ------------------------------------------------------------
+def test_p6_exhaustive_rest0_every_lower_element():
+    """Brute force: every lower element of a small matrix, storage error at REST(0), bit 60."""
+    n, nb = 24, 8
+    A = syn.spd_matrix(n, seed=11)
+    ref = oracle.potrf(A, nb)
+    for r_ in range(n):
+        for c_ in range(r_ + 1):
+            spec = dict(k=0, hook="REST", row=r_, col=c_, bit=60)
+            res = oracle.potrf(A, nb, inj=syn.inj_array([spec]))
+            assert res.status == 0
+            assert res.event_tuples() == [predict(spec, n, nb)], (r_, c_)
+            assert floor_rel(res.L, ref.L, A) <= 1e-12
+
+
+@pytest.mark.parametrize("hook", ["REST", "POTRF_OUT", "TRSM_OUT", "UPDATE_OUT"])
+def test_p6_per_iteration_injections(hook):
+    n, nb = 1024, 128
+    A = syn.spd_matrix(n)
+    specs = [s for s in syn.per_iteration_injections(n, nb, bits=(45, 61)) if s["hook"] == hook]
+    ref = oracle.potrf(A, nb)
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs))
+    assert r.status == 0
+    assert r.event_tuples() == sorted(predict(s, n, nb) for s in specs)
+    assert floor_rel(r.L, ref.L, A) <= 1e-11
+
+
+def test_p6_c2_schedule_all_hooks():
+    n, nb = 4096, 256
+    A = syn.spd_matrix(n)
+    specs = syn.per_iteration_injections(n, nb)
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs))
+    assert r.status == 0
+    pred = sorted(predict(s, n, nb) for s in specs)
+    assert r.event_tuples() == pred
+    Lref = scipy.linalg.cholesky(A, lower=True)
+    assert floor_rel(r.L, Lref, A) <= 1e-11
+
+
+@pytest.mark.parametrize("cr_off", [0, 1])
+def test_p6_checksum_row_errors_leave_L_bit_identical(cr_off):
+    n, nb = 512, 64
+    A = syn.spd_matrix(n)
+    specs = [dict(k=1, hook="REST", target="CHK", row=2 * 5 + cr_off, col=3 * nb + 7, bit=55),
+             dict(k=2, hook="REST", target="CHK", row=2 * 2 + cr_off, col=2 * nb + 9, bit=50),
+             dict(k=4, hook="REST", target="CHK", row=2 * 1 + cr_off, col=0 * nb + 3, bit=49)]
+    ref = oracle.potrf(A, nb)
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs))
+    assert r.status == 0
+    assert r.event_tuples() == sorted(predict(s, n, nb) for s in specs)
+    assert np.array_equal(r.L, ref.L)
+
+
+def test_p6_diagonal_tile_symmetric_dedupe():
+    """An error in the stored lower half of an unfactored diagonal tile appears twice in
+    sym(tril(T)) (row r of column c and row c of column r): exactly one event (reading A12)."""
+    n, nb = 256, 32
+    A = syn.spd_matrix(n, seed=5)
+    ref = oracle.potrf(A, nb)
+    for (row, col) in [(100, 97), (127, 96), (200, 200), (230, 224)]:
+        spec = dict(k=2, hook="REST", row=row, col=col, bit=57)
+        r = oracle.potrf(A, nb, inj=syn.inj_array([spec]))
+        assert r.event_tuples() == [predict(spec, n, nb)]
+        assert floor_rel(r.L, ref.L, A) <= 1e-12
+
+
+def test_p6_nonfinite_rule():
+    n, nb = 256, 64
+    A = syn.spd_matrix(n, seed=2)
+    ref = oracle.potrf(A, nb)
+    # bit 62 of an input value in [0.25, 1): exponent 0x3FD/0x3FE -> 0x7FD/0x7FE, |x| >= 4e307;
+    # with row weight >= 41 the weighted recalculation overflows -> non-finite delta ->
+    # NONFINITE, located by argmax |X|. REST(0) reads the input value itself.
+    row = next(r_ for r_ in range(192 + 40, 256) if A[r_, 150] >= 0.25)
+    spec = dict(k=0, hook="REST", row=row, col=150, bit=62)
+    r = oracle.potrf(A, nb, inj=syn.inj_array([spec]))
+    e = predict(spec, n, nb)
+    assert r.event_tuples() == [e[:6] + (KIND["NONFINITE"], 0)]
+    assert floor_rel(r.L, ref.L, A) <= 1e-12
+    # a mask that turns the stored value into a NaN (exponent all ones, mantissa != 0)
+    nanmask = int(np.float64(A[200, 150]).view(np.uint64)) ^ 0x7FF8000000000001
+    spec = dict(k=0, hook="REST", row=200, col=150, xor_mask=nanmask)
+    r = oracle.potrf(A, nb, inj=syn.inj_array([spec]))
+    assert [t[6] for t in r.event_tuples()] == [KIND["NONFINITE"]]
+    assert floor_rel(r.L, ref.L, A) <= 1e-12
+
+
+def test_p6_two_errors_one_column_is_uncorrectable():
+    n, nb = 256, 64
+    A = syn.spd_matrix(n, seed=2)
+    specs = [dict(k=1, hook="REST", row=200, col=150, bit=55),
+             dict(k=1, hook="REST", row=220, col=150, bit=56)]
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs))
+    assert r.status == 1
+    assert [t[6] for t in r.event_tuples()] == [KIND["UNCORRECTABLE"]]
+    assert r.event_tuples()[0][:5] == (1, V["V5"], 2, 3, 150 - 128)
+
+
+def test_p6_masked_small_injection_produces_no_event():
+    n, nb = 512, 64
+    A = syn.spd_matrix(n)
+    spec = dict(k=1, hook="REST", row=300, col=200, bit=2)   # |Delta| ~ 1e-16 << tau
+    r = oracle.potrf(A, nb, inj=syn.inj_array([spec]))
+    assert r.status == 0 and len(r.events) == 0
+
+
+def test_p6_factored_L_storage_error_caught_by_v6():
+    n, nb = 512, 64
+    A = syn.spd_matrix(n)
+    ref = oracle.potrf(A, nb)
+    specs = [dict(k=5, hook="REST", row=300, col=20, bit=50),     # finished panel 0
+             dict(k=8, hook="REST", row=70, col=70, bit=50)]      # finished diagonal L_11 (k = N)
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs))
+    assert r.event_tuples() == sorted(predict(s, n, nb) for s in specs)
+    assert floor_rel(r.L, ref.L, A) <= 1e-12
+
+
+# ---- multi-rank simulation and Opt. 3 --------------------------------------------------------
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_nranks_simulation_matches_single_rank(P):
+    n, nb = 1024, 128
+    A = syn.spd_matrix(n)
+    specs = syn.per_iteration_injections(n, nb, bits=(45, 61))
+    r1 = oracle.potrf(A, nb, inj=syn.inj_array(specs))
+    rP = oracle.potrf(A, nb, inj=syn.inj_array(specs), nranks=P)
+    assert np.array_equal(r1.L, rP.L)
+    assert r1.event_tuples() == [e for e in rP.event_tuples() if e[1] != V["V4R"]]
+
+
+def test_recv_injection_caught_by_receiver():
+    n, nb, P = 1024, 128, 4
+    A = syn.spd_matrix(n)
+    ref = oracle.potrf(A, nb)
+    specs = [dict(k=1, hook="RECV", row=700, col=150, bit=50, rank=3),
+             dict(k=2, hook="RECV", target="CHK", row=2 * 6 + 1, col=2 * nb + 5, bit=50, rank=0)]
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs), nranks=P)
+    assert r.event_tuples() == sorted(predict(s, n, nb) for s in specs)
+    assert floor_rel(r.L, ref.L, A) <= 1e-12
+
+
+@pytest.mark.parametrize("K", [3, 5])
+def test_opt3_verify_every_K(K):
+    n, nb = 1024, 64
+    A = syn.spd_matrix(n)
+    ref = oracle.potrf(A, nb)
+    rK = oracle.potrf(A, nb, K=K)
+    assert np.array_equal(rK.L, ref.L) and len(rK.events) == 0
+    specs = [dict(k=2, hook="REST", row=900, col=700, bit=50),
+             dict(k=4, hook="UPDATE_OUT", row=600, col=330, bit=52)]
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs), K=K)
+    assert r.event_tuples() == sorted(predict(s, n, nb, K=K) for s in specs)
+    assert rK.counts["flops_check"] < ref.counts["flops_check"]
+
+
+# ---- P8: overhead bookkeeping vs the paper's closed forms (Tables III, V) ----------
+def test_p8_counters_leading_terms():
+    n, nb = 2048, 128
+    A = syn.spd_matrix(n)
+    r = oracle.potrf(A, nb)
+    c = r.counts
+    assert abs(c["flops_factor"] / (n ** 3 / 3) - 1) < 3 * nb / n        # N_Cho = n^3/3
+    assert abs(c["flops_chkupd"] / (2 * n ** 3 / (3 * nb)) - 1) < 6 * nb / n  # GEMM row, Table III
+    assert abs(c["flops_encode"] / (2 * n ** 2) - 1) < 2 * nb / n
+    # V5 recalculation ~ 2n^3/(3B) (Table V GEMM, K=1) + O(n^2) for V1-V4, V6
+    assert abs(c["flops_check"] / (2 * n ** 3 / (3 * nb)) - 1) < 12 * nb / n
+
+
+# ---- P9: threshold margin (C_tau = 64 is parity-unpinned by the paper) --------------------
+@pytest.mark.parametrize("n,nb", [(1024, 64), (2048, 512), (2048, 1024), (4096, 256)])
+def test_p9_noise_margin(n, nb):
+    """Fault-free rounding noise, normalised by the threshold, stays below 2^-6 (SURVEY SX2:
+    <= 0.064 eps*scale for n <= 8192, i.e. >= 640x margin to C_tau = 64)."""
+    A = syn.spd_matrix(n)
+    r = oracle.potrf(A, nb)
+    assert r.status == 0 and len(r.events) == 0
+    assert r.counts["max_ratio"] <= 2.0 ** -6
+
+
+def test_verify_entry_detects_and_corrects():
+    n, nb = 256, 64
+    A = np.asfortranarray(np.tril(syn.spd_matrix(n, seed=4)))
+    chk, scl = oracle.encode(A, nb)
+    st, ev, _ = oracle.verify(A.copy(order="F"), nb, chk.copy(order="F"), scl)
+    assert st == 0 and len(ev) == 0
+    B = A.copy(order="F")
+    B[150, 70] += 3.0
+    st, ev, _ = oracle.verify(B, nb, chk.copy(order="F"), scl)
+    assert st == 0 and len(ev) == 1
+    assert (ev[0]["tile_i"], ev[0]["tile_j"], ev[0]["row"], ev[0]["col"]) == (2, 1, 150 - 128, 70 - 64)
+    assert abs(ev[0]["delta1"] - 3.0) < 1e-9 and abs(ev[0]["delta2"] - 3.0 * (150 - 128 + 1)) < 1e-8
+    assert abs(B[150, 70] - A[150, 70]) < 1e-13
