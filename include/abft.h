@@ -1,0 +1,165 @@
+/*
+ * abft.h — C-ABI of the B200-native Enhanced Online-ABFT Cholesky (libabft.so).
+ *
+ * Operation (§III, §IV): factor an SPD n x n FP64 matrix A = L L^T while the
+ * matrix carries two column checksums per nb x nb block (chk1 = v1^T T, chk2 = v2^T T with
+ * v1 = [1..1], v2 = [1, 2, .., nb]; §IV.A). The checksums are carried through
+ * POTRF (Alg. 2), TRSM and the SYRK/GEMM trailing update
+ * (PAPER.md:137-153). Every block is re-verified before it is read (V1-V6 schedule,
+ * SURVEY.md §8c / DESIGN.md §2); a detected error is located from d2/d1
+ * and corrected in place. The MAGMA dpotrf_gpu interface is kept: the
+ * matrix is already in GPU memory, lower storage, overwritten by L.
+ *
+ * Conventions for every entry point:
+ *  - FP64, column-major, lower triangle (uplo = 'L'). The strictly upper triangle of A is
+ *    never read or written.
+ *  - Pointers are DEVICE pointers unless stated otherwise; `stream` is a cudaStream_t
+ *    (declared here as struct CUstream_st* so that this header needs no CUDA include).
+ *  - Everything is stream-ordered on `stream`. A call synchronises the stream exactly once,
+ *    at its end, and only when it must fill a host report (rep != NULL).
+ *  - Return value: 0 OK; -i if argument i is invalid (LAPACK style, 1-based);
+ *    ABFT_UNCORRECTABLE (1); ABFT_NOT_SPD (2); ABFT_ERR_CUDA (3); ABFT_ERR_NCCL (4).
+ *    No C++ exception crosses this boundary. When rep == NULL the call is fully asynchronous
+ *    and statuses 1/2 are not observable (use a report to learn them).
+ *  - Version-1 restriction: n % nb == 0 (all of the paper's sizes are multiples);
+ *    otherwise the nb argument is reported invalid.
+ */
+#ifndef ABFT_H
+#define ABFT_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+struct CUstream_st;
+typedef struct CUstream_st* abft_stream_t;
+
+/* status codes */
+#define ABFT_OK 0
+#define ABFT_UNCORRECTABLE 1
+#define ABFT_NOT_SPD 2
+#define ABFT_ERR_CUDA 3
+#define ABFT_ERR_NCCL 4
+
+/* injection hooks ("computation error" = output
+ * corruption of an operation, "memory error" = storage corruption between verification and use) */
+#define ABFT_HOOK_REST 0       /* storage error at the start of iteration k (k = N: before V6)  */
+#define ABFT_HOOK_POTRF_OUT 1  /* corrupt the output of POTRF(k) / Alg. 2                         */
+#define ABFT_HOOK_TRSM_OUT 2   /* corrupt the output of the panel TRSM(k)                          */
+#define ABFT_HOOK_UPDATE_OUT 3 /* corrupt the output of the trailing update of iteration k        */
+#define ABFT_HOOK_RECV 4       /* (multi-GPU) corrupt rank `rank`'s received copy of panel k      */
+#define ABFT_TGT_DATA 0        /* row, col = global element of A (row >= col)                     */
+#define ABFT_TGT_CHK 1         /* row = checksum row 2I + {0,1}, col = global column (col/nb <= I) */
+
+/* checks (where an event was raised) and event kinds */
+#define ABFT_V1 1   /* pre-read check of the diagonal tile (k,k) before POTRF                */
+#define ABFT_V2 2   /* pre-read check of panel tiles (i>k, k) before TRSM                     */
+#define ABFT_V3 3   /* check of L_kk against the Alg.-2 checksums                             */
+#define ABFT_V4 4   /* check of the solved panel before the trailing update reads it          */
+#define ABFT_V5 5   /* check of every trailing tile after update k                            */
+#define ABFT_V6 6   /* final sweep over L                                                      */
+#define ABFT_V4R 7  /* (multi-GPU) receiver re-check of the broadcast panel                   */
+#define ABFT_KIND_DATA 1          /* one data element located (row = d2/d1 - 1) and corrected   */
+#define ABFT_KIND_NONFINITE 2     /* non-finite delta; located by argmax |X| and corrected       */
+#define ABFT_KIND_CHK1 3          /* checksum row 1 corrupted; recomputed from the data          */
+#define ABFT_KIND_CHK2 4          /* checksum row 2 corrupted; recomputed from the data          */
+#define ABFT_KIND_UNCORRECTABLE 5 /* more than one error in a tile column: abort (status 1)      */
+
+typedef struct abft_inject_spec {
+    int32_t k, hook, target, pad0;
+    int64_t row, col;
+    uint64_t xor_mask;  /* XOR-ed into the 64-bit pattern of the stored double */
+    int32_t rank, pad1; /* RECV only */
+} abft_inject_spec_t;   /* host array, terminated by an entry with k = -1 */
+
+typedef struct abft_event {
+    int32_t k, check, tile_i, tile_j;
+    int32_t row, col;   /* inside the tile; the stored (lower) element for diagonal tiles;
+                           row = -1 / -2 for CHK1 / CHK2, -3 for UNCORRECTABLE              */
+    int32_t kind, rank;
+    double delta1, delta2;
+} abft_event_t;
+
+typedef struct abft_report {
+    int64_t info;       /* LAPACK info: 1-based order of the first non-positive leading minor */
+    int64_t n_checks, n_detected, n_data, n_nonfinite, n_chk1, n_chk2, n_uncorrectable;
+    int64_t n_events;   /* events raised (may exceed cap; only cap are stored)               */
+    int64_t cap;        /* capacity of `events` (set by the caller)                          */
+    abft_event_t* events; /* HOST array owned by the caller, sorted by (k, check, J, I, col, row) */
+    double seconds;     /* device time of the call (CUDA events on `stream`)                 */
+} abft_report_t;
+
+typedef struct abft_options {
+    int32_t abft_enabled; /* 1: Enhanced Online-ABFT; 0: the same kernels with every checksum
+                             operation, check and encode removed (overhead baseline)            */
+    int32_t K;            /* Opt. 3: V5 every K iterations; 1 = every one   */
+    double c_tau;         /* threshold constant C_tau of reading A4 (default 64)               */
+    int32_t lookahead;    /* reserved (0/1)                                                    */
+    int32_t pad;
+} abft_options_t;
+
+/* Checksum encoding (§IV.A, cost 2n^2).
+ * A: n x n lower (lda >= max(1,n)); chk: 2N x n output (ldchk >= 2N, N = n/nb): row 2I is
+ * v1^T T(I,J), row 2I+1 is v2^T T(I,J) for I >= J (diagonal tiles as sym(tril(T)));
+ * scales: output, n + 2N doubles = [s_i = sqrt(A_ii) | S1_I | S2_I] (threshold scales, A4).
+ * Errors: -1 n<0, -2 nb<1 or n%nb, -3 A NULL, -4 lda, -5 chk NULL, -6 ldchk, -7 scales NULL. */
+int abft_encode(int64_t n, int64_t nb, const double* A, int64_t lda, double* chk, int64_t ldchk,
+                double* scales, abft_stream_t stream);
+
+/* One detect/locate/correct sweep (§IV.C) over every lower tile I >= J.
+ * factored = 1 checks L (diagonal tiles as tril), 0 checks an unfactored matrix (sym).
+ * correct = 0 only reports. Events carry k = -1, check = V6 (factored) or V5.
+ * rep may be NULL (no sync). Errors as abft_encode, -8 factored, -9 correct. */
+int abft_verify(int64_t n, int64_t nb, double* A, int64_t lda, double* chk, int64_t ldchk,
+                const double* scales, int factored, int correct, abft_stream_t stream,
+                abft_report_t* rep);
+
+/* Enhanced Online-ABFT Cholesky, A = L L^T in place (lower). Workspace (checksums, scales,
+ * panel buffer, event buffer: about n*nb + 2n^2/nb doubles) is allocated with cudaMallocAsync
+ * on `stream` and freed before return. inj: HOST list (NULL = none), validated up front
+ * (-6 on an out-of-range target/hook). rep: HOST report (NULL = asynchronous, no report).
+ * Errors: -1 n, -2 nb, -3 A, -4 lda, -6 inj. */
+int abft_potrf(int64_t n, int64_t nb, double* A, int64_t lda, abft_stream_t stream,
+               const abft_inject_spec_t* inj, abft_report_t* rep);
+
+/* As abft_potrf with options (NULL = defaults: ABFT on, K = 1, C_tau = 64). -8 bad options. */
+int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft_stream_t stream,
+                  const abft_inject_spec_t* inj, abft_report_t* rep, const abft_options_t* opt);
+
+/* End-to-end variant on HOST memory (A_host: n x n column-major, lda >= n; pinned memory
+ * recommended): copies A to the device, factors with abft_potrf_ex, copies L back, all on
+ * `stream`, then synchronises. Same errors as abft_potrf_ex. */
+int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t lda, abft_stream_t stream,
+                    const abft_inject_spec_t* inj, abft_report_t* rep, const abft_options_t* opt);
+
+/* Synthetic SPD input of reading A15 (the same counter-based generator as synthetic/):
+ * A[i,j] = A[j,i] = U(splitmix64(seed*n^2 + max(i,j)*n + min(i,j))), A[i,i] += n.
+ * Writes the full n x n matrix. Errors: -1 n, -3 A, -4 lda. */
+int abft_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, abft_stream_t stream);
+
+/* ---- multi-GPU (one process per GPU, 1D block-cyclic block columns, NCCL panel broadcast) ---
+ * abft_nccl_id: fill 128 bytes (ncclUniqueId) on rank 0, share them out of band.
+ * abft_comm_init: create the communicator for `rank` of `nranks` on the current device.
+ * abft_potrf_dist: rank r owns block columns {j : j mod nranks == r}, stored contiguously in
+ * A_local (n x (n_local_cols) column-major, lda_local >= n, local block column t is global
+ * block column t*nranks + r). Same semantics and report as abft_potrf; events of all ranks are
+ * gathered into rank 0's report (other ranks report their own). Errors as abft_potrf, 4 NCCL. */
+int abft_nccl_id(void* id128);
+int abft_comm_init(void** comm, int nranks, const void* id128, int rank);
+int abft_comm_destroy(void* comm);
+int abft_potrf_dist(int64_t n, int64_t nb, double* A_local, int64_t lda_local, void* comm, int rank,
+                    int nranks, abft_stream_t stream, const abft_inject_spec_t* inj,
+                    abft_report_t* rep, const abft_options_t* opt);
+
+/* Diagnostics: kernel launches issued by the last call on this thread, a static version string,
+ * and the text of the last CUDA error seen on this thread (empty if none). */
+int64_t abft_last_launch_count(void);
+const char* abft_version(void);
+const char* abft_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ABFT_H */

@@ -1,0 +1,248 @@
+"""Thin ctypes binding of libabft.so (include/abft.h) — argument marshalling only.
+
+Every step of the factorisation runs in the CUDA kernels of csrc/; this module never computes
+anything itself and has no CPU fallback: importing it on a machine where libabft.so is missing
+raises, and calling into it without a CUDA device fails inside the library.
+
+Names follow the C-ABI: abft_potrf, abft_potrf_ex, abft_potrf_host, abft_encode, abft_verify,
+abft_gen_spd, abft_nccl_id, abft_comm_init, abft_comm_destroy, abft_potrf_dist.
+Device buffers are passed as torch CUDA tensors (float64, column-major = a transposed view of a
+contiguous row-major tensor, or any tensor whose column stride is 1) or as raw integer device
+pointers; streams default to torch's current stream.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libabft.so")
+
+# Codes restated from include/abft.h
+OK, UNCORRECTABLE, NOT_SPD, ERR_CUDA, ERR_NCCL = 0, 1, 2, 3, 4
+HOOK = {"REST": 0, "POTRF_OUT": 1, "TRSM_OUT": 2, "UPDATE_OUT": 3, "RECV": 4}
+CHECK = {1: "V1", 2: "V2", 3: "V3", 4: "V4", 5: "V5", 6: "V6", 7: "V4R"}
+KIND = {1: "DATA", 2: "NONFINITE", 3: "CHK1", 4: "CHK2", 5: "UNCORRECTABLE"}
+
+EVENT_DTYPE = np.dtype([
+    ("k", "<i4"), ("check", "<i4"), ("tile_i", "<i4"), ("tile_j", "<i4"),
+    ("row", "<i4"), ("col", "<i4"), ("kind", "<i4"), ("rank", "<i4"),
+    ("delta1", "<f8"), ("delta2", "<f8"),
+])
+INJ_DTYPE = np.dtype([
+    ("k", "<i4"), ("hook", "<i4"), ("target", "<i4"), ("pad0", "<i4"),
+    ("row", "<i8"), ("col", "<i8"), ("xor_mask", "<u8"), ("rank", "<i4"), ("pad1", "<i4"),
+])
+
+
+class Event(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int32) for n in ("k", "check", "tile_i", "tile_j", "row", "col", "kind", "rank")] + \
+               [("delta1", ctypes.c_double), ("delta2", ctypes.c_double)]
+
+
+class Report(ctypes.Structure):
+    _fields_ = [("info", ctypes.c_int64), ("n_checks", ctypes.c_int64), ("n_detected", ctypes.c_int64),
+                ("n_data", ctypes.c_int64), ("n_nonfinite", ctypes.c_int64), ("n_chk1", ctypes.c_int64),
+                ("n_chk2", ctypes.c_int64), ("n_uncorrectable", ctypes.c_int64), ("n_events", ctypes.c_int64),
+                ("cap", ctypes.c_int64), ("events", ctypes.c_void_p), ("seconds", ctypes.c_double)]
+
+
+class Options(ctypes.Structure):
+    _fields_ = [("abft_enabled", ctypes.c_int32), ("K", ctypes.c_int32), ("c_tau", ctypes.c_double),
+                ("lookahead", ctypes.c_int32), ("pad", ctypes.c_int32)]
+
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"libabft.so not built ({LIB_PATH}); run `python paper_conf_ipps_chenlc16_b200/build.py` "
+                      "(there is no CPU fallback)")
+_lib = ctypes.CDLL(LIB_PATH)
+_i64, _i32, _vp, _dbl = ctypes.c_int64, ctypes.c_int, ctypes.c_void_p, ctypes.c_double
+_lib.abft_encode.argtypes = [_i64, _i64, _vp, _i64, _vp, _i64, _vp, _vp]
+_lib.abft_verify.argtypes = [_i64, _i64, _vp, _i64, _vp, _i64, _vp, _i32, _i32, _vp, _vp]
+_lib.abft_potrf.argtypes = [_i64, _i64, _vp, _i64, _vp, _vp, _vp]
+_lib.abft_potrf_ex.argtypes = [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _vp]
+_lib.abft_potrf_host.argtypes = [_i64, _i64, _vp, _i64, _vp, _vp, _vp, _vp]
+_lib.abft_gen_spd.argtypes = [_i64, ctypes.c_uint64, _vp, _i64, _vp]
+_lib.abft_nccl_id.argtypes = [_vp]
+_lib.abft_comm_init.argtypes = [ctypes.POINTER(_vp), _i32, _vp, _i32]
+_lib.abft_comm_destroy.argtypes = [_vp]
+_lib.abft_potrf_dist.argtypes = [_i64, _i64, _vp, _i64, _vp, _i32, _i32, _vp, _vp, _vp, _vp]
+_lib.abft_last_launch_count.restype = _i64
+_lib.abft_version.restype = ctypes.c_char_p
+_lib.abft_last_error.restype = ctypes.c_char_p
+for _f in ("abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
+           "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist"):
+    getattr(_lib, _f).restype = _i32
+
+EXPORTS = ["abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
+           "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist",
+           "abft_last_launch_count", "abft_version", "abft_last_error"]
+
+
+def lib():
+    return _lib
+
+
+# ---- marshalling helpers ---------------------------------------------------------------------
+def _dev(x):
+    """(pointer, leading dimension) of a column-major float64 CUDA tensor, or (int, None)."""
+    if x is None:
+        return None, None
+    if isinstance(x, int):
+        return x, None
+    import torch
+    assert x.is_cuda and x.dtype == torch.float64, "expected a float64 CUDA tensor"
+    if x.dim() == 1:
+        return x.data_ptr(), None
+    assert x.stride(0) == 1, "expected column-major storage (stride(0) == 1)"
+    return x.data_ptr(), x.stride(1)
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        return torch.cuda.current_stream().cuda_stream
+    return getattr(stream, "cuda_stream", stream)
+
+
+def _inj(inj):
+    if inj is None:
+        return None, None
+    arr = np.ascontiguousarray(inj, dtype=INJ_DTYPE)
+    if len(arr) == 0 or arr[-1]["k"] != -1:
+        arr = np.concatenate([arr, np.zeros(1, INJ_DTYPE)])
+        arr[-1]["k"] = -1
+    return arr, arr.ctypes.data
+
+
+def _new_report(cap):
+    ev = np.zeros(max(cap, 1), dtype=EVENT_DTYPE)
+    rep = Report()
+    rep.cap = cap
+    rep.events = ev.ctypes.data
+    return rep, ev
+
+
+def _report_dict(rep, ev):
+    n = min(rep.n_events, rep.cap)
+    return dict(info=rep.info, n_checks=rep.n_checks, n_detected=rep.n_detected, n_data=rep.n_data,
+                n_nonfinite=rep.n_nonfinite, n_chk1=rep.n_chk1, n_chk2=rep.n_chk2,
+                n_uncorrectable=rep.n_uncorrectable, n_events=rep.n_events, events=ev[:n].copy(),
+                seconds=rep.seconds)
+
+
+def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0):
+    return Options(int(bool(abft_enabled)), int(K), float(c_tau), int(lookahead), 0)
+
+
+# ---- entry points (same names as the C-ABI) --------------------------------------------------
+def abft_potrf_ex(n, nb, A, lda=None, stream=None, inj=None, report=True, cap=1 << 16, opt=None):
+    """Factor A (n x n float64 CUDA, column-major) in place. Returns (status, report|None)."""
+    p, ld = _dev(A)
+    lda = lda if lda is not None else (ld if ld is not None else n)
+    arr, pinj = _inj(inj)
+    rep, ev = _new_report(cap) if report else (None, None)
+    o = opt if opt is not None else options()
+    st = _lib.abft_potrf_ex(n, nb, p, lda, _stream(stream), pinj, ctypes.byref(rep) if rep else None,
+                            ctypes.byref(o))
+    return st, (_report_dict(rep, ev) if rep else None)
+
+
+def abft_potrf(n, nb, A, lda=None, stream=None, inj=None, report=True, cap=1 << 16):
+    return abft_potrf_ex(n, nb, A, lda, stream, inj, report, cap, None)
+
+
+def abft_potrf_host(n, nb, A_host, lda=None, stream=None, inj=None, report=True, cap=1 << 16, opt=None):
+    """A_host: numpy float64 array, Fortran order (or a raw pointer + lda). Pinned memory is the
+    caller's choice (e.g. a torch pinned tensor's .numpy() view)."""
+    if isinstance(A_host, np.ndarray):
+        assert A_host.dtype == np.float64 and A_host.flags.f_contiguous
+        p, lda = A_host.ctypes.data, (lda or A_host.shape[0])
+    else:
+        p = A_host
+    arr, pinj = _inj(inj)
+    rep, ev = _new_report(cap) if report else (None, None)
+    o = opt if opt is not None else options()
+    st = _lib.abft_potrf_host(n, nb, p, lda, _stream(stream), pinj, ctypes.byref(rep) if rep else None,
+                              ctypes.byref(o))
+    return st, (_report_dict(rep, ev) if rep else None)
+
+
+def abft_encode(n, nb, A, chk, scales, lda=None, ldchk=None, stream=None):
+    pa, la = _dev(A)
+    pc, lc = _dev(chk)
+    ps, _ = _dev(scales)
+    return _lib.abft_encode(n, nb, pa, lda or la or n, pc, ldchk or lc or max(1, 2 * (n // nb)), ps,
+                            _stream(stream))
+
+
+def abft_verify(n, nb, A, chk, scales, factored=False, correct=True, lda=None, ldchk=None, stream=None,
+                report=True, cap=1 << 16):
+    pa, la = _dev(A)
+    pc, lc = _dev(chk)
+    ps, _ = _dev(scales)
+    rep, ev = _new_report(cap) if report else (None, None)
+    st = _lib.abft_verify(n, nb, pa, lda or la or n, pc, ldchk or lc or max(1, 2 * (n // nb)), ps,
+                          int(factored), int(correct), _stream(stream), ctypes.byref(rep) if rep else None)
+    return st, (_report_dict(rep, ev) if rep else None)
+
+
+def abft_gen_spd(n, A, seed=None, lda=None, stream=None):
+    p, ld = _dev(A)
+    return _lib.abft_gen_spd(n, n if seed is None else seed, p, lda or ld or n, _stream(stream))
+
+
+def abft_nccl_id():
+    buf = ctypes.create_string_buffer(128)
+    st = _lib.abft_nccl_id(buf)
+    return st, bytes(buf.raw)
+
+
+def abft_comm_init(nranks, id128, rank):
+    comm = ctypes.c_void_p()
+    buf = ctypes.create_string_buffer(bytes(id128), 128)
+    st = _lib.abft_comm_init(ctypes.byref(comm), nranks, buf, rank)
+    return st, comm.value
+
+
+def abft_comm_destroy(comm):
+    return _lib.abft_comm_destroy(comm)
+
+
+def abft_potrf_dist(n, nb, A_local, comm, rank, nranks, lda=None, stream=None, inj=None, report=True,
+                    cap=1 << 16, opt=None):
+    p, ld = _dev(A_local)
+    arr, pinj = _inj(inj)
+    rep, ev = _new_report(cap) if report else (None, None)
+    o = opt if opt is not None else options()
+    st = _lib.abft_potrf_dist(n, nb, p, lda or ld or n, comm, rank, nranks, _stream(stream), pinj,
+                              ctypes.byref(rep) if rep else None, ctypes.byref(o))
+    return st, (_report_dict(rep, ev) if rep else None)
+
+
+def abft_last_launch_count():
+    return int(_lib.abft_last_launch_count())
+
+
+def abft_version():
+    return _lib.abft_version().decode()
+
+
+def sorted_event_tuples(events):
+    """(k, V, J, I, col, row, kind, rank) — the parity key shared with the oracle's tests."""
+    return sorted((int(e["k"]), int(e["check"]), int(e["tile_j"]), int(e["tile_i"]), int(e["col"]),
+                   int(e["row"]), int(e["kind"]), int(e["rank"])) for e in events)
+
+
+def colmajor(A_np, device="cuda"):
+    """Upload a numpy (any order) n x n matrix as a column-major float64 CUDA tensor view."""
+    import torch
+    t = torch.from_numpy(np.ascontiguousarray(np.asarray(A_np, dtype=np.float64).T)).to(device)
+    return t.T   # stride(0) == 1
+
+
+def to_numpy_colmajor(At):
+    """Download a column-major CUDA tensor view into a Fortran-ordered numpy array."""
+    return np.asfortranarray(At.T.contiguous().cpu().numpy().T)

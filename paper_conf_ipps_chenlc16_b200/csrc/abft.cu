@@ -1,0 +1,391 @@
+// abft.cu — the C-ABI entry points and the single-GPU factorisation driver.
+//
+// Iteration k of the right-looking Enhanced Online-ABFT Cholesky (reading A1; the paper's
+// Alg. 1 is left-looking), with verification before every read
+// in the V1..V6 schedule of DESIGN.md §2:
+//   REST(k) hook -> V1/V2 check of block column k (pre-read, unfactored)
+//   POTRF + inv(L_kk)  (potrf.cu)
+//   TRSM: W = [A(k+1:N,k); chk(k:N,k)] * inv(L_kk)^T  -- one DMMA GEMM that also performs Alg. 2
+//         on the checksum rows of tile (k,k)
+//   POTRF_OUT hook -> V3 (L_kk vs Alg.-2 checksums);  TRSM_OUT hook -> V4 (solved panel, in W)
+//   write-back W -> A panel, chk
+//   trailing SYRK/GEMM: A(trail) -= W_d W_d^T (lower), chk(trail) -= W_c W_d^T
+//   UPDATE_OUT hook -> V5 (every trailing tile, every K-th iteration: Opt. 3)
+// then REST(N) -> V6 over L. Everything is stream-ordered; the only host sync is the final
+// report copy. An UNCORRECTABLE / NOT_SPD sets a device abort flag that every later kernel
+// checks at entry.
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <vector>
+
+#include "common.cuh"
+
+using namespace abft;
+
+int launch_check(const StageArgs& a, cudaStream_t s);
+int launch_scales(int64_t n, int64_t nb, const double* A, int64_t lda, double* scl, cudaStream_t s);
+int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
+                int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
+                int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
+                cudaStream_t s, int force_tile = 0);
+int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,
+                const int32_t* abort_flag, cudaStream_t s);
+int launch_zero(int64_t rows, int64_t cols, double* dst, int64_t ldd, cudaStream_t s);
+int launch_chol_inv(double* T, int64_t ldt, double* Li, int64_t B, int64_t info_off, double* tmp,
+                    DevState* st, cudaStream_t s);
+int launch_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, cudaStream_t s);
+int launch_inject(int nops, double* const* ptrs, const uint64_t* masks, const int32_t* abort_flag,
+                  cudaStream_t s);
+
+// ---- diagnostics --------------------------------------------------------------------------
+static thread_local int64_t g_launches = 0;
+static thread_local char g_err[256] = {0};
+void abft_count_launch(int n) { g_launches += n; }
+void abft_set_error(cudaError_t e, const char* what) {
+    snprintf(g_err, sizeof g_err, "%s: %s", what, cudaGetErrorString(e));
+}
+extern "C" int64_t abft_last_launch_count(void) { return g_launches; }
+extern "C" const char* abft_version(void) {
+    return "libabft 0.1 (sm_100a, DMMA f64; Enhanced Online-ABFT Cholesky, Chen-Liang-Chen IPDPS'16)";
+}
+extern "C" const char* abft_last_error(void) { return g_err; }
+
+// ---- argument checking ----------------------------------------------------------------------
+static int check_common(int64_t n, int64_t nb, const void* A, int64_t lda) {
+    if (n < 0) return -1;
+    if (nb < 1 || n % nb != 0) return -2;
+    if (A == nullptr && n > 0) return -3;
+    if (lda < std::max<int64_t>(1, n)) return -4;
+    return 0;
+}
+
+// Injection specs: validated against the region their hook can touch.
+static int collect_inj(const abft_inject_spec_t* inj, int64_t n, int64_t nb, std::vector<abft_inject_spec_t>& out) {
+    out.clear();
+    if (!inj) return 0;
+    const int64_t N = n / nb;
+    for (int t = 0; inj[t].k != -1; ++t) {
+        const abft_inject_spec_t& s = inj[t];
+        if (t > 1 << 20) return -1;
+        if (s.hook < ABFT_HOOK_REST || s.hook > ABFT_HOOK_RECV) return -1;
+        if (s.target != ABFT_TGT_DATA && s.target != ABFT_TGT_CHK) return -1;
+        if (s.k < 0 || s.k > N || (s.hook != ABFT_HOOK_REST && s.k >= N)) return -1;
+        int64_t I, J;
+        if (s.target == ABFT_TGT_DATA) {
+            if (s.col < 0 || s.row < s.col || s.row >= n) return -1;
+            I = s.row / nb; J = s.col / nb;
+        } else {
+            if (s.row < 0 || s.row >= 2 * N || s.col < 0 || s.col >= n) return -1;
+            I = s.row / 2; J = s.col / nb;
+            if (J > I) return -1;
+        }
+        const int64_t k = s.k;
+        switch (s.hook) {
+            case ABFT_HOOK_POTRF_OUT: if (!(I == k && J == k)) return -1; break;
+            case ABFT_HOOK_TRSM_OUT: if (!(J == k && I > k)) return -1; break;
+            case ABFT_HOOK_UPDATE_OUT: if (!(J > k)) return -1; break;
+            case ABFT_HOOK_RECV: if (!(J == k && I > k)) return -1; break;
+            default: break;
+        }
+        out.push_back(s);
+    }
+    return 0;
+}
+
+// ---- workspace -------------------------------------------------------------------------------
+struct Work {
+    int64_t n, nb, N;
+    double* chk = nullptr; int64_t ldc = 1;
+    double* scl = nullptr;
+    double* W = nullptr;
+    double* Li = nullptr;
+    double* tmp = nullptr;
+    DevState* st = nullptr;
+    abft_event_t* ev = nullptr; int64_t ev_cap = 0;
+};
+
+static int work_alloc(Work& w, int64_t n, int64_t nb, int64_t ncols_local, int64_t ev_cap, bool abft, cudaStream_t s) {
+    w.n = n; w.nb = nb; w.N = n / nb;
+    const int64_t N = w.N;
+    w.ldc = std::max<int64_t>(1, 2 * N);
+    if (abft) {
+        ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.chk, sizeof(double) * (size_t)(w.ldc * std::max<int64_t>(1, ncols_local)), s));
+        ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.scl, sizeof(double) * (size_t)(n + 2 * N + 1), s));
+    }
+    const int64_t wrows = (N - 1) * nb + 2 * N + 2;
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.W, sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb), s));
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.Li, sizeof(double) * (size_t)(nb * nb), s));
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.tmp, sizeof(double) * (size_t)(((nb + 1) / 2 + 64) * ((nb + 1) / 2 + 64)), s));
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.st, sizeof(DevState), s));
+    ABFT_CUDA_TRY(cudaMemsetAsync(w.st, 0, sizeof(DevState), s));
+    w.ev_cap = std::max<int64_t>(ev_cap, 1);
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.ev, sizeof(abft_event_t) * (size_t)w.ev_cap, s));
+    return 0;
+}
+
+static void work_free(Work& w, cudaStream_t s) {
+    if (w.chk) cudaFreeAsync(w.chk, s);
+    if (w.scl) cudaFreeAsync(w.scl, s);
+    if (w.W) cudaFreeAsync(w.W, s);
+    if (w.Li) cudaFreeAsync(w.Li, s);
+    if (w.tmp) cudaFreeAsync(w.tmp, s);
+    if (w.st) cudaFreeAsync(w.st, s);
+    if (w.ev) cudaFreeAsync(w.ev, s);
+    w = Work();
+}
+
+static StageArgs stage_base(const Work& w, double* A, int64_t lda, double c_tau, int kind, int V, int k) {
+    StageArgs a;
+    memset(&a, 0, sizeof a);
+    a.kind = kind; a.V = V; a.k = k; a.factored = 0; a.correct = 1; a.rank = 0; a.encode = 0;
+    a.n = w.n; a.nb = w.nb; a.N = w.N;
+    a.A = A; a.lda = lda; a.chk = w.chk; a.ldc = w.ldc; a.W = w.W; a.ldw = 1; a.mB = 0;
+    a.s = w.scl; a.S1 = w.scl ? w.scl + w.n : nullptr; a.S2 = w.scl ? w.scl + w.n + w.N : nullptr;
+    a.c_tau = c_tau; a.col_owner_mod = 1; a.col_owner_rank = 0;
+    a.st = w.st; a.ev = w.ev; a.ev_cap = w.ev_cap;
+    return a;
+}
+
+// Fill the host report from the device state (the one synchronisation of a call).
+static int finish_report(const Work& w, abft_report_t* rep, cudaStream_t s, int* status_out) {
+    DevState hs;
+    ABFT_CUDA_TRY(cudaMemcpyAsync(&hs, w.st, offsetof(DevState, flags), cudaMemcpyDeviceToHost, s));
+    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+    const int64_t nev = (int64_t)hs.nev;
+    if (rep) {
+        rep->info = hs.info;
+        rep->n_checks = (int64_t)hs.n_checks; rep->n_detected = hs.n_detected; rep->n_data = hs.n_data;
+        rep->n_nonfinite = hs.n_nonfinite; rep->n_chk1 = hs.n_chk1; rep->n_chk2 = hs.n_chk2;
+        rep->n_uncorrectable = hs.n_unc; rep->n_events = nev;
+        const int64_t ncopy = std::min<int64_t>(std::min<int64_t>(nev, w.ev_cap), std::max<int64_t>(rep->cap, 0));
+        if (ncopy > 0 && rep->events) {
+            ABFT_CUDA_TRY(cudaMemcpy(rep->events, w.ev, sizeof(abft_event_t) * (size_t)ncopy, cudaMemcpyDeviceToHost));
+            std::sort(rep->events, rep->events + ncopy, [](const abft_event_t& x, const abft_event_t& y) {
+                if (x.k != y.k) return x.k < y.k;
+                if (x.check != y.check) return x.check < y.check;
+                if (x.tile_j != y.tile_j) return x.tile_j < y.tile_j;
+                if (x.tile_i != y.tile_i) return x.tile_i < y.tile_i;
+                if (x.col != y.col) return x.col < y.col;
+                if (x.row != y.row) return x.row < y.row;
+                return x.rank < y.rank;
+            });
+        }
+    }
+    *status_out = hs.status;
+    return 0;
+}
+
+// Injection pointer at hook time (where the element lives at that moment).
+struct Loc { double* A; int64_t lda; double* chk; int64_t ldc; double* W; int64_t ldw; int64_t mB; };
+
+static double* inj_ptr(const abft_inject_spec_t& s, int64_t k, int64_t nb, const Loc& L) {
+    const int hook = s.hook;
+    if (hook == ABFT_HOOK_TRSM_OUT || hook == ABFT_HOOK_POTRF_OUT) {
+        if (s.target == ABFT_TGT_DATA) {
+            if (hook == ABFT_HOOK_TRSM_OUT)
+                return L.W + (s.col - k * nb) * L.ldw + (s.row - (k + 1) * nb);
+            return L.A + s.col * L.lda + s.row;
+        }
+        return L.W + (s.col - k * nb) * L.ldw + L.mB + (s.row - 2 * k);
+    }
+    if (s.target == ABFT_TGT_DATA) return L.A + s.col * L.lda + s.row;
+    return L.chk + s.col * L.ldc + s.row;
+}
+
+static void do_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, int hook, int64_t nb, const Loc& L,
+                      const int32_t* ab, cudaStream_t s) {
+    std::vector<double*> ptrs; std::vector<uint64_t> masks;
+    for (const auto& sp : list)
+        if (sp.k == k && sp.hook == hook) { ptrs.push_back(inj_ptr(sp, k, nb, L)); masks.push_back(sp.xor_mask); }
+    if (!ptrs.empty()) launch_inject((int)ptrs.size(), ptrs.data(), masks.data(), ab, s);
+}
+
+static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t s,
+                     const std::vector<abft_inject_spec_t>& inj, abft_report_t* rep, const abft_options_t& o) {
+    const bool abft = o.abft_enabled != 0;
+    const int K = std::max(1, o.K);
+    Work w;
+    int rc = work_alloc(w, n, nb, n, rep ? std::max<int64_t>(rep->cap, 1) : 1024, abft, s);
+    if (rc) return rc;
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (rep) { cudaEventCreate(&e0); cudaEventCreate(&e1); cudaEventRecord(e0, s); }
+    const int64_t N = w.N, B = nb;
+    const int32_t* ab = &w.st->abort;
+    launch_zero(B, B, w.Li, B, s);
+    if (abft) {   // encode
+        launch_scales(n, nb, A, lda, w.scl, s);
+        StageArgs a = stage_base(w, A, lda, o.c_tau, SK_ALL, 0, -1);
+        a.encode = 1;
+        launch_check(a, s);
+    }
+    for (int64_t k = 0; k < N; ++k) {
+        const int64_t m = N - k - 1, mB = m * B;
+        const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
+        double* Akk = A + k * B * lda + k * B;
+        const Loc L{A, lda, w.chk, w.ldc, w.W, ldw, mB};
+        if (abft) {
+            do_inject(inj, k, ABFT_HOOK_REST, B, L, ab, s);
+            launch_check(stage_base(w, A, lda, o.c_tau, SK_COLUMN, ABFT_V2, (int)k), s);   // V1, V2
+        }
+        launch_chol_inv(Akk, lda, w.Li, B, k * B, w.tmp, w.st, s);
+        // TRSM (+ Alg. 2 on the checksum rows of tile (k,k)): one GEMM per row segment
+        launch_gemm(mB, B, B, Akk + B, lda, w.Li, B, w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, s);
+        if (abft) {
+            launch_gemm(2 * m + 2, B, B, w.chk + k * B * w.ldc + 2 * k, w.ldc, w.Li, B, w.W + mB, ldw, 1.0, 0.0,
+                        true, 0, 1, 0, 0, 0, ab, s);
+            do_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, L, ab, s);
+            StageArgs a3 = stage_base(w, A, lda, o.c_tau, SK_DIAG_FACT, ABFT_V3, (int)k);
+            a3.W = w.W; a3.ldw = ldw; a3.mB = mB;
+            launch_check(a3, s);                                                          // V3
+            do_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, L, ab, s);
+            StageArgs a4 = stage_base(w, A, lda, o.c_tau, SK_PANEL, ABFT_V4, (int)k);
+            a4.W = w.W; a4.ldw = ldw; a4.mB = mB;
+            launch_check(a4, s);                                                          // V4
+        }
+        launch_copy(mB, B, w.W, ldw, Akk + B, lda, ab, s);                                // L panel
+        if (abft) launch_copy(2 * m + 2, B, w.W + mB, ldw, w.chk + k * B * w.ldc + 2 * k, w.ldc, ab, s);
+        if (m > 0) {
+            double* Atr = Akk + B * lda + B;
+            launch_gemm(mB, mB, B, w.W, ldw, w.W, ldw, Atr, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
+            if (abft) {
+                launch_gemm(2 * m, mB, B, w.W + mB + 2, ldw, w.W, ldw, w.chk + (k + 1) * B * w.ldc + 2 * (k + 1),
+                            w.ldc, -1.0, 1.0, true, 2, 0, B, 0, 0, ab, s);
+                do_inject(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s);
+                if (((k + 1) % K == 0) || k == N - 2)
+                    launch_check(stage_base(w, A, lda, o.c_tau, SK_TRAIL, ABFT_V5, (int)k), s);  // V5
+            }
+        }
+    }
+    if (abft) {
+        const Loc L{A, lda, w.chk, w.ldc, w.W, 1, 0};
+        do_inject(inj, N, ABFT_HOOK_REST, B, L, ab, s);
+        StageArgs a6 = stage_base(w, A, lda, o.c_tau, SK_ALL, ABFT_V6, (int)N);
+        a6.factored = 1;
+        launch_check(a6, s);                                                              // V6
+    }
+    ABFT_CUDA_TRY(cudaGetLastError());
+    int status = 0;
+    if (rep) {
+        cudaEventRecord(e1, s);
+        rc = finish_report(w, rep, s, &status);
+        float ms = 0; cudaEventElapsedTime(&ms, e0, e1);
+        rep->seconds = ms * 1e-3;
+        cudaEventDestroy(e0); cudaEventDestroy(e1);
+    }
+    work_free(w, s);
+    if (rc) return rc;
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return status;
+}
+
+static abft_options_t default_options() {
+    abft_options_t o;
+    memset(&o, 0, sizeof o);
+    o.abft_enabled = 1; o.K = 1; o.c_tau = 64.0; o.lookahead = 0;
+    return o;
+}
+
+extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft_stream_t stream,
+                             const abft_inject_spec_t* inj, abft_report_t* rep, const abft_options_t* opt) {
+    g_launches = 0;
+    int rc = check_common(n, nb, A, lda);
+    if (rc) return rc;
+    abft_options_t o = opt ? *opt : default_options();
+    if (o.K < 1 || !(o.c_tau > 0)) return -8;
+    std::vector<abft_inject_spec_t> list;
+    if (collect_inj(inj, n, nb, list)) return -6;
+    if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; }
+    if (n == 0) return 0;
+    return run_potrf(n, nb, A, lda, (cudaStream_t)stream, list, rep, o);
+}
+
+extern "C" int abft_potrf(int64_t n, int64_t nb, double* A, int64_t lda, abft_stream_t stream,
+                          const abft_inject_spec_t* inj, abft_report_t* rep) {
+    return abft_potrf_ex(n, nb, A, lda, stream, inj, rep, nullptr);
+}
+
+extern "C" int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t lda, abft_stream_t stream,
+                               const abft_inject_spec_t* inj, abft_report_t* rep, const abft_options_t* opt) {
+    int rc = check_common(n, nb, A_host, lda);
+    if (rc) return rc;
+    if (n == 0) return 0;
+    cudaStream_t s = (cudaStream_t)stream;
+    double* dA = nullptr;
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&dA, sizeof(double) * (size_t)(n * n), s));
+    ABFT_CUDA_TRY(cudaMemcpy2DAsync(dA, n * sizeof(double), A_host, lda * sizeof(double), n * sizeof(double), n,
+                                    cudaMemcpyHostToDevice, s));
+    rc = abft_potrf_ex(n, nb, dA, n, stream, inj, rep, opt);
+    if (rc >= 0 && rc != ABFT_ERR_CUDA)
+        ABFT_CUDA_TRY(cudaMemcpy2DAsync(A_host, lda * sizeof(double), dA, n * sizeof(double), n * sizeof(double), n,
+                                        cudaMemcpyDeviceToHost, s));
+    cudaFreeAsync(dA, s);
+    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+    return rc;
+}
+
+extern "C" int abft_encode(int64_t n, int64_t nb, const double* A, int64_t lda, double* chk, int64_t ldchk,
+                           double* scales, abft_stream_t stream) {
+    g_launches = 0;
+    int rc = check_common(n, nb, A, lda);
+    if (rc) return rc;
+    if (!chk && n > 0) return -5;
+    const int64_t N = n / nb;
+    if (ldchk < std::max<int64_t>(1, 2 * N)) return -6;
+    if (!scales && n > 0) return -7;
+    if (n == 0) return 0;
+    cudaStream_t s = (cudaStream_t)stream;
+    DevState* st = nullptr;
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&st, sizeof(DevState), s));
+    ABFT_CUDA_TRY(cudaMemsetAsync(st, 0, sizeof(DevState), s));
+    launch_scales(n, nb, A, lda, scales, s);
+    Work w; w.n = n; w.nb = nb; w.N = N; w.chk = chk; w.ldc = ldchk; w.scl = scales; w.st = st;
+    StageArgs a = stage_base(w, (double*)A, lda, 64.0, SK_ALL, 0, -1);
+    a.encode = 1;
+    launch_check(a, s);
+    cudaFreeAsync(st, s);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return 0;
+}
+
+extern "C" int abft_verify(int64_t n, int64_t nb, double* A, int64_t lda, double* chk, int64_t ldchk,
+                           const double* scales, int factored, int correct, abft_stream_t stream,
+                           abft_report_t* rep) {
+    g_launches = 0;
+    int rc = check_common(n, nb, A, lda);
+    if (rc) return rc;
+    if (!chk && n > 0) return -5;
+    const int64_t N = n / nb;
+    if (ldchk < std::max<int64_t>(1, 2 * N)) return -6;
+    if (!scales && n > 0) return -7;
+    if (factored != 0 && factored != 1) return -8;
+    if (correct != 0 && correct != 1) return -9;
+    if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; }
+    if (n == 0) return 0;
+    cudaStream_t s = (cudaStream_t)stream;
+    Work w; w.n = n; w.nb = nb; w.N = N;
+    w.ldc = ldchk; w.chk = chk; w.scl = (double*)scales;
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.st, sizeof(DevState), s));
+    ABFT_CUDA_TRY(cudaMemsetAsync(w.st, 0, sizeof(DevState), s));
+    w.ev_cap = rep ? std::max<int64_t>(rep->cap, 1) : 1;
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.ev, sizeof(abft_event_t) * (size_t)w.ev_cap, s));
+    StageArgs a = stage_base(w, A, lda, 64.0, SK_ALL, factored ? ABFT_V6 : ABFT_V5, -1);
+    a.factored = factored; a.correct = correct;
+    launch_check(a, s);
+    int status = 0;
+    if (rep) rc = finish_report(w, rep, s, &status);
+    cudaFreeAsync(w.st, s); cudaFreeAsync(w.ev, s);
+    if (rc) return rc;
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return status;
+}
+
+extern "C" int abft_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, abft_stream_t stream) {
+    g_launches = 0;
+    if (n < 0) return -1;
+    if (!A && n > 0) return -3;
+    if (lda < std::max<int64_t>(1, n)) return -4;
+    launch_gen_spd(n, seed, A, lda, (cudaStream_t)stream);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return 0;
+}

@@ -1,0 +1,320 @@
+// check.cu — checksum encoding, recalculation (phase 1) and detect/locate/correct (phase 2).
+//
+// PAPER.md:121-129 (§IV.A encoding), :180-195 (§IV.C detection / location / correction),
+// with the readings A4-A12 of DESIGN.md §3. The paper's checksum recalculation is a set of
+// BLAS-2 dgemv calls spread over N CUDA streams (Opt. 1); here one
+// bandwidth-bound launch covers every tile of a check stage: one warp per tile column,
+// coalesced column loads and warp-shuffle reductions (the mirrored half of an unfactored
+// diagonal tile is read row-wise, also coalesced).
+#include "common.cuh"
+
+namespace abft {
+
+constexpr int kChkThreads = 256;  // 8 warps
+constexpr int kChkCols = 64;      // tile columns per CTA (8 per warp)
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// Phase 1: recompute r1 = v1^T X[:,c], r2 = v2^T X[:,c] for every column of every tile of the
+// stage. encode = 1: store them as the checksums. Otherwise compare, flag columns
+// with |d| > tau or non-finite d, and append them to the flag list.
+__global__ void __launch_bounds__(kChkThreads) k_check_phase1(StageArgs a) {
+    if (a.st->abort) return;
+    const int64_t B = a.nb;
+    const int64_t chunks = (B + kChkCols - 1) / kChkCols;
+    const int64_t t = blockIdx.x / chunks;
+    const int64_t c0 = (blockIdx.x % chunks) * kChkCols;
+    int64_t I, J;
+    stage_tile(a, t, I, J);
+    if (J % a.col_owner_mod != a.col_owner_rank) return;  // dist: not this rank's column
+    const TileView v = stage_view(a, I, J);
+    const int cw = (int)((B - c0) < kChkCols ? (B - c0) : kChkCols);
+    __shared__ double s_r1[kChkCols], s_r2[kChkCols];
+    __shared__ double s_m1[kChkThreads], s_m2[kChkThreads];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+    // column part: rows r >= c for diagonal tiles, all rows otherwise
+    for (int cc = warp; cc < cw; cc += kChkThreads / 32) {
+        const int64_t c = c0 + cc;
+        const double* col = v.T + c * v.ldt;
+        const int64_t rbeg = v.diag ? c : 0;
+        double r1 = 0.0, r2 = 0.0;
+        int64_t r = rbeg + lane;
+#pragma unroll 4
+        for (; r < B; r += 32) {
+            const double x = col[r];
+            r1 += x;
+            r2 = fma((double)(r + 1), x, r2);
+        }
+        r1 = warp_sum(r1);
+        r2 = warp_sum(r2);
+        if (lane == 0) { s_r1[cc] = r1; s_r2[cc] = r2; }
+    }
+    // mirrored part of an unfactored diagonal tile: X[r,c] = T[c,r] for r < c (row c of T)
+    if (v.diag && !v.factored) {
+        const int ngroups = kChkThreads / kChkCols;
+        const int cc = threadIdx.x % kChkCols, grp = threadIdx.x / kChkCols;
+        double m1 = 0.0, m2 = 0.0;
+        if (cc < cw) {
+            const int64_t c = c0 + cc;
+            for (int64_t r = grp; r < c; r += ngroups) {
+                const double x = v.T[r * v.ldt + c];
+                m1 += x;
+                m2 = fma((double)(r + 1), x, m2);
+            }
+        }
+        s_m1[threadIdx.x] = m1; s_m2[threadIdx.x] = m2;
+        __syncthreads();
+        if (threadIdx.x < cw) {
+            double a1 = 0.0, a2 = 0.0;
+            for (int g = 0; g < ngroups; ++g) { a1 += s_m1[g * kChkCols + threadIdx.x]; a2 += s_m2[g * kChkCols + threadIdx.x]; }
+            s_r1[threadIdx.x] += a1; s_r2[threadIdx.x] += a2;
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && c0 == 0 && !a.encode) atomicAdd(&a.st->n_checks, 1ull);
+    if (threadIdx.x >= cw) return;
+    const int64_t c = c0 + threadIdx.x;
+    const double r1 = s_r1[threadIdx.x], r2 = s_r2[threadIdx.x];
+    if (a.encode) { v.c1[c * v.ldc] = r1; v.c2[c * v.ldc] = r2; return; }
+    const double d1 = __dsub_rn(r1, v.c1[c * v.ldc]);
+    const double d2 = __dsub_rn(r2, v.c2[c * v.ldc]);
+    double tau1, tau2;
+    thresholds(a, I, J * B + c, v.factored, tau1, tau2);
+    const bool f1 = !dfinite(d1) || fabs(d1) > tau1;        // P:195 + A5
+    const bool f2 = !dfinite(d2) || fabs(d2) > tau2;
+    if (!(f1 || f2)) return;
+    const int slot = atomicAdd(&a.st->nflag, 1);
+    if (slot >= kFlagCap) { a.st->flag_overflow = 1; return; }
+    Flag& f = a.st->flags[slot];
+    f.I = (int32_t)I; f.J = (int32_t)J; f.c = (int32_t)c;
+    f.d1 = d1; f.d2 = d2; f.r1 = r1; f.r2 = r2;
+}
+
+// Block-wide reductions used by phase 2 (one CTA).
+__device__ double block_sum(double v, double* red) {
+    v = warp_sum(v);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+    __syncthreads();
+    if (lane == 0) red[warp] = v;
+    __syncthreads();
+    double s = 0.0;
+    for (int w = 0; w < nw; ++w) s += red[w];
+    return s;
+}
+
+// argmax over r of (non-finite -> +inf, else |x|), lowest r on ties (reading A9)
+__device__ int64_t block_argmax(const TileView& v, int64_t c, int64_t B, double* redv, long long* redi) {
+    double best = -1.0; long long bi = 0x7fffffffffffffffll;
+    for (int64_t r = threadIdx.x; r < B; r += blockDim.x) {
+        const double x = view_x(v, r, c);
+        const double m = dfinite(x) ? fabs(x) : INFINITY;
+        if (m > best || (m == best && r < bi)) { best = m; bi = r; }
+    }
+    __syncthreads();
+    redv[threadIdx.x] = best; redi[threadIdx.x] = bi;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double b = -1.0; long long i = 0x7fffffffffffffffll;
+        for (int u = 0; u < (int)blockDim.x; ++u)
+            if (redv[u] > b || (redv[u] == b && redi[u] < i)) { b = redv[u]; i = redi[u]; }
+        redi[0] = i;
+    }
+    __syncthreads();
+    const int64_t r = redi[0];
+    __syncthreads();
+    return r;
+}
+
+struct Fix { double* p; double* p2; double val; };
+
+// Phase 2: resolve the flagged columns in the oracle's order (tile, then column): decide
+// DATA / NONFINITE / CHK1 / CHK2 / UNCORRECTABLE, dedupe diagonal-tile mirrors, compute the
+// corrections from the pre-correction tile, apply them per tile, log events. One CTA.
+__global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
+    DevState* st = a.st;
+    __shared__ int s_n;
+    __shared__ Fix s_fix[64];
+    __shared__ int s_nfix, s_unc, s_stop;
+    __shared__ double redv[256];
+    __shared__ long long redi[256];
+    if (threadIdx.x == 0) {
+        s_n = min(st->nflag, kFlagCap);
+        if (st->abort) s_n = 0;
+        if (st->flag_overflow && !st->abort) {   // more flagged columns than we can resolve
+            st->status = ABFT_UNCORRECTABLE; st->abort = 1; s_n = 0;
+            const long long e = (long long)atomicAdd(&st->nev, 1ull);
+            if (e < a.ev_cap) {
+                abft_event_t& ev = a.ev[e];
+                ev.k = a.k; ev.check = a.V; ev.tile_i = -1; ev.tile_j = -1; ev.row = -3; ev.col = -1;
+                ev.kind = ABFT_KIND_UNCORRECTABLE; ev.rank = a.rank; ev.delta1 = 0; ev.delta2 = 0;
+            }
+            st->n_unc++;
+        }
+        // insertion sort by (J, I, c): the oracle's check order
+        Flag* F = st->flags;
+        for (int i = 1; i < s_n; ++i) {
+            Flag x = F[i]; int j = i - 1;
+            auto key = [](const Flag& f) { return ((long long)f.J << 40) | ((long long)f.I << 20) | f.c; };
+            while (j >= 0 && key(F[j]) > key(x)) { F[j + 1] = F[j]; --j; }
+            F[j + 1] = x;
+        }
+        s_stop = 0;
+    }
+    __syncthreads();
+    const int n = s_n;
+    const int64_t B = a.nb;
+    int i0 = 0;
+    while (i0 < n && !s_stop) {
+        // entries [i0, i1) belong to one tile
+        const Flag first = st->flags[i0];
+        int i1 = i0;
+        while (i1 < n && st->flags[i1].I == first.I && st->flags[i1].J == first.J) ++i1;
+        const TileView v = stage_view(a, first.I, first.J);
+        if (threadIdx.x == 0) { s_nfix = 0; s_unc = 0; }
+        __syncthreads();
+        for (int e = i0; e < i1; ++e) {
+            const Flag f = st->flags[e];
+            const int64_t c = f.c;
+            double tau1, tau2;
+            thresholds(a, f.I, (int64_t)f.J * B + c, v.factored, tau1, tau2);
+            const bool f1 = !dfinite(f.d1) || fabs(f.d1) > tau1;
+            const bool f2 = !dfinite(f.d2) || fabs(f.d2) > tau2;
+            int kind; int64_t row = -1;
+            if (!dfinite(f.d1) || !dfinite(f.d2)) {
+                kind = ABFT_KIND_NONFINITE;
+                row = block_argmax(v, c, B, redv, redi);
+            } else if (f1) {
+                const double q = __ddiv_rn(f.d2, f.d1);
+                const double j = rint(q);                       // half-to-even
+                kind = f2 ? ABFT_KIND_UNCORRECTABLE : ABFT_KIND_CHK1;
+                if (j >= 1.0 && j <= (double)B) {
+                    const double jd1 = __dmul_rn(j, f.d1);
+                    if (fabs(__dsub_rn(f.d2, jd1)) <= __dadd_rn(tau2, __dmul_rn(ABFT_RHO, fabs(jd1)))) {
+                        kind = ABFT_KIND_DATA; row = (int64_t)j - 1;
+                    }
+                }
+            } else {
+                kind = ABFT_KIND_CHK2;
+            }
+            if (kind == ABFT_KIND_DATA || kind == ABFT_KIND_NONFINITE) {
+                double* p = view_store(v, row, c);
+                bool dup = false;
+                for (int u = 0; u < s_nfix; ++u) dup |= (s_fix[u].p == p);
+                if (dup) continue;                              // corrected once, logged once
+                double part = 0.0;
+                for (int64_t r = threadIdx.x; r < B; r += blockDim.x)
+                    if (r != row) part += view_x(v, r, c);
+                const double sum = block_sum(part, redv);
+                if (threadIdx.x == 0) {
+                    const double val = __dsub_rn(v.c1[c * v.ldc], sum);   // A8
+                    if (s_nfix < 64) { s_fix[s_nfix].p = p; s_fix[s_nfix].p2 = nullptr; s_fix[s_nfix].val = val; s_nfix++; }
+                    else s_unc = 1;
+                    int64_t sr = row, sc = c;
+                    if (v.diag && !v.factored && sr < sc) { const int64_t t = sr; sr = sc; sc = t; }
+                    const long long ev_i = (long long)atomicAdd(&st->nev, 1ull);
+                    if (ev_i < a.ev_cap) {
+                        abft_event_t& ev = a.ev[ev_i];
+                        ev.k = a.k; ev.check = (a.kind == SK_COLUMN && f.I == a.k) ? ABFT_V1 : a.V;
+                        ev.tile_i = f.I; ev.tile_j = f.J;
+                        ev.row = (int32_t)sr; ev.col = (int32_t)sc; ev.kind = kind; ev.rank = a.rank;
+                        ev.delta1 = f.d1; ev.delta2 = f.d2;
+                    }
+                    st->n_detected++;
+                    if (kind == ABFT_KIND_DATA) st->n_data++; else st->n_nonfinite++;
+                }
+                __syncthreads();
+            } else if (threadIdx.x == 0) {
+                const long long ev_i = (long long)atomicAdd(&st->nev, 1ull);
+                if (ev_i < a.ev_cap) {
+                    abft_event_t& ev = a.ev[ev_i];
+                    ev.k = a.k; ev.check = (a.kind == SK_COLUMN && f.I == a.k) ? ABFT_V1 : a.V;
+                    ev.tile_i = f.I; ev.tile_j = f.J;
+                    ev.row = kind == ABFT_KIND_CHK1 ? -1 : kind == ABFT_KIND_CHK2 ? -2 : -3;
+                    ev.col = (int32_t)c; ev.kind = kind; ev.rank = a.rank;
+                    ev.delta1 = f.d1; ev.delta2 = f.d2;
+                }
+                st->n_detected++;
+                if (kind == ABFT_KIND_CHK1 || kind == ABFT_KIND_CHK2) {
+                    if (kind == ABFT_KIND_CHK1) st->n_chk1++; else st->n_chk2++;
+                    if (s_nfix < 64) {
+                        s_fix[s_nfix].p = kind == ABFT_KIND_CHK1 ? &v.c1[c * v.ldc] : &v.c2[c * v.ldc];
+                        s_fix[s_nfix].p2 = nullptr;
+                        s_fix[s_nfix].val = kind == ABFT_KIND_CHK1 ? f.r1 : f.r2;   // chk := v^T X
+                        s_nfix++;
+                    } else s_unc = 1;
+                } else {
+                    st->n_unc++;
+                    s_unc = 1;
+                }
+            }
+            __syncthreads();
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            if (a.correct)
+                for (int u = 0; u < s_nfix; ++u) *s_fix[u].p = s_fix[u].val;
+            if (s_unc) { st->status = ABFT_UNCORRECTABLE; st->abort = 1; s_stop = 1; }
+        }
+        __syncthreads();
+        i0 = i1;
+    }
+    if (threadIdx.x == 0) { st->nflag = 0; st->flag_overflow = 0; }
+}
+
+// Threshold scales of reading A4: s_i = sqrt(A_ii); S1_I = sum s_i, S2_I = sum (i+1) s_i over
+// block I, summed sequentially in ascending order with explicit round-to-nearest operations.
+__global__ void k_scales_diag(int64_t n, const double* A, int64_t lda, double* s) {
+    const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (i < n) s[i] = __dsqrt_rn(A[i * lda + i]);
+}
+__global__ void k_scales_block(int64_t N, int64_t B, const double* s, double* S1, double* S2) {
+    const int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    if (I >= N) return;
+    double a = 0.0, b = 0.0;
+    for (int64_t r = 0; r < B; ++r) {
+        a = __dadd_rn(a, s[I * B + r]);
+        b = __dadd_rn(b, __dmul_rn((double)(r + 1), s[I * B + r]));
+    }
+    S1[I] = a; S2[I] = b;
+}
+
+}  // namespace abft
+
+// ---- host launchers ---------------------------------------------------------------------
+using namespace abft;
+
+int launch_check(const StageArgs& a, cudaStream_t s) {
+    int64_t count;
+    {
+        const int64_t N = a.N, k = a.k;
+        switch (a.kind) {
+            case SK_COLUMN: count = N - k; break;
+            case SK_DIAG_FACT: count = 1; break;
+            case SK_PANEL: count = N - k - 1; break;
+            case SK_TRAIL: { int64_t m = N - k - 1; count = m * (m + 1) / 2; break; }
+            default: count = N * (N + 1) / 2;
+        }
+    }
+    if (count <= 0) return 0;
+    const int64_t chunks = (a.nb + kChkCols - 1) / kChkCols;
+    k_check_phase1<<<(unsigned)(count * chunks), kChkThreads, 0, s>>>(a);
+    abft_count_launch();
+    if (a.encode) return 0;
+    k_check_phase2<<<1, 256, 0, s>>>(a);
+    abft_count_launch();
+    return 0;
+}
+
+int launch_scales(int64_t n, int64_t nb, const double* A, int64_t lda, double* scl, cudaStream_t s) {
+    const int64_t N = n / nb;
+    if (n == 0) return 0;
+    k_scales_diag<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(n, A, lda, scl);
+    k_scales_block<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(N, nb, scl, scl + n, scl + n + N);
+    abft_count_launch(2);
+    return 0;
+}

@@ -1,0 +1,159 @@
+// common.cuh — shared device-side types of libabft (CUDA path only; the oracle has its own).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "../../include/abft.h"
+
+#define ABFT_EPS 0x1p-52  /* DBL_EPSILON (reading A17) */
+#define ABFT_RHO 0x1p-30  /* relative slack of the location test (reading A6) */
+
+namespace abft {
+
+// A flagged column produced by a check's recalculation pass (phase 1), resolved by phase 2.
+struct Flag {
+    int32_t I, J, c, pad;
+    double d1, d2, r1, r2;
+};
+
+constexpr int kFlagCap = 8192;
+
+// Device-resident run state. One per abft_* call.
+struct DevState {
+    int32_t abort;        // set by UNCORRECTABLE / NOT_SPD: every later kernel returns at entry
+    int32_t status;       // ABFT_OK / ABFT_UNCORRECTABLE / ABFT_NOT_SPD
+    long long info;       // LAPACK info (1-based)
+    int32_t nflag;        // flagged columns pending resolution (phase 1 -> phase 2)
+    int32_t flag_overflow;
+    unsigned long long nev;        // events raised
+    unsigned long long n_checks;   // tile checks run
+    long long n_detected, n_data, n_nonfinite, n_chk1, n_chk2, n_unc;
+    Flag flags[kFlagCap];
+};
+
+// Where the tiles of a check stage live (DESIGN.md §5 "data layout").
+enum StageKind : int32_t {
+    SK_COLUMN = 0,     // V1/V2: tiles (k..N-1, k) in A, unfactored; checksums in chk
+    SK_DIAG_FACT = 1,  // V3: tile (k,k) in A, factored; checksums in W rows mB, mB+1
+    SK_PANEL = 2,      // V4/V4R: tiles (k+1..N-1, k) in W (data rows), checksums in W (chk rows)
+    SK_TRAIL = 3,      // V5: tiles (I,J), k < J <= I, in A, unfactored; checksums in chk
+    SK_ALL = 4,        // V6 / abft_verify: all tiles I >= J in A; factored per flag
+};
+
+struct StageArgs {
+    int32_t kind, V, k, factored;   // k: iteration (-1 for abft_verify); V: event check code
+    int32_t correct, rank, encode, pad;
+    int64_t n, nb, N;
+    double* A; int64_t lda;         // global matrix (or local columns in dist mode)
+    double* chk; int64_t ldc;       // checksum matrix 2N x n(local)
+    double* W; int64_t ldw;         // packed panel buffer (SK_DIAG_FACT, SK_PANEL)
+    int64_t mB;                     // rows of data in W (m * nb)
+    const double* s; const double* S1; const double* S2;  // threshold scales
+    double c_tau;
+    int32_t col_owner_mod, col_owner_rank;  // dist: local column mapping (1, 0 on one GPU)
+    DevState* st;
+    abft_event_t* ev; int64_t ev_cap;
+};
+
+// Tile view: data pointer, leading dim, checksum row pointers with stride.
+struct TileView {
+    double* T; int64_t ldt;
+    double* c1; double* c2; int64_t ldc;
+    bool diag, factored;
+};
+
+__device__ __forceinline__ int64_t stage_count(const StageArgs& a) {
+    const int64_t N = a.N, k = a.k;
+    switch (a.kind) {
+        case SK_COLUMN: return N - k;
+        case SK_DIAG_FACT: return 1;
+        case SK_PANEL: return N - k - 1;
+        case SK_TRAIL: { int64_t m = N - k - 1; return m * (m + 1) / 2; }
+        default: return N * (N + 1) / 2;
+    }
+}
+
+// t-th tile of the stage, in the oracle's check order (column-major over tiles).
+__device__ __forceinline__ void stage_tile(const StageArgs& a, int64_t t, int64_t& I, int64_t& J) {
+    const int64_t N = a.N, k = a.k;
+    switch (a.kind) {
+        case SK_COLUMN: I = k + t; J = k; return;
+        case SK_DIAG_FACT: I = k; J = k; return;
+        case SK_PANEL: I = k + 1 + t; J = k; return;
+        default: {
+            const int64_t j0 = (a.kind == SK_TRAIL) ? k + 1 : 0;
+            const int64_t m = N - j0;
+            int64_t jj = 0, rem = t;
+            while (rem >= m - jj) { rem -= m - jj; ++jj; }
+            J = j0 + jj; I = J + rem; return;
+        }
+    }
+}
+
+// Local column offset of global block column J (1D block-cyclic in dist mode).
+__device__ __forceinline__ int64_t local_col(const StageArgs& a, int64_t J) {
+    return (J / a.col_owner_mod) * a.nb;
+}
+
+__device__ __forceinline__ TileView stage_view(const StageArgs& a, int64_t I, int64_t J) {
+    TileView v;
+    const int64_t B = a.nb;
+    v.diag = (I == J);
+    switch (a.kind) {
+        case SK_DIAG_FACT:
+            v.T = a.A + local_col(a, J) * a.lda + I * B; v.ldt = a.lda;
+            v.c1 = a.W + a.mB; v.c2 = v.c1 + 1; v.ldc = a.ldw;
+            v.factored = true; break;
+        case SK_PANEL:
+            v.T = a.W + (I - a.k - 1) * B; v.ldt = a.ldw;
+            v.c1 = a.W + a.mB + 2 + 2 * (I - a.k - 1); v.c2 = v.c1 + 1; v.ldc = a.ldw;
+            v.diag = false; v.factored = true; break;
+        case SK_COLUMN:
+        case SK_TRAIL:
+            v.T = a.A + local_col(a, J) * a.lda + I * B; v.ldt = a.lda;
+            v.c1 = a.chk + local_col(a, J) * a.ldc + 2 * I; v.c2 = v.c1 + 1; v.ldc = a.ldc;
+            v.factored = false; break;
+        default:
+            v.T = a.A + local_col(a, J) * a.lda + I * B; v.ldt = a.lda;
+            v.c1 = a.chk + local_col(a, J) * a.ldc + 2 * I; v.c2 = v.c1 + 1; v.ldc = a.ldc;
+            v.factored = a.factored != 0; break;
+    }
+    return v;
+}
+
+// X(r,c) of the check: sym(tril(T)) for an unfactored diagonal tile, tril(T) if factored.
+__device__ __forceinline__ double view_x(const TileView& v, int64_t r, int64_t c) {
+    if (v.diag) {
+        if (r >= c) return v.T[c * v.ldt + r];
+        return v.factored ? 0.0 : v.T[r * v.ldt + c];
+    }
+    return v.T[c * v.ldt + r];
+}
+__device__ __forceinline__ double* view_store(const TileView& v, int64_t r, int64_t c) {
+    if (v.diag && r < c) return &v.T[r * v.ldt + c];
+    return &v.T[c * v.ldt + r];
+}
+
+// Thresholds of reading A4, evaluated with explicit round-to-nearest ops (no FMA contraction)
+// so that a decision depends only on (d1, d2) and the scales.
+__device__ __forceinline__ void thresholds(const StageArgs& a, int64_t I, int64_t g, bool factored,
+                                           double& tau1, double& tau2) {
+    const double base = a.c_tau * ABFT_EPS;  // exact: power-of-two scaling
+    const double sc = factored ? 1.0 : a.s[g];
+    tau1 = __dmul_rn(__dmul_rn(base, a.S1[I]), sc);
+    tau2 = __dmul_rn(__dmul_rn(base, a.S2[I]), sc);
+}
+
+__device__ __forceinline__ bool dfinite(double x) { return isfinite(x); }
+
+}  // namespace abft
+
+// Host helpers
+#define ABFT_CUDA_TRY(expr)                                   \
+    do {                                                      \
+        cudaError_t _e = (expr);                              \
+        if (_e != cudaSuccess) { abft_set_error(_e, #expr); return ABFT_ERR_CUDA; } \
+    } while (0)
+
+void abft_set_error(cudaError_t e, const char* what);
+void abft_count_launch(int n = 1);

@@ -1,0 +1,291 @@
+// gemm.cu — FP64 tensor-core (DMMA) GEMM for the trailing SYRK/GEMM update, the panel TRSM
+// (as a product with the inverted diagonal block) and the recursive diagonal-block POTRF.
+//
+//   C[m,n] = beta * C[m,n] + alpha * sum_k A[m,k] * opB[k,n]
+//   A : M x K column-major (lda);  opB = Bm^T with Bm N x K (TRANS_B, "NT") or Bm K x N ("NN").
+//
+// FP64 tensor work on sm_100a is warp-level DMMA (mma.sync.m8n8k4.f64 -> DMMA.8x8x4);
+// tcgen05 has no kind::f64 (ptxas rejects it), so TMEM/UMMA do not apply to this path.
+// Operands are staged global -> shared memory with a multi-stage cp.async (LDGSTS) pipeline;
+// fragments are read with conflict-free 64-bit shared loads (row pitch = tile + 4 doubles,
+// which is 4 mod 16 8-byte banks).
+//
+// Output masks:
+//   MASK_NONE  : all of M x N
+//   MASK_LOWER : only r >= c (SYRK of the trailing lower triangle; CTA tiles with tile-row <
+//                tile-col are not launched). PAPER.md:137-153: A' = A - LC LC^T, B' = B - LD LC^T
+//   MASK_CHK   : checksum rows: row q belongs to block I = q_tile0 + q/2, column c to block
+//                J = c_tile0 + c/nb; written iff I >= J (chk(B') = chk(B) - chk(LD) LC^T)
+// K-range restrictions exploit triangular operands (zeros are never multiplied):
+//   KR_LE_N  : k < n0 + BN   (opB = inv(L)^T, lower inverse: TRSM)
+//   KR_GE_N  : k >= n0       (opB = inv(L), NN)
+//   KR_LE_M  : k < m0 + BM   (A = inv(L) lower, NN)
+#include "common.cuh"
+
+namespace abft {
+
+enum { MASK_NONE = 0, MASK_LOWER = 1, MASK_CHK = 2 };
+enum { KR_FULL = 0, KR_LE_N = 1, KR_GE_N = 2, KR_LE_M = 3 };
+
+struct GemmArgs {
+    int64_t M, N, K;
+    const double* A; int64_t lda;
+    const double* B; int64_t ldb;
+    double* C; int64_t ldc;
+    double alpha, beta;
+    int32_t mask, krange;
+    int64_t nb, q_tile0, c_tile0;   // MASK_CHK geometry
+    int64_t tiles_n;                // number of column tiles (rect grid)
+    const int32_t* abort;
+    int32_t vecA, vecB;             // 16-byte cp.async allowed for A / B
+};
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(src_bytes));
+}
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem, int src_bytes) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;\n" ::"r"(s), "l"(gmem), "r"(src_bytes));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
+__device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(c0), "+d"(c1) : "d"(a), "d"(b));
+}
+
+template <int BM, int BN, int BK, int WM, int WN, int STAGES, bool TB>
+struct GemmCfg {
+    static constexpr int WARPS_M = BM / WM, WARPS_N = BN / WN;
+    static constexpr int THREADS = WARPS_M * WARPS_N * 32;
+    static constexpr int PA = BM + 4;                    // sA[k][m], pitch PA
+    static constexpr int PB_T = BN + 4;                  // TB: sB[k][n]
+    static constexpr int PB_N = BK + 4;                  // NN: sB[n][k]
+    static constexpr int SA = BK * PA;
+    static constexpr int SB = TB ? BK * PB_T : BN * PB_N;
+    static constexpr size_t SMEM = (size_t)STAGES * (SA + SB) * sizeof(double);
+    static constexpr int FM = WM / 8, FN = WN / 8;
+};
+
+template <int BM, int BN, int BK, int WM, int WN, int STAGES, bool TB>
+__global__ void __launch_bounds__(GemmCfg<BM, BN, BK, WM, WN, STAGES, TB>::THREADS, 1)
+k_gemm_dmma(GemmArgs g) {
+    using Cfg = GemmCfg<BM, BN, BK, WM, WN, STAGES, TB>;
+    if (*(volatile const int32_t*)g.abort) return;
+    // ---- tile mapping ----
+    int64_t tm, tn;
+    if (g.mask == MASK_LOWER) {  // lower-triangular tile enumeration, row-major
+        const int64_t idx = blockIdx.x;
+        int64_t a = (int64_t)((sqrt(8.0 * (double)idx + 1.0) - 1.0) * 0.5);
+        while (a * (a + 1) / 2 > idx) --a;
+        while ((a + 1) * (a + 2) / 2 <= idx) ++a;
+        tm = a; tn = idx - a * (a + 1) / 2;
+    } else {
+        tm = blockIdx.x / g.tiles_n; tn = blockIdx.x % g.tiles_n;
+    }
+    const int64_t m0 = tm * BM, n0 = tn * BN;
+    if (g.mask == MASK_CHK) {  // skip tiles where no row reaches the column blocks
+        const int64_t qmax = min(g.M, m0 + BM) - 1;
+        const int64_t Imax = g.q_tile0 + qmax / 2, Jmin = g.c_tile0 + n0 / g.nb;
+        if (Imax < Jmin) return;
+    }
+    int64_t kb = 0, ke = g.K;
+    if (g.krange == KR_LE_N) ke = min(g.K, n0 + BN);
+    else if (g.krange == KR_GE_N) kb = (n0 / BK) * BK;
+    else if (g.krange == KR_LE_M) ke = min(g.K, m0 + BM);
+    const int ktiles = (int)((ke - kb + BK - 1) / BK);
+
+    extern __shared__ __align__(16) double smem[];
+    double* sA = smem;
+    double* sB = smem + STAGES * Cfg::SA;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int wm = warp / Cfg::WARPS_N, wn = warp % Cfg::WARPS_N;
+
+    auto load_stage = [&](int stage, int kt) {
+        const int64_t k0 = kb + (int64_t)kt * BK;
+        double* dA = sA + stage * Cfg::SA;
+        double* dB = sB + stage * Cfg::SB;
+        // A: BK columns of BM rows
+        if (g.vecA) {
+            constexpr int CH = BK * BM / 2;
+            for (int i = tid; i < CH; i += Cfg::THREADS) {
+                const int kk = i / (BM / 2), mm = (i % (BM / 2)) * 2;
+                const int64_t gm = m0 + mm, gk = k0 + kk;
+                int bytes = 0;
+                if (gk < ke && gm < g.M) bytes = (gm + 1 < g.M) ? 16 : 8;
+                const double* src = bytes ? g.A + gk * g.lda + gm : g.A;
+                cp_async16(dA + kk * Cfg::PA + mm, src, bytes);
+            }
+        } else {
+            constexpr int CH = BK * BM;
+            for (int i = tid; i < CH; i += Cfg::THREADS) {
+                const int kk = i / BM, mm = i % BM;
+                const int64_t gm = m0 + mm, gk = k0 + kk;
+                const bool ok = gk < ke && gm < g.M;
+                cp_async8(dA + kk * Cfg::PA + mm, ok ? g.A + gk * g.lda + gm : g.A, ok ? 8 : 0);
+            }
+        }
+        if (TB) {  // Bm is N x K: column k holds n contiguous
+            if (g.vecB) {
+                constexpr int CH = BK * BN / 2;
+                for (int i = tid; i < CH; i += Cfg::THREADS) {
+                    const int kk = i / (BN / 2), nn = (i % (BN / 2)) * 2;
+                    const int64_t gn = n0 + nn, gk = k0 + kk;
+                    int bytes = 0;
+                    if (gk < ke && gn < g.N) bytes = (gn + 1 < g.N) ? 16 : 8;
+                    cp_async16(dB + kk * Cfg::PB_T + nn, bytes ? g.B + gk * g.ldb + gn : g.B, bytes);
+                }
+            } else {
+                constexpr int CH = BK * BN;
+                for (int i = tid; i < CH; i += Cfg::THREADS) {
+                    const int kk = i / BN, nn = i % BN;
+                    const int64_t gn = n0 + nn, gk = k0 + kk;
+                    const bool ok = gk < ke && gn < g.N;
+                    cp_async8(dB + kk * Cfg::PB_T + nn, ok ? g.B + gk * g.ldb + gn : g.B, ok ? 8 : 0);
+                }
+            }
+        } else {   // Bm is K x N: column n holds k contiguous
+            if (g.vecB) {
+                constexpr int CH = BN * BK / 2;
+                for (int i = tid; i < CH; i += Cfg::THREADS) {
+                    const int nn = i / (BK / 2), kk = (i % (BK / 2)) * 2;
+                    const int64_t gn = n0 + nn, gk = k0 + kk;
+                    int bytes = 0;
+                    if (gn < g.N && gk < ke) bytes = (gk + 1 < ke) ? 16 : 8;
+                    cp_async16(dB + nn * Cfg::PB_N + kk, bytes ? g.B + gn * g.ldb + gk : g.B, bytes);
+                }
+            } else {
+                constexpr int CH = BN * BK;
+                for (int i = tid; i < CH; i += Cfg::THREADS) {
+                    const int nn = i / BK, kk = i % BK;
+                    const int64_t gn = n0 + nn, gk = k0 + kk;
+                    const bool ok = gn < g.N && gk < ke;
+                    cp_async8(dB + nn * Cfg::PB_N + kk, ok ? g.B + gn * g.ldb + gk : g.B, ok ? 8 : 0);
+                }
+            }
+        }
+    };
+
+    double acc[Cfg::FM][Cfg::FN][2];
+#pragma unroll
+    for (int i = 0; i < Cfg::FM; ++i)
+#pragma unroll
+        for (int j = 0; j < Cfg::FN; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+
+#pragma unroll
+    for (int s = 0; s < STAGES - 1; ++s) {
+        if (s < ktiles) load_stage(s, s);
+        cp_async_commit();
+    }
+    const int fr = lane >> 2, fc = lane & 3;   // fragment row (groupID) / k (thread in group)
+    for (int kt = 0; kt < ktiles; ++kt) {
+        cp_async_wait<STAGES - 2>();
+        __syncthreads();
+        {   // prefetch stage kt + STAGES - 1 (its buffer was consumed at iteration kt - 1)
+            const int nk = kt + STAGES - 1;
+            if (nk < ktiles) load_stage(nk % STAGES, nk);
+            cp_async_commit();
+        }
+        const double* cA = sA + (kt % STAGES) * Cfg::SA + wm * WM + fr;
+        const double* cB = sB + (kt % STAGES) * Cfg::SB;
+#pragma unroll
+        for (int kk = 0; kk < BK; kk += 4) {
+            double af[Cfg::FM], bf[Cfg::FN];
+#pragma unroll
+            for (int i = 0; i < Cfg::FM; ++i) af[i] = cA[(kk + fc) * Cfg::PA + i * 8];
+#pragma unroll
+            for (int j = 0; j < Cfg::FN; ++j) {
+                const int nn = wn * WN + j * 8 + fr;
+                bf[j] = TB ? cB[(kk + fc) * Cfg::PB_T + nn] : cB[nn * Cfg::PB_N + kk + fc];
+            }
+#pragma unroll
+            for (int i = 0; i < Cfg::FM; ++i)
+#pragma unroll
+                for (int j = 0; j < Cfg::FN; ++j) dmma(acc[i][j][0], acc[i][j][1], af[i], bf[j]);
+        }
+    }
+    cp_async_wait<0>();
+
+    // ---- epilogue: C = beta C + alpha acc, masked ----
+#pragma unroll
+    for (int i = 0; i < Cfg::FM; ++i) {
+        const int64_t r = m0 + wm * WM + i * 8 + fr;
+        if (r >= g.M) continue;
+#pragma unroll
+        for (int j = 0; j < Cfg::FN; ++j) {
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
+                if (c >= g.N) continue;
+                if (g.mask == MASK_LOWER && r < c) continue;
+                if (g.mask == MASK_CHK && (g.q_tile0 + r / 2) < (g.c_tile0 + c / g.nb)) continue;
+                double* p = g.C + c * g.ldc + r;
+                const double v = g.alpha * acc[i][j][h];
+                *p = (g.beta == 0.0) ? v : fma(g.beta, *p, v);
+            }
+        }
+    }
+}
+
+template <int BM, int BN, int BK, int WM, int WN, int STAGES, bool TB>
+static int run_cfg(GemmArgs g, cudaStream_t s) {
+    using Cfg = GemmCfg<BM, BN, BK, WM, WN, STAGES, TB>;
+    auto kern = k_gemm_dmma<BM, BN, BK, WM, WN, STAGES, TB>;
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Cfg::SMEM);
+        attr = true;
+    }
+    const int64_t tm = (g.M + BM - 1) / BM, tn = (g.N + BN - 1) / BN;
+    g.tiles_n = tn;
+    int64_t grid;
+    if (g.mask == MASK_LOWER) grid = tm * (tm + 1) / 2;
+    else grid = tm * tn;
+    if (grid <= 0) return 0;
+    kern<<<(unsigned)grid, Cfg::THREADS, Cfg::SMEM, s>>>(g);
+    abft_count_launch();
+    return 0;
+}
+
+}  // namespace abft
+
+using namespace abft;
+
+static bool aligned16(const void* p) { return ((uintptr_t)p & 15) == 0; }
+
+// Public-to-the-library launcher. Picks the CTA tile from the problem size so that small
+// GEMMs inside the diagonal-block factorisation still spread over the SMs.
+int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
+                int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
+                int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
+                cudaStream_t s, int force_tile = 0) {
+    if (M <= 0 || N <= 0) return 0;
+    GemmArgs g;
+    g.M = M; g.N = N; g.K = K; g.A = A; g.lda = lda; g.B = B; g.ldb = ldb; g.C = C; g.ldc = ldc;
+    g.alpha = alpha; g.beta = beta; g.mask = mask; g.krange = krange; g.nb = nb;
+    g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
+    g.vecA = aligned16(A) && (lda % 2 == 0);
+    g.vecB = aligned16(B) && (ldb % 2 == 0);
+    auto tiles = [&](int64_t t) {
+        const int64_t tm = (M + t - 1) / t, tn = (N + t - 1) / t;
+        return mask == MASK_LOWER ? tm * (tm + 1) / 2 : tm * tn;
+    };
+    int tile = force_tile;
+    if (!tile) {
+        if (tiles(128) >= 148) tile = 128;
+        else if (tiles(64) >= 148) tile = 64;
+        else tile = 32;
+    }
+    if (transB) {
+        if (tile == 128) return run_cfg<128, 128, 16, 64, 32, 4, true>(g, s);
+        if (tile == 64) return run_cfg<64, 64, 16, 32, 32, 4, true>(g, s);
+        return run_cfg<32, 32, 16, 16, 16, 4, true>(g, s);
+    } else {
+        if (tile == 128) return run_cfg<128, 128, 16, 64, 32, 4, false>(g, s);
+        if (tile == 64) return run_cfg<64, 64, 16, 32, 32, 4, false>(g, s);
+        return run_cfg<32, 32, 16, 16, 16, 4, false>(g, s);
+    }
+}

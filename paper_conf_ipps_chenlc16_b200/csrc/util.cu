@@ -1,0 +1,68 @@
+// util.cu — synthetic SPD generator (reading A15, the same counter-based generator as the
+// Python module synthetic/, implemented independently here) and the fault-injection kernel.
+#include "common.cuh"
+
+#include <algorithm>
+
+namespace abft {
+
+__device__ __forceinline__ uint64_t splitmix64(uint64_t x) {
+    uint64_t z = x + 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+// A[i,j] = A[j,i] = U(key(max, min)), A[i,i] += n; full matrix written, columns coalesced.
+__global__ void k_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda) {
+    const uint64_t nn = (uint64_t)n;
+    const uint64_t base = seed * nn * nn;
+    const int64_t total = n * n;
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t j = t / n, i = t % n;
+        const uint64_t hi = (uint64_t)(i > j ? i : j), lo = (uint64_t)(i > j ? j : i);
+        const uint64_t z = splitmix64(base + hi * nn + lo);
+        double u = (double)(z >> 11) * 0x1p-53;
+        if (i == j) u += (double)n;
+        A[j * lda + i] = u;
+    }
+}
+
+struct InjOp { double* p; uint64_t mask; };
+struct InjBatch { int n; InjOp op[16]; };
+
+// XOR masks into stored doubles (the harness of PAPER.md:383-385). Stream-ordered between
+// the producing kernel and the next check; skipped after an abort.
+__global__ void k_inject(InjBatch b, const int32_t* abort_flag) {
+    if (*abort_flag) return;
+    if (threadIdx.x != 0) return;
+    for (int i = 0; i < b.n; ++i) {   // sequential: two specs may hit the same element
+        unsigned long long* p = reinterpret_cast<unsigned long long*>(b.op[i].p);
+        *p ^= (unsigned long long)b.op[i].mask;
+    }
+}
+
+}  // namespace abft
+
+using namespace abft;
+
+int launch_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, cudaStream_t s) {
+    if (n == 0) return 0;
+    const int64_t total = n * n;
+    const int64_t blocks = std::min<int64_t>((total + 255) / 256, 148 * 32);
+    k_gen_spd<<<(unsigned)blocks, 256, 0, s>>>(n, seed, A, lda);
+    abft_count_launch();
+    return 0;
+}
+
+int launch_inject(int nops, double* const* ptrs, const uint64_t* masks, const int32_t* abort_flag,
+                  cudaStream_t s) {
+    for (int base = 0; base < nops; base += 16) {
+        InjBatch b;
+        b.n = std::min(16, nops - base);
+        for (int i = 0; i < b.n; ++i) { b.op[i].p = ptrs[base + i]; b.op[i].mask = masks[base + i]; }
+        k_inject<<<1, 32, 0, s>>>(b, abort_flag);
+        abft_count_launch();
+    }
+    return 0;
+}
