@@ -193,12 +193,12 @@ def test_nonfinite_and_checksum_row_errors(P):
 def test_uncorrectable_aborts_like_oracle(P):
     n, nb = 512, 64
     A = syn.spd_matrix(n, seed=2)
-    specs = [dict(k=1, hook="REST", row=300, col=150, bit=55),
-             dict(k=1, hook="REST", row=320, col=150, bit=56)]
+    specs = [dict(k=1, hook="REST", row=300, col=150, bit=55),     # both in tile (4, 2), column 22
+             dict(k=1, hook="REST", row=310, col=150, bit=56)]
     inj = syn.inj_array(specs)
     ref = oracle.potrf(A, nb, inj=inj)
     st, rep, _ = run_gpu(P, A, nb, inj=inj)
-    assert st == 1 == ref.status
+    assert ref.status == 1 and st == 1
     assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
 
 
