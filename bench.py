@@ -1,0 +1,302 @@
+#!/usr/bin/env python
+"""bench.py — FP64 GFLOP/s (n^3/3) of the Enhanced Online-ABFT Cholesky on B200, ABFT overhead %.
+
+Default workload (BASELINE.json configs[3] at N=1, the north_star's headline point):
+n = 32768, nb = 512, random SPD (reading A15 generator, seed = n), fault-free, ABFT on.
+A "step" is one complete abft_potrf (encode, V1-V6, POTRF, TRSM, trailing update) over a fresh
+copy of the matrix, resident in HBM (8 GiB > 126 MB L2, so no L2 flush is needed).
+
+Timing: W warm-up steps, then exactly K steps, each bracketed by CUDA events on the launching
+stream (the restore of the input between steps is outside the events); barrier + synchronize
+before and after the timed loop; max over ranks. nvidia-smi samples clocks during the timed loop.
+
+Extra measurements reported on the same line (same workload, not part of `value`):
+  abft_off       the same kernels with every checksum operation removed (overhead %)
+  injected       C3-style computing + storage errors, one of each per iteration
+  e2e            abft_potrf_host on pinned host memory: H2D + factorisation + D2H per step
+  roofline       dominant kernel (trailing DMMA update) from the library's per-phase CUDA events
+  cpu_baseline   the CPU oracle on a bounded sample (rank 0, N=1)
+  cusolver       torch.linalg.cholesky (cuSOLVER dpotrf, vendor context, no ABFT)
+
+--impl reference: the oracle (the only reference implementation this paper-only tier has), timed
+on the host cores on a bounded sample of the same workload per step.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+FP64_DMMA_PEAK_TFLOPS = 37.1   # measured: tools/fp64_peak.cu, register-resident DMMA (profiles/fp64_peak_r01.txt)
+HBM_PEAK_FALLBACK = 6555.8
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=32768)
+    ap.add_argument("--nb", type=int, default=512)
+    ap.add_argument("--no-extras", action="store_true", help="main metric only (for ncu launch lists)")
+    ap.add_argument("--oracle-n", type=int, default=6144, help="cpu_baseline sample size")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+# ---- clocks sampler ----------------------------------------------------------------------
+class Clocks:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index=0):
+        self.index, self.lines, self.proc = index, [], None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 7:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = float(parts[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---- the oracle as CPU baseline / reference arm ---------------------------------------------
+def oracle_sample(n_s, nb):
+    import numpy as np
+    import oracle
+    import synthetic as syn
+    A = syn.spd_matrix(n_s)
+    t0 = time.perf_counter()
+    r = oracle.potrf(A, nb)
+    dt = time.perf_counter() - t0
+    assert r.status == 0
+    return n_s ** 3 / 3 / dt / 1e9, dt, oracle.num_threads()
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    n_s = min(args.n, 4096)
+    vals = []
+    for i in range(args.warmup + args.steps):
+        g, dt, cores = oracle_sample(n_s, args.nb)
+        if i >= args.warmup:
+            vals.append((g, dt))
+    value = statistics.median(v[0] for v in vals)
+    sample = f"oracle potrf n={n_s} nb={args.nb} per step (bounded sample of the n={args.n} workload), fault-free, ABFT on"
+    line = {"impl": "reference", "metric": "FP64 GFLOP/s (n^3/3) with online ABFT", "value": round(value, 3),
+            "unit": "GFLOP/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(1e3 * statistics.median(v[1] for v in vals), 3), "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": f"C4: n={args.n} nb={args.nb} random SPD (A15), fault-free", "n": args.n,
+                       "nb": args.nb},
+            "cpu_baseline": {"value": round(value, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+                             "sample": sample},
+            "e2e": {"value": round(value, 3), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---- our arm -------------------------------------------------------------------------------
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+
+    import numpy as np
+    import torch
+    import paper_conf_ipps_chenlc16_b200 as P
+
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    torch.cuda.set_device(local)
+    dist = world > 1
+    if dist:
+        import torch.distributed as tdist
+        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    n, nb = args.n, args.nb
+    flops = n ** 3 / 3
+    stream = torch.cuda.current_stream()
+    # input: generated on the device by the A15 generator, kept pristine for restores
+    A0 = torch.empty(n, n, dtype=torch.float64, device="cuda").T
+    assert P.abft_gen_spd(n, A0) == 0
+    A = torch.empty_like(A0.T).T
+
+    def barrier():
+        if dist:
+            import torch.distributed as tdist
+            tdist.barrier()
+        torch.cuda.synchronize()
+
+    def run_steps(opt, inj=None, steps=args.steps, warmup=args.warmup, check=True):
+        times, reps = [], []
+        for i in range(warmup + steps):
+            A.copy_(A0)
+            if i == warmup:
+                barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            st, rep = P.abft_potrf_ex(n, nb, A, inj=inj, opt=opt, report=True, cap=4096)
+            e1.record(stream)
+            e1.synchronize()
+            if check:
+                assert st == 0, f"abft_potrf status {st}"
+            if i >= warmup:
+                times.append(e0.elapsed_time(e1))
+                reps.append(rep)
+        barrier()
+        return times, reps
+
+    # ---- main metric: ABFT on, fault-free, per-phase profile on -------------------------
+    with Clocks(local) as clk:
+        times, reps = run_steps(P.options(profile=True))
+    prof = P.abft_last_profile()
+    launches = P.abft_last_launch_count()
+    ms_local = sum(times) / len(times)
+    ms = ms_local
+    if dist:
+        import torch.distributed as tdist
+        t = torch.tensor([ms_local], device="cuda")
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+        ms = t.item()
+    # single GPU: each rank factors its own matrix (replicas) until the 1D-cyclic dist path lands
+    value = world * flops / (ms * 1e-3) / 1e9
+    upd = prof.get("update", {})
+    achieved = upd["flops"] / (upd["ms"] * 1e-3) / 1e12 if upd.get("ms") else None
+    line = {
+        "metric": "FP64 GFLOP/s (n^3/3) with online ABFT", "value": round(value, 2), "unit": "GFLOP/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 3),
+        "higher_is_better": True, "scaling": "weak" if world > 1 else "strong", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"C4: n={n} nb={nb} random SPD (A15 generator, seed=n), fault-free, Enhanced "
+                               f"Online-ABFT on (K=1), 1 GPU per rank", "n": n, "nb": nb,
+                   "l2": "inputs (8 GiB) larger than L2; restore copy between steps outside the CUDA events",
+                   "parallelism": f"replicas x{world}" if world > 1 else "single GPU"},
+        "gpu_launches": int(launches) * args.steps,
+        "roofline": {"bound": "tensor", "kernel": "k_gemm_dmma<128,128,16,64,32,4,NT> trailing SYRK update",
+                     "achieved": round(achieved, 3) if achieved else None,
+                     "peak": FP64_DMMA_PEAK_TFLOPS, "unit": "TFLOP/s",
+                     "frac": round(achieved / FP64_DMMA_PEAK_TFLOPS, 4) if achieved else None,
+                     "traffic": None,
+                     "peak_source": "measured FP64 DMMA register-resident loop on this pool's B200 "
+                                    "(MEASURED_PEAKS.json has no FP64 entry)",
+                     "share_of_step": round(upd["ms"] / ms_local, 4) if upd.get("ms") else None},
+        "whole_path_frac_of_fp64_peak": round(value / world / 1e3 / FP64_DMMA_PEAK_TFLOPS, 4),
+        "phases_ms_per_step": {k: round(v["ms"], 3) for k, v in prof.items()},
+    }
+    line["clocks"] = clk.summary()
+
+    if not args.no_extras and rank == 0:
+        # ABFT off: the same kernels without checksum work
+        t_off, _ = run_steps(P.options(abft_enabled=False), steps=max(1, args.steps), warmup=1)
+        ms_off = sum(t_off) / len(t_off)
+        line["abft_off"] = {"value": round(flops / (ms_off * 1e-3) / 1e9, 2), "ms_per_step": round(ms_off, 3)}
+        line["abft_overhead_pct"] = round(100 * (ms_local - ms_off) / ms_off, 3)
+        # injected: one storage + one computing error per iteration (C3-style)
+        import synthetic as syn
+        specs = [s for s in syn.mixed_injections(n, nb) if s["hook"] != "RECV"]
+        inj = syn.inj_array(specs)
+        t_inj, rep_inj = run_steps(P.options(), inj=inj, steps=max(1, args.steps), warmup=1, check=False)
+        r0 = rep_inj[-1]
+        line["injected"] = {"value": round(flops / (sum(t_inj) / len(t_inj) * 1e-3) / 1e9, 2),
+                            "injections": len(specs), "events": int(r0["n_events"]),
+                            "corrected": int(r0["n_data"] + r0["n_nonfinite"] + r0["n_chk1"] + r0["n_chk2"]),
+                            "uncorrectable": int(r0["n_uncorrectable"])}
+        # e2e through the host C-ABI entry (pinned host memory, H2D + D2H inside the timing)
+        del A
+        torch.cuda.empty_cache()
+        h0 = torch.empty(n * n, dtype=torch.float64, pin_memory=True)
+        h = torch.empty(n * n, dtype=torch.float64, pin_memory=True)
+        h0.copy_(A0.T.contiguous().view(-1))     # row-major of A0^T == column-major of A0
+        e2e_t = []
+        for i in range(1 + max(1, args.steps)):
+            h.copy_(h0)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            st, _ = P.abft_potrf_host(n, nb, h.data_ptr(), lda=n, report=True, cap=16)
+            t1 = time.perf_counter()
+            assert st == 0
+            if i >= 1:
+                e2e_t.append(t1 - t0)
+        te = sum(e2e_t) / len(e2e_t)
+        line["e2e"] = {"value": round(flops / te / 1e9, 2), "unit": "GFLOP/s", "h2d_bytes_per_step": 8 * n * n,
+                       "d2h_bytes_per_step": 8 * n * n, "ms_per_step": round(te * 1e3, 3)}
+        del h, h0
+        # vendor context: cuSOLVER dpotrf via torch (no ABFT)
+        try:
+            X = A0.T.contiguous()
+            torch.linalg.cholesky(X)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(); torch.linalg.cholesky(X); e1.record(); e1.synchronize()
+            line["cusolver_dpotrf_context"] = {"value": round(flops / (e0.elapsed_time(e1) * 1e-3) / 1e9, 2),
+                                               "note": "vendor library, no ABFT, context only"}
+            del X
+        except Exception as ex:  # pragma: no cover
+            line["cusolver_dpotrf_context"] = {"error": str(ex)[:100]}
+        # CPU oracle, bounded sample
+        if world == 1:
+            g, dt, cores = oracle_sample(args.oracle_n, nb)
+            line["cpu_baseline"] = {"value": round(g, 3), "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
+                                    "sample": f"oracle potrf n={args.oracle_n} nb={nb} (same nb, "
+                                              f"{(args.oracle_n / n) ** 3:.4f} of the workload's flops), "
+                                              f"fault-free, ABFT on, {dt:.1f} s"}
+        line["paper_context"] = {"Bulldozer64_K40c_n30720_nb512": "1092.4 GFLOP/s (Enhanced, no error, PAPER.md:374)",
+                                 "Tardis_M2075_n20480_nb256": "268.7 GFLOP/s (PAPER.md:366)"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if dist:
+        import torch.distributed as tdist
+        tdist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

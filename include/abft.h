@@ -97,8 +97,23 @@ typedef struct abft_options {
     int32_t K;            /* Opt. 3: V5 every K iterations; 1 = every one   */
     double c_tau;         /* threshold constant C_tau of reading A4 (default 64)               */
     int32_t lookahead;    /* reserved (0/1)                                                    */
-    int32_t pad;
+    int32_t profile;      /* 1: time every phase with CUDA events on `stream` (abft_last_profile) */
 } abft_options_t;
+
+/* Per-phase device time of the last abft_potrf* call on this thread with options.profile = 1.
+ * Phases: 0 encode, 1 V1/V2, 2 POTRF+inverse, 3 TRSM (+Alg. 2 rows), 4 V3, 5 V4, 6 panel
+ * write-back, 7 trailing update (data rows), 8 trailing update (checksum rows), 9 V5, 10 V6,
+ * 11 injection. flops / bytes are the ALGORITHMIC counts of DESIGN.md §6 (not executed ones). */
+#define ABFT_NPHASE 12
+typedef struct abft_profile {
+    int32_t nphase, pad;
+    double ms[16];
+    int64_t launches[16];   /* event-timed instances of the phase */
+    double flops[16];
+    double bytes[16];
+} abft_profile_t;
+int abft_last_profile(abft_profile_t* out);
+const char* abft_phase_name(int phase);
 
 /* Checksum encoding (§IV.A, cost 2n^2).
  * A: n x n lower (lda >= max(1,n)); chk: 2N x n output (ldchk >= 2N, N = n/nb): row 2I is

@@ -51,7 +51,12 @@ class Report(ctypes.Structure):
 
 class Options(ctypes.Structure):
     _fields_ = [("abft_enabled", ctypes.c_int32), ("K", ctypes.c_int32), ("c_tau", ctypes.c_double),
-                ("lookahead", ctypes.c_int32), ("pad", ctypes.c_int32)]
+                ("lookahead", ctypes.c_int32), ("profile", ctypes.c_int32)]
+
+
+class Profile(ctypes.Structure):
+    _fields_ = [("nphase", ctypes.c_int32), ("pad", ctypes.c_int32), ("ms", ctypes.c_double * 16),
+                ("launches", ctypes.c_int64 * 16), ("flops", ctypes.c_double * 16), ("bytes", ctypes.c_double * 16)]
 
 
 if not os.path.exists(LIB_PATH):
@@ -72,13 +77,17 @@ _lib.abft_potrf_dist.argtypes = [_i64, _i64, _vp, _i64, _vp, _i32, _i32, _vp, _v
 _lib.abft_last_launch_count.restype = _i64
 _lib.abft_version.restype = ctypes.c_char_p
 _lib.abft_last_error.restype = ctypes.c_char_p
+_lib.abft_phase_name.restype = ctypes.c_char_p
+_lib.abft_phase_name.argtypes = [_i32]
+_lib.abft_last_profile.argtypes = [_vp]
 for _f in ("abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
            "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist"):
     getattr(_lib, _f).restype = _i32
 
 EXPORTS = ["abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
            "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist",
-           "abft_last_launch_count", "abft_version", "abft_last_error"]
+           "abft_last_launch_count", "abft_version", "abft_last_error", "abft_last_profile",
+           "abft_phase_name"]
 
 
 def lib():
@@ -133,8 +142,19 @@ def _report_dict(rep, ev):
                 seconds=rep.seconds)
 
 
-def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0):
-    return Options(int(bool(abft_enabled)), int(K), float(c_tau), int(lookahead), 0)
+def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False):
+    return Options(int(bool(abft_enabled)), int(K), float(c_tau), int(lookahead), int(bool(profile)))
+
+
+def abft_last_profile():
+    """{phase name: dict(ms, launches, flops, bytes)} of the last profiled call on this thread."""
+    pr = Profile()
+    _lib.abft_last_profile(ctypes.byref(pr))
+    out = {}
+    for i in range(pr.nphase):
+        out[_lib.abft_phase_name(i).decode()] = dict(ms=pr.ms[i], launches=int(pr.launches[i]),
+                                                      flops=pr.flops[i], bytes=pr.bytes[i])
+    return out
 
 
 # ---- entry points (same names as the C-ABI) --------------------------------------------------

@@ -201,6 +201,57 @@ static void do_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, in
     if (!ptrs.empty()) launch_inject((int)ptrs.size(), ptrs.data(), masks.data(), ab, s);
 }
 
+// ---- per-phase profiler (options.profile) ----------------------------------------------------
+enum { PH_ENCODE, PH_V12, PH_POTRF, PH_TRSM, PH_V3, PH_V4, PH_WB, PH_UPD, PH_UPDC, PH_V5, PH_V6, PH_INJ };
+static const char* kPhaseNames[ABFT_NPHASE] = {"encode", "v1v2", "potrf_inv", "trsm", "v3", "v4", "writeback",
+                                               "update", "update_chk", "v5", "v6", "inject"};
+static thread_local abft_profile_t g_prof;
+
+struct Profiler {
+    bool on = false;
+    cudaStream_t s = nullptr;
+    struct Rec { int ph; cudaEvent_t a, b; double flops, bytes; };
+    std::vector<Rec> recs;
+    std::vector<cudaEvent_t> pool;
+    size_t used = 0;
+    int open_ph = -1; cudaEvent_t open_ev = nullptr;
+    cudaEvent_t get() {
+        if (used == pool.size()) { cudaEvent_t e; cudaEventCreate(&e); pool.push_back(e); }
+        return pool[used++];
+    }
+    void begin(int ph) {
+        if (!on) return;
+        open_ph = ph; open_ev = get(); cudaEventRecord(open_ev, s);
+    }
+    void end(double flops = 0, double bytes = 0) {
+        if (!on || open_ph < 0) return;
+        cudaEvent_t e = get(); cudaEventRecord(e, s);
+        recs.push_back({open_ph, open_ev, e, flops, bytes});
+        open_ph = -1;
+    }
+    void finish() {   // after a stream sync
+        if (!on) return;
+        memset(&g_prof, 0, sizeof g_prof);
+        g_prof.nphase = ABFT_NPHASE;
+        for (auto& r : recs) {
+            float ms = 0; cudaEventElapsedTime(&ms, r.a, r.b);
+            g_prof.ms[r.ph] += ms; g_prof.launches[r.ph] += 1;
+            g_prof.flops[r.ph] += r.flops; g_prof.bytes[r.ph] += r.bytes;
+        }
+        for (auto e : pool) cudaEventDestroy(e);
+        pool.clear(); recs.clear(); used = 0;
+    }
+};
+
+extern "C" int abft_last_profile(abft_profile_t* out) {
+    if (!out) return -1;
+    *out = g_prof;
+    return 0;
+}
+extern "C" const char* abft_phase_name(int phase) {
+    return (phase >= 0 && phase < ABFT_NPHASE) ? kPhaseNames[phase] : "";
+}
+
 static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t s,
                      const std::vector<abft_inject_spec_t>& inj, abft_report_t* rep, const abft_options_t& o) {
     const bool abft = o.abft_enabled != 0;
@@ -211,49 +262,77 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     cudaEvent_t e0 = nullptr, e1 = nullptr;
     if (rep) { cudaEventCreate(&e0); cudaEventCreate(&e1); cudaEventRecord(e0, s); }
     const int64_t N = w.N, B = nb;
+    const double Bd = (double)B;
     const int32_t* ab = &w.st->abort;
+    Profiler prof; prof.on = o.profile != 0; prof.s = s;
+    const double lowerB = Bd * (Bd + 1) / 2;                 // elements of a tril tile
     launch_zero(B, B, w.Li, B, s);
     if (abft) {   // encode
+        prof.begin(PH_ENCODE);
         launch_scales(n, nb, A, lda, w.scl, s);
         StageArgs a = stage_base(w, A, lda, o.c_tau, SK_ALL, 0, -1);
         a.encode = 1;
         launch_check(a, s);
+        const double el = (double)(N * (N - 1) / 2) * Bd * Bd + (double)N * lowerB;
+        prof.end(4.0 * el, 8.0 * el);
     }
     for (int64_t k = 0; k < N; ++k) {
         const int64_t m = N - k - 1, mB = m * B;
         const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
         double* Akk = A + k * B * lda + k * B;
         const Loc L{A, lda, w.chk, w.ldc, w.W, ldw, mB};
+        const double md = (double)m, mBd = (double)mB;
         if (abft) {
             do_inject(inj, k, ABFT_HOOK_REST, B, L, ab, s);
+            prof.begin(PH_V12);
             launch_check(stage_base(w, A, lda, o.c_tau, SK_COLUMN, ABFT_V2, (int)k), s);   // V1, V2
+            prof.end(4.0 * (lowerB + mBd * Bd), 8.0 * (lowerB + mBd * Bd));
         }
+        prof.begin(PH_POTRF);
         launch_chol_inv(Akk, lda, w.Li, B, k * B, w.tmp, w.st, s);
+        prof.end(2.0 * Bd * Bd * Bd / 3.0, 0);                    // B^3/3 (POTRF) + B^3/3 (TRTRI)
         // TRSM (+ Alg. 2 on the checksum rows of tile (k,k)): one GEMM per row segment
+        prof.begin(PH_TRSM);
         launch_gemm(mB, B, B, Akk + B, lda, w.Li, B, w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, s);
-        if (abft) {
+        if (abft)
             launch_gemm(2 * m + 2, B, B, w.chk + k * B * w.ldc + 2 * k, w.ldc, w.Li, B, w.W + mB, ldw, 1.0, 0.0,
                         true, 0, 1, 0, 0, 0, ab, s);
+        prof.end((mBd + (abft ? 2 * md + 2 : 0)) * Bd * Bd, 0);
+        if (abft) {
             do_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, L, ab, s);
             StageArgs a3 = stage_base(w, A, lda, o.c_tau, SK_DIAG_FACT, ABFT_V3, (int)k);
             a3.W = w.W; a3.ldw = ldw; a3.mB = mB;
+            prof.begin(PH_V3);
             launch_check(a3, s);                                                          // V3
+            prof.end(4.0 * lowerB, 8.0 * lowerB);
             do_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, L, ab, s);
             StageArgs a4 = stage_base(w, A, lda, o.c_tau, SK_PANEL, ABFT_V4, (int)k);
             a4.W = w.W; a4.ldw = ldw; a4.mB = mB;
+            prof.begin(PH_V4);
             launch_check(a4, s);                                                          // V4
+            prof.end(4.0 * mBd * Bd, 8.0 * mBd * Bd);
         }
+        prof.begin(PH_WB);
         launch_copy(mB, B, w.W, ldw, Akk + B, lda, ab, s);                                // L panel
         if (abft) launch_copy(2 * m + 2, B, w.W + mB, ldw, w.chk + k * B * w.ldc + 2 * k, w.ldc, ab, s);
+        prof.end(0, 16.0 * (mBd + (abft ? 2 * md + 2 : 0)) * Bd);
         if (m > 0) {
             double* Atr = Akk + B * lda + B;
+            prof.begin(PH_UPD);
             launch_gemm(mB, mB, B, w.W, ldw, w.W, ldw, Atr, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
+            prof.end(mBd * (mBd + 1) * Bd, 8.0 * (mBd * Bd + mBd * (mBd + 1)));   // SYRK: B mB (mB+1)
             if (abft) {
+                prof.begin(PH_UPDC);
                 launch_gemm(2 * m, mB, B, w.W + mB + 2, ldw, w.W, ldw, w.chk + (k + 1) * B * w.ldc + 2 * (k + 1),
                             w.ldc, -1.0, 1.0, true, 2, 0, B, 0, 0, ab, s);
+                prof.end(4.0 * Bd * Bd * md * (md + 1) / 2, 0);
                 do_inject(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s);
-                if (((k + 1) % K == 0) || k == N - 2)
+                if (((k + 1) % K == 0) || k == N - 2) {
+                    prof.begin(PH_V5);
                     launch_check(stage_base(w, A, lda, o.c_tau, SK_TRAIL, ABFT_V5, (int)k), s);  // V5
+                    const double el = md * (md - 1) / 2 * Bd * Bd + md * lowerB;
+                    prof.end(4.0 * el, 8.0 * el);
+                }
             }
         }
     }
@@ -262,7 +341,10 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         do_inject(inj, N, ABFT_HOOK_REST, B, L, ab, s);
         StageArgs a6 = stage_base(w, A, lda, o.c_tau, SK_ALL, ABFT_V6, (int)N);
         a6.factored = 1;
+        prof.begin(PH_V6);
         launch_check(a6, s);                                                              // V6
+        const double el = (double)(N * (N - 1) / 2) * Bd * Bd + (double)N * lowerB;
+        prof.end(4.0 * el, 8.0 * el);
     }
     ABFT_CUDA_TRY(cudaGetLastError());
     int status = 0;
@@ -273,6 +355,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         rep->seconds = ms * 1e-3;
         cudaEventDestroy(e0); cudaEventDestroy(e1);
     }
+    if (prof.on) { cudaStreamSynchronize(s); prof.finish(); }
     work_free(w, s);
     if (rc) return rc;
     ABFT_CUDA_TRY(cudaGetLastError());
@@ -282,7 +365,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
 static abft_options_t default_options() {
     abft_options_t o;
     memset(&o, 0, sizeof o);
-    o.abft_enabled = 1; o.K = 1; o.c_tau = 64.0; o.lookahead = 0;
+    o.abft_enabled = 1; o.K = 1; o.c_tau = 64.0; o.lookahead = 0; o.profile = 0;
     return o;
 }
 
