@@ -74,6 +74,7 @@ template <int BM, int BN, int BK, int WM, int WN, int STAGES, bool TB>
 __global__ void __launch_bounds__(GemmCfg<BM, BN, BK, WM, WN, STAGES, TB>::THREADS, 1)
 k_gemm_dmma(GemmArgs g) {
     using Cfg = GemmCfg<BM, BN, BK, WM, WN, STAGES, TB>;
+    constexpr int T = Cfg::THREADS;
     if (*(volatile const int32_t*)g.abort) return;
     // ---- tile mapping ----
     int64_t tm, tn;
@@ -104,24 +105,34 @@ k_gemm_dmma(GemmArgs g) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int wm = warp / Cfg::WARPS_N, wn = warp % Cfg::WARPS_N;
 
+    // ---- per-thread loader geometry (16-byte path): fixed row pair, k stepped by a constant ----
+    static_assert(T % (BM / 2) == 0 && T % (BN / 2) == 0 && T % (BK / 2) == 0, "loader mapping");
+    constexpr int A_KSTEP = T / (BM / 2), A_PER = BK / A_KSTEP;
+    const int a_mm = (tid % (BM / 2)) * 2, a_kk = tid / (BM / 2);
+    const int64_t a_gm = m0 + a_mm;
+    const int a_bytes = (a_gm < g.M) ? ((a_gm + 1 < g.M) ? 16 : 8) : 0;
+    const double* a_src = g.A + a_gm;                 // + k * lda
+    constexpr int BT_KSTEP = T / (BN / 2), BT_PER = BK / BT_KSTEP;
+    const int bt_nn = (tid % (BN / 2)) * 2, bt_kk = tid / (BN / 2);
+    const int64_t bt_gn = n0 + bt_nn;
+    const int bt_bytes = (bt_gn < g.N) ? ((bt_gn + 1 < g.N) ? 16 : 8) : 0;
+    constexpr int BN_NSTEP = T / (BK / 2), BN_PER = BN / BN_NSTEP;
+    const int bn_kk = (tid % (BK / 2)) * 2, bn_nn = tid / (BK / 2);
+
     auto load_stage = [&](int stage, int kt) {
         const int64_t k0 = kb + (int64_t)kt * BK;
         double* dA = sA + stage * Cfg::SA;
         double* dB = sB + stage * Cfg::SB;
-        // A: BK columns of BM rows
         if (g.vecA) {
-            constexpr int CH = BK * BM / 2;
-            for (int i = tid; i < CH; i += Cfg::THREADS) {
-                const int kk = i / (BM / 2), mm = (i % (BM / 2)) * 2;
-                const int64_t gm = m0 + mm, gk = k0 + kk;
-                int bytes = 0;
-                if (gk < ke && gm < g.M) bytes = (gm + 1 < g.M) ? 16 : 8;
-                const double* src = bytes ? g.A + gk * g.lda + gm : g.A;
-                cp_async16(dA + kk * Cfg::PA + mm, src, bytes);
+#pragma unroll
+            for (int q = 0; q < A_PER; ++q) {
+                const int kk = a_kk + q * A_KSTEP;
+                const int64_t gk = k0 + kk;
+                const int bytes = gk < ke ? a_bytes : 0;
+                cp_async16(dA + kk * Cfg::PA + a_mm, bytes ? a_src + gk * g.lda : g.A, bytes);
             }
         } else {
-            constexpr int CH = BK * BM;
-            for (int i = tid; i < CH; i += Cfg::THREADS) {
+            for (int i = tid; i < BK * BM; i += T) {
                 const int kk = i / BM, mm = i % BM;
                 const int64_t gm = m0 + mm, gk = k0 + kk;
                 const bool ok = gk < ke && gm < g.M;
@@ -130,17 +141,15 @@ k_gemm_dmma(GemmArgs g) {
         }
         if (TB) {  // Bm is N x K: column k holds n contiguous
             if (g.vecB) {
-                constexpr int CH = BK * BN / 2;
-                for (int i = tid; i < CH; i += Cfg::THREADS) {
-                    const int kk = i / (BN / 2), nn = (i % (BN / 2)) * 2;
-                    const int64_t gn = n0 + nn, gk = k0 + kk;
-                    int bytes = 0;
-                    if (gk < ke && gn < g.N) bytes = (gn + 1 < g.N) ? 16 : 8;
-                    cp_async16(dB + kk * Cfg::PB_T + nn, bytes ? g.B + gk * g.ldb + gn : g.B, bytes);
+#pragma unroll
+                for (int q = 0; q < BT_PER; ++q) {
+                    const int kk = bt_kk + q * BT_KSTEP;
+                    const int64_t gk = k0 + kk;
+                    const int bytes = gk < ke ? bt_bytes : 0;
+                    cp_async16(dB + kk * Cfg::PB_T + bt_nn, bytes ? g.B + gk * g.ldb + bt_gn : g.B, bytes);
                 }
             } else {
-                constexpr int CH = BK * BN;
-                for (int i = tid; i < CH; i += Cfg::THREADS) {
+                for (int i = tid; i < BK * BN; i += T) {
                     const int kk = i / BN, nn = i % BN;
                     const int64_t gn = n0 + nn, gk = k0 + kk;
                     const bool ok = gk < ke && gn < g.N;
@@ -149,17 +158,16 @@ k_gemm_dmma(GemmArgs g) {
             }
         } else {   // Bm is K x N: column n holds k contiguous
             if (g.vecB) {
-                constexpr int CH = BN * BK / 2;
-                for (int i = tid; i < CH; i += Cfg::THREADS) {
-                    const int nn = i / (BK / 2), kk = (i % (BK / 2)) * 2;
-                    const int64_t gn = n0 + nn, gk = k0 + kk;
+#pragma unroll
+                for (int q = 0; q < BN_PER; ++q) {
+                    const int nn = bn_nn + q * BN_NSTEP;
+                    const int64_t gn = n0 + nn, gk = k0 + bn_kk;
                     int bytes = 0;
                     if (gn < g.N && gk < ke) bytes = (gk + 1 < ke) ? 16 : 8;
-                    cp_async16(dB + nn * Cfg::PB_N + kk, bytes ? g.B + gn * g.ldb + gk : g.B, bytes);
+                    cp_async16(dB + nn * Cfg::PB_N + bn_kk, bytes ? g.B + gn * g.ldb + gk : g.B, bytes);
                 }
             } else {
-                constexpr int CH = BN * BK;
-                for (int i = tid; i < CH; i += Cfg::THREADS) {
+                for (int i = tid; i < BN * BK; i += T) {
                     const int nn = i / BK, kk = i % BK;
                     const int64_t gn = n0 + nn, gk = k0 + kk;
                     const bool ok = gn < g.N && gk < ke;
@@ -208,24 +216,60 @@ k_gemm_dmma(GemmArgs g) {
         }
     }
     cp_async_wait<0>();
+    __syncthreads();
 
-    // ---- epilogue: C = beta C + alpha acc, masked ----
+    // ---- epilogue: stage the tile in shared memory (column-major, pitch BM+2), then a coalesced
+    // 16-byte read-modify-write of C, four independent column segments in flight per thread ----
+    constexpr int PC = BM + 2;
+    static_assert((size_t)BN * PC * sizeof(double) <= Cfg::SMEM, "epilogue staging fits");
+    double* sC = smem;
 #pragma unroll
-    for (int i = 0; i < Cfg::FM; ++i) {
-        const int64_t r = m0 + wm * WM + i * 8 + fr;
-        if (r >= g.M) continue;
+    for (int i = 0; i < Cfg::FM; ++i)
 #pragma unroll
-        for (int j = 0; j < Cfg::FN; ++j) {
+        for (int j = 0; j < Cfg::FN; ++j)
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
-                if (c >= g.N) continue;
-                if (g.mask == MASK_LOWER && r < c) continue;
-                if (g.mask == MASK_CHK && (g.q_tile0 + r / 2) < (g.c_tile0 + c / g.nb)) continue;
-                double* p = g.C + c * g.ldc + r;
-                const double v = g.alpha * acc[i][j][h];
-                *p = (g.beta == 0.0) ? v : fma(g.beta, *p, v);
+            for (int h = 0; h < 2; ++h)
+                sC[(wn * WN + j * 8 + fc * 2 + h) * PC + wm * WM + i * 8 + fr] = acc[i][j][h];
+    __syncthreads();
+    constexpr int RP = BM / 2;                 // row pairs per column
+    constexpr int ITEMS = BN * RP;             // row pairs in the tile
+    constexpr int BATCH = 4;
+    static_assert(ITEMS % (T * BATCH) == 0, "epilogue batching");
+    const bool vecC = ((((uintptr_t)g.C) & 15) == 0) && (g.ldc % 2 == 0);
+    const double alpha = g.alpha, beta = g.beta;
+    for (int base = tid; base < ITEMS; base += T * BATCH) {
+        double2 old[BATCH];
+        bool ok0[BATCH], ok1[BATCH];
+        double* ptr[BATCH];
+#pragma unroll
+        for (int b = 0; b < BATCH; ++b) {
+            const int idx = base + b * T;
+            const int c = idx / RP, rp = (idx % RP) * 2;
+            const int64_t gr = m0 + rp, gc = n0 + c;
+            bool o0 = gr < g.M && gc < g.N, o1 = gr + 1 < g.M && gc < g.N;
+            if (g.mask == MASK_LOWER) { o0 = o0 && gr >= gc; o1 = o1 && gr + 1 >= gc; }
+            else if (g.mask == MASK_CHK) {
+                const int64_t J = g.c_tile0 + gc / g.nb;
+                o0 = o0 && (g.q_tile0 + gr / 2) >= J;
+                o1 = o1 && (g.q_tile0 + (gr + 1) / 2) >= J;
             }
+            ok0[b] = o0; ok1[b] = o1;
+            ptr[b] = g.C + gc * g.ldc + gr;
+            old[b] = make_double2(0.0, 0.0);
+            if (beta != 0.0) {
+                if (o0 && o1 && vecC) old[b] = *reinterpret_cast<const double2*>(ptr[b]);
+                else { if (o0) old[b].x = ptr[b][0]; if (o1) old[b].y = ptr[b][1]; }
+            }
+        }
+#pragma unroll
+        for (int b = 0; b < BATCH; ++b) {
+            const int idx = base + b * T;
+            const int c = idx / RP, rp = (idx % RP) * 2;
+            const double v0 = alpha * sC[c * PC + rp], v1 = alpha * sC[c * PC + rp + 1];
+            const double r0 = beta == 0.0 ? v0 : fma(beta, old[b].x, v0);
+            const double r1 = beta == 0.0 ? v1 : fma(beta, old[b].y, v1);
+            if (ok0[b] && ok1[b] && vecC) *reinterpret_cast<double2*>(ptr[b]) = make_double2(r0, r1);
+            else { if (ok0[b]) ptr[b][0] = r0; if (ok1[b]) ptr[b][1] = r1; }
         }
     }
 }
