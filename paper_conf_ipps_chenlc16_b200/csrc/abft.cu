@@ -144,13 +144,15 @@ static StageArgs stage_base(const Work& w, double* A, int64_t lda, double c_tau,
     a.s = w.scl; a.S1 = w.scl ? w.scl + w.n : nullptr; a.S2 = w.scl ? w.scl + w.n + w.N : nullptr;
     a.c_tau = c_tau; a.col_owner_mod = 1; a.col_owner_rank = 0;
     a.st = w.st; a.ev = w.ev; a.ev_cap = w.ev_cap;
+    a.flist = 0; a.j_lo = k + 1; a.j_hi = w.N;
     return a;
 }
 
 // Fill the host report from the device state (the one synchronisation of a call).
 static int finish_report(const Work& w, abft_report_t* rep, cudaStream_t s, int* status_out) {
-    DevState hs;
-    ABFT_CUDA_TRY(cudaMemcpyAsync(&hs, w.st, offsetof(DevState, flags), cudaMemcpyDeviceToHost, s));
+    std::vector<char> hbuf(sizeof(DevState));
+    DevState& hs = *reinterpret_cast<DevState*>(hbuf.data());
+    ABFT_CUDA_TRY(cudaMemcpyAsync(&hs, w.st, offsetof(DevState, fl), cudaMemcpyDeviceToHost, s));
     ABFT_CUDA_TRY(cudaStreamSynchronize(s));
     const int64_t nev = (int64_t)hs.nev;
     if (rep) {
@@ -209,25 +211,23 @@ static thread_local abft_profile_t g_prof;
 
 struct Profiler {
     bool on = false;
-    cudaStream_t s = nullptr;
     struct Rec { int ph; cudaEvent_t a, b; double flops, bytes; };
     std::vector<Rec> recs;
     std::vector<cudaEvent_t> pool;
     size_t used = 0;
-    int open_ph = -1; cudaEvent_t open_ev = nullptr;
     cudaEvent_t get() {
         if (used == pool.size()) { cudaEvent_t e; cudaEventCreate(&e); pool.push_back(e); }
         return pool[used++];
     }
-    void begin(int ph) {
-        if (!on) return;
-        open_ph = ph; open_ev = get(); cudaEventRecord(open_ev, s);
+    // begin() returns a token; end() closes it (phases may be open on two streams at once)
+    cudaEvent_t begin(cudaStream_t s) {
+        if (!on) return nullptr;
+        cudaEvent_t e = get(); cudaEventRecord(e, s); return e;
     }
-    void end(double flops = 0, double bytes = 0) {
-        if (!on || open_ph < 0) return;
+    void end(cudaEvent_t tok, int ph, cudaStream_t s, double flops = 0, double bytes = 0) {
+        if (!on || !tok) return;
         cudaEvent_t e = get(); cudaEventRecord(e, s);
-        recs.push_back({open_ph, open_ev, e, flops, bytes});
-        open_ph = -1;
+        recs.push_back({ph, tok, e, flops, bytes});
     }
     void finish() {   // after a stream sync
         if (!on) return;
@@ -252,6 +252,28 @@ extern "C" const char* abft_phase_name(int phase) {
     return (phase >= 0 && phase < ABFT_NPHASE) ? kPhaseNames[phase] : "";
 }
 
+// Column-block filter for an injection (which block column J its target lives in).
+static int64_t inj_col_block(const abft_inject_spec_t& sp, int64_t nb) { return sp.col / nb; }
+
+static void do_inject_if(const std::vector<abft_inject_spec_t>& list, int64_t k, int hook, int64_t nb, const Loc& L,
+                         const int32_t* ab, cudaStream_t s, int64_t jlo, int64_t jhi, bool inside) {
+    std::vector<double*> ptrs; std::vector<uint64_t> masks;
+    for (const auto& sp : list) {
+        if (sp.k != k || sp.hook != hook) continue;
+        const int64_t J = inj_col_block(sp, nb);
+        const bool in = J >= jlo && J < jhi;
+        if (in != inside) continue;
+        ptrs.push_back(inj_ptr(sp, k, nb, L)); masks.push_back(sp.xor_mask);
+    }
+    if (!ptrs.empty()) launch_inject((int)ptrs.size(), ptrs.data(), masks.data(), ab, s);
+}
+
+// The single-GPU driver with depth-1 look-ahead: the panel of iteration k+1
+// (V1/V2, POTRF + inverse, TRSM, V3, V4, write-back) runs on a high-priority stream P as soon
+// as block column k+1 has received update k and its V5 check, while the main stream S applies
+// the rest of update k and V5 to the trailing matrix. Hook timing and the set of events are
+// those of the sequential schedule: injections and checks are split by block column exactly
+// where the two streams split the work.
 static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t s,
                      const std::vector<abft_inject_spec_t>& inj, abft_report_t* rep, const abft_options_t& o) {
     const bool abft = o.abft_enabled != 0;
@@ -259,81 +281,152 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     Work w;
     int rc = work_alloc(w, n, nb, n, rep ? std::max<int64_t>(rep->cap, 1) : 1024, abft, s);
     if (rc) return rc;
-    cudaEvent_t e0 = nullptr, e1 = nullptr;
-    if (rep) { cudaEventCreate(&e0); cudaEventCreate(&e1); cudaEventRecord(e0, s); }
     const int64_t N = w.N, B = nb;
     const double Bd = (double)B;
     const int32_t* ab = &w.st->abort;
-    Profiler prof; prof.on = o.profile != 0; prof.s = s;
+    // second panel buffer for the look-ahead
+    double* Wbuf[2] = {w.W, nullptr};
+    const int64_t wrows = (N - 1) * nb + 2 * N + 2;
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&Wbuf[1], sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb), s));
+    cudaStream_t P = nullptr;
+    int lo_prio = 0, hi_prio = 0;
+    cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio);
+    ABFT_CUDA_TRY(cudaStreamCreateWithPriority(&P, cudaStreamNonBlocking, hi_prio));
+    std::vector<cudaEvent_t> evs;
+    auto new_event = [&]() { cudaEvent_t e; cudaEventCreateWithFlags(&e, cudaEventDisableTiming); evs.push_back(e); return e; };
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (rep) { cudaEventCreate(&e0); cudaEventCreate(&e1); cudaEventRecord(e0, s); }
+    Profiler prof; prof.on = o.profile != 0;
     const double lowerB = Bd * (Bd + 1) / 2;                 // elements of a tril tile
     launch_zero(B, B, w.Li, B, s);
     if (abft) {   // encode
-        prof.begin(PH_ENCODE);
+        cudaEvent_t t = prof.begin(s);
         launch_scales(n, nb, A, lda, w.scl, s);
         StageArgs a = stage_base(w, A, lda, o.c_tau, SK_ALL, 0, -1);
         a.encode = 1;
         launch_check(a, s);
         const double el = (double)(N * (N - 1) / 2) * Bd * Bd + (double)N * lowerB;
-        prof.end(4.0 * el, 8.0 * el);
+        prof.end(t, PH_ENCODE, s, 4.0 * el, 8.0 * el);
     }
-    for (int64_t k = 0; k < N; ++k) {
+    {   // P starts after everything enqueued on S so far
+        cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(P, e, 0);
+    }
+
+    // ---- the panel of iteration k, on stream P ----
+    auto panel = [&](int64_t k) {
         const int64_t m = N - k - 1, mB = m * B;
         const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
+        double* W = Wbuf[k & 1];
         double* Akk = A + k * B * lda + k * B;
-        const Loc L{A, lda, w.chk, w.ldc, w.W, ldw, mB};
+        const Loc L{A, lda, w.chk, w.ldc, W, ldw, mB};
         const double md = (double)m, mBd = (double)mB;
+        Work wk = w; wk.W = W;
         if (abft) {
-            do_inject(inj, k, ABFT_HOOK_REST, B, L, ab, s);
-            prof.begin(PH_V12);
-            launch_check(stage_base(w, A, lda, o.c_tau, SK_COLUMN, ABFT_V2, (int)k), s);   // V1, V2
-            prof.end(4.0 * (lowerB + mBd * Bd), 8.0 * (lowerB + mBd * Bd));
+            do_inject_if(inj, k, ABFT_HOOK_REST, B, L, ab, P, k, k + 1, true);   // REST(k) into column k
+            StageArgs a = stage_base(wk, A, lda, o.c_tau, SK_COLUMN, ABFT_V2, (int)k);
+            a.flist = 1;
+            cudaEvent_t t = prof.begin(P);
+            launch_check(a, P);                                                  // V1, V2
+            prof.end(t, PH_V12, P, 4.0 * (lowerB + mBd * Bd), 8.0 * (lowerB + mBd * Bd));
         }
-        prof.begin(PH_POTRF);
-        launch_chol_inv(Akk, lda, w.Li, B, k * B, w.tmp, w.st, s);
-        prof.end(2.0 * Bd * Bd * Bd / 3.0, 0);                    // B^3/3 (POTRF) + B^3/3 (TRTRI)
+        cudaEvent_t t = prof.begin(P);
+        launch_chol_inv(Akk, lda, w.Li, B, k * B, w.tmp, w.st, P);
+        prof.end(t, PH_POTRF, P, 2.0 * Bd * Bd * Bd / 3.0, 0);
         // TRSM (+ Alg. 2 on the checksum rows of tile (k,k)): one GEMM per row segment
-        prof.begin(PH_TRSM);
-        launch_gemm(mB, B, B, Akk + B, lda, w.Li, B, w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, s);
+        t = prof.begin(P);
+        launch_gemm(mB, B, B, Akk + B, lda, w.Li, B, W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, P);
         if (abft)
-            launch_gemm(2 * m + 2, B, B, w.chk + k * B * w.ldc + 2 * k, w.ldc, w.Li, B, w.W + mB, ldw, 1.0, 0.0,
-                        true, 0, 1, 0, 0, 0, ab, s);
-        prof.end((mBd + (abft ? 2 * md + 2 : 0)) * Bd * Bd, 0);
+            launch_gemm(2 * m + 2, B, B, w.chk + k * B * w.ldc + 2 * k, w.ldc, w.Li, B, W + mB, ldw, 1.0, 0.0,
+                        true, 0, 1, 0, 0, 0, ab, P);
+        prof.end(t, PH_TRSM, P, (mBd + (abft ? 2 * md + 2 : 0)) * Bd * Bd, 0);
         if (abft) {
-            do_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, L, ab, s);
-            StageArgs a3 = stage_base(w, A, lda, o.c_tau, SK_DIAG_FACT, ABFT_V3, (int)k);
-            a3.W = w.W; a3.ldw = ldw; a3.mB = mB;
-            prof.begin(PH_V3);
-            launch_check(a3, s);                                                          // V3
-            prof.end(4.0 * lowerB, 8.0 * lowerB);
-            do_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, L, ab, s);
-            StageArgs a4 = stage_base(w, A, lda, o.c_tau, SK_PANEL, ABFT_V4, (int)k);
-            a4.W = w.W; a4.ldw = ldw; a4.mB = mB;
-            prof.begin(PH_V4);
-            launch_check(a4, s);                                                          // V4
-            prof.end(4.0 * mBd * Bd, 8.0 * mBd * Bd);
+            do_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, L, ab, P);
+            StageArgs a3 = stage_base(wk, A, lda, o.c_tau, SK_DIAG_FACT, ABFT_V3, (int)k);
+            a3.ldw = ldw; a3.mB = mB; a3.flist = 1;
+            t = prof.begin(P);
+            launch_check(a3, P);                                                 // V3
+            prof.end(t, PH_V3, P, 4.0 * lowerB, 8.0 * lowerB);
+            do_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, L, ab, P);
+            StageArgs a4 = stage_base(wk, A, lda, o.c_tau, SK_PANEL, ABFT_V4, (int)k);
+            a4.ldw = ldw; a4.mB = mB; a4.flist = 1;
+            t = prof.begin(P);
+            launch_check(a4, P);                                                 // V4
+            prof.end(t, PH_V4, P, 4.0 * mBd * Bd, 8.0 * mBd * Bd);
         }
-        prof.begin(PH_WB);
-        launch_copy(mB, B, w.W, ldw, Akk + B, lda, ab, s);                                // L panel
-        if (abft) launch_copy(2 * m + 2, B, w.W + mB, ldw, w.chk + k * B * w.ldc + 2 * k, w.ldc, ab, s);
-        prof.end(0, 16.0 * (mBd + (abft ? 2 * md + 2 : 0)) * Bd);
-        if (m > 0) {
-            double* Atr = Akk + B * lda + B;
-            prof.begin(PH_UPD);
-            launch_gemm(mB, mB, B, w.W, ldw, w.W, ldw, Atr, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
-            prof.end(mBd * (mBd + 1) * Bd, 8.0 * (mBd * Bd + mBd * (mBd + 1)));   // SYRK: B mB (mB+1)
+        t = prof.begin(P);
+        launch_copy(mB, B, W, ldw, Akk + B, lda, ab, P);                        // L panel
+        if (abft) launch_copy(2 * m + 2, B, W + mB, ldw, w.chk + k * B * w.ldc + 2 * k, w.ldc, ab, P);
+        prof.end(t, PH_WB, P, 0, 16.0 * (mBd + (abft ? 2 * md + 2 : 0)) * Bd);
+        cudaEvent_t e = new_event(); cudaEventRecord(e, P);
+        return e;
+    };
+
+    // ---- trailing update of iteration k restricted to block columns [jlo, jhi), on S ----
+    auto update_cols = [&](int64_t k, int64_t jlo, int64_t jhi) {
+        const int64_t m = N - k - 1, mB = m * B;
+        const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
+        double* W = Wbuf[k & 1];
+        const int64_t c0 = (jlo - k - 1) * B, nc = (jhi - jlo) * B;   // W row offset of column block jlo
+        const int64_t rows = mB - c0;                                   // data rows from block jlo down
+        double* C = A + jlo * B * lda + jlo * B;
+        const double r = (double)rows, c = (double)nc;
+        cudaEvent_t t = prof.begin(s);
+        // C[rows x nc] -= W[c0:, :] W[c0:c0+nc, :]^T, lower (r >= c)
+        launch_gemm(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
+        prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd, 0);
+        if (abft) {
+            // checksum rows of tiles I >= jlo: chk[2I+t, cols] -= W_chk(I) W[c0:c0+nc]^T, I >= J
+            const int64_t q0 = 2 * (jlo - k - 1);                       // first chk row of tile jlo in W
+            const int64_t nq = 2 * (N - jlo);
+            t = prof.begin(s);
+            launch_gemm(nq, nc, B, W + mB + 2 + q0, ldw, W + c0, ldw, w.chk + jlo * B * w.ldc + 2 * jlo, w.ldc,
+                        -1.0, 1.0, true, 2, 0, B, 0, 0, ab, s);
+            const double mm = (double)(N - jlo), jj = (double)(jhi - jlo);
+            prof.end(t, PH_UPDC, s, 4.0 * Bd * Bd * (jj * mm - jj * (jj - 1) / 2), 0);
+        }
+    };
+    auto v5_cols = [&](int64_t k, int64_t jlo, int64_t jhi) {
+        StageArgs a = stage_base(w, A, lda, o.c_tau, SK_TRAIL, ABFT_V5, (int)k);
+        a.j_lo = jlo; a.j_hi = jhi; a.flist = 0;
+        const double el = (double)stage_count(a) * Bd * Bd - (double)(jhi - jlo) * Bd * (Bd - 1) / 2;
+        cudaEvent_t t = prof.begin(s);
+        launch_check(a, s);
+        prof.end(t, PH_V5, s, 4.0 * el, 8.0 * el);
+    };
+
+    std::vector<cudaEvent_t> pan(N, nullptr);
+    if (abft) {   // REST(0) outside block column 0 (column 0 is handled by the panel stream)
+        const Loc L0{A, lda, w.chk, w.ldc, Wbuf[0], 1, 0};
+        do_inject_if(inj, 0, ABFT_HOOK_REST, B, L0, ab, s, 0, 1, false);
+    }
+    pan[0] = panel(0);
+    for (int64_t k = 0; k < N; ++k) {
+        cudaStreamWaitEvent(s, pan[k], 0);
+        const int64_t m = N - k - 1, mB = m * B;
+        if (m == 0) break;
+        const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
+        const Loc L{A, lda, w.chk, w.ldc, Wbuf[k & 1], ldw, mB};
+        const bool gated = ((k + 1) % K == 0) || k == N - 2;
+        // (a) block column k+1 first: update, UPDATE_OUT hook, V5 -> hand it to the panel stream
+        update_cols(k, k + 1, k + 2);
+        if (abft) {
+            do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 1, k + 2, true);
+            if (gated) v5_cols(k, k + 1, k + 2);
+        }
+        cudaEvent_t ec = new_event(); cudaEventRecord(ec, s);
+        cudaStreamWaitEvent(P, ec, 0);
+        pan[k + 1] = panel(k + 1);
+        // (b) the rest of the trailing matrix
+        if (m > 1) {
+            update_cols(k, k + 2, N);
             if (abft) {
-                prof.begin(PH_UPDC);
-                launch_gemm(2 * m, mB, B, w.W + mB + 2, ldw, w.W, ldw, w.chk + (k + 1) * B * w.ldc + 2 * (k + 1),
-                            w.ldc, -1.0, 1.0, true, 2, 0, B, 0, 0, ab, s);
-                prof.end(4.0 * Bd * Bd * md * (md + 1) / 2, 0);
-                do_inject(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s);
-                if (((k + 1) % K == 0) || k == N - 2) {
-                    prof.begin(PH_V5);
-                    launch_check(stage_base(w, A, lda, o.c_tau, SK_TRAIL, ABFT_V5, (int)k), s);  // V5
-                    const double el = md * (md - 1) / 2 * Bd * Bd + md * lowerB;
-                    prof.end(4.0 * el, 8.0 * el);
-                }
+                do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 2, N, true);
+                if (gated) v5_cols(k, k + 2, N);
             }
+        }
+        if (abft) {   // REST(k+1) outside block column k+1 (that one was applied on P)
+            const Loc L1{A, lda, w.chk, w.ldc, Wbuf[(k + 1) & 1], 1, 0};
+            do_inject_if(inj, k + 1, ABFT_HOOK_REST, B, L1, ab, s, k + 1, k + 2, false);
         }
     }
     if (abft) {
@@ -341,10 +434,10 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         do_inject(inj, N, ABFT_HOOK_REST, B, L, ab, s);
         StageArgs a6 = stage_base(w, A, lda, o.c_tau, SK_ALL, ABFT_V6, (int)N);
         a6.factored = 1;
-        prof.begin(PH_V6);
+        cudaEvent_t t = prof.begin(s);
         launch_check(a6, s);                                                              // V6
         const double el = (double)(N * (N - 1) / 2) * Bd * Bd + (double)N * lowerB;
-        prof.end(4.0 * el, 8.0 * el);
+        prof.end(t, PH_V6, s, 4.0 * el, 8.0 * el);
     }
     ABFT_CUDA_TRY(cudaGetLastError());
     int status = 0;
@@ -356,7 +449,10 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         cudaEventDestroy(e0); cudaEventDestroy(e1);
     }
     if (prof.on) { cudaStreamSynchronize(s); prof.finish(); }
+    cudaFreeAsync(Wbuf[1], s);
     work_free(w, s);
+    for (auto e : evs) cudaEventDestroy(e);
+    cudaStreamDestroy(P);
     if (rc) return rc;
     ABFT_CUDA_TRY(cudaGetLastError());
     return status;

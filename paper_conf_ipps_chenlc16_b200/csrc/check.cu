@@ -88,9 +88,10 @@ __global__ void __launch_bounds__(kChkThreads) k_check_phase1(StageArgs a) {
     const bool f1 = !dfinite(d1) || fabs(d1) > tau1;        // P:195 + A5
     const bool f2 = !dfinite(d2) || fabs(d2) > tau2;
     if (!(f1 || f2)) return;
-    const int slot = atomicAdd(&a.st->nflag, 1);
-    if (slot >= kFlagCap) { a.st->flag_overflow = 1; return; }
-    Flag& f = a.st->flags[slot];
+    FlagList& FL = a.st->fl[a.flist];
+    const int slot = atomicAdd(&FL.nflag, 1);
+    if (slot >= kFlagCap) { FL.overflow = 1; return; }
+    Flag& f = FL.flags[slot];
     f.I = (int32_t)I; f.J = (int32_t)J; f.c = (int32_t)c;
     f.d1 = d1; f.d2 = d2; f.r1 = r1; f.r2 = r2;
 }
@@ -137,15 +138,16 @@ struct Fix { double* p; double* p2; double val; };
 // corrections from the pre-correction tile, apply them per tile, log events. One CTA.
 __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
     DevState* st = a.st;
+    FlagList& FL = st->fl[a.flist];
     __shared__ int s_n;
     __shared__ Fix s_fix[64];
     __shared__ int s_nfix, s_unc, s_stop;
     __shared__ double redv[256];
     __shared__ long long redi[256];
     if (threadIdx.x == 0) {
-        s_n = min(st->nflag, kFlagCap);
+        s_n = min(FL.nflag, kFlagCap);
         if (st->abort) s_n = 0;
-        if (st->flag_overflow && !st->abort) {   // more flagged columns than we can resolve
+        if (FL.overflow && !st->abort) {   // more flagged columns than we can resolve
             st->status = ABFT_UNCORRECTABLE; st->abort = 1; s_n = 0;
             const long long e = (long long)atomicAdd(&st->nev, 1ull);
             if (e < a.ev_cap) {
@@ -156,7 +158,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
             st->n_unc++;
         }
         // insertion sort by (J, I, c): the oracle's check order
-        Flag* F = st->flags;
+        Flag* F = FL.flags;
         for (int i = 1; i < s_n; ++i) {
             Flag x = F[i]; int j = i - 1;
             auto key = [](const Flag& f) { return ((long long)f.J << 40) | ((long long)f.I << 20) | f.c; };
@@ -171,14 +173,14 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
     int i0 = 0;
     while (i0 < n && !s_stop) {
         // entries [i0, i1) belong to one tile
-        const Flag first = st->flags[i0];
+        const Flag first = FL.flags[i0];
         int i1 = i0;
-        while (i1 < n && st->flags[i1].I == first.I && st->flags[i1].J == first.J) ++i1;
+        while (i1 < n && FL.flags[i1].I == first.I && FL.flags[i1].J == first.J) ++i1;
         const TileView v = stage_view(a, first.I, first.J);
         if (threadIdx.x == 0) { s_nfix = 0; s_unc = 0; }
         __syncthreads();
         for (int e = i0; e < i1; ++e) {
-            const Flag f = st->flags[e];
+            const Flag f = FL.flags[e];
             const int64_t c = f.c;
             double tau1, tau2;
             thresholds(a, f.I, (int64_t)f.J * B + c, v.factored, tau1, tau2);
@@ -263,7 +265,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
         __syncthreads();
         i0 = i1;
     }
-    if (threadIdx.x == 0) { st->nflag = 0; st->flag_overflow = 0; }
+    if (threadIdx.x == 0) { FL.nflag = 0; FL.overflow = 0; }
 }
 
 // Threshold scales of reading A4: s_i = sqrt(A_ii); S1_I = sum s_i, S2_I = sum (i+1) s_i over
@@ -289,17 +291,7 @@ __global__ void k_scales_block(int64_t N, int64_t B, const double* s, double* S1
 using namespace abft;
 
 int launch_check(const StageArgs& a, cudaStream_t s) {
-    int64_t count;
-    {
-        const int64_t N = a.N, k = a.k;
-        switch (a.kind) {
-            case SK_COLUMN: count = N - k; break;
-            case SK_DIAG_FACT: count = 1; break;
-            case SK_PANEL: count = N - k - 1; break;
-            case SK_TRAIL: { int64_t m = N - k - 1; count = m * (m + 1) / 2; break; }
-            default: count = N * (N + 1) / 2;
-        }
-    }
+    const int64_t count = stage_count(a);
     if (count <= 0) return 0;
     const int64_t chunks = (a.nb + kChkCols - 1) / kChkCols;
     k_check_phase1<<<(unsigned)(count * chunks), kChkThreads, 0, s>>>(a);

@@ -18,17 +18,21 @@ struct Flag {
 
 constexpr int kFlagCap = 8192;
 
+// Flagged columns pending resolution (phase 1 -> phase 2). One list per concurrent stream.
+struct FlagList {
+    int32_t nflag, overflow;
+    Flag flags[kFlagCap];
+};
+
 // Device-resident run state. One per abft_* call.
 struct DevState {
     int32_t abort;        // set by UNCORRECTABLE / NOT_SPD: every later kernel returns at entry
     int32_t status;       // ABFT_OK / ABFT_UNCORRECTABLE / ABFT_NOT_SPD
     long long info;       // LAPACK info (1-based)
-    int32_t nflag;        // flagged columns pending resolution (phase 1 -> phase 2)
-    int32_t flag_overflow;
     unsigned long long nev;        // events raised
     unsigned long long n_checks;   // tile checks run
     long long n_detected, n_data, n_nonfinite, n_chk1, n_chk2, n_unc;
-    Flag flags[kFlagCap];
+    FlagList fl[2];       // [0]: main stream, [1]: look-ahead panel stream
 };
 
 // Where the tiles of a check stage live (DESIGN.md §5 "data layout").
@@ -51,6 +55,8 @@ struct StageArgs {
     const double* s; const double* S1; const double* S2;  // threshold scales
     double c_tau;
     int32_t col_owner_mod, col_owner_rank;  // dist: local column mapping (1, 0 on one GPU)
+    int32_t flist, pad2;            // flag list used by this stage (one per stream)
+    int64_t j_lo, j_hi;             // SK_TRAIL: block columns [j_lo, j_hi)
     DevState* st;
     abft_event_t* ev; int64_t ev_cap;
 };
@@ -62,13 +68,16 @@ struct TileView {
     bool diag, factored;
 };
 
-__device__ __forceinline__ int64_t stage_count(const StageArgs& a) {
+__host__ __device__ __forceinline__ int64_t stage_count(const StageArgs& a) {
     const int64_t N = a.N, k = a.k;
     switch (a.kind) {
         case SK_COLUMN: return N - k;
         case SK_DIAG_FACT: return 1;
         case SK_PANEL: return N - k - 1;
-        case SK_TRAIL: { int64_t m = N - k - 1; return m * (m + 1) / 2; }
+        case SK_TRAIL: {
+            const int64_t lo = a.j_lo, hi = a.j_hi;
+            return hi <= lo ? 0 : (hi - lo) * N - (hi * (hi - 1) - lo * (lo - 1)) / 2;
+        }
         default: return N * (N + 1) / 2;
     }
 }
@@ -81,7 +90,7 @@ __device__ __forceinline__ void stage_tile(const StageArgs& a, int64_t t, int64_
         case SK_DIAG_FACT: I = k; J = k; return;
         case SK_PANEL: I = k + 1 + t; J = k; return;
         default: {
-            const int64_t j0 = (a.kind == SK_TRAIL) ? k + 1 : 0;
+            const int64_t j0 = (a.kind == SK_TRAIL) ? a.j_lo : 0;
             const int64_t m = N - j0;
             int64_t jj = 0, rem = t;
             while (rem >= m - jj) { rem -= m - jj; ++jj; }

@@ -78,12 +78,16 @@ k_gemm_dmma(GemmArgs g) {
     if (*(volatile const int32_t*)g.abort) return;
     // ---- tile mapping ----
     int64_t tm, tn;
-    if (g.mask == MASK_LOWER) {  // lower-triangular tile enumeration, row-major
-        const int64_t idx = blockIdx.x;
-        int64_t a = (int64_t)((sqrt(8.0 * (double)idx + 1.0) - 1.0) * 0.5);
-        while (a * (a + 1) / 2 > idx) --a;
-        while ((a + 1) * (a + 2) / 2 <= idx) ++a;
-        tm = a; tn = idx - a * (a + 1) / 2;
+    if (g.mask == MASK_LOWER) {  // lower trapezoid (tile row >= tile col, col < tiles_n), row-major
+        const int64_t idx = blockIdx.x, TN = g.tiles_n, tri = TN * (TN + 1) / 2;
+        if (idx < tri) {
+            int64_t a = (int64_t)((sqrt(8.0 * (double)idx + 1.0) - 1.0) * 0.5);
+            while (a * (a + 1) / 2 > idx) --a;
+            while ((a + 1) * (a + 2) / 2 <= idx) ++a;
+            tm = a; tn = idx - a * (a + 1) / 2;
+        } else {
+            tm = TN + (idx - tri) / TN; tn = (idx - tri) % TN;
+        }
     } else {
         tm = blockIdx.x / g.tiles_n; tn = blockIdx.x % g.tiles_n;
     }
@@ -286,7 +290,7 @@ static int run_cfg(GemmArgs g, cudaStream_t s) {
     const int64_t tm = (g.M + BM - 1) / BM, tn = (g.N + BN - 1) / BN;
     g.tiles_n = tn;
     int64_t grid;
-    if (g.mask == MASK_LOWER) grid = tm * (tm + 1) / 2;
+    if (g.mask == MASK_LOWER) grid = tn * (tn + 1) / 2 + (tm - tn) * tn;   // requires N <= M
     else grid = tm * tn;
     if (grid <= 0) return 0;
     kern<<<(unsigned)grid, Cfg::THREADS, Cfg::SMEM, s>>>(g);
@@ -315,7 +319,7 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
     g.vecB = aligned16(B) && (ldb % 2 == 0);
     auto tiles = [&](int64_t t) {
         const int64_t tm = (M + t - 1) / t, tn = (N + t - 1) / t;
-        return mask == MASK_LOWER ? tm * (tm + 1) / 2 : tm * tn;
+        return mask == MASK_LOWER ? tn * (tn + 1) / 2 + (tm - tn) * tn : tm * tn;
     };
     int tile = force_tile;
     if (!tile) {
