@@ -22,6 +22,9 @@
 //   KR_LE_M  : k < m0 + BM   (A = inv(L) lower, NN)
 #include "common.cuh"
 
+#include <algorithm>
+#include <cstdlib>
+
 namespace abft {
 
 enum { MASK_NONE = 0, MASK_LOWER = 1, MASK_CHK = 2 };
@@ -298,6 +301,214 @@ static int run_cfg(GemmArgs g, cudaStream_t s) {
     return 0;
 }
 
+// ============================================================================================
+// Warp-specialised persistent variant (the hot path: trailing update and panel TRSM).
+//
+// One CTA per SM loops over output tiles. Warp 8 is the producer: one elected lane arms an
+// mbarrier with the stage's byte count, then the 32 lanes issue one cp.async.bulk per operand
+// column (1 KB each, straight into the padded, conflict-free layout) that completes on that
+// mbarrier; it also prefetches the next tile's C columns into L2. Warps 0-7 consume: wait on
+// the stage's "full" barrier, run the DMMA k-steps, release the stage with one arrive per warp
+// on its "empty" barrier. No CTA-wide barrier in the main loop. C is read into the
+// accumulators at the start of a tile (acc = alpha*beta*C, alpha = +-1) so that the epilogue is
+// a stream of fire-and-forget stores and never exposes load latency.
+// ============================================================================================
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    uint32_t done;
+    do {
+        asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+                     : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void prefetch_l2(const void* src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(src), "r"(bytes) : "memory");
+}
+
+struct WsCfg {
+    static constexpr int BM = 128, BN = 128, BK = 32, WM = 64, WN = 32, STAGES = 3;
+    static constexpr int WARPS_M = BM / WM, WARPS_N = BN / WN, CONSUMERS = WARPS_M * WARPS_N;
+    static constexpr int THREADS = (CONSUMERS + 4) * 32;   // + one producer warpgroup (setmaxnreg)
+    static constexpr int PA = BM + 4, PB = BN + 4;
+    static constexpr int SA = BK * PA, SB = BK * PB;
+    static constexpr size_t SMEM = (size_t)STAGES * (SA + SB) * sizeof(double) + 2 * STAGES * sizeof(uint64_t);
+    static constexpr int FM = WM / 8, FN = WN / 8;
+};
+
+// tile index -> (tm, tn) for the three masks; returns false for tiles with nothing to write
+__device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t& m0, int64_t& n0) {
+    constexpr int BM = WsCfg::BM, BN = WsCfg::BN;
+    int64_t tm, tn;
+    if (g.mask == MASK_LOWER) {
+        const int64_t TN = g.tiles_n, tri = TN * (TN + 1) / 2;
+        if (idx < tri) {
+            int64_t a = (int64_t)((sqrt(8.0 * (double)idx + 1.0) - 1.0) * 0.5);
+            while (a * (a + 1) / 2 > idx) --a;
+            while ((a + 1) * (a + 2) / 2 <= idx) ++a;
+            tm = a; tn = idx - a * (a + 1) / 2;
+        } else {
+            tm = TN + (idx - tri) / TN; tn = (idx - tri) % TN;
+        }
+    } else {
+        tm = idx / g.tiles_n; tn = idx % g.tiles_n;
+    }
+    m0 = tm * BM; n0 = tn * BN;
+    if (g.mask == MASK_CHK) {
+        const int64_t qmax = min(g.M, m0 + BM) - 1;
+        if (g.q_tile0 + qmax / 2 < g.c_tile0 + n0 / g.nb) return false;
+    }
+    return true;
+}
+
+__global__ void __launch_bounds__(WsCfg::THREADS, 1) k_gemm_ws(GemmArgs g, int64_t ntiles) {
+    using C_ = WsCfg;
+    constexpr int BM = C_::BM, BN = C_::BN, BK = C_::BK, WM = C_::WM, WN = C_::WN, STAGES = C_::STAGES;
+    if (*(volatile const int32_t*)g.abort) return;
+    extern __shared__ __align__(16) double smem[];
+    double* sA = smem;
+    double* sB = smem + STAGES * C_::SA;
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * (C_::SA + C_::SB));
+    uint64_t* empty = full + STAGES;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) {
+        for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], C_::CONSUMERS); }
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    __syncthreads();
+
+    if (warp >= C_::CONSUMERS) {
+        // ------------------------------- producer -------------------------------
+        asm volatile("setmaxnreg.dec.sync.aligned.u32 40;\n" ::: "memory");
+        if (warp != C_::CONSUMERS) return;
+        uint32_t it = 0;
+        for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+            int64_t m0, n0;
+            if (!ws_tile(g, t, m0, n0)) continue;
+            const int64_t ke = (g.krange == KR_LE_N) ? min(g.K, n0 + BN) : g.K;
+            const int kt_n = (int)(ke / BK);
+            const uint32_t rowsA = (uint32_t)(g.M - m0 < BM ? g.M - m0 : BM), rowsB = (uint32_t)(g.N - n0 < BN ? g.N - n0 : BN);
+            // warm L2 with the C columns of this tile (they are read at the tile's start)
+            if (g.beta != 0.0) {
+                for (int c = lane; c < (int)rowsB; c += 32) prefetch_l2(g.C + (n0 + c) * g.ldc + m0, rowsA * 8);
+            }
+            for (int kt = 0; kt < kt_n; ++kt, ++it) {
+                const int st = it % STAGES;
+                const uint32_t ph = (it / STAGES) & 1;
+                if (lane == 0) {
+                    mbar_wait(&empty[st], ph ^ 1);
+                    mbar_expect_tx(&full[st], (uint32_t)BK * (rowsA + rowsB) * 8);
+                }
+                __syncwarp();
+                const int64_t k0 = (int64_t)kt * BK;
+                for (int kk = lane; kk < BK; kk += 32) {
+                    bulk_g2s(sA + st * C_::SA + kk * C_::PA, g.A + (k0 + kk) * g.lda + m0, rowsA * 8, &full[st]);
+                    bulk_g2s(sB + st * C_::SB + kk * C_::PB, g.B + (k0 + kk) * g.ldb + n0, rowsB * 8, &full[st]);
+                }
+            }
+        }
+        return;
+    }
+    // ------------------------------- consumers -------------------------------
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 232;\n" ::: "memory");
+    const int wm = warp / C_::WARPS_N, wn = warp % C_::WARPS_N;
+    const int fr = lane >> 2, fc = lane & 3;
+    const double ab = g.alpha * g.beta, alpha = g.alpha;
+    uint32_t it = 0;
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        int64_t m0, n0;
+        if (!ws_tile(g, t, m0, n0)) continue;
+        const int64_t ke = (g.krange == KR_LE_N) ? min(g.K, n0 + BN) : g.K;
+        const int kt_n = (int)(ke / BK);
+        double acc[C_::FM][C_::FN][2];
+        // acc = alpha*beta*C on the elements this tile owns (masked / out-of-range: 0)
+#pragma unroll
+        for (int i = 0; i < C_::FM; ++i) {
+            const int64_t r = m0 + wm * WM + i * 8 + fr;
+#pragma unroll
+            for (int j = 0; j < C_::FN; ++j)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
+                    bool ok = r < g.M && c < g.N;
+                    if (g.mask == MASK_LOWER) ok = ok && r >= c;
+                    else if (g.mask == MASK_CHK) ok = ok && (g.q_tile0 + r / 2) >= (g.c_tile0 + c / g.nb);
+                    acc[i][j][h] = (ok && ab != 0.0) ? ab * g.C[c * g.ldc + r] : 0.0;
+                }
+        }
+        for (int kt = 0; kt < kt_n; ++kt, ++it) {
+            const int st = it % STAGES;
+            mbar_wait(&full[st], (it / STAGES) & 1);
+            const double* cA = sA + st * C_::SA + wm * WM + fr;
+            const double* cB = sB + st * C_::SB + wn * WN + fr;
+#pragma unroll
+            for (int kk = 0; kk < BK; kk += 4) {
+                double af[C_::FM], bf[C_::FN];
+#pragma unroll
+                for (int i = 0; i < C_::FM; ++i) af[i] = cA[(kk + fc) * C_::PA + i * 8];
+#pragma unroll
+                for (int j = 0; j < C_::FN; ++j) bf[j] = cB[(kk + fc) * C_::PB + j * 8];
+#pragma unroll
+                for (int i = 0; i < C_::FM; ++i)
+#pragma unroll
+                    for (int j = 0; j < C_::FN; ++j) dmma(acc[i][j][0], acc[i][j][1], af[i], bf[j]);
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&empty[st]);
+        }
+        // epilogue: C = alpha * acc, masked stores only
+#pragma unroll
+        for (int i = 0; i < C_::FM; ++i) {
+            const int64_t r = m0 + wm * WM + i * 8 + fr;
+#pragma unroll
+            for (int j = 0; j < C_::FN; ++j)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
+                    bool ok = r < g.M && c < g.N;
+                    if (g.mask == MASK_LOWER) ok = ok && r >= c;
+                    else if (g.mask == MASK_CHK) ok = ok && (g.q_tile0 + r / 2) >= (g.c_tile0 + c / g.nb);
+                    if (ok) g.C[c * g.ldc + r] = alpha * acc[i][j][h];
+                }
+        }
+    }
+}
+
+static int run_ws(GemmArgs g, cudaStream_t s) {
+    static bool attr = false;
+    static int nsm = 148;
+    if (!attr) {
+        cudaFuncSetAttribute(k_gemm_ws, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)WsCfg::SMEM);
+        int dev = 0; cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        attr = true;
+    }
+    const int64_t tm = (g.M + WsCfg::BM - 1) / WsCfg::BM, tn = (g.N + WsCfg::BN - 1) / WsCfg::BN;
+    g.tiles_n = tn;
+    const int64_t ntiles = (g.mask == MASK_LOWER) ? tn * (tn + 1) / 2 + (tm - tn) * tn : tm * tn;
+    if (ntiles <= 0) return 0;
+    // tiles per CTA: 1 lets the block scheduler interleave the high-priority look-ahead stream's
+    // kernels as CTAs retire; a fully persistent grid (tpc = inf) would starve that stream.
+    static int64_t tpc = -1;
+    if (tpc < 0) { const char* e = getenv("ABFT_WS_TPC"); tpc = e ? std::max(1, atoi(e)) : 1; }
+    const int64_t grid = std::max<int64_t>(1, (ntiles + tpc - 1) / tpc);
+    k_gemm_ws<<<(unsigned)grid, WsCfg::THREADS, WsCfg::SMEM, s>>>(g, ntiles);
+    abft_count_launch();
+    return 0;
+}
+
 }  // namespace abft
 
 using namespace abft;
@@ -327,12 +538,20 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
         else if (tiles(64) >= 148) tile = 64;
         else tile = 32;
     }
+    static int variant = -1;
+    if (variant < 0) { const char* e = getenv("ABFT_GEMM_VARIANT"); variant = e ? atoi(e) : 0; }
+    // warp-specialised persistent fast path: NT, 16-byte aligned operands with even leading
+    // dimensions, even M and N, alpha = +-1, whole BK-deep k-tiles (K % 32 == 0, k from 0)
+    const bool ws_ok = transB && g.vecA && g.vecB && (M % 2 == 0) && (N % 2 == 0) && (K % WsCfg::BK == 0) &&
+                       (krange == KR_FULL || krange == KR_LE_N) && (alpha == 1.0 || alpha == -1.0) &&
+                       (mask != MASK_LOWER || N <= M);
     if (transB) {
-        if (tile == 128) return run_cfg<128, 128, 16, 64, 32, 4, true>(g, s);
+        if (tile == 128 && ws_ok && variant != 2) return run_ws(g, s);
+        if (tile == 128) return run_cfg<128, 128, 32, 64, 32, 3, true>(g, s);
         if (tile == 64) return run_cfg<64, 64, 16, 32, 32, 4, true>(g, s);
         return run_cfg<32, 32, 16, 16, 16, 4, true>(g, s);
     } else {
-        if (tile == 128) return run_cfg<128, 128, 16, 64, 32, 4, false>(g, s);
+        if (tile == 128) return run_cfg<128, 128, 32, 64, 32, 3, false>(g, s);
         if (tile == 64) return run_cfg<64, 64, 16, 32, 32, 4, false>(g, s);
         return run_cfg<32, 32, 16, 16, 16, 4, false>(g, s);
     }
