@@ -24,11 +24,8 @@
 using namespace abft;
 
 int launch_check(const StageArgs& a, cudaStream_t s);
+int launch_check_v5_fused(const StageArgs& diag, const StageArgs& off, cudaStream_t s);
 int launch_scales(int64_t n, int64_t nb, const double* A, int64_t lda, double* scl, cudaStream_t s);
-int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
-                int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
-                int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
-                cudaStream_t s, int force_tile = 0);
 int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,
                 const int32_t* abort_flag, cudaStream_t s);
 int launch_zero(int64_t rows, int64_t cols, double* dst, int64_t ldd, cudaStream_t s);
@@ -103,6 +100,7 @@ struct Work {
     double* tmp = nullptr;
     DevState* st = nullptr;
     abft_event_t* ev = nullptr; int64_t ev_cap = 0;
+    double* cs = nullptr; int64_t cs_nslab = 0;   // fused-V5 partials (nb % 128 == 0)
 };
 
 static int work_alloc(Work& w, int64_t n, int64_t nb, int64_t ncols_local, int64_t ev_cap, bool abft, cudaStream_t s) {
@@ -132,6 +130,7 @@ static void work_free(Work& w, cudaStream_t s) {
     if (w.tmp) cudaFreeAsync(w.tmp, s);
     if (w.st) cudaFreeAsync(w.st, s);
     if (w.ev) cudaFreeAsync(w.ev, s);
+    if (w.cs) cudaFreeAsync(w.cs, s);
     w = Work();
 }
 
@@ -284,6 +283,12 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     const int64_t N = w.N, B = nb;
     const double Bd = (double)B;
     const int32_t* ab = &w.st->abort;
+    // fused V5 partials: 64-row slabs x n columns x {v1, v2}
+    const bool can_fuse = abft && (nb % 128 == 0) && (lda % 2 == 0) && (((uintptr_t)A & 15) == 0);
+    if (can_fuse) {
+        w.cs_nslab = n / 64;
+        ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n), s));
+    }
     // second panel buffer for the look-ahead
     double* Wbuf[2] = {w.W, nullptr};
     const int64_t wrows = (N - 1) * nb + 2 * N + 2;
@@ -362,7 +367,8 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     };
 
     // ---- trailing update of iteration k restricted to block columns [jlo, jhi), on S ----
-    auto update_cols = [&](int64_t k, int64_t jlo, int64_t jhi) {
+    // Returns true when the GEMM epilogue produced the fused V5 partials for these columns.
+    auto update_cols = [&](int64_t k, int64_t jlo, int64_t jhi) -> bool {
         const int64_t m = N - k - 1, mB = m * B;
         const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
         double* W = Wbuf[k & 1];
@@ -372,7 +378,12 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         const double r = (double)rows, c = (double)nc;
         cudaEvent_t t = prof.begin(s);
         // C[rows x nc] -= W[c0:, :] W[c0:c0+nc, :]^T, lower (r >= c)
-        launch_gemm(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
+        bool inj_here = false;
+        for (const auto& sp : inj)
+            if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && sp.col / nb >= jlo && sp.col / nb < jhi) inj_here = true;
+        ColSumOut cso{w.cs, n, w.cs_nslab, jlo * B, jlo * B, B};
+        const int fused = launch_gemm(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab,
+                                      s, 0, (can_fuse && !inj_here) ? &cso : nullptr);
         prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd, 0);
         if (abft) {
             // checksum rows of tiles I >= jlo: chk[2I+t, cols] -= W_chk(I) W[c0:c0+nc]^T, I >= J
@@ -384,14 +395,24 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
             const double mm = (double)(N - jlo), jj = (double)(jhi - jlo);
             prof.end(t, PH_UPDC, s, 4.0 * Bd * Bd * (jj * mm - jj * (jj - 1) / 2), 0);
         }
+        return fused == 1;
     };
-    auto v5_cols = [&](int64_t k, int64_t jlo, int64_t jhi) {
+    auto v5_cols = [&](int64_t k, int64_t jlo, int64_t jhi, bool fused) {
         StageArgs a = stage_base(w, A, lda, o.c_tau, SK_TRAIL, ABFT_V5, (int)k);
         a.j_lo = jlo; a.j_hi = jhi; a.flist = 0;
         const double el = (double)stage_count(a) * Bd * Bd - (double)(jhi - jlo) * Bd * (Bd - 1) / 2;
         cudaEvent_t t = prof.begin(s);
-        launch_check(a, s);
-        prof.end(t, PH_V5, s, 4.0 * el, 8.0 * el);
+        if (fused) {
+            StageArgs d = a; d.kind = SK_TRAIL_DIAG;
+            StageArgs f = a; f.kind = SK_TRAIL_OFF;
+            f.cs = w.cs; f.cs_ld = n; f.cs_nslab = w.cs_nslab; f.cs_slab_rows = 64;
+            launch_check_v5_fused(d, f, s);
+            const double rd = (double)(jhi - jlo) * lowerB, ro = (double)stage_count(f) * Bd * 2.0 * (Bd / 64.0);
+            prof.end(t, PH_V5, s, 4.0 * el, 8.0 * (rd + ro));   // bytes actually needed by the fused check
+        } else {
+            launch_check(a, s);
+            prof.end(t, PH_V5, s, 4.0 * el, 8.0 * el);
+        }
     };
 
     std::vector<cudaEvent_t> pan(N, nullptr);
@@ -408,20 +429,20 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         const Loc L{A, lda, w.chk, w.ldc, Wbuf[k & 1], ldw, mB};
         const bool gated = ((k + 1) % K == 0) || k == N - 2;
         // (a) block column k+1 first: update, UPDATE_OUT hook, V5 -> hand it to the panel stream
-        update_cols(k, k + 1, k + 2);
+        const bool fa = update_cols(k, k + 1, k + 2);
         if (abft) {
             do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 1, k + 2, true);
-            if (gated) v5_cols(k, k + 1, k + 2);
+            if (gated) v5_cols(k, k + 1, k + 2, fa);
         }
         cudaEvent_t ec = new_event(); cudaEventRecord(ec, s);
         cudaStreamWaitEvent(P, ec, 0);
         pan[k + 1] = panel(k + 1);
         // (b) the rest of the trailing matrix
         if (m > 1) {
-            update_cols(k, k + 2, N);
+            const bool fb = update_cols(k, k + 2, N);
             if (abft) {
                 do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 2, N, true);
-                if (gated) v5_cols(k, k + 2, N);
+                if (gated) v5_cols(k, k + 2, N, fb);
             }
         }
         if (abft) {   // REST(k+1) outside block column k+1 (that one was applied on P)

@@ -96,6 +96,41 @@ __global__ void __launch_bounds__(kChkThreads) k_check_phase1(StageArgs a) {
     f.d1 = d1; f.d2 = d2; f.r1 = r1; f.r2 = r2;
 }
 
+// Phase 1 of V5 for off-diagonal trailing tiles from the partial sums the update GEMM left
+// behind (SK_TRAIL_OFF): r1 = sum of the tile's slab partials, r2 likewise. One thread per column.
+__global__ void __launch_bounds__(256) k_check_phase1_fused(StageArgs a) {
+    if (a.st->abort) return;
+    const int64_t B = a.nb;
+    const int64_t chunks = (B + 255) / 256;
+    const int64_t t = blockIdx.x / chunks;
+    const int64_t c = (blockIdx.x % chunks) * 256 + threadIdx.x;
+    int64_t I, J;
+    stage_tile(a, t, I, J);
+    if (J % a.col_owner_mod != a.col_owner_rank) return;
+    if (threadIdx.x == 0 && c == 0) atomicAdd(&a.st->n_checks, 1ull);
+    if (c >= B) return;
+    const TileView v = stage_view(a, I, J);
+    const int64_t g = J * B + c, s0 = I * B / a.cs_slab_rows, ns = B / a.cs_slab_rows;
+    double r1 = 0.0, r2 = 0.0;
+    for (int64_t q = 0; q < ns; ++q) {
+        r1 += a.cs[(s0 + q) * a.cs_ld + g];
+        r2 += a.cs[(a.cs_nslab + s0 + q) * a.cs_ld + g];
+    }
+    const double d1 = __dsub_rn(r1, v.c1[c * v.ldc]);
+    const double d2 = __dsub_rn(r2, v.c2[c * v.ldc]);
+    double tau1, tau2;
+    thresholds(a, I, g, false, tau1, tau2);
+    const bool f1 = !dfinite(d1) || fabs(d1) > tau1;
+    const bool f2 = !dfinite(d2) || fabs(d2) > tau2;
+    if (!(f1 || f2)) return;
+    FlagList& FL = a.st->fl[a.flist];
+    const int slot = atomicAdd(&FL.nflag, 1);
+    if (slot >= kFlagCap) { FL.overflow = 1; return; }
+    Flag& f = FL.flags[slot];
+    f.I = (int32_t)I; f.J = (int32_t)J; f.c = (int32_t)c;
+    f.d1 = d1; f.d2 = d2; f.r1 = r1; f.r2 = r2;
+}
+
 // Block-wide reductions used by phase 2 (one CTA).
 __device__ double block_sum(double v, double* red) {
     v = warp_sum(v);
@@ -293,11 +328,38 @@ using namespace abft;
 int launch_check(const StageArgs& a, cudaStream_t s) {
     const int64_t count = stage_count(a);
     if (count <= 0) return 0;
-    const int64_t chunks = (a.nb + kChkCols - 1) / kChkCols;
-    k_check_phase1<<<(unsigned)(count * chunks), kChkThreads, 0, s>>>(a);
+    if (a.kind == SK_TRAIL_OFF) {
+        const int64_t chunks = (a.nb + 255) / 256;
+        k_check_phase1_fused<<<(unsigned)(count * chunks), 256, 0, s>>>(a);
+    } else {
+        const int64_t chunks = (a.nb + kChkCols - 1) / kChkCols;
+        k_check_phase1<<<(unsigned)(count * chunks), kChkThreads, 0, s>>>(a);
+    }
     abft_count_launch();
     if (a.encode) return 0;
     k_check_phase2<<<1, 256, 0, s>>>(a);
+    abft_count_launch();
+    return 0;
+}
+
+// V5 with the fused recalculation: diagonal tiles re-read (sym), off-diagonal tiles from the
+// update GEMM's partials; both phase-1 kernels feed one flag list resolved by one phase 2 in
+// the oracle's tile order.
+int launch_check_v5_fused(const StageArgs& diag, const StageArgs& off, cudaStream_t s) {
+    const int64_t nd = stage_count(diag), no = stage_count(off);
+    if (nd > 0) {
+        const int64_t chunks = (diag.nb + kChkCols - 1) / kChkCols;
+        k_check_phase1<<<(unsigned)(nd * chunks), kChkThreads, 0, s>>>(diag);
+        abft_count_launch();
+    }
+    if (no > 0) {
+        const int64_t chunks = (off.nb + 255) / 256;
+        k_check_phase1_fused<<<(unsigned)(no * chunks), 256, 0, s>>>(off);
+        abft_count_launch();
+    }
+    StageArgs r = diag;
+    r.kind = SK_TRAIL;
+    k_check_phase2<<<1, 256, 0, s>>>(r);
     abft_count_launch();
     return 0;
 }

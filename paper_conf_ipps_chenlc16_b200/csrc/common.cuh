@@ -42,6 +42,8 @@ enum StageKind : int32_t {
     SK_PANEL = 2,      // V4/V4R: tiles (k+1..N-1, k) in W (data rows), checksums in W (chk rows)
     SK_TRAIL = 3,      // V5: tiles (I,J), k < J <= I, in A, unfactored; checksums in chk
     SK_ALL = 4,        // V6 / abft_verify: all tiles I >= J in A; factored per flag
+    SK_TRAIL_OFF = 5,  // V5, off-diagonal trailing tiles, recalculation from the GEMM's fused partials
+    SK_TRAIL_DIAG = 6, // V5, diagonal trailing tiles (J, J), J in [j_lo, j_hi), re-read as sym(tril)
 };
 
 struct StageArgs {
@@ -56,7 +58,8 @@ struct StageArgs {
     double c_tau;
     int32_t col_owner_mod, col_owner_rank;  // dist: local column mapping (1, 0 on one GPU)
     int32_t flist, pad2;            // flag list used by this stage (one per stream)
-    int64_t j_lo, j_hi;             // SK_TRAIL: block columns [j_lo, j_hi)
+    int64_t j_lo, j_hi;             // SK_TRAIL*: block columns [j_lo, j_hi)
+    const double* cs; int64_t cs_ld, cs_nslab, cs_slab_rows;   // SK_TRAIL_OFF: fused partials
     DevState* st;
     abft_event_t* ev; int64_t ev_cap;
 };
@@ -78,6 +81,11 @@ __host__ __device__ __forceinline__ int64_t stage_count(const StageArgs& a) {
             const int64_t lo = a.j_lo, hi = a.j_hi;
             return hi <= lo ? 0 : (hi - lo) * N - (hi * (hi - 1) - lo * (lo - 1)) / 2;
         }
+        case SK_TRAIL_DIAG: return a.j_hi > a.j_lo ? a.j_hi - a.j_lo : 0;
+        case SK_TRAIL_OFF: {
+            const int64_t lo = a.j_lo, hi = a.j_hi;
+            return hi <= lo ? 0 : (hi - lo) * (N - 1) - (hi * (hi - 1) - lo * (lo - 1)) / 2;
+        }
         default: return N * (N + 1) / 2;
     }
 }
@@ -89,6 +97,12 @@ __device__ __forceinline__ void stage_tile(const StageArgs& a, int64_t t, int64_
         case SK_COLUMN: I = k + t; J = k; return;
         case SK_DIAG_FACT: I = k; J = k; return;
         case SK_PANEL: I = k + 1 + t; J = k; return;
+        case SK_TRAIL_DIAG: I = J = a.j_lo + t; return;
+        case SK_TRAIL_OFF: {   // column-major over (I > J), J in [j_lo, j_hi)
+            int64_t jj = a.j_lo, rem = t;
+            while (rem >= N - jj - 1) { rem -= N - jj - 1; ++jj; }
+            J = jj; I = jj + 1 + rem; return;
+        }
         default: {
             const int64_t j0 = (a.kind == SK_TRAIL) ? a.j_lo : 0;
             const int64_t m = N - j0;
@@ -119,6 +133,8 @@ __device__ __forceinline__ TileView stage_view(const StageArgs& a, int64_t I, in
             v.diag = false; v.factored = true; break;
         case SK_COLUMN:
         case SK_TRAIL:
+        case SK_TRAIL_OFF:
+        case SK_TRAIL_DIAG:
             v.T = a.A + local_col(a, J) * a.lda + I * B; v.ldt = a.lda;
             v.c1 = a.chk + local_col(a, J) * a.ldc + 2 * I; v.c2 = v.c1 + 1; v.ldc = a.ldc;
             v.factored = false; break;
@@ -157,6 +173,18 @@ __device__ __forceinline__ bool dfinite(double x) { return isfinite(x); }
 
 }  // namespace abft
 
+// Per-column partial checksums of an updated trailing tile, written by the GEMM epilogue
+// (fused V5 recalculation): slab s = global_row / 128, column g (global):
+//   p[s * ld + g] = sum over the slab's rows of C_new,  p[(nslab + s) * ld + g] = weighted sum,
+// weights = (row index inside its nb-block) + 1.
+namespace abft {
+struct ColSumOut {
+    double* p; int64_t ld, nslab;
+    int64_t row0, col0;   // global row / column of C's (0, 0)
+    int64_t nb;
+};
+}  // namespace abft
+
 // Host helpers
 #define ABFT_CUDA_TRY(expr)                                   \
     do {                                                      \
@@ -166,3 +194,10 @@ __device__ __forceinline__ bool dfinite(double x) { return isfinite(x); }
 
 void abft_set_error(cudaError_t e, const char* what);
 void abft_count_launch(int n = 1);
+
+// DMMA GEMM launcher (gemm.cu). Returns 1 if the fused column partials `cs` were written
+// (warp-specialised path with 128-row tiles aligned to nb), 0 otherwise.
+int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
+                int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
+                int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
+                cudaStream_t s, int force_tile = 0, const abft::ColSumOut* cs = nullptr);

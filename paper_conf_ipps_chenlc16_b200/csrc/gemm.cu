@@ -41,6 +41,7 @@ struct GemmArgs {
     int64_t tiles_n;                // number of column tiles (rect grid)
     const int32_t* abort;
     int32_t vecA, vecB;             // 16-byte cp.async allowed for A / B
+    ColSumOut cs;                   // fused V5 partials (cs.p == nullptr: off)
 };
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
@@ -480,8 +481,40 @@ __global__ void __launch_bounds__(WsCfg::THREADS, 1) k_gemm_ws(GemmArgs g, int64
                     bool ok = r < g.M && c < g.N;
                     if (g.mask == MASK_LOWER) ok = ok && r >= c;
                     else if (g.mask == MASK_CHK) ok = ok && (g.q_tile0 + r / 2) >= (g.c_tile0 + c / g.nb);
-                    if (ok) g.C[c * g.ldc + r] = alpha * acc[i][j][h];
+                    acc[i][j][h] = alpha * acc[i][j][h];
+                    if (ok) g.C[c * g.ldc + r] = acc[i][j][h];
                 }
+        }
+        // fused V5 recalculation: per-column v1/v2 partial sums of the
+        // updated values over each warp's 64 rows (slab = global_row / 64), for tiles off the
+        // block diagonal (diagonal blocks are checked as sym(tril) by a re-read).
+        if (g.cs.p != nullptr) {
+            const int64_t gr0 = g.cs.row0 + m0 + wm * WM, gc0 = g.cs.col0 + n0;
+            if (gr0 / g.cs.nb != gc0 / g.cs.nb) {
+                const int64_t wbase = gr0 % g.cs.nb + fr + 1;   // weight (1-based) of row i = 0
+#pragma unroll
+                for (int j = 0; j < C_::FN; ++j)
+#pragma unroll
+                    for (int h = 0; h < 2; ++h) {
+                        double s1 = 0.0, s2 = 0.0;
+#pragma unroll
+                        for (int i = 0; i < C_::FM; ++i) {
+                            s1 += acc[i][j][h];
+                            s2 = fma((double)(wbase + i * 8), acc[i][j][h], s2);
+                        }
+#pragma unroll
+                        for (int o = 4; o < 32; o <<= 1) {
+                            s1 += __shfl_xor_sync(0xffffffffu, s1, o);
+                            s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+                        }
+                        if (fr == 0) {
+                            const int64_t slab = gr0 / WM;
+                            const int64_t gc = gc0 + wn * WN + j * 8 + fc * 2 + h;
+                            g.cs.p[slab * g.cs.ld + gc] = s1;
+                            g.cs.p[(g.cs.nslab + slab) * g.cs.ld + gc] = s2;
+                        }
+                    }
+            }
         }
     }
 }
@@ -520,12 +553,13 @@ static bool aligned16(const void* p) { return ((uintptr_t)p & 15) == 0; }
 int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                 int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
                 int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
-                cudaStream_t s, int force_tile = 0) {
+                cudaStream_t s, int force_tile, const ColSumOut* cs) {
     if (M <= 0 || N <= 0) return 0;
     GemmArgs g;
     g.M = M; g.N = N; g.K = K; g.A = A; g.lda = lda; g.B = B; g.ldb = ldb; g.C = C; g.ldc = ldc;
     g.alpha = alpha; g.beta = beta; g.mask = mask; g.krange = krange; g.nb = nb;
     g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
+    g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1};
     g.vecA = aligned16(A) && (lda % 2 == 0);
     g.vecB = aligned16(B) && (ldb % 2 == 0);
     auto tiles = [&](int64_t t) {
@@ -545,6 +579,11 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
     const bool ws_ok = transB && g.vecA && g.vecB && (M % 2 == 0) && (N % 2 == 0) && (K % WsCfg::BK == 0) &&
                        (krange == KR_FULL || krange == KR_LE_N) && (alpha == 1.0 || alpha == -1.0) &&
                        (mask != MASK_LOWER || N <= M);
+    if (cs) {   // fused partials need the warp-specialised kernel with nb-aligned 128-row tiles
+        if (!(ws_ok && variant != 2 && mask == MASK_LOWER && cs->nb % WsCfg::BM == 0 &&
+              cs->row0 % WsCfg::BM == 0 && cs->col0 % WsCfg::BN == 0 && M % WsCfg::BM == 0)) g.cs.p = nullptr;
+        else { run_ws(g, s); return 1; }
+    }
     if (transB) {
         if (tile == 128 && ws_ok && variant != 2) return run_ws(g, s);
         if (tile == 128) return run_cfg<128, 128, 32, 64, 32, 3, true>(g, s);

@@ -11,74 +11,89 @@
 
 #include <algorithm>
 
-int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
-                int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
-                int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
-                cudaStream_t s, int force_tile = 0);
 
 namespace abft {
 
 constexpr int kLeaf = 64;
 
 // One CTA: Cholesky of the lower triangle of T (nl x nl, nl <= 64) in shared memory, then its
-// inverse by column-wise forward substitution. Writes L (lower) into T and inv(L) (lower,
-// upper zeroed) into Li. A non-positive pivot sets NOT_SPD with info = off + j + 1 and aborts.
-__global__ void __launch_bounds__(256) k_leaf_potrf_inv(double* T, int64_t ldt, double* Li, int64_t ldi,
-                                                        int nl, int64_t info_off, DevState* st) {
+// inverse, both right-looking with ONE barrier per step: each thread owns a fixed set of <= 9
+// lower-triangle elements; step j updates them with the unscaled column j divided by the pivot
+// d_j (A22 -= a_j a_j^T / d_j, identical to l_j l_j^T), and the columns are scaled once at the
+// end. The inverse solves L X = I by forward elimination in the same owner-computes pattern.
+// Writes L (lower) into T and inv(L) (lower, upper zeroed) into Li. A non-positive pivot sets
+// NOT_SPD with info = off + j + 1 and aborts.
+constexpr int kLeafThreads = 256;
+constexpr int kLeafOwn = (kLeaf * (kLeaf + 1) / 2 + kLeafThreads - 1) / kLeafThreads;   // 9
+
+__global__ void __launch_bounds__(kLeafThreads) k_leaf_potrf_inv(double* T, int64_t ldt, double* Li, int64_t ldi,
+                                                                 int nl, int64_t info_off, DevState* st) {
     if (st->abort) return;
     extern __shared__ double leaf_smem[];
-    double (*L)[kLeaf + 1] = reinterpret_cast<double (*)[kLeaf + 1]>(leaf_smem);            // L[c][r]
-    double (*X)[kLeaf + 1] = reinterpret_cast<double (*)[kLeaf + 1]>(leaf_smem + kLeaf * (kLeaf + 1));  // X[j][i] = inv(L)[i][j]
-    __shared__ int s_fail;
+    double* L = leaf_smem;                              // L[c*(kLeaf+1) + r]
+    double* X = leaf_smem + kLeaf * (kLeaf + 1);        // X[c*(kLeaf+1) + i] = inv(L)(i, c)
+    __shared__ double dd[kLeaf];
+    constexpr int P = kLeaf + 1;
     const int tid = threadIdx.x;
-    for (int i = tid; i < nl * nl; i += blockDim.x) {
-        const int c = i / nl, r = i % nl;
-        L[c][r] = (r >= c) ? T[c * ldt + r] : 0.0;
+    const int E = nl * (nl + 1) / 2;
+    // owned elements (r, c), r >= c, enumerated column by column
+    int own_r[kLeafOwn], own_c[kLeafOwn];
+#pragma unroll
+    for (int q = 0; q < kLeafOwn; ++q) {
+        int e = tid + q * kLeafThreads, c = 0;
+        if (e < E) {
+            while (e >= nl - c) { e -= nl - c; ++c; }
+            own_r[q] = c + e; own_c[q] = c;
+        } else { own_r[q] = -1; own_c[q] = -1; }
     }
-    if (tid == 0) s_fail = 0;
-    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < kLeafOwn; ++q)
+        if (own_r[q] >= 0) {
+            const int r = own_r[q], c = own_c[q];
+            L[c * P + r] = T[c * ldt + r];
+            X[c * P + r] = (r == c) ? 1.0 : 0.0;
+        }
     for (int j = 0; j < nl; ++j) {
-        if (tid == 0) {
-            const double d = L[j][j];
-            if (!(d > 0.0)) {
-                s_fail = 1;
-                if (atomicCAS(&st->abort, 0, 1) == 0) { st->status = ABFT_NOT_SPD; st->info = info_off + j + 1; }
-            } else {
-                L[j][j] = sqrt(d);
-            }
+        __syncthreads();
+        const double d = L[j * P + j];
+        if (!(d > 0.0)) {
+            if (tid == 0 && atomicCAS(&st->abort, 0, 1) == 0) { st->status = ABFT_NOT_SPD; st->info = info_off + j + 1; }
+            return;
         }
-        __syncthreads();
-        if (s_fail) return;
-        const double piv = L[j][j];
-        for (int r = j + 1 + tid; r < nl; r += blockDim.x) L[j][r] = L[j][r] / piv;
-        __syncthreads();
-        // trailing update of the lower triangle: L[c][r] -= L[j][r] * L[j][c], j < c <= r
-        const int m = nl - j - 1;
-        for (int i = tid; i < m * m; i += blockDim.x) {
-            const int c = j + 1 + i / m, r = j + 1 + i % m;
-            if (r >= c) L[c][r] -= L[j][r] * L[j][c];
-        }
-        __syncthreads();
-    }
-    for (int i = tid; i < nl * nl; i += blockDim.x) {
-        const int c = i / nl, r = i % nl;
-        if (r >= c) T[c * ldt + r] = L[c][r];
-    }
-    // inverse: column j of inv(L) solves L x = e_j (x_i = 0 for i < j)
-    if (tid < nl) {
-        const int j = tid;
-        for (int i = 0; i < nl; ++i) X[j][i] = 0.0;
-        X[j][j] = 1.0 / L[j][j];
-        for (int i = j + 1; i < nl; ++i) {
-            double s = 0.0;
-            for (int p = j; p < i; ++p) s = fma(L[p][i], X[j][p], s);
-            X[j][i] = -s / L[i][i];
+        if (tid == 0) dd[j] = d;
+        const double inv_d = 1.0 / d;
+#pragma unroll
+        for (int q = 0; q < kLeafOwn; ++q) {
+            const int r = own_r[q], c = own_c[q];
+            if (c > j) L[c * P + r] -= L[j * P + r] * (L[j * P + c] * inv_d);
         }
     }
     __syncthreads();
-    for (int i = tid; i < nl * nl; i += blockDim.x) {
-        const int c = i / nl, r = i % nl;
-        Li[c * ldi + r] = X[c][r];   // upper part written as 0
+    // scale: l_j = a_j / sqrt(d_j)
+#pragma unroll
+    for (int q = 0; q < kLeafOwn; ++q) {
+        const int r = own_r[q], c = own_c[q];
+        if (r >= 0) {
+            const double sq = sqrt(dd[c]);
+            const double v = (r == c) ? sq : L[c * P + r] / sq;
+            L[c * P + r] = v;
+            T[c * ldt + r] = v;
+        }
+    }
+    // inverse: Y = I; step p: Y(i,:) -= L(i,p)/L(p,p) * Y(p,:) for i > p; X(i,:) = Y(i,:)/L(i,i)
+    for (int p = 0; p < nl; ++p) {
+        __syncthreads();
+        const double lpp = L[p * P + p];
+#pragma unroll
+        for (int q = 0; q < kLeafOwn; ++q) {
+            const int i = own_r[q], c = own_c[q];
+            if (i > p && p >= c) X[c * P + i] -= (L[p * P + i] / lpp) * X[c * P + p];
+        }
+    }
+    __syncthreads();
+    for (int e = tid; e < nl * nl; e += kLeafThreads) {
+        const int c = e / nl, i = e % nl;
+        Li[c * ldi + i] = (i >= c) ? X[c * P + i] / L[i * P + i] : 0.0;
     }
 }
 
@@ -132,7 +147,7 @@ static void chol_inv_rec(double* T, int64_t ldt, double* Li, int64_t ldi, int64_
         static bool attr = false;
         const int smem = 2 * kLeaf * (kLeaf + 1) * (int)sizeof(double);
         if (!attr) { cudaFuncSetAttribute(k_leaf_potrf_inv, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); attr = true; }
-        k_leaf_potrf_inv<<<1, 256, smem, s>>>(T + off * ldt + off, ldt, Li + off * ldi + off, ldi, (int)sz,
+        k_leaf_potrf_inv<<<1, kLeafThreads, smem, s>>>(T + off * ldt + off, ldt, Li + off * ldi + off, ldi, (int)sz,
                                            info_off + off, st);
         abft_count_launch();
         return;
