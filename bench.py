@@ -221,7 +221,7 @@ def main():
                    "l2": "inputs (8 GiB) larger than L2; restore copy between steps outside the CUDA events",
                    "parallelism": f"replicas x{world}" if world > 1 else "single GPU"},
         "gpu_launches": int(launches) * args.steps,
-        "roofline": {"bound": "tensor", "kernel": "k_gemm_dmma<128,128,16,64,32,4,NT> trailing SYRK update",
+        "roofline": {"bound": "tensor", "kernel": "k_gemm_ws (warp-specialised DMMA, 128x128 tiles) trailing SYRK update",
                      "achieved": round(achieved, 3) if achieved else None,
                      "peak": FP64_DMMA_PEAK_TFLOPS, "unit": "TFLOP/s",
                      "frac": round(achieved / FP64_DMMA_PEAK_TFLOPS, 4) if achieved else None,

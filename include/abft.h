@@ -168,6 +168,13 @@ int abft_potrf_dist(int64_t n, int64_t nb, double* A_local, int64_t lda_local, v
                     int nranks, abft_stream_t stream, const abft_inject_spec_t* inj,
                     abft_report_t* rep, const abft_options_t* opt);
 
+/* Diagnostics: the trailing-update GEMM on its own (for benchmarking the dominant kernel):
+ * C = beta C + alpha A B^T over the lower triangle (lower = 1: r >= c, requires N <= M) or all
+ * of C (lower = 0). A: M x K, B: N x K, column-major device buffers. Errors: -1 bad sizes. */
+int abft_dev_gemm_nt(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
+                     int64_t ldb, double* C, int64_t ldc, double alpha, double beta, int lower,
+                     abft_stream_t stream);
+
 /* Diagnostics: kernel launches issued by the last call on this thread, a static version string,
  * and the text of the last CUDA error seen on this thread (empty if none). */
 int64_t abft_last_launch_count(void);

@@ -74,6 +74,8 @@ _lib.abft_nccl_id.argtypes = [_vp]
 _lib.abft_comm_init.argtypes = [ctypes.POINTER(_vp), _i32, _vp, _i32]
 _lib.abft_comm_destroy.argtypes = [_vp]
 _lib.abft_potrf_dist.argtypes = [_i64, _i64, _vp, _i64, _vp, _i32, _i32, _vp, _vp, _vp, _vp]
+_lib.abft_dev_gemm_nt.argtypes = [_i64, _i64, _i64, _vp, _i64, _vp, _i64, _vp, _i64, _dbl, _dbl, _i32, _vp]
+_lib.abft_dev_gemm_nt.restype = _i32
 _lib.abft_last_launch_count.restype = _i64
 _lib.abft_version.restype = ctypes.c_char_p
 _lib.abft_last_error.restype = ctypes.c_char_p
@@ -86,7 +88,7 @@ for _f in ("abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_po
 
 EXPORTS = ["abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
            "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist",
-           "abft_last_launch_count", "abft_version", "abft_last_error", "abft_last_profile",
+           "abft_last_launch_count", "abft_version", "abft_last_error", "abft_last_profile", "abft_dev_gemm_nt",
            "abft_phase_name"]
 
 
@@ -240,6 +242,15 @@ def abft_potrf_dist(n, nb, A_local, comm, rank, nranks, lda=None, stream=None, i
     st = _lib.abft_potrf_dist(n, nb, p, lda or ld or n, comm, rank, nranks, _stream(stream), pinj,
                               ctypes.byref(rep) if rep else None, ctypes.byref(o))
     return st, (_report_dict(rep, ev) if rep else None)
+
+
+def abft_dev_gemm_nt(M, N, K, A, B, C, alpha=-1.0, beta=1.0, lower=True, stream=None):
+    """Diagnostics: the update GEMM alone (C = beta C + alpha A B^T, lower triangle)."""
+    pa, la = _dev(A)
+    pb, lb = _dev(B)
+    pc, lc = _dev(C)
+    return _lib.abft_dev_gemm_nt(M, N, K, pa, la or M, pb, lb or N, pc, lc or M, alpha, beta, int(lower),
+                                 _stream(stream))
 
 
 def abft_last_launch_count():

@@ -286,7 +286,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     // fused V5 partials: 64-row slabs x n columns x {v1, v2}
     const bool can_fuse = abft && (nb % 128 == 0) && (lda % 2 == 0) && (((uintptr_t)A & 15) == 0);
     if (can_fuse) {
-        w.cs_nslab = n / 64;
+        w.cs_nslab = n / 32;   // room for 32-row slabs (the smallest warp-tile height)
         ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n), s));
     }
     // second panel buffer for the look-ahead
@@ -366,6 +366,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         return e;
     };
 
+    int64_t slab_rows_used = 64;
     // ---- trailing update of iteration k restricted to block columns [jlo, jhi), on S ----
     // Returns true when the GEMM epilogue produced the fused V5 partials for these columns.
     auto update_cols = [&](int64_t k, int64_t jlo, int64_t jhi) -> bool {
@@ -381,7 +382,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         bool inj_here = false;
         for (const auto& sp : inj)
             if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && sp.col / nb >= jlo && sp.col / nb < jhi) inj_here = true;
-        ColSumOut cso{w.cs, n, w.cs_nslab, jlo * B, jlo * B, B};
+        ColSumOut cso{w.cs, n, w.cs_nslab, jlo * B, jlo * B, B, 64};
         const int fused = launch_gemm(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab,
                                       s, 0, (can_fuse && !inj_here) ? &cso : nullptr);
         prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd, 0);
@@ -395,6 +396,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
             const double mm = (double)(N - jlo), jj = (double)(jhi - jlo);
             prof.end(t, PH_UPDC, s, 4.0 * Bd * Bd * (jj * mm - jj * (jj - 1) / 2), 0);
         }
+        if (fused == 1) slab_rows_used = cso.slab_rows;
         return fused == 1;
     };
     auto v5_cols = [&](int64_t k, int64_t jlo, int64_t jhi, bool fused) {
@@ -405,9 +407,9 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         if (fused) {
             StageArgs d = a; d.kind = SK_TRAIL_DIAG;
             StageArgs f = a; f.kind = SK_TRAIL_OFF;
-            f.cs = w.cs; f.cs_ld = n; f.cs_nslab = w.cs_nslab; f.cs_slab_rows = 64;
+            f.cs = w.cs; f.cs_ld = n; f.cs_nslab = w.cs_nslab; f.cs_slab_rows = slab_rows_used;
             launch_check_v5_fused(d, f, s);
-            const double rd = (double)(jhi - jlo) * lowerB, ro = (double)stage_count(f) * Bd * 2.0 * (Bd / 64.0);
+            const double rd = (double)(jhi - jlo) * lowerB, ro = (double)stage_count(f) * Bd * 2.0 * (Bd / (double)slab_rows_used);
             prof.end(t, PH_V5, s, 4.0 * el, 8.0 * (rd + ro));   // bytes actually needed by the fused check
         } else {
             launch_check(a, s);
@@ -578,6 +580,20 @@ extern "C" int abft_verify(int64_t n, int64_t nb, double* A, int64_t lda, double
     if (rc) return rc;
     ABFT_CUDA_TRY(cudaGetLastError());
     return status;
+}
+
+extern "C" int abft_dev_gemm_nt(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
+                                int64_t ldb, double* C, int64_t ldc, double alpha, double beta, int lower,
+                                abft_stream_t stream) {
+    g_launches = 0;
+    if (M < 0 || N < 0 || K < 0 || (lower && N > M) || lda < std::max<int64_t>(1, M) ||
+        ldb < std::max<int64_t>(1, N) || ldc < std::max<int64_t>(1, M)) return -1;
+    static int32_t* zero_flag = nullptr;
+    if (!zero_flag) { ABFT_CUDA_TRY(cudaMalloc((void**)&zero_flag, sizeof(int32_t))); ABFT_CUDA_TRY(cudaMemset(zero_flag, 0, 4)); }
+    launch_gemm(M, N, K, A, lda, B, ldb, C, ldc, alpha, beta, true, lower ? 1 : 0, 0, 0, 0, 0, zero_flag,
+                (cudaStream_t)stream);
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return 0;
 }
 
 extern "C" int abft_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, abft_stream_t stream) {

@@ -174,7 +174,7 @@ __device__ __forceinline__ bool dfinite(double x) { return isfinite(x); }
 }  // namespace abft
 
 // Per-column partial checksums of an updated trailing tile, written by the GEMM epilogue
-// (fused V5 recalculation): slab s = global_row / 128, column g (global):
+// (fused V5 recalculation): slab s = global_row / slab_rows, column g (global):
 //   p[s * ld + g] = sum over the slab's rows of C_new,  p[(nslab + s) * ld + g] = weighted sum,
 // weights = (row index inside its nb-block) + 1.
 namespace abft {
@@ -182,6 +182,7 @@ struct ColSumOut {
     double* p; int64_t ld, nslab;
     int64_t row0, col0;   // global row / column of C's (0, 0)
     int64_t nb;
+    int64_t slab_rows;    // rows per slab (set by the GEMM launcher: its warp-tile height)
 };
 }  // namespace abft
 
@@ -200,4 +201,4 @@ void abft_count_launch(int n = 1);
 int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                 int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
                 int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
-                cudaStream_t s, int force_tile = 0, const abft::ColSumOut* cs = nullptr);
+                cudaStream_t s, int force_tile = 0, abft::ColSumOut* cs = nullptr);

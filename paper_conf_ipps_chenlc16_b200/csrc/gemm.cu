@@ -24,6 +24,7 @@
 
 #include <algorithm>
 #include <cstdlib>
+#include <cstring>
 
 namespace abft {
 
@@ -339,32 +340,82 @@ __device__ __forceinline__ void prefetch_l2(const void* src, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(src), "r"(bytes) : "memory");
 }
 
-struct WsCfg {
-    static constexpr int BM = 128, BN = 128, BK = 32, WM = 64, WN = 32, STAGES = 3;
+template <int BM_, int BN_, int BK_, int STAGES_, int WM_, int WN_, int REG_CONS_, int MINB_>
+struct WsCfgT {
+    static constexpr int BM = BM_, BN = BN_, BK = BK_, WM = WM_, WN = WN_, STAGES = STAGES_, MINB = MINB_;
     static constexpr int WARPS_M = BM / WM, WARPS_N = BN / WN, CONSUMERS = WARPS_M * WARPS_N;
     static constexpr int THREADS = (CONSUMERS + 4) * 32;   // + one producer warpgroup (setmaxnreg)
+    static constexpr int REG_CONS = REG_CONS_, REG_PROD = 40;
     static constexpr int PA = BM + 4, PB = BN + 4;
     static constexpr int SA = BK * PA, SB = BK * PB;
     static constexpr size_t SMEM = (size_t)STAGES * (SA + SB) * sizeof(double) + 2 * STAGES * sizeof(uint64_t);
     static constexpr int FM = WM / 8, FN = WN / 8;
+    // setmaxnreg moves registers inside the CTA's launch allocation (R0 per thread): what the
+    // producer warpgroup releases must cover what the consumers add, or .inc blocks forever.
+    static constexpr int R0 = (65536 / MINB / THREADS) / 8 * 8;
+    static_assert(CONSUMERS * 32 * (REG_CONS - R0) <= 128 * (R0 - REG_PROD), "setmaxnreg budget");
+    static_assert(SMEM * MINB <= 232448, "shared memory");
 };
+using WsCfg = WsCfgT<128, 128, 32, 3, 64, 32, 232, 1>;    // 8 consumer warps, 1 CTA/SM (default)
+using WsCfg16 = WsCfgT<128, 128, 32, 3, 32, 32, 104, 1>;  // 16 consumer warps, 32x32 warp tiles
+using WsCfg2a = WsCfgT<128, 64, 16, 4, 64, 32, 216, 2>;   // 2 CTAs/SM, 128x64 tiles, 4-stage BK=16
+using WsCfg2b = WsCfgT<128, 64, 32, 2, 64, 32, 216, 2>;   // 2 CTAs/SM, 128x64 tiles, 2-stage BK=32
 
 // tile index -> (tm, tn) for the three masks; returns false for tiles with nothing to write
+// Lower-trapezoid tile enumeration for BN = BM / R (R = 1 or 2): tile row tm holds the column
+// tiles tn < min(R (tm + 1), TN); prefix(t) = tiles in rows < t.
+template <int R>
+__host__ __device__ __forceinline__ int64_t lower_prefix(int64_t t, int64_t TN) {
+    const int64_t T0 = TN / R;   // rows whose count R(tm+1) <= TN
+    if (t <= T0) return R * t * (t + 1) / 2;
+    return R * T0 * (T0 + 1) / 2 + (t - T0) * TN;
+}
+
+// Column prefix inside a group of rows [a0, a0 + Gp) of the lower trapezoid: column u holds the
+// rows a >= max(a0, floor(u / R)); P(u) = tiles in columns < u of the group.
+template <int R>
+__device__ __forceinline__ int64_t group_col_prefix(int64_t u, int64_t a0, int64_t Gp) {
+    int64_t w = u - R * (a0 + 1);
+    int64_t S = 0;
+    if (w > 0) {
+        const int64_t p = w / R, rem = w - p * R;
+        S = R * p * (p + 1) / 2 + rem * (p + 1);
+    }
+    return u * Gp - S;
+}
+
+constexpr int kWsGroup = 8;   // tile rows per L2 group: A rows of a group stay in L2, W streams once per group
+
+// tile index -> (m0, n0) for the three masks; returns false for tiles with nothing to write.
+// Tiles are enumerated group by group (kWsGroup tile rows), column-major inside a group, so the
+// CTAs running at the same time share operand tiles in L2.
+template <int BM, int BN>
 __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t& m0, int64_t& n0) {
-    constexpr int BM = WsCfg::BM, BN = WsCfg::BN;
+    constexpr int R = BM / BN;
+    const int64_t TN = g.tiles_n, TM = (g.M + BM - 1) / BM;
     int64_t tm, tn;
     if (g.mask == MASK_LOWER) {
-        const int64_t TN = g.tiles_n, tri = TN * (TN + 1) / 2;
-        if (idx < tri) {
-            int64_t a = (int64_t)((sqrt(8.0 * (double)idx + 1.0) - 1.0) * 0.5);
-            while (a * (a + 1) / 2 > idx) --a;
-            while ((a + 1) * (a + 2) / 2 <= idx) ++a;
-            tm = a; tn = idx - a * (a + 1) / 2;
-        } else {
-            tm = TN + (idx - tri) / TN; tn = (idx - tri) % TN;
+        // group q: the last q with lower_prefix(q G) <= idx
+        int64_t lo = 0, hi = (TM + kWsGroup - 1) / kWsGroup;
+        while (hi - lo > 1) {
+            const int64_t mid = (lo + hi) / 2;
+            if (lower_prefix<R>(mid * kWsGroup, TN) <= idx) lo = mid; else hi = mid;
         }
+        const int64_t a0 = lo * kWsGroup, Gp = ((TM - a0) < kWsGroup ? (TM - a0) : (int64_t)kWsGroup);
+        const int64_t e = idx - lower_prefix<R>(a0, TN);
+        const int64_t ncol = ((R * (a0 + Gp)) < TN ? (R * (a0 + Gp)) : TN);
+        int64_t ul = 0, uh = ncol;   // column u: P(u) <= e < P(u + 1)
+        while (uh - ul > 1) {
+            const int64_t mid = (ul + uh) / 2;
+            if (group_col_prefix<R>(mid, a0, Gp) <= e) ul = mid; else uh = mid;
+        }
+        tn = ul;
+        const int64_t first = ((ul / R) > a0 ? (ul / R) : a0);
+        tm = first + (e - group_col_prefix<R>(ul, a0, Gp));
     } else {
-        tm = idx / g.tiles_n; tn = idx % g.tiles_n;
+        const int64_t q = idx / (kWsGroup * TN), a0 = q * kWsGroup, Gp = ((TM - a0) < kWsGroup ? (TM - a0) : (int64_t)kWsGroup);
+        const int64_t e = idx - a0 * TN;
+        tn = e / Gp; tm = a0 + e % Gp;
     }
     m0 = tm * BM; n0 = tn * BN;
     if (g.mask == MASK_CHK) {
@@ -374,8 +425,8 @@ __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t&
     return true;
 }
 
-__global__ void __launch_bounds__(WsCfg::THREADS, 1) k_gemm_ws(GemmArgs g, int64_t ntiles) {
-    using C_ = WsCfg;
+template <class C_>
+__global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, int64_t ntiles) {
     constexpr int BM = C_::BM, BN = C_::BN, BK = C_::BK, WM = C_::WM, WN = C_::WN, STAGES = C_::STAGES;
     if (*(volatile const int32_t*)g.abort) return;
     extern __shared__ __align__(16) double smem[];
@@ -392,12 +443,12 @@ __global__ void __launch_bounds__(WsCfg::THREADS, 1) k_gemm_ws(GemmArgs g, int64
 
     if (warp >= C_::CONSUMERS) {
         // ------------------------------- producer -------------------------------
-        asm volatile("setmaxnreg.dec.sync.aligned.u32 40;\n" ::: "memory");
+        asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;\n" ::"n"(C_::REG_PROD) : "memory");
         if (warp != C_::CONSUMERS) return;
         uint32_t it = 0;
         for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
             int64_t m0, n0;
-            if (!ws_tile(g, t, m0, n0)) continue;
+            if (!ws_tile<BM, BN>(g, t, m0, n0)) continue;
             const int64_t ke = (g.krange == KR_LE_N) ? min(g.K, n0 + BN) : g.K;
             const int kt_n = (int)(ke / BK);
             const uint32_t rowsA = (uint32_t)(g.M - m0 < BM ? g.M - m0 : BM), rowsB = (uint32_t)(g.N - n0 < BN ? g.N - n0 : BN);
@@ -423,14 +474,14 @@ __global__ void __launch_bounds__(WsCfg::THREADS, 1) k_gemm_ws(GemmArgs g, int64
         return;
     }
     // ------------------------------- consumers -------------------------------
-    asm volatile("setmaxnreg.inc.sync.aligned.u32 232;\n" ::: "memory");
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;\n" ::"n"(C_::REG_CONS) : "memory");
     const int wm = warp / C_::WARPS_N, wn = warp % C_::WARPS_N;
     const int fr = lane >> 2, fc = lane & 3;
     const double ab = g.alpha * g.beta, alpha = g.alpha;
     uint32_t it = 0;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
         int64_t m0, n0;
-        if (!ws_tile(g, t, m0, n0)) continue;
+        if (!ws_tile<BM, BN>(g, t, m0, n0)) continue;
         const int64_t ke = (g.krange == KR_LE_N) ? min(g.K, n0 + BN) : g.K;
         const int kt_n = (int)(ke / BK);
         double acc[C_::FM][C_::FN][2];
@@ -508,7 +559,7 @@ __global__ void __launch_bounds__(WsCfg::THREADS, 1) k_gemm_ws(GemmArgs g, int64
                             s2 += __shfl_xor_sync(0xffffffffu, s2, o);
                         }
                         if (fr == 0) {
-                            const int64_t slab = gr0 / WM;
+                            const int64_t slab = gr0 / g.cs.slab_rows;
                             const int64_t gc = gc0 + wn * WN + j * 8 + fc * 2 + h;
                             g.cs.p[slab * g.cs.ld + gc] = s1;
                             g.cs.p[(g.cs.nslab + slab) * g.cs.ld + gc] = s2;
@@ -519,27 +570,48 @@ __global__ void __launch_bounds__(WsCfg::THREADS, 1) k_gemm_ws(GemmArgs g, int64
     }
 }
 
+template <class C_>
 static int run_ws(GemmArgs g, cudaStream_t s) {
     static bool attr = false;
-    static int nsm = 148;
     if (!attr) {
-        cudaFuncSetAttribute(k_gemm_ws, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)WsCfg::SMEM);
-        int dev = 0; cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        cudaFuncSetAttribute(k_gemm_ws<C_>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::SMEM);
         attr = true;
     }
-    const int64_t tm = (g.M + WsCfg::BM - 1) / WsCfg::BM, tn = (g.N + WsCfg::BN - 1) / WsCfg::BN;
+    const int64_t tm = (g.M + C_::BM - 1) / C_::BM, tn = (g.N + C_::BN - 1) / C_::BN;
     g.tiles_n = tn;
-    const int64_t ntiles = (g.mask == MASK_LOWER) ? tn * (tn + 1) / 2 + (tm - tn) * tn : tm * tn;
+    const int64_t ntiles = (g.mask == MASK_LOWER) ? lower_prefix<C_::BM / C_::BN>(tm, tn) : tm * tn;
     if (ntiles <= 0) return 0;
     // tiles per CTA: 1 lets the block scheduler interleave the high-priority look-ahead stream's
-    // kernels as CTAs retire; a fully persistent grid (tpc = inf) would starve that stream.
+    // kernels as CTAs retire; a fully persistent grid would starve that stream.
     static int64_t tpc = -1;
     if (tpc < 0) { const char* e = getenv("ABFT_WS_TPC"); tpc = e ? std::max(1, atoi(e)) : 1; }
     const int64_t grid = std::max<int64_t>(1, (ntiles + tpc - 1) / tpc);
-    k_gemm_ws<<<(unsigned)grid, WsCfg::THREADS, WsCfg::SMEM, s>>>(g, ntiles);
+    k_gemm_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles);
     abft_count_launch();
     return 0;
+}
+
+static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CTA/SM), 16, 2a
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("ABFT_WS");
+        v = 22;
+        if (e && !strcmp(e, "1")) v = 0;
+        if (e && !strcmp(e, "16")) v = 16;
+        if (e && !strcmp(e, "2a")) v = 21;
+        if (e && !strcmp(e, "2b")) v = 22;
+    }
+    return v;
+}
+static int ws_slab_rows() { return ws_variant() == 16 ? WsCfg16::WM : 64; }
+static int run_ws_any(GemmArgs g, cudaStream_t s) {
+    g.cs.slab_rows = ws_slab_rows();
+    switch (ws_variant()) {
+        case 16: return run_ws<WsCfg16>(g, s);
+        case 21: return run_ws<WsCfg2a>(g, s);
+        case 22: return run_ws<WsCfg2b>(g, s);
+        default: return run_ws<WsCfg>(g, s);
+    }
 }
 
 }  // namespace abft
@@ -553,13 +625,13 @@ static bool aligned16(const void* p) { return ((uintptr_t)p & 15) == 0; }
 int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                 int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
                 int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
-                cudaStream_t s, int force_tile, const ColSumOut* cs) {
+                cudaStream_t s, int force_tile, ColSumOut* cs) {
     if (M <= 0 || N <= 0) return 0;
     GemmArgs g;
     g.M = M; g.N = N; g.K = K; g.A = A; g.lda = lda; g.B = B; g.ldb = ldb; g.C = C; g.ldc = ldc;
     g.alpha = alpha; g.beta = beta; g.mask = mask; g.krange = krange; g.nb = nb;
     g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
-    g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1};
+    g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64};
     g.vecA = aligned16(A) && (lda % 2 == 0);
     g.vecB = aligned16(B) && (ldb % 2 == 0);
     auto tiles = [&](int64_t t) {
@@ -582,10 +654,10 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
     if (cs) {   // fused partials need the warp-specialised kernel with nb-aligned 128-row tiles
         if (!(ws_ok && variant != 2 && mask == MASK_LOWER && cs->nb % WsCfg::BM == 0 &&
               cs->row0 % WsCfg::BM == 0 && cs->col0 % WsCfg::BN == 0 && M % WsCfg::BM == 0)) g.cs.p = nullptr;
-        else { run_ws(g, s); return 1; }
+        else { run_ws_any(g, s); cs->slab_rows = ws_slab_rows(); return 1; }
     }
     if (transB) {
-        if (tile == 128 && ws_ok && variant != 2) return run_ws(g, s);
+        if (tile == 128 && ws_ok && variant != 2) return run_ws_any(g, s);
         if (tile == 128) return run_cfg<128, 128, 32, 64, 32, 3, true>(g, s);
         if (tile == 64) return run_cfg<64, 64, 16, 32, 32, 4, true>(g, s);
         return run_cfg<32, 32, 16, 16, 16, 4, true>(g, s);

@@ -83,11 +83,11 @@ __global__ void __launch_bounds__(kLeafThreads) k_leaf_potrf_inv(double* T, int6
     // inverse: Y = I; step p: Y(i,:) -= L(i,p)/L(p,p) * Y(p,:) for i > p; X(i,:) = Y(i,:)/L(i,i)
     for (int p = 0; p < nl; ++p) {
         __syncthreads();
-        const double lpp = L[p * P + p];
+        const double rpp = 1.0 / L[p * P + p];       // one FP64 division per step, not per element
 #pragma unroll
         for (int q = 0; q < kLeafOwn; ++q) {
             const int i = own_r[q], c = own_c[q];
-            if (i > p && p >= c) X[c * P + i] -= (L[p * P + i] / lpp) * X[c * P + p];
+            if (i > p && p >= c) X[c * P + i] -= (L[p * P + i] * rpp) * X[c * P + p];
         }
     }
     __syncthreads();
