@@ -103,8 +103,9 @@ typedef struct abft_options {
 /* Per-phase device time of the last abft_potrf* call on this thread with options.profile = 1.
  * Phases: 0 encode, 1 V1/V2, 2 POTRF+inverse, 3 TRSM (+Alg. 2 rows), 4 V3, 5 V4, 6 panel
  * write-back, 7 trailing update (data rows), 8 trailing update (checksum rows), 9 V5, 10 V6,
- * 11 injection. flops / bytes are the ALGORITHMIC counts of DESIGN.md §6 (not executed ones). */
-#define ABFT_NPHASE 12
+ * 11 injection, 12 main stream waiting for the look-ahead panel. flops / bytes are the
+ * ALGORITHMIC counts of DESIGN.md §6 (not executed ones). */
+#define ABFT_NPHASE 13
 typedef struct abft_profile {
     int32_t nphase, pad;
     double ms[16];

@@ -203,9 +203,9 @@ static void do_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, in
 }
 
 // ---- per-phase profiler (options.profile) ----------------------------------------------------
-enum { PH_ENCODE, PH_V12, PH_POTRF, PH_TRSM, PH_V3, PH_V4, PH_WB, PH_UPD, PH_UPDC, PH_V5, PH_V6, PH_INJ };
+enum { PH_ENCODE, PH_V12, PH_POTRF, PH_TRSM, PH_V3, PH_V4, PH_WB, PH_UPD, PH_UPDC, PH_V5, PH_V6, PH_INJ, PH_WAIT };
 static const char* kPhaseNames[ABFT_NPHASE] = {"encode", "v1v2", "potrf_inv", "trsm", "v3", "v4", "writeback",
-                                               "update", "update_chk", "v5", "v6", "inject"};
+                                               "update", "update_chk", "v5", "v6", "inject", "wait_panel"};
 static thread_local abft_profile_t g_prof;
 
 struct Profiler {
@@ -424,7 +424,11 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     }
     pan[0] = panel(0);
     for (int64_t k = 0; k < N; ++k) {
-        cudaStreamWaitEvent(s, pan[k], 0);
+        {
+            cudaEvent_t t = prof.begin(s);
+            cudaStreamWaitEvent(s, pan[k], 0);
+            prof.end(t, PH_WAIT, s);
+        }
         const int64_t m = N - k - 1, mB = m * B;
         if (m == 0) break;
         const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);

@@ -16,27 +16,27 @@ namespace abft {
 
 constexpr int kLeaf = 64;
 
-// One CTA: Cholesky of the lower triangle of T (nl x nl, nl <= 64) in shared memory, then its
-// inverse, both right-looking with ONE barrier per step: each thread owns a fixed set of <= 9
-// lower-triangle elements; step j updates them with the unscaled column j divided by the pivot
-// d_j (A22 -= a_j a_j^T / d_j, identical to l_j l_j^T), and the columns are scaled once at the
-// end. The inverse solves L X = I by forward elimination in the same owner-computes pattern.
+// One CTA: Cholesky of the lower triangle of T (nl x nl, nl <= 64) and its inverse, in shared
+// memory, with ONE barrier per column: each thread owns a fixed set of lower-triangle elements.
+// Interval j runs Cholesky step j (A22 -= a_j a_j^T / d_j with the unscaled column a_j, which is
+// l_j l_j^T) and forward-elimination step j of L X = I (Y(i,:) -= a_ij / d_j * Y(j,:), which is
+// l_ij / l_jj); both only read column j, final since interval j-1. Columns and rows are scaled
+// once at the end (l_j = a_j / sqrt(d_j), X(i,:) = Y(i,:) / sqrt(d_i)).
 // Writes L (lower) into T and inv(L) (lower, upper zeroed) into Li. A non-positive pivot sets
 // NOT_SPD with info = off + j + 1 and aborts.
-constexpr int kLeafThreads = 256;
-constexpr int kLeafOwn = (kLeaf * (kLeaf + 1) / 2 + kLeafThreads - 1) / kLeafThreads;   // 9
+constexpr int kLeafThreads = 512;
+constexpr int kLeafOwn = (kLeaf * (kLeaf + 1) / 2 + kLeafThreads - 1) / kLeafThreads;   // 5
 
 __global__ void __launch_bounds__(kLeafThreads) k_leaf_potrf_inv(double* T, int64_t ldt, double* Li, int64_t ldi,
                                                                  int nl, int64_t info_off, DevState* st) {
     if (st->abort) return;
     extern __shared__ double leaf_smem[];
-    double* L = leaf_smem;                              // L[c*(kLeaf+1) + r]
-    double* X = leaf_smem + kLeaf * (kLeaf + 1);        // X[c*(kLeaf+1) + i] = inv(L)(i, c)
-    __shared__ double dd[kLeaf];
     constexpr int P = kLeaf + 1;
+    double* L = leaf_smem;                 // L[c*P + r]: unscaled a, then l
+    double* Y = leaf_smem + kLeaf * P;     // Y[c*P + i]: forward elimination of L X = I
+    __shared__ double rdd[kLeaf];          // 1 / d_j
     const int tid = threadIdx.x;
     const int E = nl * (nl + 1) / 2;
-    // owned elements (r, c), r >= c, enumerated column by column
     int own_r[kLeafOwn], own_c[kLeafOwn];
 #pragma unroll
     for (int q = 0; q < kLeafOwn; ++q) {
@@ -44,14 +44,14 @@ __global__ void __launch_bounds__(kLeafThreads) k_leaf_potrf_inv(double* T, int6
         if (e < E) {
             while (e >= nl - c) { e -= nl - c; ++c; }
             own_r[q] = c + e; own_c[q] = c;
-        } else { own_r[q] = -1; own_c[q] = -1; }
+        } else { own_r[q] = -1; own_c[q] = kLeaf; }
     }
 #pragma unroll
     for (int q = 0; q < kLeafOwn; ++q)
         if (own_r[q] >= 0) {
             const int r = own_r[q], c = own_c[q];
             L[c * P + r] = T[c * ldt + r];
-            X[c * P + r] = (r == c) ? 1.0 : 0.0;
+            Y[c * P + r] = (r == c) ? 1.0 : 0.0;
         }
     for (int j = 0; j < nl; ++j) {
         __syncthreads();
@@ -60,40 +60,30 @@ __global__ void __launch_bounds__(kLeafThreads) k_leaf_potrf_inv(double* T, int6
             if (tid == 0 && atomicCAS(&st->abort, 0, 1) == 0) { st->status = ABFT_NOT_SPD; st->info = info_off + j + 1; }
             return;
         }
-        if (tid == 0) dd[j] = d;
         const double inv_d = 1.0 / d;
+        if (tid == 0) rdd[j] = inv_d;
+        const double* colj = L + j * P;
+        const double* rowj = Y + j;          // Y(j, c) at rowj[c * P]
 #pragma unroll
         for (int q = 0; q < kLeafOwn; ++q) {
             const int r = own_r[q], c = own_c[q];
-            if (c > j) L[c * P + r] -= L[j * P + r] * (L[j * P + c] * inv_d);
+            if (c > j) L[c * P + r] -= colj[r] * (colj[c] * inv_d);             // Cholesky step j
+            if (r > j && j >= c) Y[c * P + r] -= (colj[r] * inv_d) * rowj[c * P]; // elimination step j
         }
     }
     __syncthreads();
-    // scale: l_j = a_j / sqrt(d_j)
 #pragma unroll
     for (int q = 0; q < kLeafOwn; ++q) {
         const int r = own_r[q], c = own_c[q];
         if (r >= 0) {
-            const double sq = sqrt(dd[c]);
-            const double v = (r == c) ? sq : L[c * P + r] / sq;
-            L[c * P + r] = v;
-            T[c * ldt + r] = v;
+            const double sc = sqrt(rdd[c]);                 // 1 / sqrt(d_c)
+            T[c * ldt + r] = (r == c) ? 1.0 / sc : L[c * P + r] * sc;
+            Li[c * ldi + r] = Y[c * P + r] * sqrt(rdd[r]);
         }
     }
-    // inverse: Y = I; step p: Y(i,:) -= L(i,p)/L(p,p) * Y(p,:) for i > p; X(i,:) = Y(i,:)/L(i,i)
-    for (int p = 0; p < nl; ++p) {
-        __syncthreads();
-        const double rpp = 1.0 / L[p * P + p];       // one FP64 division per step, not per element
-#pragma unroll
-        for (int q = 0; q < kLeafOwn; ++q) {
-            const int i = own_r[q], c = own_c[q];
-            if (i > p && p >= c) X[c * P + i] -= (L[p * P + i] * rpp) * X[c * P + p];
-        }
-    }
-    __syncthreads();
-    for (int e = tid; e < nl * nl; e += kLeafThreads) {
+    for (int e = tid; e < nl * nl; e += kLeafThreads) {    // upper part of the inverse: zeros
         const int c = e / nl, i = e % nl;
-        Li[c * ldi + i] = (i >= c) ? X[c * P + i] / L[i * P + i] : 0.0;
+        if (i < c) Li[c * ldi + i] = 0.0;
     }
 }
 
