@@ -78,7 +78,7 @@ typedef struct abft_event {
     int32_t k, check, tile_i, tile_j;
     int32_t row, col;   /* inside the tile; the stored (lower) element for diagonal tiles;
                            row = -1 / -2 for CHK1 / CHK2, -3 for UNCORRECTABLE              */
-    int32_t kind, rank;
+    int32_t kind, rank;   /* rank that ran the check: owner of block column tile_j (receiver for V4R) */
     double delta1, delta2;
 } abft_event_t;
 
@@ -168,6 +168,19 @@ int abft_comm_destroy(void* comm);
 int abft_potrf_dist(int64_t n, int64_t nb, double* A_local, int64_t lda_local, void* comm, int rank,
                     int nranks, abft_stream_t stream, const abft_inject_spec_t* inj,
                     abft_report_t* rep, const abft_options_t* opt);
+/* abft_potrf_dist errors: -1 n, -2 nb, -3 A_local, -4 lda_local, -5 comm (or its rank/size
+ * disagree with rank/nranks), -6 rank, -7 nranks, -9 inj, -11 options; ABFT_ERR_NCCL on a failed
+ * collective. No look-ahead across ranks yet. */
+
+/* Test harness of the multi-GPU algorithm on ONE device: runs the nranks ranks of
+ * abft_potrf_dist in one process, in lock-step, with the NCCL broadcast replaced by device-to-
+ * device copies (A_locals[r]: rank r's local block columns, same layout as abft_potrf_dist).
+ * Everything else — ownership, the owner's panel, the receivers' RECV hook and V4R re-check,
+ * the per-rank trailing updates, V5/V6 on owned tiles, the merged report — is the code the NCCL
+ * path runs. Errors: -1 n, -2 nb, -3 nranks, -4 A_locals, -5 lda_local, -6 inj (as -9 there). */
+int abft_potrf_dist_sim(int64_t n, int64_t nb, int nranks, double* const* A_locals, int64_t lda_local,
+                        abft_stream_t stream, const abft_inject_spec_t* inj, abft_report_t* rep,
+                        const abft_options_t* opt);
 
 /* Diagnostics: the trailing-update GEMM on its own (for benchmarking the dominant kernel):
  * C = beta C + alpha A B^T over the lower triangle (lower = 1: r >= c, requires N <= M) or all

@@ -107,6 +107,7 @@ typedef struct { int64_t c; int kind; int64_t row; double d1, d2, r1, r2; } odec
 
 static int check_tile(octx_t* x, const tview_t* v, int k, int V, int rank) {
     const int64_t B = x->B;
+    if (V != O_V4R) rank = (int)(v->J % x->nranks);    /* the owner of block column J runs the check */
     odec_t* dec = (odec_t*)malloc(sizeof(odec_t) * (size_t)B);
     int64_t nd = 0;
     x->cnt->n_checks++;
@@ -503,6 +504,7 @@ int oracle_encode(int64_t n, int64_t nb, const double* A, int64_t lda, double* c
     ocount_t c; memset(&c, 0, sizeof c); x->cnt = &c;
     x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = ldc;
     x->A = (double*)A; x->chk = chk; x->s = scl; x->S1 = scl + n; x->S2 = scl + n + x->N;
+    x->nranks = 1;
     if (n == 0) return 0;
     scales(x); encode(x);
     return 0;
@@ -521,7 +523,7 @@ int oracle_verify(int64_t n, int64_t nb, double* A, int64_t lda, double* chk, in
     x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = ldc;
     x->A = A; x->chk = chk; x->s = (double*)scl; x->S1 = (double*)scl + n; x->S2 = (double*)scl + n + x->N;
     x->c_tau = c_tau > 0 ? c_tau : 64.0; x->rho = 0x1p-30; x->correct = correct;
-    x->ev = ev; x->cap = cap;
+    x->ev = ev; x->cap = cap; x->nranks = 1;
     for (int64_t J = 0; J < x->N; ++J)
         for (int64_t I = J; I < x->N; ++I) {
             tview_t v = gview(x, I, J, factored);

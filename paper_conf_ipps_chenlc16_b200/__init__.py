@@ -74,6 +74,8 @@ _lib.abft_nccl_id.argtypes = [_vp]
 _lib.abft_comm_init.argtypes = [ctypes.POINTER(_vp), _i32, _vp, _i32]
 _lib.abft_comm_destroy.argtypes = [_vp]
 _lib.abft_potrf_dist.argtypes = [_i64, _i64, _vp, _i64, _vp, _i32, _i32, _vp, _vp, _vp, _vp]
+_lib.abft_potrf_dist_sim.argtypes = [_i64, _i64, _i32, _vp, _i64, _vp, _vp, _vp, _vp]
+_lib.abft_potrf_dist_sim.restype = _i32
 _lib.abft_dev_gemm_nt.argtypes = [_i64, _i64, _i64, _vp, _i64, _vp, _i64, _vp, _i64, _dbl, _dbl, _i32, _vp]
 _lib.abft_dev_gemm_nt.restype = _i32
 _lib.abft_last_launch_count.restype = _i64
@@ -89,6 +91,7 @@ for _f in ("abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_po
 EXPORTS = ["abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
            "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist",
            "abft_last_launch_count", "abft_version", "abft_last_error", "abft_last_profile", "abft_dev_gemm_nt",
+           "abft_potrf_dist_sim",
            "abft_phase_name"]
 
 
@@ -251,6 +254,59 @@ def abft_dev_gemm_nt(M, N, K, A, B, C, alpha=-1.0, beta=1.0, lower=True, stream=
     pc, lc = _dev(C)
     return _lib.abft_dev_gemm_nt(M, N, K, pa, la or M, pb, lb or N, pc, lc or M, alpha, beta, int(lower),
                                  _stream(stream))
+
+
+def abft_potrf_dist_sim(n, nb, A_locals, lda=None, stream=None, inj=None, report=True, cap=1 << 16, opt=None):
+    """Multi-GPU algorithm with nranks = len(A_locals) simulated ranks on one device (tests)."""
+    ptrs = [(_dev(a)[0] if a is not None else None) or 0 for a in A_locals]
+    lds = [_dev(a)[1] for a in A_locals if a is not None and _dev(a)[1] is not None]
+    arrp = (ctypes.c_void_p * len(ptrs))(*ptrs)
+    arr, pinj = _inj(inj)
+    rep, ev = _new_report(cap) if report else (None, None)
+    o = opt if opt is not None else options()
+    st = _lib.abft_potrf_dist_sim(n, nb, len(ptrs), arrp, lda or (lds[0] if lds else n), _stream(stream), pinj,
+                                  ctypes.byref(rep) if rep else None, ctypes.byref(o))
+    return st, (_report_dict(rep, ev) if rep else None)
+
+
+def owned_blocks(N, rank, nranks):
+    """Block columns rank `rank` owns in the 1D block-cyclic layout (J mod nranks == rank)."""
+    return list(range(rank, N, nranks))
+
+
+def nccl_id_exchange(group=None):
+    """Host plumbing of the multi-GPU path: rank 0 creates the NCCL unique id through the C-ABI
+    and every rank of the torch.distributed group receives the same 128 bytes."""
+    import torch.distributed as dist
+    obj = [None]
+    if dist.get_rank(group) == 0:
+        st, nid = abft_nccl_id()
+        assert st == 0, "abft_nccl_id failed"
+        obj[0] = nid
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
+def block_cyclic_split(A, nb, nranks):
+    """Global column-major matrix (numpy, n x n) -> per-rank local block columns (F-order arrays)."""
+    n = A.shape[0]
+    N = n // nb
+    out = []
+    for r in range(nranks):
+        cols = [np.arange(J * nb, (J + 1) * nb) for J in range(r, N, nranks)]
+        idx = np.concatenate(cols) if cols else np.zeros(0, dtype=np.int64)
+        out.append(np.asfortranarray(A[:, idx]))
+    return out
+
+
+def block_cyclic_join(locals_, nb, n):
+    """Inverse of block_cyclic_split."""
+    P = len(locals_)
+    A = np.zeros((n, n), order="F")
+    for r, L in enumerate(locals_):
+        for t, J in enumerate(range(r, n // nb, P)):
+            A[:, J * nb:(J + 1) * nb] = L[:, t * nb:(t + 1) * nb]
+    return A
 
 
 def abft_last_launch_count():

@@ -34,6 +34,11 @@ int launch_chol_inv(double* T, int64_t ldt, double* Li, int64_t B, int64_t info_
 int launch_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, cudaStream_t s);
 int launch_inject(int nops, double* const* ptrs, const uint64_t* masks, const int32_t* abort_flag,
                   cudaStream_t s);
+int launch_axpy(int64_t n, const double* x, double* y, cudaStream_t s);
+int launch_abort_to_slot(const int32_t* abort_flag, double* slot, cudaStream_t s);
+int launch_abort_from_slot(const double* slot, DevState* st, cudaStream_t s);
+int launch_scales_diag(int64_t nrows, const double* Adiag, int64_t lda, double* s_out, cudaStream_t s);
+int launch_scales_blocks(int64_t N, int64_t nb, const double* sv, double* S1, double* S2, cudaStream_t s);
 
 // ---- diagnostics --------------------------------------------------------------------------
 static thread_local int64_t g_launches = 0;
@@ -382,7 +387,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         bool inj_here = false;
         for (const auto& sp : inj)
             if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && sp.col / nb >= jlo && sp.col / nb < jhi) inj_here = true;
-        ColSumOut cso{w.cs, n, w.cs_nslab, jlo * B, jlo * B, B, 64};
+        ColSumOut cso{w.cs, n, w.cs_nslab, jlo * B, jlo * B, B, 64, jlo * B};
         const int fused = launch_gemm(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab,
                                       s, 0, (can_fuse && !inj_here) ? &cso : nullptr);
         prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd, 0);
@@ -483,6 +488,313 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     if (rc) return rc;
     ABFT_CUDA_TRY(cudaGetLastError());
     return status;
+}
+
+
+// =============================================================================================
+// 1D block-cyclic multi-GPU driver. Rank r owns block columns {J : J mod P = r},
+// stored contiguously (local block t = global block t*P + r). Per iteration k the owner of block
+// column k runs V1/V2, POTRF + inverse, TRSM (+ Alg. 2 rows), V3, V4 and the write-back exactly as
+// on one GPU, then broadcasts the packed panel W = [L(k+1:N,k); chk rows 2k..2N-1] (plus one
+// slot carrying its abort flag); every receiver re-checks its copy (RECV hook -> V4R, rank r)
+// and all ranks apply the trailing update to their own block columns, checksum rows included,
+// followed by V5 on their own tiles. Decisions are owner-local, so the event multiset is the
+// single-GPU one plus V4R events (the oracle's P-rank simulation reproduces it).
+// =============================================================================================
+namespace {
+struct RankState {
+    int r;
+    double* A; int64_t lda;
+    int64_t nblk, ncl;        // local block columns, local columns
+    Work w;
+    double* xslot = nullptr;  // abort flag slot right after the packed panel inside W
+};
+}
+
+static int64_t dist_lc(int64_t J, int P, int64_t nb) { return (J / P) * nb; }   // local column of block J
+
+static double* dist_inj_ptr(const abft_inject_spec_t& sp, int64_t k, int64_t nb, int P, const RankState& R,
+                            int64_t ldw, int64_t mB) {
+    const int hook = sp.hook;
+    const int64_t Jc = sp.col / nb, lcol = dist_lc(Jc, P, nb) + sp.col % nb;
+    if (hook == ABFT_HOOK_TRSM_OUT || hook == ABFT_HOOK_RECV) {
+        if (sp.target == ABFT_TGT_DATA) return R.w.W + (sp.col - k * nb) * ldw + (sp.row - (k + 1) * nb);
+        return R.w.W + (sp.col - k * nb) * ldw + mB + (sp.row - 2 * k);
+    }
+    if (hook == ABFT_HOOK_POTRF_OUT && sp.target == ABFT_TGT_CHK)
+        return R.w.W + (sp.col - k * nb) * ldw + mB + (sp.row - 2 * k);
+    if (sp.target == ABFT_TGT_DATA) return R.A + lcol * R.lda + sp.row;
+    return R.w.chk + lcol * R.w.ldc + sp.row;
+}
+
+static void dist_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, int hook, int64_t nb, int P,
+                        const RankState& R, int64_t ldw, int64_t mB, cudaStream_t s) {
+    std::vector<double*> ptrs; std::vector<uint64_t> masks;
+    for (const auto& sp : list) {
+        if (sp.k != k || sp.hook != hook) continue;
+        if (hook == ABFT_HOOK_RECV) { if (sp.rank != R.r) continue; }
+        else if ((sp.col / nb) % P != R.r) continue;       // the owner of the target's block column
+        ptrs.push_back(dist_inj_ptr(sp, k, nb, P, R, ldw, mB)); masks.push_back(sp.xor_mask);
+    }
+    if (!ptrs.empty()) launch_inject((int)ptrs.size(), ptrs.data(), masks.data(), &R.w.st->abort, s);
+}
+
+int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, DistTransport* tp,
+             cudaStream_t s, const abft_inject_spec_t* inj_c, abft_report_t* rep, const abft_options_t* opt) {
+    abft_options_t o = opt ? *opt : abft_options_t{1, 1, 64.0, 0, 0};
+    if (o.K < 1 || !(o.c_tau > 0)) return -11;
+    std::vector<abft_inject_spec_t> inj;
+    if (collect_inj(inj_c, n, nb, inj)) return -9;
+    if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; }
+    if (n == 0) return 0;
+    const bool abft = o.abft_enabled != 0;
+    const int K = std::max(1, o.K);
+    const int64_t N = n / nb, B = nb;
+    std::vector<RankState> R(nlocal);
+    const int64_t evcap = rep ? std::max<int64_t>(rep->cap, 1) : 1024;
+    for (int i = 0; i < nlocal; ++i) {
+        RankState& q = R[i];
+        q.r = locals[i].rank; q.A = locals[i].A; q.lda = locals[i].lda;
+        q.nblk = (N - q.r + P - 1) / P; q.ncl = q.nblk * B;
+        int rc = work_alloc(q.w, n, nb, std::max<int64_t>(q.ncl, 1), evcap, abft, s);
+        if (rc) return rc;
+        // W with one extra slot for the owner's abort flag
+        cudaFreeAsync(q.w.W, s);
+        const int64_t wrows = (N - 1) * nb + 2 * N + 2;
+        ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.w.W, sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb + 1), s));
+        if (abft && nb % 128 == 0 && q.lda % 2 == 0 && ((uintptr_t)q.A & 15) == 0) {
+            q.w.cs_nslab = n / 32;
+            ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.w.cs, sizeof(double) * (size_t)(2 * q.w.cs_nslab * std::max<int64_t>(q.ncl, 1)), s));
+        }
+        launch_zero(B, B, q.w.Li, B, s);
+    }
+    auto stage = [&](RankState& q, int kind, int V, int k) {
+        StageArgs a = stage_base(q.w, q.A, q.lda, o.c_tau, kind, V, k);
+        a.col_owner_mod = P; a.col_owner_rank = q.r; a.rank = q.r;
+        return a;
+    };
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (rep) { cudaEventCreate(&e0); cudaEventCreate(&e1); cudaEventRecord(e0, s); }
+    // ---- encode: scales need every diagonal block -> all-reduce of the owner-local parts ----
+    if (abft) {
+        for (auto& q : R) {
+            cudaMemsetAsync(q.w.scl, 0, sizeof(double) * (size_t)(n + 2 * N), s);
+            for (int64_t J = q.r; J < N; J += P)
+                launch_scales_diag(B, q.A + dist_lc(J, P, B) * q.lda + J * B, q.lda, q.w.scl + J * B, s);
+        }
+        if (tp) {
+            if (tp->allreduce_sum(R[0].w.scl, (size_t)n, s)) return ABFT_ERR_NCCL;
+        } else {
+            for (int i = 1; i < nlocal; ++i) launch_axpy(n, R[i].w.scl, R[0].w.scl, s);
+            for (int i = 1; i < nlocal; ++i)
+                cudaMemcpyAsync(R[i].w.scl, R[0].w.scl, sizeof(double) * (size_t)n, cudaMemcpyDeviceToDevice, s);
+        }
+        for (auto& q : R) {
+            launch_scales_blocks(N, B, q.w.scl, q.w.scl + n, q.w.scl + n + N, s);
+            StageArgs a = stage(q, SK_ALL, 0, -1);
+            a.encode = 1;
+            launch_check(a, s);
+        }
+    }
+    for (int64_t k = 0; k < N; ++k) {
+        const int owner = (int)(k % P);
+        const int64_t m = N - k - 1, mB = m * B;
+        const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
+        const size_t wcount = (size_t)(ldw * B);
+        for (auto& q : R) if (abft) dist_inject(inj, k, ABFT_HOOK_REST, B, P, q, ldw, mB, s);
+        for (auto& q : R) {
+            if (q.r != owner) continue;
+            const int32_t* ab = &q.w.st->abort;
+            double* Akk = q.A + dist_lc(k, P, B) * q.lda + k * B;
+            double* ckk = q.w.chk + dist_lc(k, P, B) * q.w.ldc;
+            q.xslot = q.w.W + wcount;
+            if (abft) launch_check(stage(q, SK_COLUMN, ABFT_V2, (int)k), s);          // V1, V2
+            launch_chol_inv(Akk, q.lda, q.w.Li, B, k * B, q.w.tmp, q.w.st, s);
+            launch_gemm(mB, B, B, Akk + B, q.lda, q.w.Li, B, q.w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, s);
+            if (abft) {
+                launch_gemm(2 * m + 2, B, B, ckk + 2 * k, q.w.ldc, q.w.Li, B, q.w.W + mB, ldw, 1.0, 0.0, true, 0, 1,
+                            0, 0, 0, ab, s);
+                dist_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, P, q, ldw, mB, s);
+                StageArgs a3 = stage(q, SK_DIAG_FACT, ABFT_V3, (int)k);
+                a3.ldw = ldw; a3.mB = mB;
+                launch_check(a3, s);                                                   // V3
+                dist_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, P, q, ldw, mB, s);
+                StageArgs a4 = stage(q, SK_PANEL, ABFT_V4, (int)k);
+                a4.ldw = ldw; a4.mB = mB;
+                launch_check(a4, s);                                                   // V4
+            }
+            launch_copy(mB, B, q.w.W, ldw, Akk + B, q.lda, ab, s);
+            if (abft) launch_copy(2 * m + 2, B, q.w.W + mB, ldw, ckk + 2 * k, q.w.ldc, ab, s);
+            launch_abort_to_slot(ab, q.xslot, s);
+        }
+        if (m == 0) continue;
+        // ---- broadcast of the packed panel (+ abort slot) from the owner ----
+        if (tp) {
+            if (tp->bcast(R[0].w.W, (wcount + 1) * sizeof(double), owner, s)) return ABFT_ERR_NCCL;
+        } else {
+            const RankState* src = nullptr;
+            for (auto& q : R) if (q.r == owner) src = &q;
+            for (auto& q : R)
+                if (q.r != owner)
+                    cudaMemcpyAsync(q.w.W, src->w.W, (wcount + 1) * sizeof(double), cudaMemcpyDeviceToDevice, s);
+        }
+        for (auto& q : R) {
+            if (q.r == owner) continue;
+            launch_abort_from_slot(q.w.W + wcount, q.w.st, s);
+            if (abft) {
+                dist_inject(inj, k, ABFT_HOOK_RECV, B, P, q, ldw, mB, s);
+                StageArgs a = stage(q, SK_PANEL, ABFT_V4R, (int)k);                   // V4R
+                a.ldw = ldw; a.mB = mB; a.col_owner_mod = 1; a.col_owner_rank = 0;
+                launch_check(a, s);
+            }
+        }
+        // ---- trailing update of each rank's own block columns ----
+        const bool gated = ((k + 1) % K == 0) || k == N - 2;
+        for (auto& q : R) {
+            const int32_t* ab = &q.w.st->abort;
+            bool inj_here = false;
+            for (const auto& sp : inj)
+                if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && (sp.col / B) % P == q.r) inj_here = true;
+            bool all_fused = q.w.cs != nullptr && !inj_here;
+            for (int64_t J = k + 1; J < N; ++J) {
+                if (J % P != q.r) continue;
+                const int64_t t = J / P;
+                double* W0 = q.w.W + (J - k - 1) * B;
+                double* C = q.A + t * B * q.lda + J * B;
+                ColSumOut cso{q.w.cs, q.ncl, q.w.cs_nslab, J * B, t * B, B, 64, J * B};
+                const int f = launch_gemm((N - J) * B, B, B, W0, ldw, W0, ldw, C, q.lda, -1.0, 1.0, true, 1, 0, 0, 0,
+                                          0, ab, s, 0, all_fused ? &cso : nullptr);
+                if (f != 1) all_fused = false;
+                if (abft)
+                    launch_gemm(2 * (N - J), B, B, q.w.W + mB + 2 + 2 * (J - k - 1), ldw, W0, ldw,
+                                q.w.chk + t * B * q.w.ldc + 2 * J, q.w.ldc, -1.0, 1.0, true, 2, 0, B, 0, 0, ab, s);
+            }
+            if (!abft) continue;
+            dist_inject(inj, k, ABFT_HOOK_UPDATE_OUT, B, P, q, ldw, mB, s);
+            if (gated) {
+                StageArgs a = stage(q, SK_TRAIL, ABFT_V5, (int)k);
+                a.j_lo = k + 1; a.j_hi = N;
+                if (all_fused) {
+                    StageArgs d = a; d.kind = SK_TRAIL_DIAG;
+                    StageArgs f = a; f.kind = SK_TRAIL_OFF;
+                    f.cs = q.w.cs; f.cs_ld = q.ncl; f.cs_nslab = q.w.cs_nslab; f.cs_slab_rows = 64;
+                    launch_check_v5_fused(d, f, s);                                    // V5 (fused)
+                } else {
+                    launch_check(a, s);                                                // V5
+                }
+            }
+        }
+    }
+    if (abft) {
+        for (auto& q : R) {
+            dist_inject(inj, N, ABFT_HOOK_REST, B, P, q, 1, 0, s);
+            StageArgs a6 = stage(q, SK_ALL, ABFT_V6, (int)N);
+            a6.factored = 1;
+            launch_check(a6, s);                                                       // V6
+        }
+    }
+    ABFT_CUDA_TRY(cudaGetLastError());
+    // ---- report: counters summed, status/info maxed, events of every rank merged ----
+    int status = 0;
+    {
+        const int nc = 8;
+        std::vector<double> cnt(nc * nlocal, 0.0), mx(2 * nlocal, 0.0);
+        std::vector<abft_event_t> evs;
+        constexpr int64_t CAPG = 2048;
+        double* dbuf = nullptr;     // device staging for the collectives
+        abft_event_t* evg = nullptr;
+        const int nr = tp ? tp->nranks : 1;
+        if (tp) {
+            ABFT_CUDA_TRY(cudaMallocAsync((void**)&dbuf, sizeof(double) * 16, s));
+            ABFT_CUDA_TRY(cudaMallocAsync((void**)&evg, sizeof(abft_event_t) * (size_t)(CAPG * (nr + 1)), s));
+        }
+        std::vector<char> hbuf(sizeof(DevState));
+        DevState& hs = *reinterpret_cast<DevState*>(hbuf.data());
+        double tot[8] = {0}, smax[2] = {0, 0};
+        for (auto& q : R) {
+            ABFT_CUDA_TRY(cudaMemcpyAsync(&hs, q.w.st, offsetof(DevState, fl), cudaMemcpyDeviceToHost, s));
+            ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+            const double v[8] = {(double)hs.n_checks, (double)hs.n_detected, (double)hs.n_data, (double)hs.n_nonfinite,
+                                 (double)hs.n_chk1, (double)hs.n_chk2, (double)hs.n_unc, (double)hs.nev};
+            for (int i = 0; i < 8; ++i) tot[i] += v[i];
+            smax[0] = std::max(smax[0], (double)hs.status); smax[1] = std::max(smax[1], (double)hs.info);
+            const int64_t ne = std::min<int64_t>((int64_t)hs.nev, q.w.ev_cap);
+            std::vector<abft_event_t> tmp(ne);
+            if (ne > 0) ABFT_CUDA_TRY(cudaMemcpy(tmp.data(), q.w.ev, sizeof(abft_event_t) * (size_t)ne, cudaMemcpyDeviceToHost));
+            evs.insert(evs.end(), tmp.begin(), tmp.end());
+        }
+        if (tp) {
+            double hb[16] = {0};
+            for (int i = 0; i < 8; ++i) hb[i] = tot[i];
+            ABFT_CUDA_TRY(cudaMemcpyAsync(dbuf, hb, sizeof(double) * 8, cudaMemcpyHostToDevice, s));
+            if (tp->allreduce_sum(dbuf, 8, s)) return ABFT_ERR_NCCL;
+            ABFT_CUDA_TRY(cudaMemcpyAsync(hb, dbuf, sizeof(double) * 8, cudaMemcpyDeviceToHost, s));
+            double hm[2] = {smax[0], smax[1]};
+            ABFT_CUDA_TRY(cudaMemcpyAsync(dbuf + 8, hm, sizeof(double) * 2, cudaMemcpyHostToDevice, s));
+            if (tp->allreduce_max(dbuf + 8, 2, s)) return ABFT_ERR_NCCL;
+            ABFT_CUDA_TRY(cudaMemcpyAsync(hm, dbuf + 8, sizeof(double) * 2, cudaMemcpyDeviceToHost, s));
+            // events: fixed CAPG block per rank
+            std::vector<abft_event_t> mine(CAPG);
+            memset(mine.data(), 0, sizeof(abft_event_t) * CAPG);
+            const int64_t nm = std::min<int64_t>((int64_t)evs.size(), CAPG);
+            for (int64_t i = 0; i < nm; ++i) mine[i] = evs[i];
+            for (int64_t i = nm; i < CAPG; ++i) mine[i].k = -2;   // padding marker
+            ABFT_CUDA_TRY(cudaMemcpyAsync(evg + CAPG * nr, mine.data(), sizeof(abft_event_t) * CAPG, cudaMemcpyHostToDevice, s));
+            if (tp->allgather(evg + CAPG * nr, evg, sizeof(abft_event_t) * CAPG, s)) return ABFT_ERR_NCCL;
+            std::vector<abft_event_t> all((size_t)(CAPG * nr));
+            ABFT_CUDA_TRY(cudaMemcpyAsync(all.data(), evg, sizeof(abft_event_t) * (size_t)(CAPG * nr), cudaMemcpyDeviceToHost, s));
+            ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+            evs.clear();
+            for (auto& e : all) if (e.k != -2) evs.push_back(e);
+            for (int i = 0; i < 8; ++i) tot[i] = hb[i];
+            smax[0] = hm[0]; smax[1] = hm[1];
+            cudaFreeAsync(dbuf, s); cudaFreeAsync(evg, s);
+        }
+        status = (int)smax[0];
+        if (rep) {
+            rep->info = (int64_t)smax[1];
+            rep->n_checks = (int64_t)tot[0]; rep->n_detected = (int64_t)tot[1]; rep->n_data = (int64_t)tot[2];
+            rep->n_nonfinite = (int64_t)tot[3]; rep->n_chk1 = (int64_t)tot[4]; rep->n_chk2 = (int64_t)tot[5];
+            rep->n_uncorrectable = (int64_t)tot[6]; rep->n_events = (int64_t)tot[7];
+            std::sort(evs.begin(), evs.end(), [](const abft_event_t& x, const abft_event_t& y) {
+                if (x.k != y.k) return x.k < y.k;
+                if (x.check != y.check) return x.check < y.check;
+                if (x.tile_j != y.tile_j) return x.tile_j < y.tile_j;
+                if (x.tile_i != y.tile_i) return x.tile_i < y.tile_i;
+                if (x.col != y.col) return x.col < y.col;
+                if (x.row != y.row) return x.row < y.row;
+                return x.rank < y.rank;
+            });
+            const int64_t nc2 = std::min<int64_t>((int64_t)evs.size(), std::max<int64_t>(rep->cap, 0));
+            if (rep->events) for (int64_t i = 0; i < nc2; ++i) rep->events[i] = evs[i];
+            cudaEventRecord(e1, s);
+            cudaEventSynchronize(e1);
+            float ms = 0; cudaEventElapsedTime(&ms, e0, e1);
+            rep->seconds = ms * 1e-3;
+            cudaEventDestroy(e0); cudaEventDestroy(e1);
+        }
+        (void)cnt; (void)mx;
+    }
+    for (auto& q : R) work_free(q.w, s);
+    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+    return status;
+}
+
+extern "C" int abft_potrf_dist_sim(int64_t n, int64_t nb, int nranks, double* const* A_locals, int64_t lda_local,
+                                   abft_stream_t stream, const abft_inject_spec_t* inj, abft_report_t* rep,
+                                   const abft_options_t* opt) {
+    g_launches = 0;
+    if (n < 0) return -1;
+    if (nb < 1 || n % nb) return -2;
+    if (nranks < 1) return -3;
+    if (!A_locals) return -4;
+    if (lda_local < std::max<int64_t>(1, n)) return -5;
+    std::vector<DistLocal> L(nranks);
+    for (int r = 0; r < nranks; ++r) {
+        if (!A_locals[r] && (n / nb - r + nranks - 1) / nranks > 0) return -4;
+        L[r] = DistLocal{r, A_locals[r], lda_local};
+    }
+    return run_dist(n, nb, nranks, L.data(), nranks, nullptr, (cudaStream_t)stream, inj, rep, opt);
 }
 
 static abft_options_t default_options() {

@@ -110,7 +110,7 @@ __global__ void __launch_bounds__(256) k_check_phase1_fused(StageArgs a) {
     if (threadIdx.x == 0 && c == 0) atomicAdd(&a.st->n_checks, 1ull);
     if (c >= B) return;
     const TileView v = stage_view(a, I, J);
-    const int64_t g = J * B + c, s0 = I * B / a.cs_slab_rows, ns = B / a.cs_slab_rows;
+    const int64_t g = local_col(a, J) + c, s0 = I * B / a.cs_slab_rows, ns = B / a.cs_slab_rows;
     double r1 = 0.0, r2 = 0.0;
     for (int64_t q = 0; q < ns; ++q) {
         r1 += a.cs[(s0 + q) * a.cs_ld + g];
@@ -119,7 +119,7 @@ __global__ void __launch_bounds__(256) k_check_phase1_fused(StageArgs a) {
     const double d1 = __dsub_rn(r1, v.c1[c * v.ldc]);
     const double d2 = __dsub_rn(r2, v.c2[c * v.ldc]);
     double tau1, tau2;
-    thresholds(a, I, g, false, tau1, tau2);
+    thresholds(a, I, J * B + c, false, tau1, tau2);
     const bool f1 = !dfinite(d1) || fabs(d1) > tau1;
     const bool f2 = !dfinite(d2) || fabs(d2) > tau2;
     if (!(f1 || f2)) return;
@@ -360,6 +360,19 @@ int launch_check_v5_fused(const StageArgs& diag, const StageArgs& off, cudaStrea
     StageArgs r = diag;
     r.kind = SK_TRAIL;
     k_check_phase2<<<1, 256, 0, s>>>(r);
+    abft_count_launch();
+    return 0;
+}
+
+int launch_scales_diag(int64_t nrows, const double* Adiag, int64_t lda, double* s_out, cudaStream_t s) {
+    if (nrows <= 0) return 0;
+    k_scales_diag<<<(unsigned)((nrows + 255) / 256), 256, 0, s>>>(nrows, Adiag, lda, s_out);
+    abft_count_launch();
+    return 0;
+}
+int launch_scales_blocks(int64_t N, int64_t nb, const double* sv, double* S1, double* S2, cudaStream_t s) {
+    if (N <= 0) return 0;
+    k_scales_block<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(N, nb, sv, S1, S2);
     abft_count_launch();
     return 0;
 }

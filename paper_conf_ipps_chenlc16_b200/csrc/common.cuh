@@ -180,8 +180,9 @@ __device__ __forceinline__ bool dfinite(double x) { return isfinite(x); }
 namespace abft {
 struct ColSumOut {
     double* p; int64_t ld, nslab;
-    int64_t row0, col0;   // global row / column of C's (0, 0)
+    int64_t row0, col0;   // global row of C's row 0; partial-array column of C's column 0
     int64_t nb;
+    int64_t colg0;        // GLOBAL column of C's column 0 (block-diagonal test; = col0 on one GPU)
     int64_t slab_rows;    // rows per slab (set by the GEMM launcher: its warp-tile height)
 };
 }  // namespace abft
@@ -195,6 +196,22 @@ struct ColSumOut {
 
 void abft_set_error(cudaError_t e, const char* what);
 void abft_count_launch(int n = 1);
+
+// Collective transport of the multi-GPU path: NCCL (dist.cu) — one rank per process.
+struct DistTransport {
+    int rank = 0, nranks = 1;
+    virtual ~DistTransport() {}
+    virtual int bcast(void* buf, size_t bytes, int root, cudaStream_t s) = 0;       // in place
+    virtual int allreduce_sum(double* buf, size_t count, cudaStream_t s) = 0;
+    virtual int allreduce_max(double* buf, size_t count, cudaStream_t s) = 0;
+    virtual int allgather(const void* send, void* recv, size_t bytes, cudaStream_t s) = 0;
+};
+// The 1D block-cyclic driver (abft.cu). ranks: local ranks driven by this call — one with a
+// transport (NCCL, one process per GPU) or all P of them with tp == nullptr (single-process
+// simulation on one device: the broadcast becomes a device-to-device copy).
+struct DistLocal { int rank; double* A; int64_t lda; };
+int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, DistTransport* tp,
+             cudaStream_t s, const abft_inject_spec_t* inj, abft_report_t* rep, const abft_options_t* opt);
 
 // DMMA GEMM launcher (gemm.cu). Returns 1 if the fused column partials `cs` were written
 // (warp-specialised path with 128-row tiles aligned to nb), 0 otherwise.

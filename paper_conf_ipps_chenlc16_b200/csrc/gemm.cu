@@ -541,7 +541,7 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
         // block diagonal (diagonal blocks are checked as sym(tril) by a re-read).
         if (g.cs.p != nullptr) {
             const int64_t gr0 = g.cs.row0 + m0 + wm * WM, gc0 = g.cs.col0 + n0;
-            if (gr0 / g.cs.nb != gc0 / g.cs.nb) {
+            if (gr0 / g.cs.nb != (g.cs.colg0 + n0) / g.cs.nb) {
                 const int64_t wbase = gr0 % g.cs.nb + fr + 1;   // weight (1-based) of row i = 0
 #pragma unroll
                 for (int j = 0; j < C_::FN; ++j)
@@ -631,7 +631,7 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
     g.M = M; g.N = N; g.K = K; g.A = A; g.lda = lda; g.B = B; g.ldb = ldb; g.C = C; g.ldc = ldc;
     g.alpha = alpha; g.beta = beta; g.mask = mask; g.krange = krange; g.nb = nb;
     g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
-    g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64};
+    g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
     g.vecA = aligned16(A) && (lda % 2 == 0);
     g.vecB = aligned16(B) && (ldb % 2 == 0);
     auto tiles = [&](int64_t t) {
@@ -653,7 +653,7 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
                        (mask != MASK_LOWER || N <= M);
     if (cs) {   // fused partials need the warp-specialised kernel with nb-aligned 128-row tiles
         if (!(ws_ok && variant != 2 && mask == MASK_LOWER && cs->nb % WsCfg::BM == 0 &&
-              cs->row0 % WsCfg::BM == 0 && cs->col0 % WsCfg::BN == 0 && M % WsCfg::BM == 0)) g.cs.p = nullptr;
+              cs->row0 % WsCfg::BM == 0 && cs->colg0 % WsCfg::BN == 0 && M % WsCfg::BM == 0)) g.cs.p = nullptr;
         else { run_ws_any(g, s); cs->slab_rows = ws_slab_rows(); return 1; }
     }
     if (transB) {

@@ -42,9 +42,31 @@ __global__ void k_inject(InjBatch b, const int32_t* abort_flag) {
     }
 }
 
+__global__ void k_axpy1(int64_t n, const double* x, double* y) {   // y += x
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+        y[i] += x[i];
+}
+__global__ void k_abort_to_slot(const int32_t* abort_flag, double* slot) { *slot = (double)*abort_flag; }
+__global__ void k_abort_from_slot(const double* slot, DevState* st) {
+    if (*slot != 0.0 && st->abort == 0) st->abort = 1;   // the owner aborted: stop this rank too
+}
+
 }  // namespace abft
 
 using namespace abft;
+
+int launch_axpy(int64_t n, const double* x, double* y, cudaStream_t s) {
+    if (n <= 0) return 0;
+    k_axpy1<<<(unsigned)std::min<int64_t>((n + 255) / 256, 1024), 256, 0, s>>>(n, x, y);
+    abft_count_launch();
+    return 0;
+}
+int launch_abort_to_slot(const int32_t* abort_flag, double* slot, cudaStream_t s) {
+    k_abort_to_slot<<<1, 1, 0, s>>>(abort_flag, slot); abft_count_launch(); return 0;
+}
+int launch_abort_from_slot(const double* slot, DevState* st, cudaStream_t s) {
+    k_abort_from_slot<<<1, 1, 0, s>>>(slot, st); abft_count_launch(); return 0;
+}
 
 int launch_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, cudaStream_t s) {
     if (n == 0) return 0;
