@@ -207,6 +207,38 @@ static void do_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, in
     if (!ptrs.empty()) launch_inject((int)ptrs.size(), ptrs.data(), masks.data(), ab, s);
 }
 
+// ---- per-thread caches: the look-ahead stream and CUDA events are created once and reused, so
+// a call's host-side set-up / tear-down stays a few microseconds (it is inside the caller's timing)
+struct EventPool {
+    std::vector<cudaEvent_t> ev; size_t used = 0; unsigned flags;
+    explicit EventPool(unsigned f) : flags(f) {}
+    cudaEvent_t get() {
+        if (used == ev.size()) { cudaEvent_t e; cudaEventCreateWithFlags(&e, flags); ev.push_back(e); }
+        return ev[used++];
+    }
+    void reset() { used = 0; }
+};
+struct ThreadCache {
+    int device = -1;
+    cudaStream_t P = nullptr;
+    EventPool sync{cudaEventDisableTiming};
+    EventPool timing{cudaEventDefault};
+};
+static thread_local ThreadCache g_tc;
+static ThreadCache& thread_cache() {
+    int dev = 0; cudaGetDevice(&dev);
+    if (g_tc.device != dev) {   // first use on this device (events/streams belong to a device)
+        g_tc.sync = EventPool(cudaEventDisableTiming);
+        g_tc.timing = EventPool(cudaEventDefault);
+        int lo = 0, hi = 0;
+        cudaDeviceGetStreamPriorityRange(&lo, &hi);
+        cudaStreamCreateWithPriority(&g_tc.P, cudaStreamNonBlocking, hi);
+        g_tc.device = dev;
+    }
+    g_tc.sync.reset(); g_tc.timing.reset();
+    return g_tc;
+}
+
 // ---- per-phase profiler (options.profile) ----------------------------------------------------
 enum { PH_ENCODE, PH_V12, PH_POTRF, PH_TRSM, PH_V3, PH_V4, PH_WB, PH_UPD, PH_UPDC, PH_V5, PH_V6, PH_INJ, PH_WAIT };
 static const char* kPhaseNames[ABFT_NPHASE] = {"encode", "v1v2", "potrf_inv", "trsm", "v3", "v4", "writeback",
@@ -215,22 +247,17 @@ static thread_local abft_profile_t g_prof;
 
 struct Profiler {
     bool on = false;
+    EventPool* pool = nullptr;
     struct Rec { int ph; cudaEvent_t a, b; double flops, bytes; };
     std::vector<Rec> recs;
-    std::vector<cudaEvent_t> pool;
-    size_t used = 0;
-    cudaEvent_t get() {
-        if (used == pool.size()) { cudaEvent_t e; cudaEventCreate(&e); pool.push_back(e); }
-        return pool[used++];
-    }
     // begin() returns a token; end() closes it (phases may be open on two streams at once)
     cudaEvent_t begin(cudaStream_t s) {
         if (!on) return nullptr;
-        cudaEvent_t e = get(); cudaEventRecord(e, s); return e;
+        cudaEvent_t e = pool->get(); cudaEventRecord(e, s); return e;
     }
     void end(cudaEvent_t tok, int ph, cudaStream_t s, double flops = 0, double bytes = 0) {
         if (!on || !tok) return;
-        cudaEvent_t e = get(); cudaEventRecord(e, s);
+        cudaEvent_t e = pool->get(); cudaEventRecord(e, s);
         recs.push_back({ph, tok, e, flops, bytes});
     }
     void finish() {   // after a stream sync
@@ -242,8 +269,7 @@ struct Profiler {
             g_prof.ms[r.ph] += ms; g_prof.launches[r.ph] += 1;
             g_prof.flops[r.ph] += r.flops; g_prof.bytes[r.ph] += r.bytes;
         }
-        for (auto e : pool) cudaEventDestroy(e);
-        pool.clear(); recs.clear(); used = 0;
+        recs.clear();
     }
 };
 
@@ -298,15 +324,12 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     double* Wbuf[2] = {w.W, nullptr};
     const int64_t wrows = (N - 1) * nb + 2 * N + 2;
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&Wbuf[1], sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb), s));
-    cudaStream_t P = nullptr;
-    int lo_prio = 0, hi_prio = 0;
-    cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio);
-    ABFT_CUDA_TRY(cudaStreamCreateWithPriority(&P, cudaStreamNonBlocking, hi_prio));
-    std::vector<cudaEvent_t> evs;
-    auto new_event = [&]() { cudaEvent_t e; cudaEventCreateWithFlags(&e, cudaEventDisableTiming); evs.push_back(e); return e; };
+    ThreadCache& tc = thread_cache();
+    cudaStream_t P = tc.P;
+    auto new_event = [&]() { return tc.sync.get(); };
     cudaEvent_t e0 = nullptr, e1 = nullptr;
-    if (rep) { cudaEventCreate(&e0); cudaEventCreate(&e1); cudaEventRecord(e0, s); }
-    Profiler prof; prof.on = o.profile != 0;
+    if (rep) { e0 = tc.timing.get(); e1 = tc.timing.get(); cudaEventRecord(e0, s); }
+    Profiler prof; prof.on = o.profile != 0; prof.pool = &tc.timing;
     const double lowerB = Bd * (Bd + 1) / 2;                 // elements of a tril tile
     launch_zero(B, B, w.Li, B, s);
     if (abft) {   // encode
@@ -478,13 +501,10 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         rc = finish_report(w, rep, s, &status);
         float ms = 0; cudaEventElapsedTime(&ms, e0, e1);
         rep->seconds = ms * 1e-3;
-        cudaEventDestroy(e0); cudaEventDestroy(e1);
     }
     if (prof.on) { cudaStreamSynchronize(s); prof.finish(); }
     cudaFreeAsync(Wbuf[1], s);
     work_free(w, s);
-    for (auto e : evs) cudaEventDestroy(e);
-    cudaStreamDestroy(P);
     if (rc) return rc;
     ABFT_CUDA_TRY(cudaGetLastError());
     return status;
