@@ -21,7 +21,7 @@ from __future__ import annotations
 import numpy as np
 
 __all__ = [
-    "splitmix64", "spd_matrix", "pascal_mod2", "pascal", "HOOK", "TARGET",
+    "splitmix64", "spd_matrix", "spd_diag", "pascal_mod2", "pascal", "HOOK", "TARGET",
     "inj_array", "INJ_DTYPE", "bit_mask", "c1_injections", "per_iteration_injections",
     "mixed_injections",
 ]
@@ -64,6 +64,16 @@ def spd_matrix(n: int, seed: int | None = None, dtype=np.float64) -> np.ndarray:
             A[:, c0:c1] = _u01(base + hi * nn + lo)
     A[np.arange(n), np.arange(n)] += float(n)
     return A
+
+
+def spd_diag(n: int, seed: int | None = None) -> np.ndarray:
+    """The diagonal of spd_matrix(n, seed) without forming the matrix (for full-size checks)."""
+    if seed is None:
+        seed = n
+    nn = np.uint64(n)
+    i = np.arange(n, dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        return _u01(np.uint64(seed % (1 << 64)) * nn * nn + i * nn + i) + float(n)
 
 
 def pascal_mod2(n: int) -> np.ndarray:

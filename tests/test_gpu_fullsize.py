@@ -1,0 +1,111 @@
+"""Full-size configurations on the GPU, in the launch configuration bench.py times (default
+options: Enhanced Online-ABFT, K = 1, look-ahead, fused V5): C4 n=32768 nb=512 and C5
+n=98304 nb=1024 on one B200. The oracle cannot factor these in seconds, so parity is checked on
+what it can compute one by one and on properties that hold at any size:
+  * the leading lead x lead block of L (it depends only on the leading block of A) vs the oracle,
+  * every injected error is reported exactly where the verification schedule predicts
+    (tests/_predict.py) and corrected,
+  * the backward error ||A X - L (L^T X)|| / ||A X|| on 8 random probes <= 10 n eps, with A
+    reassembled block by block from its untouched strict upper triangle and its known diagonal.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synthetic as syn
+from tests._predict import predict
+
+pytestmark = pytest.mark.gpu
+EPS = 2.0 ** -52
+
+
+def floor_rel(L, Lref, A):
+    s = np.sqrt(np.diag(A))[:, None]
+    return float(np.max(np.abs(np.tril(L) - np.tril(Lref)) / np.maximum(np.abs(np.tril(Lref)), 1e-3 * s)))
+
+
+def residual_probe(At, n, seed, nprobe=8, blk=4096):
+    """||A X - L L^T X|| / ||A X|| using only the stored upper triangle (never written) and diag."""
+    import torch
+    g = torch.Generator(device="cuda").manual_seed(1)
+    X = torch.randn(n, nprobe, dtype=torch.float64, device="cuda", generator=g)
+    d = torch.from_numpy(syn.spd_diag(n, seed)).cuda()
+    AX = torch.zeros_like(X)
+    LtX = torch.zeros_like(X)
+    for c0 in range(0, n, blk):
+        c1 = min(n, c0 + blk)
+        S = At[:, c0:c1]                              # column block of the stored matrix
+        # A[:, c0:c1]: rows < c0 from the upper triangle, diag block symmetric, rows >= c1 mirrored
+        Acol = torch.empty(n, c1 - c0, dtype=torch.float64, device="cuda")
+        Acol[:c0] = S[:c0]
+        D = torch.triu(S[c0:c1], 1)
+        Acol[c0:c1] = D + D.T + torch.diag(d[c0:c1])
+        Acol[c1:] = At[c0:c1, c1:].T
+        AX += Acol @ X[c0:c1]
+        Lcol = torch.tril(S, -c0)                     # rows >= col: lower part of the block column
+        LtX[c0:c1] = Lcol.T @ X
+        del Acol, Lcol, D
+    LLtX = torch.zeros_like(X)
+    for c0 in range(0, n, blk):
+        c1 = min(n, c0 + blk)
+        LLtX += torch.tril(At[:, c0:c1], -c0) @ LtX[c0:c1]
+    return ((AX - LLtX).norm() / AX.norm()).item()
+
+
+def run_full(P, n, nb, specs, lead):
+    import torch
+    At = torch.empty(n, n, dtype=torch.float64, device="cuda").T
+    assert P.abft_gen_spd(n, At) == 0
+    inj = syn.inj_array(specs)
+    st, rep = P.abft_potrf_ex(n, nb, At, inj=inj)
+    torch.cuda.synchronize()
+    assert st == 0
+    assert P.sorted_event_tuples(rep["events"]) == sorted(predict(s, n, nb) for s in specs)
+    Al = syn.spd_matrix(n)[:lead, :lead] if n <= 32768 else None
+    if Al is None:   # C5: the leading block of the A15 matrix, built directly
+        Al = np.empty((lead, lead), order="F")
+        nn = np.uint64(n)
+        r = np.arange(lead, dtype=np.uint64)
+        with np.errstate(over="ignore"):
+            hi, lo = np.maximum(r[:, None], r[None, :]), np.minimum(r[:, None], r[None, :])
+            Al[:, :] = (syn.splitmix64(np.uint64(n) * nn * nn + hi * nn + lo) >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+        Al[np.arange(lead), np.arange(lead)] += float(n)
+    ref = oracle.potrf(Al, nb, inj=syn.inj_array([s for s in specs if s["row"] < lead]))
+    Lg = At[:lead, :lead].cpu().numpy()
+    assert floor_rel(Lg, ref.L, Al) <= 1e-11
+    be = residual_probe(At, n, n)
+    assert be <= 10 * n * EPS, be
+    return rep
+
+
+@pytest.fixture(scope="module")
+def P():
+    import paper_conf_ipps_chenlc16_b200 as p
+    return p
+
+
+def test_c4_full_size_bench_configuration(P):
+    n, nb, lead = 32768, 512, 2048
+    specs = [dict(k=0, hook="REST", row=1500, col=700, bit=50),           # in the leading block
+             dict(k=1, hook="POTRF_OUT", row=600, col=520, bit=52),
+             dict(k=2, hook="TRSM_OUT", row=1900, col=1100, bit=48),
+             dict(k=5, hook="REST", row=30000, col=20000, bit=47),
+             dict(k=9, hook="UPDATE_OUT", row=32000, col=9000, bit=55),
+             dict(k=12, hook="REST", target="CHK", row=2 * 40 + 1, col=30 * nb + 7, bit=50),
+             dict(k=20, hook="TRSM_OUT", row=31000, col=20 * nb + 100, bit=53),
+             dict(k=40, hook="POTRF_OUT", row=40 * nb + 300, col=40 * nb + 2, bit=51),
+             dict(k=63, hook="REST", row=32767, col=32767, bit=50),
+             dict(k=64, hook="REST", row=20000, col=100, bit=52)]         # finished L -> V6
+    rep = run_full(P, n, nb, specs, lead)
+    assert rep["n_data"] + rep["n_chk2"] == len(specs)
+
+
+def test_c5_full_size_one_gpu(P):
+    n, nb, lead = 98304, 1024, 2048
+    specs = [dict(k=0, hook="REST", row=1800, col=900, bit=50),
+             dict(k=3, hook="UPDATE_OUT", row=90000, col=50000, bit=52),
+             dict(k=30, hook="TRSM_OUT", row=97000, col=30 * nb + 5, bit=50),
+             dict(k=50, hook="REST", target="CHK", row=2 * 80, col=60 * nb + 3, bit=50),
+             dict(k=96, hook="REST", row=98000, col=1000, bit=51)]
+    rep = run_full(P, n, nb, specs, lead)
+    assert rep["n_events"] == len(specs)
