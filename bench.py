@@ -246,6 +246,7 @@ def main():
         "whole_path_frac_of_fp64_peak": round(value / world / 1e3 / FP64_DMMA_PEAK_TFLOPS, 4),
         "abft_events": int(reps[-1]["n_events"]),
         "phases_ms_per_step": {k: round(v["ms"], 3) for k, v in prof.items()},
+        "library_device_ms": round(1e3 * sum(r["seconds"] for r in reps) / len(reps), 3),
     }
     line["clocks"] = clk.summary()
 

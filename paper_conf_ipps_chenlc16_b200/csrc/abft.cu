@@ -233,6 +233,13 @@ static ThreadCache& thread_cache() {
         int lo = 0, hi = 0;
         cudaDeviceGetStreamPriorityRange(&lo, &hi);
         cudaStreamCreateWithPriority(&g_tc.P, cudaStreamNonBlocking, hi);
+        // keep the workspace's pages mapped between calls: cudaMallocAsync / cudaFreeAsync then
+        // cost microseconds instead of re-mapping ~n*nb*8*4 bytes at every call
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            uint64_t keep = UINT64_MAX;
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+        }
         g_tc.device = dev;
     }
     g_tc.sync.reset(); g_tc.timing.reset();
