@@ -418,18 +418,20 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         for (const auto& sp : inj)
             if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && sp.col / nb >= jlo && sp.col / nb < jhi) inj_here = true;
         ColSumOut cso{w.cs, n, w.cs_nslab, jlo * B, jlo * B, B, 64, jlo * B};
-        const int fused = launch_gemm(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab,
-                                      s, 0, (can_fuse && !inj_here) ? &cso : nullptr);
-        prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd, 0);
+        int fused;
         if (abft) {
-            // checksum rows of tiles I >= jlo: chk[2I+t, cols] -= W_chk(I) W[c0:c0+nc]^T, I >= J
+            // checksum rows of tiles I >= jlo: chk[2I+t, cols] -= W_chk(I) W[c0:c0+nc]^T, I >= J,
+            // appended to the same launch as a second row segment
             const int64_t q0 = 2 * (jlo - k - 1);                       // first chk row of tile jlo in W
             const int64_t nq = 2 * (N - jlo);
-            t = prof.begin(s);
-            launch_gemm(nq, nc, B, W + mB + 2 + q0, ldw, W + c0, ldw, w.chk + jlo * B * w.ldc + 2 * jlo, w.ldc,
-                        -1.0, 1.0, true, 2, 0, B, 0, 0, ab, s);
+            fused = launch_update_with_chk(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, nq, W + mB + 2 + q0,
+                                           w.chk + jlo * B * w.ldc + 2 * jlo, w.ldc, B, ab, s,
+                                           (can_fuse && !inj_here) ? &cso : nullptr);
             const double mm = (double)(N - jlo), jj = (double)(jhi - jlo);
-            prof.end(t, PH_UPDC, s, 4.0 * Bd * Bd * (jj * mm - jj * (jj - 1) / 2), 0);
+            prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd + 4.0 * Bd * Bd * (jj * mm - jj * (jj - 1) / 2), 0);
+        } else {
+            fused = launch_gemm(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
+            prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd, 0);
         }
         if (fused == 1) slab_rows_used = cso.slab_rows;
         return fused == 1;
@@ -623,6 +625,7 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             launch_check(a, s);
         }
     }
+    int64_t dist_slab_rows = 64;
     for (int64_t k = 0; k < N; ++k) {
         const int owner = (int)(k % P);
         const int64_t m = N - k - 1, mB = m * B;
@@ -689,12 +692,15 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
                 double* W0 = q.w.W + (J - k - 1) * B;
                 double* C = q.A + t * B * q.lda + J * B;
                 ColSumOut cso{q.w.cs, q.ncl, q.w.cs_nslab, J * B, t * B, B, 64, J * B};
-                const int f = launch_gemm((N - J) * B, B, B, W0, ldw, W0, ldw, C, q.lda, -1.0, 1.0, true, 1, 0, 0, 0,
-                                          0, ab, s, 0, all_fused ? &cso : nullptr);
-                if (f != 1) all_fused = false;
+                int f;
                 if (abft)
-                    launch_gemm(2 * (N - J), B, B, q.w.W + mB + 2 + 2 * (J - k - 1), ldw, W0, ldw,
-                                q.w.chk + t * B * q.w.ldc + 2 * J, q.w.ldc, -1.0, 1.0, true, 2, 0, B, 0, 0, ab, s);
+                    f = launch_update_with_chk((N - J) * B, B, B, W0, ldw, W0, ldw, C, q.lda, 2 * (N - J),
+                                               q.w.W + mB + 2 + 2 * (J - k - 1), q.w.chk + t * B * q.w.ldc + 2 * J,
+                                               q.w.ldc, B, ab, s, all_fused ? &cso : nullptr);
+                else
+                    f = launch_gemm((N - J) * B, B, B, W0, ldw, W0, ldw, C, q.lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
+                if (f != 1) all_fused = false;
+                if (f == 1) dist_slab_rows = cso.slab_rows;
             }
             if (!abft) continue;
             dist_inject(inj, k, ABFT_HOOK_UPDATE_OUT, B, P, q, ldw, mB, s);
@@ -704,7 +710,7 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
                 if (all_fused) {
                     StageArgs d = a; d.kind = SK_TRAIL_DIAG;
                     StageArgs f = a; f.kind = SK_TRAIL_OFF;
-                    f.cs = q.w.cs; f.cs_ld = q.ncl; f.cs_nslab = q.w.cs_nslab; f.cs_slab_rows = 64;
+                    f.cs = q.w.cs; f.cs_ld = q.ncl; f.cs_nslab = q.w.cs_nslab; f.cs_slab_rows = dist_slab_rows;
                     launch_check_v5_fused(d, f, s);                                    // V5 (fused)
                 } else {
                     launch_check(a, s);                                                // V5

@@ -182,8 +182,8 @@ struct ColSumOut {
     double* p; int64_t ld, nslab;
     int64_t row0, col0;   // global row of C's row 0; partial-array column of C's column 0
     int64_t nb;
-    int64_t colg0;        // GLOBAL column of C's column 0 (block-diagonal test; = col0 on one GPU)
     int64_t slab_rows;    // rows per slab (set by the GEMM launcher: its warp-tile height)
+    int64_t colg0;        // GLOBAL column of C's column 0 (block-diagonal test; = col0 on one GPU)
 };
 }  // namespace abft
 
@@ -219,3 +219,8 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
                 int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
                 int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
                 cudaStream_t s, int force_tile = 0, abft::ColSumOut* cs = nullptr);
+// The trailing update with the checksum rows as a second row segment of the same launch.
+int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
+                           int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
+                           int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s,
+                           abft::ColSumOut* cs);

@@ -25,6 +25,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
+#include <cstdio>
 
 namespace abft {
 
@@ -43,6 +44,10 @@ struct GemmArgs {
     const int32_t* abort;
     int32_t vecA, vecB;             // 16-byte cp.async allowed for A / B
     ColSumOut cs;                   // fused V5 partials (cs.p == nullptr: off)
+    // optional second row segment (ws kernel only): the checksum rows appended to the update as
+    // extra GEMM rows. Rows [0, M2) of A2 (lda) update C2 (ldc2) under MASK_CHK with
+    // q_tile0 = c_tile0 = 0; their tiles follow the first segment's tiles.
+    int64_t M2; const double* A2; double* C2; int64_t ldc2;
 };
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
@@ -386,14 +391,27 @@ __device__ __forceinline__ int64_t group_col_prefix(int64_t u, int64_t a0, int64
 
 constexpr int kWsGroup = 8;   // tile rows per L2 group: A rows of a group stay in L2, W streams once per group
 
-// tile index -> (m0, n0) for the three masks; returns false for tiles with nothing to write.
-// Tiles are enumerated group by group (kWsGroup tile rows), column-major inside a group, so the
-// CTAs running at the same time share operand tiles in L2.
+// One output tile of the warp-specialised kernel: which row segment, where its operands live.
+struct WsTile {
+    int64_t m0, n0;         // m0 relative to its segment
+    bool seg2;              // checksum-row segment: A2 / C2 / ldc2 / M2, MASK_CHK with tile offsets 0
+};
+
+// tile index -> tile; returns false for tiles with nothing to write. Segment-1 tiles are
+// enumerated group by group (kWsGroup tile rows), column-major inside a group, so the CTAs
+// running at the same time share operand tiles in L2; the checksum-row segment follows.
 template <int BM, int BN>
-__device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t& m0, int64_t& n0) {
+__device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t n1tiles, WsTile& T) {
     constexpr int R = BM / BN;
     const int64_t TN = g.tiles_n, TM = (g.M + BM - 1) / BM;
     int64_t tm, tn;
+    if (idx >= n1tiles) {   // second segment: checksum rows, rectangular, row-major
+        const int64_t e = idx - n1tiles;
+        tm = e / TN; tn = e % TN;
+        T.m0 = tm * BM; T.n0 = tn * BN; T.seg2 = true;
+        const int64_t qmax = min(g.M2, T.m0 + BM) - 1;
+        return qmax / 2 >= T.n0 / g.nb;
+    }
     if (g.mask == MASK_LOWER) {
         // group q: the last q with lower_prefix(q G) <= idx
         int64_t lo = 0, hi = (TM + kWsGroup - 1) / kWsGroup;
@@ -417,16 +435,16 @@ __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t&
         const int64_t e = idx - a0 * TN;
         tn = e / Gp; tm = a0 + e % Gp;
     }
-    m0 = tm * BM; n0 = tn * BN;
+    T.m0 = tm * BM; T.n0 = tn * BN; T.seg2 = false;
     if (g.mask == MASK_CHK) {
-        const int64_t qmax = min(g.M, m0 + BM) - 1;
-        if (g.q_tile0 + qmax / 2 < g.c_tile0 + n0 / g.nb) return false;
+        const int64_t qmax = min(g.M, T.m0 + BM) - 1;
+        if (g.q_tile0 + qmax / 2 < g.c_tile0 + T.n0 / g.nb) return false;
     }
     return true;
 }
 
 template <class C_>
-__global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, int64_t ntiles) {
+__global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, int64_t ntiles, int64_t n1tiles) {
     constexpr int BM = C_::BM, BN = C_::BN, BK = C_::BK, WM = C_::WM, WN = C_::WN, STAGES = C_::STAGES;
     if (*(volatile const int32_t*)g.abort) return;
     extern __shared__ __align__(16) double smem[];
@@ -447,14 +465,19 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
         if (warp != C_::CONSUMERS) return;
         uint32_t it = 0;
         for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-            int64_t m0, n0;
-            if (!ws_tile<BM, BN>(g, t, m0, n0)) continue;
+            WsTile T;
+            if (!ws_tile<BM, BN>(g, t, n1tiles, T)) continue;
+            const int64_t m0 = T.m0, n0 = T.n0;
             const int64_t ke = (g.krange == KR_LE_N) ? min(g.K, n0 + BN) : g.K;
             const int kt_n = (int)(ke / BK);
-            const uint32_t rowsA = (uint32_t)(g.M - m0 < BM ? g.M - m0 : BM), rowsB = (uint32_t)(g.N - n0 < BN ? g.N - n0 : BN);
+            const int64_t Ms = T.seg2 ? g.M2 : g.M;
+            const double* Ap = T.seg2 ? g.A2 : g.A;
+            double* Cp = T.seg2 ? g.C2 : g.C;
+            const int64_t ldcp = T.seg2 ? g.ldc2 : g.ldc;
+            const uint32_t rowsA = (uint32_t)(Ms - m0 < BM ? Ms - m0 : BM), rowsB = (uint32_t)(g.N - n0 < BN ? g.N - n0 : BN);
             // warm L2 with the C columns of this tile (they are read at the tile's start)
             if (g.beta != 0.0) {
-                for (int c = lane; c < (int)rowsB; c += 32) prefetch_l2(g.C + (n0 + c) * g.ldc + m0, rowsA * 8);
+                for (int c = lane; c < (int)rowsB; c += 32) prefetch_l2(Cp + (n0 + c) * ldcp + m0, rowsA * 8);
             }
             for (int kt = 0; kt < kt_n; ++kt, ++it) {
                 const int st = it % STAGES;
@@ -466,7 +489,7 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
                 __syncwarp();
                 const int64_t k0 = (int64_t)kt * BK;
                 for (int kk = lane; kk < BK; kk += 32) {
-                    bulk_g2s(sA + st * C_::SA + kk * C_::PA, g.A + (k0 + kk) * g.lda + m0, rowsA * 8, &full[st]);
+                    bulk_g2s(sA + st * C_::SA + kk * C_::PA, Ap + (k0 + kk) * g.lda + m0, rowsA * 8, &full[st]);
                     bulk_g2s(sB + st * C_::SB + kk * C_::PB, g.B + (k0 + kk) * g.ldb + n0, rowsB * 8, &full[st]);
                 }
             }
@@ -480,10 +503,32 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
     const double ab = g.alpha * g.beta, alpha = g.alpha;
     uint32_t it = 0;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        int64_t m0, n0;
-        if (!ws_tile<BM, BN>(g, t, m0, n0)) continue;
+        WsTile T;
+        if (!ws_tile<BM, BN>(g, t, n1tiles, T)) continue;
+        const int64_t m0 = T.m0, n0 = T.n0;
         const int64_t ke = (g.krange == KR_LE_N) ? min(g.K, n0 + BN) : g.K;
         const int kt_n = (int)(ke / BK);
+        const bool seg2 = T.seg2;
+        // ownership of element (r, c): r < Mlim and r >= rmin(c), rmin precomputed per owned column
+        // (no per-element 64-bit division: the epilogue must stay short and I-cache friendly)
+        const int64_t Mlim = seg2 ? g.M2 : g.M;
+        int64_t rmin[C_::FN][2];
+#pragma unroll
+        for (int j = 0; j < C_::FN; ++j)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
+                int64_t v;
+                if (c >= g.N) v = INT64_MAX;
+                else if (seg2) v = 2 * (c / g.nb);                                   // q/2 >= c/nb
+                else if (g.mask == MASK_LOWER) v = c;                                 // r >= c
+                else if (g.mask == MASK_CHK) v = 2 * (g.c_tile0 + c / g.nb - g.q_tile0);
+                else v = 0;
+                rmin[j][h] = v;
+            }
+        auto owns = [&](int64_t r, int j, int h) { return r < Mlim && r >= rmin[j][h]; };
+        double* Cp = seg2 ? g.C2 : g.C;
+        const int64_t ldcp = seg2 ? g.ldc2 : g.ldc;
         double acc[C_::FM][C_::FN][2];
         // acc = alpha*beta*C on the elements this tile owns (masked / out-of-range: 0)
 #pragma unroll
@@ -494,10 +539,7 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
 #pragma unroll
                 for (int h = 0; h < 2; ++h) {
                     const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
-                    bool ok = r < g.M && c < g.N;
-                    if (g.mask == MASK_LOWER) ok = ok && r >= c;
-                    else if (g.mask == MASK_CHK) ok = ok && (g.q_tile0 + r / 2) >= (g.c_tile0 + c / g.nb);
-                    acc[i][j][h] = (ok && ab != 0.0) ? ab * g.C[c * g.ldc + r] : 0.0;
+                    acc[i][j][h] = (owns(r, j, h) && ab != 0.0) ? ab * Cp[c * ldcp + r] : 0.0;
                 }
         }
         for (int kt = 0; kt < kt_n; ++kt, ++it) {
@@ -529,43 +571,42 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
 #pragma unroll
                 for (int h = 0; h < 2; ++h) {
                     const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
-                    bool ok = r < g.M && c < g.N;
-                    if (g.mask == MASK_LOWER) ok = ok && r >= c;
-                    else if (g.mask == MASK_CHK) ok = ok && (g.q_tile0 + r / 2) >= (g.c_tile0 + c / g.nb);
                     acc[i][j][h] = alpha * acc[i][j][h];
-                    if (ok) g.C[c * g.ldc + r] = acc[i][j][h];
+                    if (owns(r, j, h)) Cp[c * ldcp + r] = acc[i][j][h];
                 }
         }
         // fused V5 recalculation: per-column v1/v2 partial sums of the
         // updated values over each warp's 64 rows (slab = global_row / 64), for tiles off the
-        // block diagonal (diagonal blocks are checked as sym(tril) by a re-read).
-        if (g.cs.p != nullptr) {
+        // block diagonal (diagonal blocks are checked as sym(tril) by a re-read). Data rows only.
+        if (g.cs.p != nullptr && t < n1tiles) {
             const int64_t gr0 = g.cs.row0 + m0 + wm * WM, gc0 = g.cs.col0 + n0;
-            if (gr0 / g.cs.nb != (g.cs.colg0 + n0) / g.cs.nb) {
-                const int64_t wbase = gr0 % g.cs.nb + fr + 1;   // weight (1-based) of row i = 0
+            // warp-uniform; the shuffles below stay outside any branch so that they compile to
+            // plain SHFLs (inside a possibly divergent branch they become WARPSYNC collectives)
+            const bool offdiag = gr0 / g.cs.nb != (g.cs.colg0 + n0) / g.cs.nb;
+            const int64_t wbase = gr0 % g.cs.nb + fr + 1;   // weight (1-based) of row i = 0
+            const int64_t slab = gr0 / g.cs.slab_rows;
+            __syncwarp();
 #pragma unroll
-                for (int j = 0; j < C_::FN; ++j)
+            for (int j = 0; j < C_::FN; ++j)
 #pragma unroll
-                    for (int h = 0; h < 2; ++h) {
-                        double s1 = 0.0, s2 = 0.0;
+                for (int h = 0; h < 2; ++h) {
+                    double s1 = 0.0, s2 = 0.0;
 #pragma unroll
-                        for (int i = 0; i < C_::FM; ++i) {
-                            s1 += acc[i][j][h];
-                            s2 = fma((double)(wbase + i * 8), acc[i][j][h], s2);
-                        }
-#pragma unroll
-                        for (int o = 4; o < 32; o <<= 1) {
-                            s1 += __shfl_xor_sync(0xffffffffu, s1, o);
-                            s2 += __shfl_xor_sync(0xffffffffu, s2, o);
-                        }
-                        if (fr == 0) {
-                            const int64_t slab = gr0 / g.cs.slab_rows;
-                            const int64_t gc = gc0 + wn * WN + j * 8 + fc * 2 + h;
-                            g.cs.p[slab * g.cs.ld + gc] = s1;
-                            g.cs.p[(g.cs.nslab + slab) * g.cs.ld + gc] = s2;
-                        }
+                    for (int i = 0; i < C_::FM; ++i) {
+                        s1 += acc[i][j][h];
+                        s2 = fma((double)(wbase + i * 8), acc[i][j][h], s2);
                     }
-            }
+#pragma unroll
+                    for (int o = 4; o < 32; o <<= 1) {
+                        s1 += __shfl_xor_sync(0xffffffffu, s1, o);
+                        s2 += __shfl_xor_sync(0xffffffffu, s2, o);
+                    }
+                    if (offdiag && fr == 0) {
+                        const int64_t gc = gc0 + wn * WN + j * 8 + fc * 2 + h;
+                        g.cs.p[slab * g.cs.ld + gc] = s1;
+                        g.cs.p[(g.cs.nslab + slab) * g.cs.ld + gc] = s2;
+                    }
+                }
         }
     }
 }
@@ -579,14 +620,15 @@ static int run_ws(GemmArgs g, cudaStream_t s) {
     }
     const int64_t tm = (g.M + C_::BM - 1) / C_::BM, tn = (g.N + C_::BN - 1) / C_::BN;
     g.tiles_n = tn;
-    const int64_t ntiles = (g.mask == MASK_LOWER) ? lower_prefix<C_::BM / C_::BN>(tm, tn) : tm * tn;
+    const int64_t n1 = (g.mask == MASK_LOWER) ? lower_prefix<C_::BM / C_::BN>(tm, tn) : tm * tn;
+    const int64_t ntiles = n1 + (g.M2 > 0 ? ((g.M2 + C_::BM - 1) / C_::BM) * tn : 0);
     if (ntiles <= 0) return 0;
     // tiles per CTA: 1 lets the block scheduler interleave the high-priority look-ahead stream's
     // kernels as CTAs retire; a fully persistent grid would starve that stream.
     static int64_t tpc = -1;
     if (tpc < 0) { const char* e = getenv("ABFT_WS_TPC"); tpc = e ? std::max(1, atoi(e)) : 1; }
     const int64_t grid = std::max<int64_t>(1, (ntiles + tpc - 1) / tpc);
-    k_gemm_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles);
+    k_gemm_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
     abft_count_launch();
     return 0;
 }
@@ -632,6 +674,7 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
     g.alpha = alpha; g.beta = beta; g.mask = mask; g.krange = krange; g.nb = nb;
     g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
     g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
+    g.M2 = 0; g.A2 = nullptr; g.C2 = nullptr; g.ldc2 = 1;
     g.vecA = aligned16(A) && (lda % 2 == 0);
     g.vecB = aligned16(B) && (ldb % 2 == 0);
     auto tiles = [&](int64_t t) {
@@ -666,4 +709,36 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
         if (tile == 64) return run_cfg<64, 64, 16, 32, 32, 4, false>(g, s);
         return run_cfg<32, 32, 16, 16, 16, 4, false>(g, s);
     }
+}
+
+// Trailing update with the checksum rows appended as a second row segment of the same launch
+// (chk(A') = chk(A) - chk(LC) LC^T as extra GEMM rows). Falls back to two
+// launches when the warp-specialised kernel cannot take the shapes. Returns 1 if the fused V5
+// partials were written.
+int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
+                           int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
+                           int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s, ColSumOut* cs) {
+    const bool ok = M > 0 && N > 0 && (M % 2 == 0) && (N % 2 == 0) && (M2 % 2 == 0) && (K % WsCfg::BK == 0) &&
+                    aligned16(A) && aligned16(B) && aligned16(A2) && lda % 2 == 0 && ldb % 2 == 0 && N <= M &&
+                    M % WsCfg::BM == 0 && getenv("ABFT_GEMM_VARIANT") == nullptr;
+    if (!ok) {
+        const int f = launch_gemm(M, N, K, A, lda, B, ldb, C, ldc, -1.0, 1.0, true, MASK_LOWER, KR_FULL, 0, 0, 0,
+                                  abort_flag, s, 0, cs);
+        if (M2 > 0)
+            launch_gemm(M2, N, K, A2, lda, B, ldb, C2, ldc2, -1.0, 1.0, true, MASK_CHK, KR_FULL, nb, 0, 0, abort_flag, s);
+        return f;
+    }
+    GemmArgs g;
+    g.M = M; g.N = N; g.K = K; g.A = A; g.lda = lda; g.B = B; g.ldb = ldb; g.C = C; g.ldc = ldc;
+    g.alpha = -1.0; g.beta = 1.0; g.mask = MASK_LOWER; g.krange = KR_FULL; g.nb = nb;
+    g.q_tile0 = 0; g.c_tile0 = 0; g.tiles_n = 1; g.abort = abort_flag; g.vecA = 1; g.vecB = 1;
+    g.cs = ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
+    int fused = 0;
+    if (cs && cs->nb % WsCfg::BM == 0 && cs->row0 % WsCfg::BM == 0 && cs->colg0 % WsCfg::BN == 0) {
+        g.cs = *cs; fused = 1;
+    }
+    g.M2 = M2; g.A2 = A2; g.C2 = C2; g.ldc2 = ldc2;
+    run_ws_any(g, s);
+    if (fused) cs->slab_rows = ws_slab_rows();
+    return fused;
 }
