@@ -249,6 +249,17 @@ def main():
         "library_device_ms": round(1e3 * sum(r["seconds"] for r in reps) / len(reps), 3),
     }
     line["clocks"] = clk.summary()
+    # bandwidth-bound check kernels: algorithmic bytes / device time (events around each phase)
+    hbm_peak = measured_peaks().get("hbm_gbs", HBM_PEAK_FALLBACK)
+    hbm = {}
+    for ph in ("encode", "v6", "v1v2", "v4", "v5", "writeback"):
+        v = prof.get(ph)
+        if v and v["ms"] > 0 and v["bytes"] > 0:
+            gbs = v["bytes"] / (v["ms"] * 1e-3) / 1e9
+            hbm[ph] = {"GB/s": round(gbs, 1), "frac": round(gbs / hbm_peak, 3)}
+    line["hbm_kernels"] = {"peak_GBps": hbm_peak, "peak_source": "MEASURED_PEAKS.json hbm_gbs", **hbm,
+                           "note": "v1v2/v4/writeback run on the look-ahead stream concurrently with the "
+                                   "update GEMM, so their device time includes waiting for SM slots"}
 
     if not args.no_extras and world == 1:   # extras are single-GPU runs (no collectives)
         # ABFT off: the same kernels without checksum work
@@ -305,6 +316,33 @@ def main():
                                     "sample": f"oracle potrf n={args.oracle_n} nb={nb} (same nb, "
                                               f"{(args.oracle_n / n) ** 3:.4f} of the workload's flops), "
                                               f"fault-free, ABFT on, {dt:.1f} s"}
+        # the other BASELINE configurations, one GPU, fault-free, ABFT on (median of the steps)
+        others = {}
+        for (cn, cnb, cst) in ((4096, 256, 5), (16384, 512, 5), (98304, 1024, 1)):
+            try:
+                del A0, A
+            except NameError:
+                pass
+            torch.cuda.empty_cache()
+            Ac = torch.empty(cn, cn, dtype=torch.float64, device="cuda").T
+            Ac0 = torch.empty_like(Ac.T).T
+            P.abft_gen_spd(cn, Ac0)
+            ts = []
+            for i in range(1 + cst):
+                Ac.copy_(Ac0)
+                torch.cuda.synchronize()
+                e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+                e0.record(stream)
+                st, _ = P.abft_potrf_ex(cn, cnb, Ac, report=True, cap=16)
+                e1.record(stream); e1.synchronize()
+                assert st == 0
+                if i >= 1:
+                    ts.append(e0.elapsed_time(e1))
+            tm = statistics.median(ts)
+            others[f"n{cn}_nb{cnb}"] = {"value": round(cn ** 3 / 3 / (tm * 1e-3) / 1e9, 1), "unit": "GFLOP/s",
+                                        "ms": round(tm, 3), "steps": cst}
+            del Ac, Ac0
+        line["other_configs"] = others
         line["paper_context"] = {"Bulldozer64_K40c_n30720_nb512": "1092.4 GFLOP/s (Enhanced, no error, PAPER.md:374)",
                                  "Tardis_M2075_n20480_nb256": "268.7 GFLOP/s (PAPER.md:366)"}
     if rank == 0:
