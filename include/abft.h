@@ -189,6 +189,11 @@ int abft_dev_gemm_nt(int64_t M, int64_t N, int64_t K, const double* A, int64_t l
                      int64_t ldb, double* C, int64_t ldc, double alpha, double beta, int lower,
                      abft_stream_t stream);
 
+/* Diagnostics: the diagonal-block factorisation alone (POTRF + inverse of an nb x nb SPD block):
+ * A (lower, overwritten by L), Li (nb x nb, ld nb) receives inv(L). Returns ABFT_NOT_SPD (2) on a
+ * non-positive pivot. Synchronises `stream`. */
+int abft_dev_chol_inv(int64_t nb, double* A, int64_t lda, double* Li, abft_stream_t stream);
+
 /* Diagnostics: kernel launches issued by the last call on this thread, a static version string,
  * and the text of the last CUDA error seen on this thread (empty if none). */
 int64_t abft_last_launch_count(void);

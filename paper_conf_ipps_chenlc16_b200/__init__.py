@@ -76,6 +76,8 @@ _lib.abft_comm_destroy.argtypes = [_vp]
 _lib.abft_potrf_dist.argtypes = [_i64, _i64, _vp, _i64, _vp, _i32, _i32, _vp, _vp, _vp, _vp]
 _lib.abft_potrf_dist_sim.argtypes = [_i64, _i64, _i32, _vp, _i64, _vp, _vp, _vp, _vp]
 _lib.abft_potrf_dist_sim.restype = _i32
+_lib.abft_dev_chol_inv.argtypes = [_i64, _vp, _i64, _vp, _vp]
+_lib.abft_dev_chol_inv.restype = _i32
 _lib.abft_dev_gemm_nt.argtypes = [_i64, _i64, _i64, _vp, _i64, _vp, _i64, _vp, _i64, _dbl, _dbl, _i32, _vp]
 _lib.abft_dev_gemm_nt.restype = _i32
 _lib.abft_last_launch_count.restype = _i64
@@ -90,7 +92,7 @@ for _f in ("abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_po
 
 EXPORTS = ["abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
            "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist",
-           "abft_last_launch_count", "abft_version", "abft_last_error", "abft_last_profile", "abft_dev_gemm_nt",
+           "abft_last_launch_count", "abft_version", "abft_last_error", "abft_last_profile", "abft_dev_gemm_nt", "abft_dev_chol_inv",
            "abft_potrf_dist_sim",
            "abft_phase_name"]
 
@@ -307,6 +309,13 @@ def block_cyclic_join(locals_, nb, n):
         for t, J in enumerate(range(r, n // nb, P)):
             A[:, J * nb:(J + 1) * nb] = L[:, t * nb:(t + 1) * nb]
     return A
+
+
+def abft_dev_chol_inv(nb, A, Li, stream=None):
+    """Diagnostics: POTRF + inverse of one nb x nb block (A lower -> L, Li <- inv(L))."""
+    pa, la = _dev(A)
+    pl, _ = _dev(Li)
+    return _lib.abft_dev_chol_inv(nb, pa, la or nb, pl, _stream(stream))
 
 
 def abft_last_launch_count():

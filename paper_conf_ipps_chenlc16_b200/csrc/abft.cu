@@ -945,6 +945,23 @@ extern "C" int abft_dev_gemm_nt(int64_t M, int64_t N, int64_t K, const double* A
     return 0;
 }
 
+extern "C" int abft_dev_chol_inv(int64_t nb, double* A, int64_t lda, double* Li, abft_stream_t stream) {
+    g_launches = 0;
+    if (nb < 1 || !A || !Li || lda < nb) return -1;
+    cudaStream_t s = (cudaStream_t)stream;
+    DevState* st = nullptr;
+    double* tmp = nullptr;
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&st, sizeof(DevState), s));
+    ABFT_CUDA_TRY(cudaMemsetAsync(st, 0, offsetof(DevState, fl), s));
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&tmp, sizeof(double) * (size_t)(((nb + 1) / 2 + 64) * ((nb + 1) / 2 + 64)), s));
+    launch_chol_inv(A, lda, Li, nb, 0, tmp, st, s);
+    int32_t status = 0;
+    ABFT_CUDA_TRY(cudaMemcpyAsync(&status, &st->status, sizeof status, cudaMemcpyDeviceToHost, s));
+    cudaFreeAsync(tmp, s); cudaFreeAsync(st, s);
+    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+    return status;
+}
+
 extern "C" int abft_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, abft_stream_t stream) {
     g_launches = 0;
     if (n < 0) return -1;
