@@ -277,6 +277,26 @@ def main():
                             "injections": len(specs), "events": int(r0["n_events"]),
                             "corrected": int(r0["n_data"] + r0["n_nonfinite"] + r0["n_chk1"] + r0["n_chk2"]),
                             "uncorrectable": int(r0["n_uncorrectable"])}
+        # Table VII/VIII analog on B200 (NEXT-2): the three schemes x {no error, computation error,
+        # memory error between verification and access}; Online/Offline re-do the factorisation
+        # when an error propagated
+        B_ = nb
+        faults = {"no_error": [], "computation_error": [dict(k=2, hook="UPDATE_OUT", row=n - 700, col=n // 2, bit=50)],
+                  "memory_error": [dict(k=3, hook="REST", row=3 * B_ + 100, col=3 * B_ + 50, bit=50)]}
+        table = {}
+        for mode in ("enhanced", "online", "offline"):
+            table[mode] = {}
+            for fname, specs in faults.items():
+                injf = syn.inj_array(specs) if specs else None
+                tf, rf = run_steps(P.options(mode=mode), inj=injf, steps=1, warmup=1, check=True)
+                table[mode][fname] = {"ms": round(tf[0], 2), "value": round(flops / (tf[0] * 1e-3) / 1e9, 1),
+                                      "reruns": int(rf[0]["reruns"]), "events": int(rf[0]["n_events"])}
+        table["paper_context_seconds"] = {
+            "Tardis_M2075_n20480": {"enhanced": [10.6572, 10.6614, 10.6678], "online": [10.5067, 10.5244, 22.625],
+                                    "offline": [10.4489, 21.3942, 21.2631], "src": "PAPER.md:366-368"},
+            "Bulldozer64_K40c_n30720": {"enhanced": [8.84598, 8.92538, 8.914928], "online": [8.64649, 8.69622, 21.4162],
+                                        "offline": [8.64265, 21.4472, 21.3511], "src": "PAPER.md:374-377"}}
+        line["schemes_table"] = table
         # e2e through the host C-ABI entry (pinned host memory, H2D + D2H inside the timing)
         del A
         torch.cuda.empty_cache()

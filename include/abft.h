@@ -89,6 +89,7 @@ typedef struct abft_report {
     int64_t cap;        /* capacity of `events` (set by the caller)                          */
     abft_event_t* events; /* HOST array owned by the caller, sorted by (k, check, J, I, col, row) */
     double seconds;     /* device time of the call (CUDA events on `stream`)                 */
+    int64_t reruns;     /* Online / Offline schemes: re-executions after an uncorrectable error */
 } abft_report_t;
 
 typedef struct abft_options {
@@ -98,7 +99,19 @@ typedef struct abft_options {
     double c_tau;         /* threshold constant C_tau of reading A4 (default 64)               */
     int32_t lookahead;    /* reserved (0/1)                                                    */
     int32_t profile;      /* 1: time every phase with CUDA events on `stream` (abft_last_profile) */
+    int32_t mode;         /* ABFT_MODE_ENHANCED (default), ABFT_MODE_ONLINE or ABFT_MODE_OFFLINE  */
+    int32_t pad;
 } abft_options_t;
+
+/* Schemes (§II.B, §III; Table VII/VIII compare them):
+ *  ENHANCED  verify every block before it is read (V1..V6) — errors are corrected in place.
+ *  ONLINE    verify each operation's result after it (V3, V4, V5) + a final sweep (V6): computing
+ *            errors are corrected; a storage error between a verification and the next read
+ *            propagates, and the call re-runs the factorisation once from a saved copy of A.
+ *  OFFLINE   checksums carried through, verified only at the end (V6); any detection re-runs.  */
+#define ABFT_MODE_ENHANCED 0
+#define ABFT_MODE_ONLINE 1
+#define ABFT_MODE_OFFLINE 2
 
 /* Per-phase device time of the last abft_potrf* call on this thread with options.profile = 1.
  * Phases: 0 encode, 1 V1/V2, 2 POTRF+inverse, 3 TRSM (+Alg. 2 rows), 4 V3, 5 V4, 6 panel

@@ -62,6 +62,10 @@ def lib():
         _lib.oracle_potrf.argtypes = [i64, i64, vp, i64, vp, i64, i32, i32, ctypes.c_double, i32,
                                       vp, i64, ctypes.POINTER(i64), ctypes.POINTER(i64), vp, vp, vp]
         _lib.oracle_potrf.restype = i32
+        _lib.oracle_potrf_mode.argtypes = [i64, i64, vp, i64, vp, i64, i32, i32, ctypes.c_double, i32, i32,
+                                           vp, i64, ctypes.POINTER(i64), ctypes.POINTER(i64), vp, vp, vp,
+                                           ctypes.POINTER(i32)]
+        _lib.oracle_potrf_mode.restype = i32
         _lib.oracle_encode.argtypes = [i64, i64, vp, i64, vp, i64, vp]
         _lib.oracle_encode.restype = i32
         _lib.oracle_verify.argtypes = [i64, i64, vp, i64, vp, i64, vp, i32, i32, ctypes.c_double,
@@ -96,9 +100,14 @@ def sorted_events(ev):
     return sorted(keys)
 
 
-def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, inplace=False):
-    """Enhanced Online-ABFT Cholesky of A (lower), n % nb == 0. Returns Result with L in the
-    lower triangle (upper triangle untouched), status (0/1/2), LAPACK info, sorted events."""
+MODE = {"enhanced": 0, "online": 1, "offline": 2}
+
+
+def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, inplace=False, mode="enhanced"):
+    """ABFT Cholesky of A (lower), n % nb == 0. mode: "enhanced" (the paper's scheme, default),
+    "online" or "offline" (its comparison schemes, which re-run once on an uncorrectable error).
+    Returns Result with L in the lower triangle (upper triangle untouched), status (0/1/2),
+    LAPACK info, sorted events, reruns."""
     L = _as_f(A)
     if not inplace:
         L = L.copy(order="F")
@@ -114,14 +123,18 @@ def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, in
     N = n // nb if nb > 0 else 0
     chk = np.zeros((max(2 * N, 1), n), dtype=np.float64, order="F")
     scl = np.zeros(n + 2 * N, dtype=np.float64)
-    st = lib().oracle_potrf(n, nb, _ptr(L), max(n, 1), _ptr(inj_arr), ninj, nranks, K, c_tau, int(abft),
-                            _ptr(ev), cap, ctypes.byref(nev), ctypes.byref(info), _ptr(cnt), _ptr(chk),
-                            _ptr(scl))
+    reruns = ctypes.c_int(0)
+    st = lib().oracle_potrf_mode(n, nb, _ptr(L), max(n, 1), _ptr(inj_arr), ninj, nranks, K, c_tau, int(abft),
+                                 MODE[mode] if isinstance(mode, str) else int(mode), _ptr(ev), cap,
+                                 ctypes.byref(nev), ctypes.byref(info), _ptr(cnt), _ptr(chk), _ptr(scl),
+                                 ctypes.byref(reruns))
     if st < 0:
         raise ValueError(f"oracle_potrf: invalid argument {-st}")
     ev = ev[: min(nev.value, cap)]
     order = np.lexsort((ev["row"], ev["col"], ev["tile_i"], ev["tile_j"], ev["check"], ev["k"]))
-    return Result(L, st, info.value, ev[order], cnt[0], chk, scl)
+    res = Result(L, st, info.value, ev[order], cnt[0], chk, scl)
+    res.reruns = reruns.value
+    return res
 
 
 def encode(A, nb):

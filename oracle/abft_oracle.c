@@ -62,6 +62,7 @@ typedef struct {
     double *A, *chk, *s, *S1, *S2;
     double c_tau, rho;
     int nranks, K, correct;
+    int mode;                      /* 0 Enhanced Online-ABFT, 1 Online-ABFT, 2 Offline-ABFT */
     const oinj_t* inj; int64_t ninj;
     oevent_t* ev; int64_t cap, nev;
     int status; int64_t info;
@@ -375,20 +376,17 @@ static int run_checks_column(octx_t* x, int64_t k, int factored, int V_diag, int
     return 0;
 }
 
-int oracle_potrf(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
-                 int nranks, int K, double c_tau, int abft, oevent_t* ev, int64_t cap, int64_t* nev,
-                 int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out) {
-    if (n < 0) return -1;
-    if (nb < 1) return -2;
-    if (n % nb) return -2;                          /* [A20] */
-    if (lda < (n > 1 ? n : 1)) return -4;
-    if (nranks < 1) nranks = 1;
-    if (K < 1) K = 1;
+/* One factorisation. Which checks run depends on the scheme (§II.B, §III):
+ *   mode 0 Enhanced Online-ABFT: V1..V6 (verify before every read)
+ *   mode 1 Online-ABFT: verify each operation's result after it: V3, V4, V5, + final V6
+ *   mode 2 Offline-ABFT: checksums carried, verified once at the end: V6 only        */
+static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
+                      int nranks, int K, double c_tau, int abft, int mode, oevent_t* ev, int64_t cap,
+                      int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out) {
     octx_t X_; octx_t* x = &X_;
     memset(x, 0, sizeof *x);
-    ocount_t dummy; memset(&dummy, 0, sizeof dummy);
-    x->cnt = cnt ? cnt : &dummy;
-    memset(x->cnt, 0, sizeof(ocount_t));
+    x->cnt = cnt;
+    x->mode = mode;
     x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = 2 * x->N > 0 ? 2 * x->N : 1;
     x->A = A; x->c_tau = c_tau > 0 ? c_tau : 64.0; x->rho = 0x1p-30;   /* [A4, A6] */
     x->nranks = nranks; x->K = K; x->correct = 1;
@@ -410,25 +408,25 @@ int oracle_potrf(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* in
         const int owner = (int)(k % nranks);
         if (abft) {
             inject(x, (int)k, O_HOOK_REST, 0, x->A, lda, x->chk, x->ldc);
-            if (run_checks_column(x, k, 0, O_V1, O_V2, 1)) break;          /* V1, V2 */
+            if (mode == 0 && run_checks_column(x, k, 0, O_V1, O_V2, 1)) break;   /* V1, V2 */
         }
         if (potrf_tile(x, k)) break;
         if (abft) {
             inject(x, (int)k, O_HOOK_POTRF_OUT, 0, x->A, lda, x->chk, x->ldc);
             tview_t v = gview(x, k, k, 1);
-            if (check_tile(x, &v, (int)k, O_V3, 0)) break;                   /* V3 */
+            if (mode != 2 && check_tile(x, &v, (int)k, O_V3, 0)) break;      /* V3 */
         }
         trsm_panel(x, k);
         if (abft) {
             inject(x, (int)k, O_HOOK_TRSM_OUT, 0, x->A, lda, x->chk, x->ldc);
-            if (run_checks_column(x, k, 1, 0, O_V4, 0)) break;              /* V4 */
+            if (mode != 2 && run_checks_column(x, k, 1, 0, O_V4, 0)) break;   /* V4 */
         }
         const int64_t m = N - k - 1;
         for (int r = 0; r < nranks; ++r) {
             pan[r].L = x->A + k * B * lda + (k + 1) * B; pan[r].ldl = lda;
             pan[r].C = x->chk + k * B * x->ldc + 2 * (k + 1); pan[r].ldcc = x->ldc;
         }
-        if (abft && nranks > 1 && m > 0) {                                  /* RECV + V4R */
+        if (abft && mode == 0 && nranks > 1 && m > 0) {                     /* RECV + V4R */
             int stop = 0;
             for (int r = 0; r < nranks && !stop; ++r) {
                 if (r == owner) continue;
@@ -460,7 +458,7 @@ int oracle_potrf(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* in
         if (m > 0) update(x, k, pan);
         if (abft && m > 0) {
             inject(x, (int)k, O_HOOK_UPDATE_OUT, 0, x->A, lda, x->chk, x->ldc);
-            const int do_v5 = ((k + 1) % x->K == 0) || (k == N - 2);          /* Opt. 3 [A14] */
+            const int do_v5 = mode != 2 && (((k + 1) % x->K == 0) || (k == N - 2));   /* Opt. 3 [A14] */
             if (do_v5) {
                 int stop = 0;
                 for (int64_t j = k + 1; j < N && !stop; ++j)
@@ -491,6 +489,59 @@ int oracle_potrf(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* in
     }
     free(x->chk); free(x->s); free(x->S1); free(x->S2); free(rcopy); free(rchk); free(pan);
     return x->status;
+}
+
+/* The factorisation with the scheme's recovery: Enhanced corrects in place; Online and Offline
+ * cannot correct an error that propagated ("it needs to repeat the whole decomposition
+ * again"), so an UNCORRECTABLE / NOT_SPD outcome or any detection by the final sweep re-runs the
+ * factorisation once from the saved input, without the injected faults. Events of both runs are
+ * returned in order. */
+int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
+                      int nranks, int K, double c_tau, int abft, int mode, oevent_t* ev, int64_t cap,
+                      int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out,
+                      int* reruns) {
+    if (n < 0) return -1;
+    if (nb < 1) return -2;
+    if (n % nb) return -2;                          /* [A20] */
+    if (lda < (n > 1 ? n : 1)) return -4;
+    if (mode < 0 || mode > 2) return -11;
+    if (nranks < 1) nranks = 1;
+    if (K < 1) K = 1;
+    ocount_t dummy;
+    ocount_t* c = cnt ? cnt : &dummy;
+    memset(c, 0, sizeof(ocount_t));
+    if (reruns) *reruns = 0;
+    double* A0 = NULL;
+    if (mode != 0 && n > 0) {
+        A0 = (double*)malloc(sizeof(double) * (size_t)(lda * n));
+        memcpy(A0, A, sizeof(double) * (size_t)(lda * n));
+    }
+    int64_t nev1 = 0;
+    int st = potrf_core(n, nb, A, lda, inj, ninj, nranks, K, c_tau, abft, mode, ev, cap, &nev1, info, c,
+                        chk_out, scl_out);
+    /* Online / Offline: a detection at the final sweep means an error escaped the scheme's
+     * online checks and may have propagated -> re-do. */
+    int v6_detect = 0;
+    for (int64_t e = 0; ev && e < nev1 && e < cap; ++e) v6_detect |= (ev[e].check == O_V6);
+    if (mode != 0 && (st == O_STATUS_UNCORRECTABLE || st == O_STATUS_NOT_SPD || v6_detect)) {
+        memcpy(A, A0, sizeof(double) * (size_t)(lda * n));
+        int64_t nev2 = 0;
+        const int64_t off = nev1 < cap ? nev1 : cap;
+        st = potrf_core(n, nb, A, lda, NULL, 0, nranks, K, c_tau, abft, mode, ev ? ev + off : NULL, cap - off,
+                        &nev2, info, c, chk_out, scl_out);
+        nev1 += nev2;
+        if (reruns) *reruns = 1;
+    }
+    free(A0);
+    if (nev) *nev = nev1;
+    return st;
+}
+
+int oracle_potrf(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
+                 int nranks, int K, double c_tau, int abft, oevent_t* ev, int64_t cap, int64_t* nev,
+                 int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out) {
+    return oracle_potrf_mode(n, nb, A, lda, inj, ninj, nranks, K, c_tau, abft, 0, ev, cap, nev, info, cnt, chk_out,
+                             scl_out, NULL);
 }
 
 /* ---- stand-alone steps for kernel-level parity tests ----------------------------------- */

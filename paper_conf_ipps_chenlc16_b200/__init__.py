@@ -46,12 +46,14 @@ class Report(ctypes.Structure):
     _fields_ = [("info", ctypes.c_int64), ("n_checks", ctypes.c_int64), ("n_detected", ctypes.c_int64),
                 ("n_data", ctypes.c_int64), ("n_nonfinite", ctypes.c_int64), ("n_chk1", ctypes.c_int64),
                 ("n_chk2", ctypes.c_int64), ("n_uncorrectable", ctypes.c_int64), ("n_events", ctypes.c_int64),
-                ("cap", ctypes.c_int64), ("events", ctypes.c_void_p), ("seconds", ctypes.c_double)]
+                ("cap", ctypes.c_int64), ("events", ctypes.c_void_p), ("seconds", ctypes.c_double),
+                ("reruns", ctypes.c_int64)]
 
 
 class Options(ctypes.Structure):
     _fields_ = [("abft_enabled", ctypes.c_int32), ("K", ctypes.c_int32), ("c_tau", ctypes.c_double),
-                ("lookahead", ctypes.c_int32), ("profile", ctypes.c_int32)]
+                ("lookahead", ctypes.c_int32), ("profile", ctypes.c_int32), ("mode", ctypes.c_int32),
+                ("pad", ctypes.c_int32)]
 
 
 class Profile(ctypes.Structure):
@@ -146,11 +148,15 @@ def _report_dict(rep, ev):
     return dict(info=rep.info, n_checks=rep.n_checks, n_detected=rep.n_detected, n_data=rep.n_data,
                 n_nonfinite=rep.n_nonfinite, n_chk1=rep.n_chk1, n_chk2=rep.n_chk2,
                 n_uncorrectable=rep.n_uncorrectable, n_events=rep.n_events, events=ev[:n].copy(),
-                seconds=rep.seconds)
+                seconds=rep.seconds, reruns=rep.reruns)
 
 
-def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False):
-    return Options(int(bool(abft_enabled)), int(K), float(c_tau), int(lookahead), int(bool(profile)))
+MODE = {"enhanced": 0, "online": 1, "offline": 2}
+
+
+def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False, mode="enhanced"):
+    return Options(int(bool(abft_enabled)), int(K), float(c_tau), int(lookahead), int(bool(profile)),
+                   MODE[mode] if isinstance(mode, str) else int(mode), 0)
 
 
 def abft_last_profile():

@@ -322,7 +322,9 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     const double Bd = (double)B;
     const int32_t* ab = &w.st->abort;
     // fused V5 partials: 64-row slabs x n columns x {v1, v2}
-    const bool can_fuse = abft && (nb % 128 == 0) && (lda % 2 == 0) && (((uintptr_t)A & 15) == 0);
+    const int mode = o.mode;
+    const bool can_fuse = abft && mode != ABFT_MODE_OFFLINE && (nb % 128 == 0) && (lda % 2 == 0) &&
+                          (((uintptr_t)A & 15) == 0);
     if (can_fuse) {
         w.cs_nslab = n / 32;   // room for 32-row slabs (the smallest warp-tile height)
         ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n), s));
@@ -361,8 +363,8 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         const Loc L{A, lda, w.chk, w.ldc, W, ldw, mB};
         const double md = (double)m, mBd = (double)mB;
         Work wk = w; wk.W = W;
-        if (abft) {
-            do_inject_if(inj, k, ABFT_HOOK_REST, B, L, ab, P, k, k + 1, true);   // REST(k) into column k
+        if (abft) do_inject_if(inj, k, ABFT_HOOK_REST, B, L, ab, P, k, k + 1, true);   // REST(k) into column k
+        if (abft && mode == ABFT_MODE_ENHANCED) {
             StageArgs a = stage_base(wk, A, lda, o.c_tau, SK_COLUMN, ABFT_V2, (int)k);
             a.flist = 1;
             cudaEvent_t t = prof.begin(P);
@@ -383,15 +385,19 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
             do_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, L, ab, P);
             StageArgs a3 = stage_base(wk, A, lda, o.c_tau, SK_DIAG_FACT, ABFT_V3, (int)k);
             a3.ldw = ldw; a3.mB = mB; a3.flist = 1;
-            t = prof.begin(P);
-            launch_check(a3, P);                                                 // V3
-            prof.end(t, PH_V3, P, 4.0 * lowerB, 8.0 * lowerB);
+            if (mode != ABFT_MODE_OFFLINE) {
+                t = prof.begin(P);
+                launch_check(a3, P);                                             // V3
+                prof.end(t, PH_V3, P, 4.0 * lowerB, 8.0 * lowerB);
+            }
             do_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, L, ab, P);
             StageArgs a4 = stage_base(wk, A, lda, o.c_tau, SK_PANEL, ABFT_V4, (int)k);
             a4.ldw = ldw; a4.mB = mB; a4.flist = 1;
-            t = prof.begin(P);
-            launch_check(a4, P);                                                 // V4
-            prof.end(t, PH_V4, P, 4.0 * mBd * Bd, 8.0 * mBd * Bd);
+            if (mode != ABFT_MODE_OFFLINE) {
+                t = prof.begin(P);
+                launch_check(a4, P);                                             // V4
+                prof.end(t, PH_V4, P, 4.0 * mBd * Bd, 8.0 * mBd * Bd);
+            }
         }
         t = prof.begin(P);
         launch_copy(mB, B, W, ldw, Akk + B, lda, ab, P);                        // L panel
@@ -470,7 +476,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         if (m == 0) break;
         const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
         const Loc L{A, lda, w.chk, w.ldc, Wbuf[k & 1], ldw, mB};
-        const bool gated = ((k + 1) % K == 0) || k == N - 2;
+        const bool gated = (((k + 1) % K == 0) || k == N - 2) && mode != ABFT_MODE_OFFLINE;
         // (a) block column k+1 first: update, UPDATE_OUT hook, V5 -> hand it to the panel stream
         const bool fa = update_cols(k, k + 1, k + 2);
         if (abft) {
@@ -570,8 +576,8 @@ static void dist_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, 
 
 int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, DistTransport* tp,
              cudaStream_t s, const abft_inject_spec_t* inj_c, abft_report_t* rep, const abft_options_t* opt) {
-    abft_options_t o = opt ? *opt : abft_options_t{1, 1, 64.0, 0, 0};
-    if (o.K < 1 || !(o.c_tau > 0)) return -11;
+    abft_options_t o = opt ? *opt : abft_options_t{1, 1, 64.0, 0, 0, ABFT_MODE_ENHANCED, 0};
+    if (o.K < 1 || !(o.c_tau > 0) || o.mode != ABFT_MODE_ENHANCED) return -11;   // dist: Enhanced only
     std::vector<abft_inject_spec_t> inj;
     if (collect_inj(inj_c, n, nb, inj)) return -9;
     if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; }
@@ -833,7 +839,7 @@ extern "C" int abft_potrf_dist_sim(int64_t n, int64_t nb, int nranks, double* co
 static abft_options_t default_options() {
     abft_options_t o;
     memset(&o, 0, sizeof o);
-    o.abft_enabled = 1; o.K = 1; o.c_tau = 64.0; o.lookahead = 0; o.profile = 0;
+    o.abft_enabled = 1; o.K = 1; o.c_tau = 64.0; o.lookahead = 0; o.profile = 0; o.mode = ABFT_MODE_ENHANCED;
     return o;
 }
 
@@ -846,9 +852,52 @@ extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft
     if (o.K < 1 || !(o.c_tau > 0)) return -8;
     std::vector<abft_inject_spec_t> list;
     if (collect_inj(inj, n, nb, list)) return -6;
-    if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; }
+    if (o.mode < ABFT_MODE_ENHANCED || o.mode > ABFT_MODE_OFFLINE) return -8;
+    if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; rep->reruns = 0; }
     if (n == 0) return 0;
-    return run_potrf(n, nb, A, lda, (cudaStream_t)stream, list, rep, o);
+    cudaStream_t s = (cudaStream_t)stream;
+    if (o.mode == ABFT_MODE_ENHANCED || !o.abft_enabled) return run_potrf(n, nb, A, lda, s, list, rep, o);
+    // Online / Offline: keep the input; an uncorrectable outcome or a detection by the final
+    // sweep means an error propagated -> re-do the factorisation once, without the faults
+    double* A0 = nullptr;
+    ABFT_CUDA_TRY(cudaMallocAsync((void**)&A0, sizeof(double) * (size_t)(n * n), s));
+    ABFT_CUDA_TRY(cudaMemcpy2DAsync(A0, n * sizeof(double), A, lda * sizeof(double), n * sizeof(double), n,
+                                    cudaMemcpyDeviceToDevice, s));
+    abft_report_t r1;
+    memset(&r1, 0, sizeof r1);
+    std::vector<abft_event_t> ev1(rep ? std::max<int64_t>(rep->cap, 4096) : 4096);
+    r1.cap = (int64_t)ev1.size(); r1.events = ev1.data();
+    int st = run_potrf(n, nb, A, lda, s, list, &r1, o);
+    bool v6 = false;
+    for (int64_t e = 0; e < std::min<int64_t>(r1.n_events, r1.cap); ++e) v6 |= (ev1[e].check == ABFT_V6);
+    abft_report_t r2;
+    memset(&r2, 0, sizeof r2);
+    std::vector<abft_event_t> ev2(rep ? std::max<int64_t>(rep->cap, 16) : 16);
+    r2.cap = (int64_t)ev2.size(); r2.events = ev2.data();
+    int reruns = 0;
+    if (st == ABFT_UNCORRECTABLE || st == ABFT_NOT_SPD || v6) {
+        ABFT_CUDA_TRY(cudaMemcpy2DAsync(A, lda * sizeof(double), A0, n * sizeof(double), n * sizeof(double), n,
+                                        cudaMemcpyDeviceToDevice, s));
+        const std::vector<abft_inject_spec_t> none;
+        st = run_potrf(n, nb, A, lda, s, none, &r2, o);
+        reruns = 1;
+    }
+    cudaFreeAsync(A0, s);
+    ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+    if (rep) {
+        rep->info = reruns ? r2.info : r1.info;
+        rep->n_checks = r1.n_checks + r2.n_checks; rep->n_detected = r1.n_detected + r2.n_detected;
+        rep->n_data = r1.n_data + r2.n_data; rep->n_nonfinite = r1.n_nonfinite + r2.n_nonfinite;
+        rep->n_chk1 = r1.n_chk1 + r2.n_chk1; rep->n_chk2 = r1.n_chk2 + r2.n_chk2;
+        rep->n_uncorrectable = r1.n_uncorrectable + r2.n_uncorrectable;
+        rep->n_events = r1.n_events + r2.n_events;
+        rep->seconds = r1.seconds + r2.seconds;
+        rep->reruns = reruns;
+        int64_t w = 0;
+        for (int64_t e = 0; e < std::min<int64_t>(r1.n_events, r1.cap) && w < rep->cap; ++e) rep->events[w++] = ev1[e];
+        for (int64_t e = 0; e < std::min<int64_t>(r2.n_events, r2.cap) && w < rep->cap; ++e) rep->events[w++] = ev2[e];
+    }
+    return st;
 }
 
 extern "C" int abft_potrf(int64_t n, int64_t nb, double* A, int64_t lda, abft_stream_t stream,

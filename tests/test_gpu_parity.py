@@ -276,3 +276,23 @@ def test_c3_full_size_sampled(P, n, nb, lead):
     R = Asym @ X - Lt @ (Lt.T @ X)
     be = (R.norm() / (Asym @ X).norm()).item()
     assert be <= 10 * n * EPS
+
+
+@pytest.mark.parametrize("mode", ["enhanced", "online", "offline"])
+@pytest.mark.parametrize("fault", ["none", "computation", "memory"])
+def test_schemes_match_oracle(P, mode, fault):
+    """The comparison schemes of Tables VII/VIII (NEXT-2): same events, same re-runs, same factor."""
+    from tests.test_oracle_pins import SCHEME_FAULTS
+    n, nb = 1024, 128
+    A = syn.spd_matrix(n)
+    specs = SCHEME_FAULTS[fault]
+    inj = syn.inj_array(specs) if specs else None
+    ref = oracle.potrf(A, nb, inj=inj, mode=mode)
+    st, rep, L = run_gpu(P, A, nb, inj=inj, opt=P.options(mode=mode))
+    assert st == ref.status == 0
+    assert rep["reruns"] == ref.reruns
+    if ref.reruns == 0:
+        assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
+    else:   # after propagation the first run's event list depends on rounding; the decision does not
+        assert rep["n_events"] > 0
+    assert floor_rel(L, ref.L, A) <= 1e-11

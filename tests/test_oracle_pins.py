@@ -363,3 +363,34 @@ def test_verify_entry_detects_and_corrects():
     assert (ev[0]["tile_i"], ev[0]["tile_j"], ev[0]["row"], ev[0]["col"]) == (2, 1, 150 - 128, 70 - 64)
     assert abs(ev[0]["delta1"] - 3.0) < 1e-9 and abs(ev[0]["delta2"] - 3.0 * (150 - 128 + 1)) < 1e-8
     assert abs(B[150, 70] - A[150, 70]) < 1e-13
+
+
+# ---- comparison schemes (NEXT-2): Tables VII/VIII ---------------------------
+SCHEME_FAULTS = {
+    "none": [],
+    # computation error: corrupt the output of the trailing update
+    "computation": [dict(k=2, hook="UPDATE_OUT", row=800, col=500, bit=50)],
+    # memory error "between checksum verification and data access": the diagonal block of
+    # column 3 after its last verification (V5 of iteration 2) and before POTRF(3) reads it
+    "memory": [dict(k=3, hook="REST", row=3 * 128 + 100, col=3 * 128 + 50, bit=50)],
+}
+# Enhanced corrects both kinds; Online corrects computing errors but must re-do the
+# decomposition for a memory error; Offline must re-do it for both.
+SCHEME_RERUNS = {("enhanced", "none"): 0, ("enhanced", "computation"): 0, ("enhanced", "memory"): 0,
+                 ("online", "none"): 0, ("online", "computation"): 0, ("online", "memory"): 1,
+                 ("offline", "none"): 0, ("offline", "computation"): 1, ("offline", "memory"): 1}
+
+
+@pytest.mark.parametrize("mode", ["enhanced", "online", "offline"])
+@pytest.mark.parametrize("fault", ["none", "computation", "memory"])
+def test_schemes_table_vii_capability(mode, fault):
+    n, nb = 1024, 128
+    A = syn.spd_matrix(n)
+    ref = oracle.potrf(A, nb)
+    specs = SCHEME_FAULTS[fault]
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs) if specs else None, mode=mode)
+    assert r.status == 0
+    assert r.reruns == SCHEME_RERUNS[(mode, fault)]
+    assert floor_rel(r.L, ref.L, A) <= 1e-11          # every scheme ends with the right factor
+    if mode == "enhanced" and specs:
+        assert r.event_tuples() == [predict(s, n, nb) for s in specs]
