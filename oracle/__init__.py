@@ -37,7 +37,7 @@ COUNT_DTYPE = np.dtype([
     ("flops_factor", "<f8"), ("flops_chkupd", "<f8"), ("flops_check", "<f8"),
     ("flops_encode", "<f8"), ("bytes_check", "<f8"), ("max_ratio", "<f8"),
 ])
-CHECK = {1: "V1", 2: "V2", 3: "V3", 4: "V4", 5: "V5", 6: "V6", 7: "V4R"}
+CHECK = {1: "V1", 2: "V2", 3: "V3", 4: "V4", 5: "V5", 6: "V6", 7: "V4R", 8: "V7"}
 KIND = {1: "DATA", 2: "NONFINITE", 3: "CHK1", 4: "CHK2", 5: "UNCORRECTABLE"}
 STATUS = {0: "OK", 1: "UNCORRECTABLE", 2: "NOT_SPD"}
 
@@ -62,7 +62,7 @@ def lib():
         _lib.oracle_potrf.argtypes = [i64, i64, vp, i64, vp, i64, i32, i32, ctypes.c_double, i32,
                                       vp, i64, ctypes.POINTER(i64), ctypes.POINTER(i64), vp, vp, vp]
         _lib.oracle_potrf.restype = i32
-        _lib.oracle_potrf_mode.argtypes = [i64, i64, vp, i64, vp, i64, i32, i32, ctypes.c_double, i32, i32,
+        _lib.oracle_potrf_mode.argtypes = [i64, i64, vp, i64, vp, i64, i32, i32, ctypes.c_double, i32, i32, i32,
                                            vp, i64, ctypes.POINTER(i64), ctypes.POINTER(i64), vp, vp, vp,
                                            ctypes.POINTER(i32)]
         _lib.oracle_potrf_mode.restype = i32
@@ -103,7 +103,8 @@ def sorted_events(ev):
 MODE = {"enhanced": 0, "online": 1, "offline": 2}
 
 
-def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, inplace=False, mode="enhanced"):
+def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, inplace=False, mode="enhanced",
+          order="right"):
     """ABFT Cholesky of A (lower), n % nb == 0. mode: "enhanced" (the paper's scheme, default),
     "online" or "offline" (its comparison schemes, which re-run once on an uncorrectable error).
     Returns Result with L in the lower triangle (upper triangle untouched), status (0/1/2),
@@ -125,7 +126,8 @@ def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, in
     scl = np.zeros(n + 2 * N, dtype=np.float64)
     reruns = ctypes.c_int(0)
     st = lib().oracle_potrf_mode(n, nb, _ptr(L), max(n, 1), _ptr(inj_arr), ninj, nranks, K, c_tau, int(abft),
-                                 MODE[mode] if isinstance(mode, str) else int(mode), _ptr(ev), cap,
+                                 MODE[mode] if isinstance(mode, str) else int(mode),
+                                 {"right": 0, "left": 1}[order], _ptr(ev), cap,
                                  ctypes.byref(nev), ctypes.byref(info), _ptr(cnt), _ptr(chk), _ptr(scl),
                                  ctypes.byref(reruns))
     if st < 0:

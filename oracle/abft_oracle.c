@@ -39,7 +39,7 @@
 /* ---- codes (restated from the interface contract, not included from include/) ---------- */
 enum { O_HOOK_REST = 0, O_HOOK_POTRF_OUT = 1, O_HOOK_TRSM_OUT = 2, O_HOOK_UPDATE_OUT = 3, O_HOOK_RECV = 4 };
 enum { O_TGT_DATA = 0, O_TGT_CHK = 1 };
-enum { O_V1 = 1, O_V2 = 2, O_V3 = 3, O_V4 = 4, O_V5 = 5, O_V6 = 6, O_V4R = 7 };
+enum { O_V1 = 1, O_V2 = 2, O_V3 = 3, O_V4 = 4, O_V5 = 5, O_V6 = 6, O_V4R = 7, O_V7 = 8 };
 enum { O_DATA = 1, O_NONFINITE = 2, O_CHK1 = 3, O_CHK2 = 4, O_UNCORRECTABLE = 5 };
 enum { O_OK = 0, O_STATUS_UNCORRECTABLE = 1, O_STATUS_NOT_SPD = 2 };
 
@@ -491,13 +491,125 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
     return x->status;
 }
 
+
+/* ---- left-looking order: MAGMA's Alg. 1 (garbled; reading A2) with the
+ * verification of Table I — NEXT-1 of SURVEY.md §8f ------------------------
+ * iteration j:  SYRK  A[j,j]     -= L[j,0:j] L[j,0:j]^T        verify A (V1) and C = L[j,0:j] (V7)
+ *               GEMM  A[j+1:N,j] -= L[j+1:N,0:j] L[j,0:j]^T    verify B (V2), C, D = L[j+1:N,0:j] (V7,
+ *                                                               every K iterations: Opt. 3)
+ *               POTF2 A[j,j] -> L[j,j]                         verify A (V5 on the updated column)
+ *               TRSM  L[j+1:N,j] = A[j+1:N,j] L[j,j]^-T        verify L (V3) and B (V5)
+ * Checksums: chk(A') = chk(A) - chk(LC) LC^T, chk(B') = chk(B) - chk(LD) LC^T,
+ * Alg. 2, chk(LB) = chk(B') LA^-T. Online-ABFT checks results instead (V5 after the update, V3,
+ * V4 after TRSM); Offline only V6. */
+static int potrf_core_left(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
+                           int K, double c_tau, int abft, int mode, oevent_t* ev, int64_t cap,
+                           int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out) {
+    octx_t X_; octx_t* x = &X_;
+    memset(x, 0, sizeof *x);
+    x->cnt = cnt; x->mode = mode;
+    x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = 2 * x->N > 0 ? 2 * x->N : 1;
+    x->A = A; x->c_tau = c_tau > 0 ? c_tau : 64.0; x->rho = 0x1p-30;
+    x->nranks = 1; x->K = K; x->correct = 1;
+    x->inj = inj; x->ninj = ninj; x->ev = ev; x->cap = cap;
+    if (info) *info = 0;
+    if (n == 0) { if (nev) *nev = 0; return 0; }
+    const int64_t N = x->N, B = nb;
+    x->chk = (double*)calloc((size_t)(x->ldc * n), sizeof(double));
+    x->s = (double*)malloc(sizeof(double) * (size_t)n);
+    x->S1 = (double*)malloc(sizeof(double) * (size_t)N);
+    x->S2 = (double*)malloc(sizeof(double) * (size_t)N);
+    double* tmp = (double*)malloc(sizeof(double) * (size_t)B);
+    if (abft) { scales(x); encode(x); }
+    for (int64_t j = 0; j < N && x->status == O_OK; ++j) {
+        if (abft) inject(x, (int)j, O_HOOK_REST, 0, x->A, lda, x->chk, x->ldc);
+        if (abft && mode == 0 && j > 0) {
+            int stop = 0;
+            for (int64_t p = 0; p < j && !stop; ++p)                 /* V7: C = L[j,p] and D = L[i>j,p] */
+                for (int64_t i = j; i < N && !stop; ++i) {
+                    if (i > j && !((j % K) == 0)) continue;          /* Opt. 3: D every K iterations */
+                    tview_t v = gview(x, i, p, 1);
+                    if (check_tile(x, &v, (int)j, O_V7, 0)) stop = 1;
+                }
+            if (stop) break;
+        }
+        if (abft && mode == 0 && run_checks_column(x, j, 0, O_V1, O_V2, 1)) break;   /* V1, V2 */
+        if (j > 0) {   /* SYRK + GEMM: A[j:N, j] -= L[j:N, 0:j] L[j, 0:j]^T, then the checksum rows */
+            const double* Lj = x->A + j * B;                          /* row block j, columns 0..jB */
+            for (int64_t i = j; i < N; ++i) {
+                const double* Li = x->A + i * B;
+                double* T = x->A + j * B * lda + i * B;
+                for (int64_t c = 0; c < B; ++c) {
+                    const int64_t r0 = (i == j) ? c : 0;
+                    for (int64_t r = r0; r < B; ++r) tmp[r] = 0.0;
+                    for (int64_t q = 0; q < j * B; ++q) {
+                        const double l = Lj[q * lda + c];
+                        for (int64_t r = r0; r < B; ++r) tmp[r] += Li[q * lda + r] * l;
+                    }
+                    for (int64_t r = r0; r < B; ++r) T[c * lda + r] -= tmp[r];
+                }
+                for (int t = 0; t < 2; ++t) {
+                    const double* ck = x->chk + 2 * i + t;            /* chk(i, 0:j) row */
+                    double* cd = x->chk + j * B * x->ldc + 2 * i + t;
+                    for (int64_t c = 0; c < B; ++c) {
+                        double a = 0.0;
+                        for (int64_t q = 0; q < j * B; ++q) a += ck[q * x->ldc] * Lj[q * lda + c];
+                        cd[c * x->ldc] -= a;
+                    }
+                }
+            }
+            x->cnt->flops_factor += 2.0 * (double)((N - j) * B) * B * (double)(j * B);
+            x->cnt->flops_chkupd += 4.0 * (double)(N - j) * B * (double)(j * B);
+        }
+        if (abft) inject(x, (int)j, O_HOOK_UPDATE_OUT, 0, x->A, lda, x->chk, x->ldc);
+        if (abft && mode != 2 && j > 0) {                             /* V5: the updated column j */
+            int stop = 0;
+            for (int64_t i = j; i < N && !stop; ++i) {
+                tview_t v = gview(x, i, j, 0);
+                if (check_tile(x, &v, (int)j, O_V5, 0)) stop = 1;
+            }
+            if (stop) break;
+        }
+        if (potrf_tile(x, j)) break;
+        if (abft) {
+            inject(x, (int)j, O_HOOK_POTRF_OUT, 0, x->A, lda, x->chk, x->ldc);
+            tview_t v = gview(x, j, j, 1);
+            if (mode != 2 && check_tile(x, &v, (int)j, O_V3, 0)) break;   /* V3 */
+        }
+        trsm_panel(x, j);
+        if (abft) {
+            inject(x, (int)j, O_HOOK_TRSM_OUT, 0, x->A, lda, x->chk, x->ldc);
+            if (mode == 1 && run_checks_column(x, j, 1, 0, O_V4, 0)) break;  /* Online: V4 */
+        }
+    }
+    if (abft && x->status == O_OK) {
+        inject(x, (int)N, O_HOOK_REST, 0, x->A, lda, x->chk, x->ldc);
+        int stop = 0;
+        for (int64_t J = 0; J < N && !stop; ++J)
+            for (int64_t I = J; I < N && !stop; ++I) {
+                tview_t v = gview(x, I, J, 1);
+                if (check_tile(x, &v, (int)N, O_V6, 0)) stop = 1;             /* V6 */
+            }
+    }
+    if (info) *info = x->info;
+    if (nev) *nev = x->nev;
+    if (chk_out) memcpy(chk_out, x->chk, sizeof(double) * (size_t)(x->ldc * n));
+    if (scl_out && abft) {
+        memcpy(scl_out, x->s, sizeof(double) * (size_t)n);
+        memcpy(scl_out + n, x->S1, sizeof(double) * (size_t)N);
+        memcpy(scl_out + n + N, x->S2, sizeof(double) * (size_t)N);
+    }
+    free(x->chk); free(x->s); free(x->S1); free(x->S2); free(tmp);
+    return x->status;
+}
+
 /* The factorisation with the scheme's recovery: Enhanced corrects in place; Online and Offline
  * cannot correct an error that propagated ("it needs to repeat the whole decomposition
  * again"), so an UNCORRECTABLE / NOT_SPD outcome or any detection by the final sweep re-runs the
  * factorisation once from the saved input, without the injected faults. Events of both runs are
  * returned in order. */
 int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
-                      int nranks, int K, double c_tau, int abft, int mode, oevent_t* ev, int64_t cap,
+                      int nranks, int K, double c_tau, int abft, int mode, int order, oevent_t* ev, int64_t cap,
                       int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out,
                       int* reruns) {
     if (n < 0) return -1;
@@ -516,9 +628,12 @@ int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
         A0 = (double*)malloc(sizeof(double) * (size_t)(lda * n));
         memcpy(A0, A, sizeof(double) * (size_t)(lda * n));
     }
+    if (order != 0 && nranks != 1) return -7;
     int64_t nev1 = 0;
-    int st = potrf_core(n, nb, A, lda, inj, ninj, nranks, K, c_tau, abft, mode, ev, cap, &nev1, info, c,
-                        chk_out, scl_out);
+    int st = order == 0 ? potrf_core(n, nb, A, lda, inj, ninj, nranks, K, c_tau, abft, mode, ev, cap, &nev1, info, c,
+                                     chk_out, scl_out)
+                        : potrf_core_left(n, nb, A, lda, inj, ninj, K, c_tau, abft, mode, ev, cap, &nev1, info, c,
+                                          chk_out, scl_out);
     /* Online / Offline: a detection at the final sweep means an error escaped the scheme's
      * online checks and may have propagated -> re-do. */
     int v6_detect = 0;
@@ -527,8 +642,10 @@ int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
         memcpy(A, A0, sizeof(double) * (size_t)(lda * n));
         int64_t nev2 = 0;
         const int64_t off = nev1 < cap ? nev1 : cap;
-        st = potrf_core(n, nb, A, lda, NULL, 0, nranks, K, c_tau, abft, mode, ev ? ev + off : NULL, cap - off,
-                        &nev2, info, c, chk_out, scl_out);
+        st = order == 0 ? potrf_core(n, nb, A, lda, NULL, 0, nranks, K, c_tau, abft, mode, ev ? ev + off : NULL,
+                                     cap - off, &nev2, info, c, chk_out, scl_out)
+                        : potrf_core_left(n, nb, A, lda, NULL, 0, K, c_tau, abft, mode, ev ? ev + off : NULL,
+                                          cap - off, &nev2, info, c, chk_out, scl_out);
         nev1 += nev2;
         if (reruns) *reruns = 1;
     }
@@ -540,8 +657,8 @@ int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
 int oracle_potrf(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
                  int nranks, int K, double c_tau, int abft, oevent_t* ev, int64_t cap, int64_t* nev,
                  int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out) {
-    return oracle_potrf_mode(n, nb, A, lda, inj, ninj, nranks, K, c_tau, abft, 0, ev, cap, nev, info, cnt, chk_out,
-                             scl_out, NULL);
+    return oracle_potrf_mode(n, nb, A, lda, inj, ninj, nranks, K, c_tau, abft, 0, 0, ev, cap, nev, info, cnt,
+                             chk_out, scl_out, NULL);
 }
 
 /* ---- stand-alone steps for kernel-level parity tests ----------------------------------- */

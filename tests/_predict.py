@@ -14,9 +14,47 @@ Location: d1 = Delta, d2 = (r+1) Delta -> data row r; an erro
 row 1 / row 2 shows as d1 alone / d2 alone (CHK1 / CHK2, reading A10).
 """
 
-V = {"V1": 1, "V2": 2, "V3": 3, "V4": 4, "V5": 5, "V6": 6, "V4R": 7}
+V = {"V1": 1, "V2": 2, "V3": 3, "V4": 4, "V5": 5, "V6": 6, "V4R": 7, "V7": 8}
 KIND = {"DATA": 1, "NONFINITE": 2, "CHK1": 3, "CHK2": 4, "UNCORRECTABLE": 5}
 HOOKS = {"REST": 0, "POTRF_OUT": 1, "TRSM_OUT": 2, "UPDATE_OUT": 3, "RECV": 4}
+
+
+def predict_left(spec, n, nb, K=1):
+    """Left-looking order (MAGMA Alg. 1) with Table I's verification:
+    iteration j verifies A[j,j] and B = A[j+1:,j] (V1/V2) and the L blocks it reads, C = L[j,0:j] and
+    D = L[j+1:,0:j] (V7, D every K iterations), the updated column (V5), L[j,j] (V3); V6 at the end.
+      REST(j) in tile (I,J): J == j -> V1/V2 at j; J > j -> V1/V2 at J (untouched until then);
+                             J < j -> V7 at the first j' >= j reading it (I >= j', D gated), else V6
+      UPDATE_OUT(j) -> V5 at j;  POTRF_OUT(j) -> V3 at j;  TRSM_OUT(j) -> V7 at the next read"""
+    N = n // nb
+    k = spec["k"]
+    hook = spec["hook"] if isinstance(spec["hook"], str) else {v: kk for kk, v in HOOKS.items()}[spec["hook"]]
+    r, c = spec["row"], spec["col"]
+    I, J = r // nb, c // nb
+    row, col, kind = r - I * nb, c - J * nb, KIND["DATA"]
+
+    def first_read(j0):
+        for jj in range(j0, N):
+            if jj > J and I >= jj and (I == jj or jj % K == 0):
+                return (jj, V["V7"])
+        return (N, V["V6"])
+
+    if hook == "REST":
+        if k >= N:
+            ck, v = N, V["V6"]
+        elif J >= k:
+            ck, v = J, V["V1"] if I == J else V["V2"]
+        else:
+            ck, v = first_read(k)
+    elif hook == "UPDATE_OUT":
+        ck, v = k, V["V5"]
+    elif hook == "POTRF_OUT":
+        ck, v = k, V["V3"]
+    elif hook == "TRSM_OUT":
+        ck, v = first_read(k + 1)
+    else:
+        raise ValueError(hook)
+    return (ck, v, J, I, col, row, kind, 0)
 
 
 def predict(spec, n, nb, K=1):

@@ -394,3 +394,61 @@ def test_schemes_table_vii_capability(mode, fault):
     assert floor_rel(r.L, ref.L, A) <= 1e-11          # every scheme ends with the right factor
     if mode == "enhanced" and specs:
         assert r.event_tuples() == [predict(s, n, nb) for s in specs]
+
+
+# ---- NEXT-1: the paper's own (left-looking, MAGMA Alg. 1) order with Table I's checks ------
+from tests._predict import predict_left
+
+
+@pytest.mark.parametrize("n,nb", [(512, 64), (1024, 128), (96, 24)])
+def test_left_looking_factor_matches_lapack(n, nb):
+    A = syn.spd_matrix(n)
+    r = oracle.potrf(A, nb, order="left")
+    assert r.status == 0 and len(r.events) == 0
+    assert floor_rel(r.L, scipy.linalg.cholesky(A, lower=True), A) <= 1e-11
+    assert r.counts["max_ratio"] <= 2.0 ** -6
+
+
+def test_left_looking_pascal_mod2_c1_exact():
+    A = syn.pascal_mod2(256)
+    specs = [dict(k=2, hook="REST", row=232, col=40, bit=52),      # finished L block (value 1), read by V7
+             dict(k=4, hook="UPDATE_OUT", row=230, col=130, bit=51)]
+    r = oracle.potrf(A, 32, inj=syn.inj_array(specs), order="left")
+    i = np.arange(256)
+    assert np.array_equal(np.tril(r.L), ((i[:, None] & i[None, :]) == i[None, :]).astype(float))
+    assert r.event_tuples() == sorted(predict_left(s, 256, 32) for s in specs)
+
+
+@pytest.mark.parametrize("K", [1, 3])
+def test_left_looking_injection_ground_truth(K):
+    """K = 1: each error is reported once, at its first read. K = 3 (Opt. 3): a D block is not
+    re-verified at every read, so an error there is used by the GEMM first and shows up again in
+    the updated column (caught by V5, one element per column) before V7 repairs the source."""
+    n, nb = 1024, 128
+    A = syn.spd_matrix(n)
+    ref = oracle.potrf(A, nb, order="left")
+    specs = [dict(k=2, hook="REST", row=900, col=130, bit=50),
+             dict(k=3, hook="TRSM_OUT", row=700, col=3 * nb + 5, bit=50),
+             dict(k=4, hook="UPDATE_OUT", row=800, col=4 * nb + 9, bit=52),
+             dict(k=5, hook="POTRF_OUT", row=5 * nb + 9, col=5 * nb + 2, bit=52),
+             dict(k=1, hook="REST", row=1000, col=7 * nb + 3, bit=50),
+             dict(k=8, hook="REST", row=600, col=300, bit=50)]
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs), order="left", K=K)
+    assert r.status == 0
+    if K == 1:
+        assert r.event_tuples() == sorted(predict_left(s, n, nb, K=K) for s in specs)
+    else:
+        assert set(predict_left(s, n, nb, K=K) for s in specs) <= set(r.event_tuples())
+    assert floor_rel(r.L, ref.L, A) <= 1e-11
+
+
+def test_left_looking_verifies_more_than_right_looking():
+    """Table I / P:255: the Enhanced scheme re-verifies L blocks at every read in the left-looking
+    order (O(n) verifications per block), so its check volume exceeds the right-looking one."""
+    n, nb = 1024, 64
+    A = syn.spd_matrix(n)
+    rl = oracle.potrf(A, nb)
+    ll = oracle.potrf(A, nb, order="left")
+    assert ll.counts["bytes_check"] > rl.counts["bytes_check"]
+    ll3 = oracle.potrf(A, nb, order="left", K=3)
+    assert ll3.counts["bytes_check"] < ll.counts["bytes_check"]
