@@ -61,6 +61,7 @@ typedef struct CUstream_st* abft_stream_t;
 #define ABFT_V5 5   /* check of every trailing tile after update k                            */
 #define ABFT_V6 6   /* final sweep over L                                                      */
 #define ABFT_V4R 7  /* (multi-GPU) receiver re-check of the broadcast panel                   */
+#define ABFT_V7 8   /* (left-looking order) the L blocks a SYRK/GEMM is about to read (Table I) */
 #define ABFT_KIND_DATA 1          /* one data element located (row = d2/d1 - 1) and corrected   */
 #define ABFT_KIND_NONFINITE 2     /* non-finite delta; located by argmax |X| and corrected       */
 #define ABFT_KIND_CHK1 3          /* checksum row 1 corrupted; recomputed from the data          */
@@ -100,8 +101,11 @@ typedef struct abft_options {
     int32_t lookahead;    /* reserved (0/1)                                                    */
     int32_t profile;      /* 1: time every phase with CUDA events on `stream` (abft_last_profile) */
     int32_t mode;         /* ABFT_MODE_ENHANCED (default), ABFT_MODE_ONLINE or ABFT_MODE_OFFLINE  */
-    int32_t pad;
+    int32_t order;        /* ABFT_ORDER_RIGHT (default: trailing update + look-ahead) or
+                             ABFT_ORDER_LEFT (MAGMA's Alg. 1, Table I checks)     */
 } abft_options_t;
+#define ABFT_ORDER_RIGHT 0
+#define ABFT_ORDER_LEFT 1
 
 /* Schemes (§II.B, §III; Table VII/VIII compare them):
  *  ENHANCED  verify every block before it is read (V1..V6) — errors are corrected in place.

@@ -23,7 +23,7 @@ LIB_PATH = os.path.join(_HERE, "libabft.so")
 # Codes restated from include/abft.h
 OK, UNCORRECTABLE, NOT_SPD, ERR_CUDA, ERR_NCCL = 0, 1, 2, 3, 4
 HOOK = {"REST": 0, "POTRF_OUT": 1, "TRSM_OUT": 2, "UPDATE_OUT": 3, "RECV": 4}
-CHECK = {1: "V1", 2: "V2", 3: "V3", 4: "V4", 5: "V5", 6: "V6", 7: "V4R"}
+CHECK = {1: "V1", 2: "V2", 3: "V3", 4: "V4", 5: "V5", 6: "V6", 7: "V4R", 8: "V7"}
 KIND = {1: "DATA", 2: "NONFINITE", 3: "CHK1", 4: "CHK2", 5: "UNCORRECTABLE"}
 
 EVENT_DTYPE = np.dtype([
@@ -53,7 +53,7 @@ class Report(ctypes.Structure):
 class Options(ctypes.Structure):
     _fields_ = [("abft_enabled", ctypes.c_int32), ("K", ctypes.c_int32), ("c_tau", ctypes.c_double),
                 ("lookahead", ctypes.c_int32), ("profile", ctypes.c_int32), ("mode", ctypes.c_int32),
-                ("pad", ctypes.c_int32)]
+                ("order", ctypes.c_int32)]
 
 
 class Profile(ctypes.Structure):
@@ -154,9 +154,9 @@ def _report_dict(rep, ev):
 MODE = {"enhanced": 0, "online": 1, "offline": 2}
 
 
-def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False, mode="enhanced"):
+def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False, mode="enhanced", order="right"):
     return Options(int(bool(abft_enabled)), int(K), float(c_tau), int(lookahead), int(bool(profile)),
-                   MODE[mode] if isinstance(mode, str) else int(mode), 0)
+                   MODE[mode] if isinstance(mode, str) else int(mode), {"right": 0, "left": 1}[order])
 
 
 def abft_last_profile():

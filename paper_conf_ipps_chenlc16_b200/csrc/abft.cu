@@ -63,7 +63,8 @@ static int check_common(int64_t n, int64_t nb, const void* A, int64_t lda) {
 }
 
 // Injection specs: validated against the region their hook can touch.
-static int collect_inj(const abft_inject_spec_t* inj, int64_t n, int64_t nb, std::vector<abft_inject_spec_t>& out) {
+static int collect_inj(const abft_inject_spec_t* inj, int64_t n, int64_t nb, std::vector<abft_inject_spec_t>& out,
+                       int order = ABFT_ORDER_RIGHT) {
     out.clear();
     if (!inj) return 0;
     const int64_t N = n / nb;
@@ -86,7 +87,9 @@ static int collect_inj(const abft_inject_spec_t* inj, int64_t n, int64_t nb, std
         switch (s.hook) {
             case ABFT_HOOK_POTRF_OUT: if (!(I == k && J == k)) return -1; break;
             case ABFT_HOOK_TRSM_OUT: if (!(J == k && I > k)) return -1; break;
-            case ABFT_HOOK_UPDATE_OUT: if (!(J > k)) return -1; break;
+            case ABFT_HOOK_UPDATE_OUT:   // the block columns the update of iteration k writes
+                if (order == ABFT_ORDER_LEFT ? !(J == k && k > 0) : !(J > k)) return -1;
+                break;
             case ABFT_HOOK_RECV: if (!(J == k && I > k)) return -1; break;
             default: break;
         }
@@ -577,7 +580,8 @@ static void dist_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, 
 int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, DistTransport* tp,
              cudaStream_t s, const abft_inject_spec_t* inj_c, abft_report_t* rep, const abft_options_t* opt) {
     abft_options_t o = opt ? *opt : abft_options_t{1, 1, 64.0, 0, 0, ABFT_MODE_ENHANCED, 0};
-    if (o.K < 1 || !(o.c_tau > 0) || o.mode != ABFT_MODE_ENHANCED) return -11;   // dist: Enhanced only
+    if (o.K < 1 || !(o.c_tau > 0) || o.mode != ABFT_MODE_ENHANCED || o.order != ABFT_ORDER_RIGHT)
+        return -11;   // dist: Enhanced scheme, right-looking order
     std::vector<abft_inject_spec_t> inj;
     if (collect_inj(inj_c, n, nb, inj)) return -9;
     if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; }
@@ -836,10 +840,129 @@ extern "C" int abft_potrf_dist_sim(int64_t n, int64_t nb, int nranks, double* co
     return run_dist(n, nb, nranks, L.data(), nranks, nullptr, (cudaStream_t)stream, inj, rep, opt);
 }
 
+
+// ---- left-looking order (NEXT-1): MAGMA's Alg. 1 with Table I's verification ----
+// Iteration j: V7 re-verifies the L blocks the SYRK/GEMM will read (C = L[j,0:j] always, D =
+// L[j+1:,0:j] every K-th iteration: Opt. 3), V1/V2 the column to update; one launch updates block
+// column j with its checksum rows appended (A[j:N,j] -= L[j:N,0:j] L[j,0:j]^T, K = j*nb), V5
+// checks the updated column (fused partials), then POTRF + inverse, TRSM, V3 (and V4 for the
+// Online scheme), write-back. Single stream: the next column's update needs this panel.
+static int run_potrf_left(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t s,
+                          const std::vector<abft_inject_spec_t>& inj, abft_report_t* rep, const abft_options_t& o) {
+    const bool abft = o.abft_enabled != 0;
+    const int K = std::max(1, o.K);
+    const int mode = o.mode;
+    Work w;
+    int rc = work_alloc(w, n, nb, n, rep ? std::max<int64_t>(rep->cap, 1) : 1024, abft, s);
+    if (rc) return rc;
+    const int64_t N = w.N, B = nb;
+    const int32_t* ab = &w.st->abort;
+    const bool can_fuse = abft && mode != ABFT_MODE_OFFLINE && (nb % 128 == 0) && (lda % 2 == 0) &&
+                          (((uintptr_t)A & 15) == 0);
+    if (can_fuse) {
+        w.cs_nslab = n / 32;
+        ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n), s));
+    }
+    ThreadCache& tc = thread_cache();
+    cudaEvent_t e0 = nullptr, e1 = nullptr;
+    if (rep) { e0 = tc.timing.get(); e1 = tc.timing.get(); cudaEventRecord(e0, s); }
+    launch_zero(B, B, w.Li, B, s);
+    if (abft) {
+        launch_scales(n, nb, A, lda, w.scl, s);
+        StageArgs a = stage_base(w, A, lda, o.c_tau, SK_ALL, 0, -1);
+        a.encode = 1;
+        launch_check(a, s);
+    }
+    for (int64_t j = 0; j < N; ++j) {
+        const int64_t m = N - j - 1, mB = m * B;
+        const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
+        double* Ajj = A + j * B * lda + j * B;
+        const Loc L{A, lda, w.chk, w.ldc, w.W, ldw, mB};
+        if (abft) do_inject(inj, j, ABFT_HOOK_REST, B, L, ab, s);
+        if (abft && mode == ABFT_MODE_ENHANCED && j > 0) {                       // V7: C, D
+            StageArgs a = stage_base(w, A, lda, o.c_tau, SK_LEFT_L, ABFT_V7, (int)j);
+            a.factored = 1;
+            a.j_hi = (j % K == 0) ? N - j : 1;
+            launch_check(a, s);
+        }
+        if (abft && mode == ABFT_MODE_ENHANCED)
+            launch_check(stage_base(w, A, lda, o.c_tau, SK_COLUMN, ABFT_V2, (int)j), s);   // V1, V2
+        bool fused = false;
+        if (j > 0) {   // SYRK + GEMM of block column j, checksum rows as a second row segment
+            bool inj_here = false;
+            for (const auto& sp : inj) if (sp.k == j && sp.hook == ABFT_HOOK_UPDATE_OUT) inj_here = true;
+            ColSumOut cso{w.cs, n, w.cs_nslab, j * B, j * B, B, 64, j * B};
+            if (abft)
+                fused = launch_update_with_chk((N - j) * B, B, j * B, A + j * B, lda, A + j * B, lda, Ajj, lda,
+                                               2 * (N - j), w.chk + 2 * j, w.chk + j * B * w.ldc + 2 * j, w.ldc, B,
+                                               ab, s, (can_fuse && !inj_here) ? &cso : nullptr, w.ldc) == 1;
+            else
+                launch_gemm((N - j) * B, B, j * B, A + j * B, lda, A + j * B, lda, Ajj, lda, -1.0, 1.0, true, 1, 0,
+                            0, 0, 0, ab, s);
+            if (abft) do_inject(inj, j, ABFT_HOOK_UPDATE_OUT, B, L, ab, s);
+            if (abft && mode != ABFT_MODE_OFFLINE) {                              // V5: column j
+                StageArgs a = stage_base(w, A, lda, o.c_tau, SK_TRAIL, ABFT_V5, (int)j);
+                a.j_lo = j; a.j_hi = j + 1;
+                if (fused) {
+                    StageArgs d = a; d.kind = SK_TRAIL_DIAG;
+                    StageArgs f = a; f.kind = SK_TRAIL_OFF;
+                    f.cs = w.cs; f.cs_ld = n; f.cs_nslab = w.cs_nslab; f.cs_slab_rows = cso.slab_rows;
+                    launch_check_v5_fused(d, f, s);
+                } else {
+                    launch_check(a, s);
+                }
+            }
+        }
+        launch_chol_inv(Ajj, lda, w.Li, B, j * B, w.tmp, w.st, s);
+        launch_gemm(mB, B, B, Ajj + B, lda, w.Li, B, w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, s);
+        if (abft) {
+            launch_gemm(2 * m + 2, B, B, w.chk + j * B * w.ldc + 2 * j, w.ldc, w.Li, B, w.W + mB, ldw, 1.0, 0.0,
+                        true, 0, 1, 0, 0, 0, ab, s);
+            do_inject(inj, j, ABFT_HOOK_POTRF_OUT, B, L, ab, s);
+            if (mode != ABFT_MODE_OFFLINE) {
+                StageArgs a3 = stage_base(w, A, lda, o.c_tau, SK_DIAG_FACT, ABFT_V3, (int)j);
+                a3.ldw = ldw; a3.mB = mB;
+                launch_check(a3, s);                                              // V3
+            }
+            do_inject(inj, j, ABFT_HOOK_TRSM_OUT, B, L, ab, s);
+            if (mode == ABFT_MODE_ONLINE) {
+                StageArgs a4 = stage_base(w, A, lda, o.c_tau, SK_PANEL, ABFT_V4, (int)j);
+                a4.ldw = ldw; a4.mB = mB;
+                launch_check(a4, s);                                              // V4 (Online)
+            }
+        }
+        launch_copy(mB, B, w.W, ldw, Ajj + B, lda, ab, s);
+        if (abft) launch_copy(2 * m + 2, B, w.W + mB, ldw, w.chk + j * B * w.ldc + 2 * j, w.ldc, ab, s);
+    }
+    if (abft) {
+        const Loc L{A, lda, w.chk, w.ldc, w.W, 1, 0};
+        do_inject(inj, N, ABFT_HOOK_REST, B, L, ab, s);
+        StageArgs a6 = stage_base(w, A, lda, o.c_tau, SK_ALL, ABFT_V6, (int)N);
+        a6.factored = 1;
+        launch_check(a6, s);                                                      // V6
+    }
+    ABFT_CUDA_TRY(cudaGetLastError());
+    int status = 0;
+    if (rep) {
+        cudaEventRecord(e1, s);
+        rc = finish_report(w, rep, s, &status);
+        float ms = 0; cudaEventElapsedTime(&ms, e0, e1);
+        rep->seconds = ms * 1e-3;
+    }
+    work_free(w, s);
+    if (rc) return rc;
+    ABFT_CUDA_TRY(cudaGetLastError());
+    return status;
+}
+
+using RunFn = int (*)(int64_t, int64_t, double*, int64_t, cudaStream_t, const std::vector<abft_inject_spec_t>&,
+                      abft_report_t*, const abft_options_t&);
+
 static abft_options_t default_options() {
     abft_options_t o;
     memset(&o, 0, sizeof o);
     o.abft_enabled = 1; o.K = 1; o.c_tau = 64.0; o.lookahead = 0; o.profile = 0; o.mode = ABFT_MODE_ENHANCED;
+    o.order = ABFT_ORDER_RIGHT;
     return o;
 }
 
@@ -851,12 +974,14 @@ extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft
     abft_options_t o = opt ? *opt : default_options();
     if (o.K < 1 || !(o.c_tau > 0)) return -8;
     std::vector<abft_inject_spec_t> list;
-    if (collect_inj(inj, n, nb, list)) return -6;
+    if (collect_inj(inj, n, nb, list, o.order)) return -6;
     if (o.mode < ABFT_MODE_ENHANCED || o.mode > ABFT_MODE_OFFLINE) return -8;
+    if (o.order != ABFT_ORDER_RIGHT && o.order != ABFT_ORDER_LEFT) return -8;
+    const RunFn run = o.order == ABFT_ORDER_LEFT ? run_potrf_left : run_potrf;
     if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; rep->reruns = 0; }
     if (n == 0) return 0;
     cudaStream_t s = (cudaStream_t)stream;
-    if (o.mode == ABFT_MODE_ENHANCED || !o.abft_enabled) return run_potrf(n, nb, A, lda, s, list, rep, o);
+    if (o.mode == ABFT_MODE_ENHANCED || !o.abft_enabled) return run(n, nb, A, lda, s, list, rep, o);
     // Online / Offline: keep the input; an uncorrectable outcome or a detection by the final
     // sweep means an error propagated -> re-do the factorisation once, without the faults
     double* A0 = nullptr;
@@ -867,7 +992,7 @@ extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft
     memset(&r1, 0, sizeof r1);
     std::vector<abft_event_t> ev1(rep ? std::max<int64_t>(rep->cap, 4096) : 4096);
     r1.cap = (int64_t)ev1.size(); r1.events = ev1.data();
-    int st = run_potrf(n, nb, A, lda, s, list, &r1, o);
+    int st = run(n, nb, A, lda, s, list, &r1, o);
     bool v6 = false;
     for (int64_t e = 0; e < std::min<int64_t>(r1.n_events, r1.cap); ++e) v6 |= (ev1[e].check == ABFT_V6);
     abft_report_t r2;
@@ -879,7 +1004,7 @@ extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft
         ABFT_CUDA_TRY(cudaMemcpy2DAsync(A, lda * sizeof(double), A0, n * sizeof(double), n * sizeof(double), n,
                                         cudaMemcpyDeviceToDevice, s));
         const std::vector<abft_inject_spec_t> none;
-        st = run_potrf(n, nb, A, lda, s, none, &r2, o);
+        st = run(n, nb, A, lda, s, none, &r2, o);
         reruns = 1;
     }
     cudaFreeAsync(A0, s);

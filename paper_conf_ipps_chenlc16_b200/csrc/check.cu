@@ -167,6 +167,9 @@ __device__ int64_t block_argmax(const TileView& v, int64_t c, int64_t B, double*
 }
 
 struct Fix { double* p; double* p2; double val; };
+// corrections held per tile: one per column at most (a tile has nb columns); beyond this the tile
+// is reported UNCORRECTABLE
+constexpr int kMaxFix = 1024;
 
 // Phase 2: resolve the flagged columns in the oracle's order (tile, then column): decide
 // DATA / NONFINITE / CHK1 / CHK2 / UNCORRECTABLE, dedupe diagonal-tile mirrors, compute the
@@ -175,7 +178,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
     DevState* st = a.st;
     FlagList& FL = st->fl[a.flist];
     __shared__ int s_n;
-    __shared__ Fix s_fix[64];
+    __shared__ Fix s_fix[kMaxFix];
     __shared__ int s_nfix, s_unc, s_stop;
     __shared__ double redv[256];
     __shared__ long long redi[256];
@@ -249,7 +252,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
                 const double sum = block_sum(part, redv);
                 if (threadIdx.x == 0) {
                     const double val = __dsub_rn(v.c1[c * v.ldc], sum);   // A8
-                    if (s_nfix < 64) { s_fix[s_nfix].p = p; s_fix[s_nfix].p2 = nullptr; s_fix[s_nfix].val = val; s_nfix++; }
+                    if (s_nfix < kMaxFix) { s_fix[s_nfix].p = p; s_fix[s_nfix].p2 = nullptr; s_fix[s_nfix].val = val; s_nfix++; }
                     else s_unc = 1;
                     int64_t sr = row, sc = c;
                     if (v.diag && !v.factored && sr < sc) { const int64_t t = sr; sr = sc; sc = t; }
@@ -278,7 +281,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
                 st->n_detected++;
                 if (kind == ABFT_KIND_CHK1 || kind == ABFT_KIND_CHK2) {
                     if (kind == ABFT_KIND_CHK1) st->n_chk1++; else st->n_chk2++;
-                    if (s_nfix < 64) {
+                    if (s_nfix < kMaxFix) {
                         s_fix[s_nfix].p = kind == ABFT_KIND_CHK1 ? &v.c1[c * v.ldc] : &v.c2[c * v.ldc];
                         s_fix[s_nfix].p2 = nullptr;
                         s_fix[s_nfix].val = kind == ABFT_KIND_CHK1 ? f.r1 : f.r2;   // chk := v^T X

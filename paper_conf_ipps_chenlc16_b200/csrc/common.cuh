@@ -44,6 +44,7 @@ enum StageKind : int32_t {
     SK_ALL = 4,        // V6 / abft_verify: all tiles I >= J in A; factored per flag
     SK_TRAIL_OFF = 5,  // V5, off-diagonal trailing tiles, recalculation from the GEMM's fused partials
     SK_TRAIL_DIAG = 6, // V5, diagonal trailing tiles (J, J), J in [j_lo, j_hi), re-read as sym(tril)
+    SK_LEFT_L = 7,     // V7 (left-looking): L tiles (I, J), J < k, I in [k, k + j_hi), factored
 };
 
 struct StageArgs {
@@ -82,6 +83,7 @@ __host__ __device__ __forceinline__ int64_t stage_count(const StageArgs& a) {
             return hi <= lo ? 0 : (hi - lo) * N - (hi * (hi - 1) - lo * (lo - 1)) / 2;
         }
         case SK_TRAIL_DIAG: return a.j_hi > a.j_lo ? a.j_hi - a.j_lo : 0;
+        case SK_LEFT_L: return (int64_t)a.k * a.j_hi;
         case SK_TRAIL_OFF: {
             const int64_t lo = a.j_lo, hi = a.j_hi;
             return hi <= lo ? 0 : (hi - lo) * (N - 1) - (hi * (hi - 1) - lo * (lo - 1)) / 2;
@@ -98,6 +100,7 @@ __device__ __forceinline__ void stage_tile(const StageArgs& a, int64_t t, int64_
         case SK_DIAG_FACT: I = k; J = k; return;
         case SK_PANEL: I = k + 1 + t; J = k; return;
         case SK_TRAIL_DIAG: I = J = a.j_lo + t; return;
+        case SK_LEFT_L: J = t / a.j_hi; I = k + t % a.j_hi; return;
         case SK_TRAIL_OFF: {   // column-major over (I > J), J in [j_lo, j_hi)
             int64_t jj = a.j_lo, rem = t;
             while (rem >= N - jj - 1) { rem -= N - jj - 1; ++jj; }
@@ -223,4 +226,4 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s,
-                           abft::ColSumOut* cs);
+                           abft::ColSumOut* cs, int64_t lda2 = 0);

@@ -47,7 +47,7 @@ struct GemmArgs {
     // optional second row segment (ws kernel only): the checksum rows appended to the update as
     // extra GEMM rows. Rows [0, M2) of A2 (lda) update C2 (ldc2) under MASK_CHK with
     // q_tile0 = c_tile0 = 0; their tiles follow the first segment's tiles.
-    int64_t M2; const double* A2; double* C2; int64_t ldc2;
+    int64_t M2; const double* A2; double* C2; int64_t ldc2; int64_t lda2;
 };
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
@@ -489,7 +489,7 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
                 __syncwarp();
                 const int64_t k0 = (int64_t)kt * BK;
                 for (int kk = lane; kk < BK; kk += 32) {
-                    bulk_g2s(sA + st * C_::SA + kk * C_::PA, Ap + (k0 + kk) * g.lda + m0, rowsA * 8, &full[st]);
+                    bulk_g2s(sA + st * C_::SA + kk * C_::PA, Ap + (k0 + kk) * (T.seg2 ? g.lda2 : g.lda) + m0, rowsA * 8, &full[st]);
                     bulk_g2s(sB + st * C_::SB + kk * C_::PB, g.B + (k0 + kk) * g.ldb + n0, rowsB * 8, &full[st]);
                 }
             }
@@ -674,7 +674,7 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
     g.alpha = alpha; g.beta = beta; g.mask = mask; g.krange = krange; g.nb = nb;
     g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
     g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
-    g.M2 = 0; g.A2 = nullptr; g.C2 = nullptr; g.ldc2 = 1;
+    g.M2 = 0; g.A2 = nullptr; g.C2 = nullptr; g.ldc2 = 1; g.lda2 = 1;
     g.vecA = aligned16(A) && (lda % 2 == 0);
     g.vecB = aligned16(B) && (ldb % 2 == 0);
     auto tiles = [&](int64_t t) {
@@ -717,15 +717,17 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
 // partials were written.
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
-                           int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s, ColSumOut* cs) {
+                           int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s, ColSumOut* cs,
+                           int64_t lda2) {
+    if (lda2 <= 0) lda2 = lda;
     const bool ok = M > 0 && N > 0 && (M % 2 == 0) && (N % 2 == 0) && (M2 % 2 == 0) && (K % WsCfg::BK == 0) &&
                     aligned16(A) && aligned16(B) && aligned16(A2) && lda % 2 == 0 && ldb % 2 == 0 && N <= M &&
-                    M % WsCfg::BM == 0 && getenv("ABFT_GEMM_VARIANT") == nullptr;
+                    lda2 % 2 == 0 && M % WsCfg::BM == 0 && getenv("ABFT_GEMM_VARIANT") == nullptr;
     if (!ok) {
         const int f = launch_gemm(M, N, K, A, lda, B, ldb, C, ldc, -1.0, 1.0, true, MASK_LOWER, KR_FULL, 0, 0, 0,
                                   abort_flag, s, 0, cs);
         if (M2 > 0)
-            launch_gemm(M2, N, K, A2, lda, B, ldb, C2, ldc2, -1.0, 1.0, true, MASK_CHK, KR_FULL, nb, 0, 0, abort_flag, s);
+            launch_gemm(M2, N, K, A2, lda2, B, ldb, C2, ldc2, -1.0, 1.0, true, MASK_CHK, KR_FULL, nb, 0, 0, abort_flag, s);
         return f;
     }
     GemmArgs g;
@@ -737,7 +739,7 @@ int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int
     if (cs && cs->nb % WsCfg::BM == 0 && cs->row0 % WsCfg::BM == 0 && cs->colg0 % WsCfg::BN == 0) {
         g.cs = *cs; fused = 1;
     }
-    g.M2 = M2; g.A2 = A2; g.C2 = C2; g.ldc2 = ldc2;
+    g.M2 = M2; g.A2 = A2; g.C2 = C2; g.ldc2 = ldc2; g.lda2 = lda2;
     run_ws_any(g, s);
     if (fused) cs->slab_rows = ws_slab_rows();
     return fused;

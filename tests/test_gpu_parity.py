@@ -296,3 +296,60 @@ def test_schemes_match_oracle(P, mode, fault):
     else:   # after propagation the first run's event list depends on rounding; the decision does not
         assert rep["n_events"] > 0
     assert floor_rel(L, ref.L, A) <= 1e-11
+
+
+# ---- NEXT-1: left-looking order (MAGMA Alg. 1) with Table I's verification --------------------
+@pytest.mark.parametrize("n,nb", [(1024, 128), (2048, 256), (512, 64), (96, 24)])
+def test_left_looking_fault_free(P, n, nb):
+    A = syn.spd_matrix(n)
+    ref = oracle.potrf(A, nb, order="left")
+    st, rep, L = run_gpu(P, A, nb, opt=P.options(order="left"))
+    assert st == 0 and rep["n_events"] == 0
+    assert rep["n_checks"] == ref.counts["n_checks"]
+    assert floor_rel(L, ref.L, A) <= 1e-11
+    assert backward_error(A, L) <= 10 * n * EPS
+
+
+@pytest.mark.parametrize("K", [1, 3])
+def test_left_looking_injections(P, K):
+    n, nb = 1024, 128
+    A = syn.spd_matrix(n)
+    specs = [dict(k=2, hook="REST", row=900, col=130, bit=50),
+             dict(k=3, hook="TRSM_OUT", row=700, col=3 * nb + 5, bit=50),
+             dict(k=4, hook="UPDATE_OUT", row=800, col=4 * nb + 9, bit=52),
+             dict(k=5, hook="POTRF_OUT", row=5 * nb + 9, col=5 * nb + 2, bit=52),
+             dict(k=1, hook="REST", row=1000, col=7 * nb + 3, bit=50),
+             dict(k=8, hook="REST", row=600, col=300, bit=50)]
+    inj = syn.inj_array(specs)
+    ref = oracle.potrf(A, nb, inj=inj, order="left", K=K)
+    st, rep, L = run_gpu(P, A, nb, inj=inj, opt=P.options(order="left", K=K))
+    assert st == ref.status == 0
+    assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
+    assert floor_rel(L, ref.L, A) <= 1e-11
+
+
+def test_left_looking_c1_golden_exact(P):
+    A = syn.pascal_mod2(256)
+    specs = [dict(k=2, hook="REST", row=232, col=40, bit=52), dict(k=4, hook="UPDATE_OUT", row=230, col=130, bit=51)]
+    inj = syn.inj_array(specs)
+    ref = oracle.potrf(A, 32, inj=inj, order="left")
+    st, rep, L = run_gpu(P, A, 32, inj=inj, opt=P.options(order="left"))
+    assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
+    i = np.arange(256)
+    assert np.array_equal(np.tril(L), ((i[:, None] & i[None, :]) == i[None, :]).astype(float))
+
+
+@pytest.mark.parametrize("mode", ["online", "offline"])
+def test_left_looking_schemes(P, mode):
+    from tests.test_oracle_pins import SCHEME_FAULTS
+    n, nb = 1024, 128
+    A = syn.spd_matrix(n)
+    # left-looking: the update of iteration k writes block column k
+    faults = {"computation": [dict(k=2, hook="UPDATE_OUT", row=800, col=2 * nb + 10, bit=50)],
+              "memory": SCHEME_FAULTS["memory"]}
+    for fault in ("computation", "memory"):
+        inj = syn.inj_array(faults[fault])
+        ref = oracle.potrf(A, nb, inj=inj, mode=mode, order="left")
+        st, rep, L = run_gpu(P, A, nb, inj=inj, opt=P.options(mode=mode, order="left"))
+        assert st == ref.status == 0 and rep["reruns"] == ref.reruns
+        assert floor_rel(L, ref.L, A) <= 1e-11
