@@ -277,6 +277,16 @@ def main():
                             "injections": len(specs), "events": int(r0["n_events"]),
                             "corrected": int(r0["n_data"] + r0["n_nonfinite"] + r0["n_chk1"] + r0["n_chk2"]),
                             "uncorrectable": int(r0["n_uncorrectable"])}
+        # NEXT-1: the paper's own left-looking order (MAGMA Alg. 1) with Table I's verification, and
+        # Opt. 3 (verify every K iterations), next to the right-looking default
+        orders = {}
+        for order in ("right", "left"):
+            for abft_on, Kv in ((True, 1), (True, 3), (False, 1)):
+                to, ro = run_steps(P.options(abft_enabled=abft_on, K=Kv, order=order), steps=1, warmup=1)
+                orders[f"{order}_{'abft' if abft_on else 'off'}_K{Kv}"] = {
+                    "ms": round(to[0], 2), "value": round(flops / (to[0] * 1e-3) / 1e9, 1),
+                    "tile_checks": int(ro[0]["n_checks"])}
+        line["orders"] = orders
         # Table VII/VIII analog on B200 (NEXT-2): the three schemes x {no error, computation error,
         # memory error between verification and access}; Online/Offline re-do the factorisation
         # when an error propagated
