@@ -187,7 +187,9 @@ int abft_potrf_dist(int64_t n, int64_t nb, double* A_local, int64_t lda_local, v
                     abft_report_t* rep, const abft_options_t* opt);
 /* abft_potrf_dist errors: -1 n, -2 nb, -3 A_local, -4 lda_local, -5 comm (or its rank/size
  * disagree with rank/nranks), -6 rank, -7 nranks, -9 inj, -11 options; ABFT_ERR_NCCL on a failed
- * collective. No look-ahead across ranks yet. */
+ * collective. Depth-1 look-ahead across ranks: the owner of block column k+1 updates it first and
+ * factors + broadcasts panel k+1 on a high-priority stream while every rank finishes update k
+ * (DESIGN.md §5). */
 
 /* Test harness of the multi-GPU algorithm on ONE device: runs the nranks ranks of
  * abft_potrf_dist in one process, in lock-step, with the NCCL broadcast replaced by device-to-

@@ -546,6 +546,7 @@ struct RankState {
     int64_t nblk, ncl;        // local block columns, local columns
     Work w;
     double* xslot = nullptr;  // abort flag slot right after the packed panel inside W
+    double* Wb[2] = {nullptr, nullptr};   // double-buffered panel (look-ahead)
 };
 }
 
@@ -635,99 +636,207 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             launch_check(a, s);
         }
     }
-    int64_t dist_slab_rows = 64;
-    for (int64_t k = 0; k < N; ++k) {
-        const int owner = (int)(k % P);
-        const int64_t m = N - k - 1, mB = m * B;
-        const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
-        const size_t wcount = (size_t)(ldw * B);
-        for (auto& q : R) if (abft) dist_inject(inj, k, ABFT_HOOK_REST, B, P, q, ldw, mB, s);
-        for (auto& q : R) {
-            if (q.r != owner) continue;
-            const int32_t* ab = &q.w.st->abort;
-            double* Akk = q.A + dist_lc(k, P, B) * q.lda + k * B;
-            double* ckk = q.w.chk + dist_lc(k, P, B) * q.w.ldc;
-            q.xslot = q.w.W + wcount;
-            if (abft) launch_check(stage(q, SK_COLUMN, ABFT_V2, (int)k), s);          // V1, V2
-            launch_chol_inv(Akk, q.lda, q.w.Li, B, k * B, q.w.tmp, q.w.st, s);
-            launch_gemm(mB, B, B, Akk + B, q.lda, q.w.Li, B, q.w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, s);
-            if (abft) {
-                launch_gemm(2 * m + 2, B, B, ckk + 2 * k, q.w.ldc, q.w.Li, B, q.w.W + mB, ldw, 1.0, 0.0, true, 0, 1,
-                            0, 0, 0, ab, s);
-                dist_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, P, q, ldw, mB, s);
-                StageArgs a3 = stage(q, SK_DIAG_FACT, ABFT_V3, (int)k);
-                a3.ldw = ldw; a3.mB = mB;
-                launch_check(a3, s);                                                   // V3
-                dist_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, P, q, ldw, mB, s);
-                StageArgs a4 = stage(q, SK_PANEL, ABFT_V4, (int)k);
-                a4.ldw = ldw; a4.mB = mB;
-                launch_check(a4, s);                                                   // V4
-            }
-            launch_copy(mB, B, q.w.W, ldw, Akk + B, q.lda, ab, s);
-            if (abft) launch_copy(2 * m + 2, B, q.w.W + mB, ldw, ckk + 2 * k, q.w.ldc, ab, s);
-            launch_abort_to_slot(ab, q.xslot, s);
+    // ---- look-ahead across ranks: the owner of block column k+1 updates that
+    // column with panel k first, then factors it and broadcasts panel k+1 on its panel stream
+    // while every rank applies the rest of update k on its main stream. Panel + broadcast + V4R
+    // run on the panel stream PS (high priority), updates + V5 on the main stream (the caller's).
+    // Single-process simulation: every rank shares the two streams; the broadcast is a device copy
+    // issued on the owner's panel stream.
+    ThreadCache& tc = thread_cache();
+    cudaStream_t PS = tc.P;
+    auto new_event = [&]() { return tc.sync.get(); };
+    {   // panel stream starts after the encode
+        cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(PS, e, 0);
+    }
+    for (auto& q : R) {   // second panel buffer per rank (W of iteration k lives in Wb[k & 1])
+        const int64_t wrows = (N - 1) * nb + 2 * N + 2;
+        q.Wb[0] = q.w.W;
+        ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.Wb[1], sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb + 1), s));
+    }
+    {   // Wb[1] allocated on s: the panel stream must see it
+        cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(PS, e, 0);
+    }
+    auto geom = [&](int64_t k, int64_t& m, int64_t& mB, int64_t& ldw) {
+        m = N - k - 1; mB = m * B; ldw = std::max<int64_t>(1, mB + 2 * m + 2);
+    };
+    // injections of hook REST(k) split by block column: inside [jlo, jhi) or outside it
+    auto rest_inject = [&](RankState& q, int64_t k, int64_t jlo, int64_t jhi, bool inside, cudaStream_t st) {
+        std::vector<abft_inject_spec_t> sub;
+        for (const auto& sp : inj) {
+            if (sp.k != k || sp.hook != ABFT_HOOK_REST) continue;
+            const int64_t J = sp.col / nb;
+            if ((J >= jlo && J < jhi) == inside) sub.push_back(sp);
         }
-        if (m == 0) continue;
-        // ---- broadcast of the packed panel (+ abort slot) from the owner ----
+        if (!sub.empty()) dist_inject(sub, k, ABFT_HOOK_REST, B, P, q, 1, 0, st);
+    };
+    // the panel of iteration k on the owner's panel stream (V1/V2, POTRF + inverse, TRSM with
+    // Alg. 2 rows, V3, V4, write-back, abort slot) into Wb[k & 1]
+    auto panel = [&](RankState& q, int64_t k) {
+        int64_t m, mB, ldw; geom(k, m, mB, ldw);
+        q.w.W = q.Wb[k & 1];
+        const size_t wcount = (size_t)(ldw * B);
+        const int32_t* ab = &q.w.st->abort;
+        double* Akk = q.A + dist_lc(k, P, B) * q.lda + k * B;
+        double* ckk = q.w.chk + dist_lc(k, P, B) * q.w.ldc;
+        if (abft) {
+            rest_inject(q, k, k, k + 1, true, PS);                                    // REST(k), column k
+            StageArgs a = stage(q, SK_COLUMN, ABFT_V2, (int)k); a.flist = 1;
+            launch_check(a, PS);                                                     // V1, V2
+        }
+        launch_chol_inv(Akk, q.lda, q.w.Li, B, k * B, q.w.tmp, q.w.st, PS);
+        launch_gemm(mB, B, B, Akk + B, q.lda, q.w.Li, B, q.w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, PS);
+        if (abft) {
+            launch_gemm(2 * m + 2, B, B, ckk + 2 * k, q.w.ldc, q.w.Li, B, q.w.W + mB, ldw, 1.0, 0.0, true, 0, 1,
+                        0, 0, 0, ab, PS);
+            dist_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, P, q, ldw, mB, PS);
+            StageArgs a3 = stage(q, SK_DIAG_FACT, ABFT_V3, (int)k);
+            a3.ldw = ldw; a3.mB = mB; a3.flist = 1;
+            launch_check(a3, PS);                                                    // V3
+            dist_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, P, q, ldw, mB, PS);
+            StageArgs a4 = stage(q, SK_PANEL, ABFT_V4, (int)k);
+            a4.ldw = ldw; a4.mB = mB; a4.flist = 1;
+            launch_check(a4, PS);                                                    // V4
+        }
+        launch_copy(mB, B, q.w.W, ldw, Akk + B, q.lda, ab, PS);
+        if (abft) launch_copy(2 * m + 2, B, q.w.W + mB, ldw, ckk + 2 * k, q.w.ldc, ab, PS);
+        launch_abort_to_slot(ab, q.w.W + wcount, PS);
+    };
+    // broadcast of panel k (+ abort slot) from its owner, then every receiver's RECV hook and V4R;
+    // afterwards evB[rank] marks "panel k usable on this rank"
+    std::vector<cudaEvent_t> evU(nlocal, nullptr), evUprev(nlocal, nullptr);   // after update k / k-1
+    std::vector<cudaEvent_t> evB(nlocal, nullptr);
+    auto bcast = [&](int64_t k) -> int {
+        int64_t m, mB, ldw; geom(k, m, mB, ldw);
+        const size_t wcount = (size_t)(ldw * B);
+        const int owner = (int)(k % P);
+        for (int i = 0; i < nlocal; ++i)   // the receive buffer Wb[k & 1] was last read by update k-2
+            if (evUprev[i]) cudaStreamWaitEvent(PS, evUprev[i], 0);
         if (tp) {
-            if (tp->bcast(R[0].w.W, (wcount + 1) * sizeof(double), owner, s)) return ABFT_ERR_NCCL;
+            if (tp->bcast(R[0].Wb[k & 1], (wcount + 1) * sizeof(double), owner, PS)) return ABFT_ERR_NCCL;
         } else {
             const RankState* src = nullptr;
             for (auto& q : R) if (q.r == owner) src = &q;
             for (auto& q : R)
                 if (q.r != owner)
-                    cudaMemcpyAsync(q.w.W, src->w.W, (wcount + 1) * sizeof(double), cudaMemcpyDeviceToDevice, s);
+                    cudaMemcpyAsync(q.Wb[k & 1], src->Wb[k & 1], (wcount + 1) * sizeof(double), cudaMemcpyDeviceToDevice, PS);
         }
-        for (auto& q : R) {
-            if (q.r == owner) continue;
-            launch_abort_from_slot(q.w.W + wcount, q.w.st, s);
-            if (abft) {
-                dist_inject(inj, k, ABFT_HOOK_RECV, B, P, q, ldw, mB, s);
-                StageArgs a = stage(q, SK_PANEL, ABFT_V4R, (int)k);                   // V4R
-                a.ldw = ldw; a.mB = mB; a.col_owner_mod = 1; a.col_owner_rank = 0;
-                launch_check(a, s);
-            }
-        }
-        // ---- trailing update of each rank's own block columns ----
-        const bool gated = ((k + 1) % K == 0) || k == N - 2;
-        for (auto& q : R) {
-            const int32_t* ab = &q.w.st->abort;
-            bool inj_here = false;
-            for (const auto& sp : inj)
-                if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && (sp.col / B) % P == q.r) inj_here = true;
-            bool all_fused = q.w.cs != nullptr && !inj_here;
-            for (int64_t J = k + 1; J < N; ++J) {
-                if (J % P != q.r) continue;
-                const int64_t t = J / P;
-                double* W0 = q.w.W + (J - k - 1) * B;
-                double* C = q.A + t * B * q.lda + J * B;
-                ColSumOut cso{q.w.cs, q.ncl, q.w.cs_nslab, J * B, t * B, B, 64, J * B};
-                int f;
-                if (abft)
-                    f = launch_update_with_chk((N - J) * B, B, B, W0, ldw, W0, ldw, C, q.lda, 2 * (N - J),
-                                               q.w.W + mB + 2 + 2 * (J - k - 1), q.w.chk + t * B * q.w.ldc + 2 * J,
-                                               q.w.ldc, B, ab, s, all_fused ? &cso : nullptr);
-                else
-                    f = launch_gemm((N - J) * B, B, B, W0, ldw, W0, ldw, C, q.lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
-                if (f != 1) all_fused = false;
-                if (f == 1) dist_slab_rows = cso.slab_rows;
-            }
-            if (!abft) continue;
-            dist_inject(inj, k, ABFT_HOOK_UPDATE_OUT, B, P, q, ldw, mB, s);
-            if (gated) {
-                StageArgs a = stage(q, SK_TRAIL, ABFT_V5, (int)k);
-                a.j_lo = k + 1; a.j_hi = N;
-                if (all_fused) {
-                    StageArgs d = a; d.kind = SK_TRAIL_DIAG;
-                    StageArgs f = a; f.kind = SK_TRAIL_OFF;
-                    f.cs = q.w.cs; f.cs_ld = q.ncl; f.cs_nslab = q.w.cs_nslab; f.cs_slab_rows = dist_slab_rows;
-                    launch_check_v5_fused(d, f, s);                                    // V5 (fused)
-                } else {
-                    launch_check(a, s);                                                // V5
+        for (int i = 0; i < nlocal; ++i) {
+            RankState& q = R[i];
+            q.w.W = q.Wb[k & 1];
+            if (q.r != owner) {
+                launch_abort_from_slot(q.w.W + wcount, q.w.st, PS);
+                if (abft) {
+                    dist_inject(inj, k, ABFT_HOOK_RECV, B, P, q, ldw, mB, PS);
+                    StageArgs a = stage(q, SK_PANEL, ABFT_V4R, (int)k);               // V4R
+                    a.ldw = ldw; a.mB = mB; a.col_owner_mod = 1; a.col_owner_rank = 0; a.flist = 1;
+                    launch_check(a, PS);
                 }
             }
+            evB[i] = new_event(); cudaEventRecord(evB[i], PS);
+        }
+        return 0;
+    };
+    int64_t dist_slab_rows = 64;
+    // trailing update of iteration k on rank q's block columns J in [jlo, jhi) (main stream),
+    // UPDATE_OUT hook and V5 of those columns
+    auto update = [&](RankState& q, int64_t k, int64_t jlo, int64_t jhi) {
+        int64_t m, mB, ldw; geom(k, m, mB, ldw);
+        double* W = q.Wb[k & 1];
+        const int32_t* ab = &q.w.st->abort;
+        bool any = false, inj_here = false;
+        for (int64_t J = jlo; J < jhi; ++J) any = any || (J % P == q.r);
+        if (!any) return;
+        for (const auto& sp : inj)
+            if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && (sp.col / B) % P == q.r && sp.col / B >= jlo &&
+                sp.col / B < jhi)
+                inj_here = true;
+        bool all_fused = q.w.cs != nullptr && !inj_here;
+        // the owned block columns J in [jlo, jhi) are J0, J0 + P, ...: one launch whose column
+        // block t is global block J0 + t P (cstride), checksum rows appended as its second segment
+        int64_t J0 = jlo;
+        while (J0 % P != q.r) ++J0;
+        const int64_t nt = (jhi - 1 - J0) / P + 1, t0 = J0 / P;
+        double* W0 = W + (J0 - k - 1) * B;
+        double* C = q.A + t0 * B * q.lda + J0 * B;
+        ColSumOut cso{q.w.cs, q.ncl, q.w.cs_nslab, J0 * B, t0 * B, B, 64, J0 * B};
+        const int f = abft ? launch_update_with_chk((N - J0) * B, nt * B, B, W0, ldw, W0, ldw, C, q.lda, 2 * (N - J0),
+                                                    W + mB + 2 + 2 * (J0 - k - 1), q.w.chk + t0 * B * q.w.ldc + 2 * J0,
+                                                    q.w.ldc, B, ab, s, all_fused ? &cso : nullptr, 0, P)
+                           : launch_update_with_chk((N - J0) * B, nt * B, B, W0, ldw, W0, ldw, C, q.lda, 0, W0, C,
+                                                    q.lda, B, ab, s, nullptr, 0, P);
+        if (f < 0) {   // shapes the strided launch cannot take (or ABFT off): one launch per block column
+            for (int64_t J = J0; J < jhi; J += P) {
+                const int64_t t = J / P;
+                double* Wj = W + (J - k - 1) * B;
+                double* Cj = q.A + t * B * q.lda + J * B;
+                ColSumOut csj{q.w.cs, q.ncl, q.w.cs_nslab, J * B, t * B, B, 64, J * B};
+                int fj;
+                if (abft)
+                    fj = launch_update_with_chk((N - J) * B, B, B, Wj, ldw, Wj, ldw, Cj, q.lda, 2 * (N - J),
+                                                W + mB + 2 + 2 * (J - k - 1), q.w.chk + t * B * q.w.ldc + 2 * J,
+                                                q.w.ldc, B, ab, s, all_fused ? &csj : nullptr);
+                else
+                    fj = launch_gemm((N - J) * B, B, B, Wj, ldw, Wj, ldw, Cj, q.lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
+                if (fj != 1) all_fused = false;
+                if (fj == 1) dist_slab_rows = csj.slab_rows;
+            }
+        } else {
+            if (f != 1) all_fused = false;
+            if (f == 1) dist_slab_rows = cso.slab_rows;
+        }
+        if (!abft) return;
+        {   // UPDATE_OUT injections of this rank inside [jlo, jhi)
+            std::vector<abft_inject_spec_t> sub;
+            for (const auto& sp : inj)
+                if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && sp.col / B >= jlo && sp.col / B < jhi) sub.push_back(sp);
+            if (!sub.empty()) dist_inject(sub, k, ABFT_HOOK_UPDATE_OUT, B, P, q, ldw, mB, s);
+        }
+        const bool gated = ((k + 1) % K == 0) || k == N - 2;
+        if (!gated) return;
+        StageArgs a = stage(q, SK_TRAIL, ABFT_V5, (int)k);
+        a.j_lo = jlo; a.j_hi = jhi; a.flist = 0;
+        if (all_fused) {
+            StageArgs d = a; d.kind = SK_TRAIL_DIAG;
+            StageArgs f = a; f.kind = SK_TRAIL_OFF;
+            f.cs = q.w.cs; f.cs_ld = q.ncl; f.cs_nslab = q.w.cs_nslab; f.cs_slab_rows = dist_slab_rows;
+            launch_check_v5_fused(d, f, s);                                            // V5 (fused)
+        } else {
+            launch_check(a, s);                                                        // V5
+        }
+    };
+
+    if (abft) for (auto& q : R) rest_inject(q, 0, 0, 1, false, s);   // REST(0) outside column 0
+    {   // P streams see those injections before the first panel
+        cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(PS, e, 0);
+    }
+    for (auto& q : R) if (q.r == 0) panel(q, 0);
+    if (N > 1) { int rc2 = bcast(0); if (rc2) return rc2; }
+    for (int64_t k = 0; k + 1 < N; ++k) {
+        for (int i = 0; i < nlocal; ++i) cudaStreamWaitEvent(s, evB[i], 0);      // panel k usable
+        const int o1 = (int)((k + 1) % P);
+        // (a) block column k+1 on its owner: update, UPDATE_OUT, V5 -> panel k+1 on PS
+        for (auto& q : R) {
+            if (q.r != o1) continue;
+            update(q, k, k + 1, k + 2);
+            cudaEvent_t ec = new_event(); cudaEventRecord(ec, s); cudaStreamWaitEvent(PS, ec, 0);
+            panel(q, k + 1);
+        }
+        // (b) the rest of update k on every rank (the owner of k+1 included)
+        for (auto& q : R) update(q, k, k + 2, N);
+        for (int i = 0; i < nlocal; ++i) { evUprev[i] = evU[i]; evU[i] = new_event(); cudaEventRecord(evU[i], s); }
+        // (c) REST(k+1) outside block column k+1 (column k+1's share was applied on PS)
+        if (abft) for (auto& q : R) rest_inject(q, k + 1, k + 1, k + 2, false, s);
+        // (d) broadcast panel k+1 (receivers wait for their update k-1 ... k to release the buffer)
+        if (k + 2 < N) {   // Wb[(k+1) & 1] was last read by update k-1 (evUprev)
+            int rc2 = bcast(k + 1); if (rc2) return rc2;
+        } else {
+            for (int i = 0; i < nlocal; ++i) { evB[i] = new_event(); cudaEventRecord(evB[i], PS); }
         }
     }
+    {   // main stream waits for the last panel
+        cudaEvent_t e = new_event(); cudaEventRecord(e, PS); cudaStreamWaitEvent(s, e, 0);
+    }
+    for (auto& q : R) { if (q.Wb[1]) cudaFreeAsync(q.Wb[1], s); q.Wb[1] = nullptr; q.w.W = q.Wb[0]; }
     if (abft) {
         for (auto& q : R) {
             dist_inject(inj, N, ABFT_HOOK_REST, B, P, q, 1, 0, s);

@@ -223,7 +223,9 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
                 int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
                 cudaStream_t s, int force_tile = 0, abft::ColSumOut* cs = nullptr);
 // The trailing update with the checksum rows as a second row segment of the same launch.
+// cstride > 1: C's column block t (and the B operand's row block t) is global block t * cstride
+// (a rank's 1D block-cyclic local columns in one launch); returns -1 if the shapes do not allow it.
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s,
-                           abft::ColSumOut* cs, int64_t lda2 = 0);
+                           abft::ColSumOut* cs, int64_t lda2 = 0, int64_t cstride = 1);

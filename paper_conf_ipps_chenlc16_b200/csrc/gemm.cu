@@ -48,6 +48,9 @@ struct GemmArgs {
     // extra GEMM rows. Rows [0, M2) of A2 (lda) update C2 (ldc2) under MASK_CHK with
     // q_tile0 = c_tile0 = 0; their tiles follow the first segment's tiles.
     int64_t M2; const double* A2; double* C2; int64_t ldc2; int64_t lda2;
+    // column-block stride (ws kernel, MASK_LOWER + checksum segment): column block t of C and of
+    // the B operand's rows is global block t * cstride (1D block-cyclic local columns; 1 = dense)
+    int64_t cstride;
 };
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
@@ -410,7 +413,15 @@ __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t 
         tm = e / TN; tn = e % TN;
         T.m0 = tm * BM; T.n0 = tn * BN; T.seg2 = true;
         const int64_t qmax = min(g.M2, T.m0 + BM) - 1;
-        return qmax / 2 >= T.n0 / g.nb;
+        return qmax / 2 >= (T.n0 / g.nb) * g.cstride;
+    }
+    if (g.mask == MASK_LOWER && g.cstride > 1) {   // strided columns: grouped rectangle, skip tiles above
+        const int64_t q = idx / (kWsGroup * TN), a0 = q * kWsGroup, Gp = ((TM - a0) < kWsGroup ? (TM - a0) : (int64_t)kWsGroup);
+        const int64_t e = idx - a0 * TN;
+        tn = e / Gp; tm = a0 + e % Gp;
+        T.m0 = tm * BM; T.n0 = tn * BN; T.seg2 = false;
+        const int64_t rmax = min(g.M, T.m0 + BM) - 1;
+        return rmax >= T.n0 + (T.n0 / g.nb) * g.nb * (g.cstride - 1);
     }
     if (g.mask == MASK_LOWER) {
         // group q: the last q with lower_prefix(q G) <= idx
@@ -475,6 +486,7 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
             double* Cp = T.seg2 ? g.C2 : g.C;
             const int64_t ldcp = T.seg2 ? g.ldc2 : g.ldc;
             const uint32_t rowsA = (uint32_t)(Ms - m0 < BM ? Ms - m0 : BM), rowsB = (uint32_t)(g.N - n0 < BN ? g.N - n0 : BN);
+            const int64_t bn0 = n0 + (g.cstride > 1 ? (n0 / g.nb) * g.nb * (g.cstride - 1) : 0);   // B row of column n0
             // warm L2 with the C columns of this tile (they are read at the tile's start)
             if (g.beta != 0.0) {
                 for (int c = lane; c < (int)rowsB; c += 32) prefetch_l2(Cp + (n0 + c) * ldcp + m0, rowsA * 8);
@@ -490,7 +502,7 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
                 const int64_t k0 = (int64_t)kt * BK;
                 for (int kk = lane; kk < BK; kk += 32) {
                     bulk_g2s(sA + st * C_::SA + kk * C_::PA, Ap + (k0 + kk) * (T.seg2 ? g.lda2 : g.lda) + m0, rowsA * 8, &full[st]);
-                    bulk_g2s(sB + st * C_::SB + kk * C_::PB, g.B + (k0 + kk) * g.ldb + n0, rowsB * 8, &full[st]);
+                    bulk_g2s(sB + st * C_::SB + kk * C_::PB, g.B + (k0 + kk) * g.ldb + bn0, rowsB * 8, &full[st]);
                 }
             }
         }
@@ -512,6 +524,7 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
         // ownership of element (r, c): r < Mlim and r >= rmin(c), rmin precomputed per owned column
         // (no per-element 64-bit division: the epilogue must stay short and I-cache friendly)
         const int64_t Mlim = seg2 ? g.M2 : g.M;
+        const int64_t cshift = g.cstride > 1 ? (n0 / g.nb) * g.nb * (g.cstride - 1) : 0;   // global - local col
         int64_t rmin[C_::FN][2];
 #pragma unroll
         for (int j = 0; j < C_::FN; ++j)
@@ -520,8 +533,8 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
                 const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
                 int64_t v;
                 if (c >= g.N) v = INT64_MAX;
-                else if (seg2) v = 2 * (c / g.nb);                                   // q/2 >= c/nb
-                else if (g.mask == MASK_LOWER) v = c;                                 // r >= c
+                else if (seg2) v = 2 * (c / g.nb) * g.cstride;                       // q/2 >= block of c
+                else if (g.mask == MASK_LOWER) v = c + cshift;                        // r >= global c
                 else if (g.mask == MASK_CHK) v = 2 * (g.c_tile0 + c / g.nb - g.q_tile0);
                 else v = 0;
                 rmin[j][h] = v;
@@ -582,7 +595,7 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
             const int64_t gr0 = g.cs.row0 + m0 + wm * WM, gc0 = g.cs.col0 + n0;
             // warp-uniform; the shuffles below stay outside any branch so that they compile to
             // plain SHFLs (inside a possibly divergent branch they become WARPSYNC collectives)
-            const bool offdiag = gr0 / g.cs.nb != (g.cs.colg0 + n0) / g.cs.nb;
+            const bool offdiag = gr0 / g.cs.nb != (g.cs.colg0 + n0 + cshift) / g.cs.nb;
             const int64_t wbase = gr0 % g.cs.nb + fr + 1;   // weight (1-based) of row i = 0
             const int64_t slab = gr0 / g.cs.slab_rows;
             __syncwarp();
@@ -620,7 +633,7 @@ static int run_ws(GemmArgs g, cudaStream_t s) {
     }
     const int64_t tm = (g.M + C_::BM - 1) / C_::BM, tn = (g.N + C_::BN - 1) / C_::BN;
     g.tiles_n = tn;
-    const int64_t n1 = (g.mask == MASK_LOWER) ? lower_prefix<C_::BM / C_::BN>(tm, tn) : tm * tn;
+    const int64_t n1 = (g.mask == MASK_LOWER && g.cstride <= 1) ? lower_prefix<C_::BM / C_::BN>(tm, tn) : tm * tn;
     const int64_t ntiles = n1 + (g.M2 > 0 ? ((g.M2 + C_::BM - 1) / C_::BM) * tn : 0);
     if (ntiles <= 0) return 0;
     // tiles per CTA: 1 lets the block scheduler interleave the high-priority look-ahead stream's
@@ -674,7 +687,7 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
     g.alpha = alpha; g.beta = beta; g.mask = mask; g.krange = krange; g.nb = nb;
     g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
     g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
-    g.M2 = 0; g.A2 = nullptr; g.C2 = nullptr; g.ldc2 = 1; g.lda2 = 1;
+    g.M2 = 0; g.A2 = nullptr; g.C2 = nullptr; g.ldc2 = 1; g.lda2 = 1; g.cstride = 1;
     g.vecA = aligned16(A) && (lda % 2 == 0);
     g.vecB = aligned16(B) && (ldb % 2 == 0);
     auto tiles = [&](int64_t t) {
@@ -718,11 +731,14 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s, ColSumOut* cs,
-                           int64_t lda2) {
+                           int64_t lda2, int64_t cstride) {
     if (lda2 <= 0) lda2 = lda;
+    if (cstride < 1) cstride = 1;
     const bool ok = M > 0 && N > 0 && (M % 2 == 0) && (N % 2 == 0) && (M2 % 2 == 0) && (K % WsCfg::BK == 0) &&
                     aligned16(A) && aligned16(B) && aligned16(A2) && lda % 2 == 0 && ldb % 2 == 0 && N <= M &&
-                    lda2 % 2 == 0 && M % WsCfg::BM == 0 && getenv("ABFT_GEMM_VARIANT") == nullptr;
+                    lda2 % 2 == 0 && M % WsCfg::BM == 0 && getenv("ABFT_GEMM_VARIANT") == nullptr &&
+                    (cstride == 1 || nb % WsCfg::BN == 0);
+    if (!ok && cstride > 1) return -1;   // strided columns need the warp-specialised kernel
     if (!ok) {
         const int f = launch_gemm(M, N, K, A, lda, B, ldb, C, ldc, -1.0, 1.0, true, MASK_LOWER, KR_FULL, 0, 0, 0,
                                   abort_flag, s, 0, cs);
@@ -739,7 +755,7 @@ int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int
     if (cs && cs->nb % WsCfg::BM == 0 && cs->row0 % WsCfg::BM == 0 && cs->colg0 % WsCfg::BN == 0) {
         g.cs = *cs; fused = 1;
     }
-    g.M2 = M2; g.A2 = A2; g.C2 = C2; g.ldc2 = ldc2; g.lda2 = lda2;
+    g.M2 = M2; g.A2 = A2; g.C2 = C2; g.ldc2 = ldc2; g.lda2 = lda2; g.cstride = cstride;
     run_ws_any(g, s);
     if (fused) cs->slab_rows = ws_slab_rows();
     return fused;
