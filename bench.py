@@ -108,6 +108,17 @@ class Clocks:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
+def update_traffic(n, nb):
+    """Measured DRAM bytes per update launch (ncu, committed under profiles/) for this workload."""
+    try:
+        d = json.load(open(os.path.join(ROOT, "profiles", "update_traffic_r01.json")))
+        if f"run_once.py {n} {nb}" in d.get("command", ""):
+            return round(d["traffic_bytes_per_launch"])
+    except Exception:
+        pass
+    return None
+
+
 # ---- the oracle as CPU baseline / reference arm ---------------------------------------------
 def oracle_sample(n_s, nb):
     import numpy as np
@@ -235,11 +246,14 @@ def main():
                    "l2": "inputs (8 GiB) larger than L2; restore copy between steps outside the CUDA events",
                    "parallelism": f"1D block-cyclic x{world}, NCCL panel broadcast" if world > 1 else "single GPU"},
         "gpu_launches": int(launches) * args.steps,
-        "roofline": {"bound": "tensor", "kernel": "k_gemm_ws (warp-specialised DMMA, 128x128 tiles) trailing SYRK update",
+        "roofline": {"bound": "tensor", "kernel": "k_update_ws (warp-specialised DMMA, 128x64 tiles, 2 CTAs/SM) trailing SYRK update + checksum rows",
                      "achieved": round(achieved, 3) if achieved else None,
                      "peak": FP64_DMMA_PEAK_TFLOPS, "unit": "TFLOP/s",
                      "frac": round(achieved / FP64_DMMA_PEAK_TFLOPS, 4) if achieved else None,
-                     "traffic": None,
+                     "traffic": update_traffic(n, nb),
+                     "traffic_source": "ncu dram__bytes_read.sum + dram__bytes_write.sum per k_update_ws launch, "
+                                       "averaged over every launch of one factorisation of this workload "
+                                       "(profiles/update_traffic_r01.json, cold-cache serialised replay)",
                      "peak_source": "measured FP64 DMMA register-resident loop on this pool's B200 "
                                     "(MEASURED_PEAKS.json has no FP64 entry)",
                      "share_of_step": round(upd["ms"] / ms_local, 4) if upd.get("ms") else None},
@@ -301,6 +315,16 @@ def main():
                 tf, rf = run_steps(P.options(mode=mode), inj=injf, steps=1, warmup=1, check=True)
                 table[mode][fname] = {"ms": round(tf[0], 2), "value": round(flops / (tf[0] * 1e-3) / 1e9, 1),
                                       "reruns": int(rf[0]["reruns"]), "events": int(rf[0]["n_events"])}
+        # NEXT-4: two errors in one column of a block (beyond what two checksums locate):
+        # Enhanced stops with UNCORRECTABLE; Enhanced + re-do re-runs once from the saved input
+        dbl = syn.inj_array([dict(k=3, hook="REST", row=3 * B_ + 100, col=3 * B_ + 50, bit=50),
+                             dict(k=3, hook="REST", row=3 * B_ + 140, col=3 * B_ + 50, bit=51)])
+        table["two_errors_in_a_column"] = {}
+        for mode in ("enhanced", "enhanced_redo"):
+            tf, rf = run_steps(P.options(mode=mode), inj=dbl, steps=1, warmup=1, check=False)
+            table["two_errors_in_a_column"][mode] = {
+                "ms": round(tf[0], 2), "status": "uncorrectable" if rf[0]["n_uncorrectable"] and not rf[0]["reruns"]
+                else "ok", "reruns": int(rf[0]["reruns"]), "events": int(rf[0]["n_events"])}
         table["paper_context_seconds"] = {
             "Tardis_M2075_n20480": {"enhanced": [10.6572, 10.6614, 10.6678], "online": [10.5067, 10.5244, 22.625],
                                     "offline": [10.4489, 21.3942, 21.2631], "src": "PAPER.md:366-368"},

@@ -100,7 +100,7 @@ typedef struct abft_options {
     double c_tau;         /* threshold constant C_tau of reading A4 (default 64)               */
     int32_t lookahead;    /* reserved (0/1)                                                    */
     int32_t profile;      /* 1: time every phase with CUDA events on `stream` (abft_last_profile) */
-    int32_t mode;         /* ABFT_MODE_ENHANCED (default), ABFT_MODE_ONLINE or ABFT_MODE_OFFLINE  */
+    int32_t mode;         /* ABFT_MODE_ENHANCED (default), _ONLINE, _OFFLINE or _ENHANCED_REDO    */
     int32_t order;        /* ABFT_ORDER_RIGHT (default: trailing update + look-ahead) or
                              ABFT_ORDER_LEFT (MAGMA's Alg. 1, Table I checks)     */
 } abft_options_t;
@@ -116,6 +116,9 @@ typedef struct abft_options {
 #define ABFT_MODE_ENHANCED 0
 #define ABFT_MODE_ONLINE 1
 #define ABFT_MODE_OFFLINE 2
+#define ABFT_MODE_ENHANCED_REDO 3   /* Enhanced + one re-run from a saved copy of A on UNCORRECTABLE
+                                       (more errors in a block column than two checksums locate,
+                                       PAPER.md:121; the paper's re-do)          */
 
 /* Per-phase device time of the last abft_potrf* call on this thread with options.profile = 1.
  * Phases: 0 encode, 1 V1/V2, 2 POTRF+inverse, 3 TRSM (+Alg. 2 rows), 4 V3, 5 V4, 6 panel

@@ -100,7 +100,7 @@ def sorted_events(ev):
     return sorted(keys)
 
 
-MODE = {"enhanced": 0, "online": 1, "offline": 2}
+MODE = {"enhanced": 0, "online": 1, "offline": 2, "enhanced_redo": 3}
 
 
 def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, inplace=False, mode="enhanced",

@@ -606,8 +606,10 @@ static int potrf_core_left(int64_t n, int64_t nb, double* A, int64_t lda, const 
 /* The factorisation with the scheme's recovery: Enhanced corrects in place; Online and Offline
  * cannot correct an error that propagated ("it needs to repeat the whole decomposition
  * again"), so an UNCORRECTABLE / NOT_SPD outcome or any detection by the final sweep re-runs the
- * factorisation once from the saved input, without the injected faults. Events of both runs are
- * returned in order. */
+ * factorisation once from the saved input, without the injected faults. mode 3 is the Enhanced
+ * scheme with the same re-do for what two checksums cannot correct (more than one error in a
+ * column of a block, P:121 [A11]): an UNCORRECTABLE outcome re-runs once.
+ * Events of both runs are returned in order. */
 int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
                       int nranks, int K, double c_tau, int abft, int mode, int order, oevent_t* ev, int64_t cap,
                       int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out,
@@ -616,7 +618,9 @@ int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
     if (nb < 1) return -2;
     if (n % nb) return -2;                          /* [A20] */
     if (lda < (n > 1 ? n : 1)) return -4;
-    if (mode < 0 || mode > 2) return -11;
+    if (mode < 0 || mode > 3) return -11;
+    const int redo = (mode == 3);                   /* Enhanced + re-do on UNCORRECTABLE */
+    if (redo) mode = 0;
     if (nranks < 1) nranks = 1;
     if (K < 1) K = 1;
     ocount_t dummy;
@@ -624,7 +628,7 @@ int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
     memset(c, 0, sizeof(ocount_t));
     if (reruns) *reruns = 0;
     double* A0 = NULL;
-    if (mode != 0 && n > 0) {
+    if ((mode != 0 || redo) && n > 0) {
         A0 = (double*)malloc(sizeof(double) * (size_t)(lda * n));
         memcpy(A0, A, sizeof(double) * (size_t)(lda * n));
     }
@@ -638,7 +642,8 @@ int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
      * online checks and may have propagated -> re-do. */
     int v6_detect = 0;
     for (int64_t e = 0; ev && e < nev1 && e < cap; ++e) v6_detect |= (ev[e].check == O_V6);
-    if (mode != 0 && (st == O_STATUS_UNCORRECTABLE || st == O_STATUS_NOT_SPD || v6_detect)) {
+    if ((mode != 0 && (st == O_STATUS_UNCORRECTABLE || st == O_STATUS_NOT_SPD || v6_detect)) ||
+        (redo && st == O_STATUS_UNCORRECTABLE)) {
         memcpy(A, A0, sizeof(double) * (size_t)(lda * n));
         int64_t nev2 = 0;
         const int64_t off = nev1 < cap ? nev1 : cap;

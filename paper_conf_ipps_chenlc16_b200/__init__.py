@@ -151,7 +151,7 @@ def _report_dict(rep, ev):
                 seconds=rep.seconds, reruns=rep.reruns)
 
 
-MODE = {"enhanced": 0, "online": 1, "offline": 2}
+MODE = {"enhanced": 0, "online": 1, "offline": 2, "enhanced_redo": 3}
 
 
 def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False, mode="enhanced", order="right"):

@@ -1084,15 +1084,18 @@ extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft
     if (o.K < 1 || !(o.c_tau > 0)) return -8;
     std::vector<abft_inject_spec_t> list;
     if (collect_inj(inj, n, nb, list, o.order)) return -6;
-    if (o.mode < ABFT_MODE_ENHANCED || o.mode > ABFT_MODE_OFFLINE) return -8;
+    if (o.mode < ABFT_MODE_ENHANCED || o.mode > ABFT_MODE_ENHANCED_REDO) return -8;
+    const bool redo = o.mode == ABFT_MODE_ENHANCED_REDO;   // NEXT-4: Enhanced + re-do on UNCORRECTABLE
+    if (redo) o.mode = ABFT_MODE_ENHANCED;
     if (o.order != ABFT_ORDER_RIGHT && o.order != ABFT_ORDER_LEFT) return -8;
     const RunFn run = o.order == ABFT_ORDER_LEFT ? run_potrf_left : run_potrf;
     if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; rep->reruns = 0; }
     if (n == 0) return 0;
     cudaStream_t s = (cudaStream_t)stream;
-    if (o.mode == ABFT_MODE_ENHANCED || !o.abft_enabled) return run(n, nb, A, lda, s, list, rep, o);
+    if ((o.mode == ABFT_MODE_ENHANCED && !redo) || !o.abft_enabled) return run(n, nb, A, lda, s, list, rep, o);
     // Online / Offline: keep the input; an uncorrectable outcome or a detection by the final
-    // sweep means an error propagated -> re-do the factorisation once, without the faults
+    // sweep means an error propagated -> re-do the factorisation once, without the faults.
+    // Enhanced + re-do: only an UNCORRECTABLE outcome (> 1 error in a block column) re-runs.
     double* A0 = nullptr;
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&A0, sizeof(double) * (size_t)(n * n), s));
     ABFT_CUDA_TRY(cudaMemcpy2DAsync(A0, n * sizeof(double), A, lda * sizeof(double), n * sizeof(double), n,
@@ -1109,7 +1112,7 @@ extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft
     std::vector<abft_event_t> ev2(rep ? std::max<int64_t>(rep->cap, 16) : 16);
     r2.cap = (int64_t)ev2.size(); r2.events = ev2.data();
     int reruns = 0;
-    if (st == ABFT_UNCORRECTABLE || st == ABFT_NOT_SPD || v6) {
+    if (redo ? st == ABFT_UNCORRECTABLE : (st == ABFT_UNCORRECTABLE || st == ABFT_NOT_SPD || v6)) {
         ABFT_CUDA_TRY(cudaMemcpy2DAsync(A, lda * sizeof(double), A0, n * sizeof(double), n * sizeof(double), n,
                                         cudaMemcpyDeviceToDevice, s));
         const std::vector<abft_inject_spec_t> none;

@@ -455,7 +455,7 @@ __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t 
 }
 
 template <class C_>
-__global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, int64_t ntiles, int64_t n1tiles) {
+__device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64_t n1tiles) {
     constexpr int BM = C_::BM, BN = C_::BN, BK = C_::BK, WM = C_::WM, WN = C_::WN, STAGES = C_::STAGES;
     if (*(volatile const int32_t*)g.abort) return;
     extern __shared__ __align__(16) double smem[];
@@ -624,11 +624,23 @@ __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, i
     }
 }
 
+// Two entry points with one body, so that profiles attribute the trailing update (the dominant
+// kernel of the factorisation) separately from the TRSM and the other products.
 template <class C_>
-static int run_ws(GemmArgs g, cudaStream_t s) {
+__global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, int64_t ntiles, int64_t n1tiles) {
+    ws_body<C_>(g, ntiles, n1tiles);
+}
+template <class C_>
+__global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_update_ws(GemmArgs g, int64_t ntiles, int64_t n1tiles) {
+    ws_body<C_>(g, ntiles, n1tiles);
+}
+
+template <class C_>
+static int run_ws(GemmArgs g, cudaStream_t s, bool update) {
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(k_gemm_ws<C_>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::SMEM);
+        cudaFuncSetAttribute(k_update_ws<C_>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::SMEM);
         attr = true;
     }
     const int64_t tm = (g.M + C_::BM - 1) / C_::BM, tn = (g.N + C_::BN - 1) / C_::BN;
@@ -641,7 +653,8 @@ static int run_ws(GemmArgs g, cudaStream_t s) {
     static int64_t tpc = -1;
     if (tpc < 0) { const char* e = getenv("ABFT_WS_TPC"); tpc = e ? std::max(1, atoi(e)) : 1; }
     const int64_t grid = std::max<int64_t>(1, (ntiles + tpc - 1) / tpc);
-    k_gemm_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
+    if (update) k_update_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
+    else k_gemm_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
     abft_count_launch();
     return 0;
 }
@@ -661,11 +674,12 @@ static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CT
 static int ws_slab_rows() { return ws_variant() == 16 ? WsCfg16::WM : 64; }
 static int run_ws_any(GemmArgs g, cudaStream_t s) {
     g.cs.slab_rows = ws_slab_rows();
+    const bool upd = g.mask == MASK_LOWER && g.alpha == -1.0 && g.beta == 1.0;   // a trailing update
     switch (ws_variant()) {
-        case 16: return run_ws<WsCfg16>(g, s);
-        case 21: return run_ws<WsCfg2a>(g, s);
-        case 22: return run_ws<WsCfg2b>(g, s);
-        default: return run_ws<WsCfg>(g, s);
+        case 16: return run_ws<WsCfg16>(g, s, upd);
+        case 21: return run_ws<WsCfg2a>(g, s, upd);
+        case 22: return run_ws<WsCfg2b>(g, s, upd);
+        default: return run_ws<WsCfg>(g, s, upd);
     }
 }
 

@@ -353,3 +353,22 @@ def test_left_looking_schemes(P, mode):
         st, rep, L = run_gpu(P, A, nb, inj=inj, opt=P.options(mode=mode, order="left"))
         assert st == ref.status == 0 and rep["reruns"] == ref.reruns
         assert floor_rel(L, ref.L, A) <= 1e-11
+
+
+@pytest.mark.parametrize("mode", ["enhanced", "enhanced_redo"])
+def test_two_errors_in_a_column_redo_matches_oracle(P, mode):
+    """NEXT-4: two errors in one column of a block (beyond what two checksums locate):
+    plain Enhanced aborts with UNCORRECTABLE; with re-do it re-runs once from the saved input.
+    Same status, re-runs and events as the oracle; the re-run's factor within 1e-11."""
+    from tests.test_oracle_pins import TWO_IN_A_COLUMN
+    n, nb = 512, 64
+    A = syn.spd_matrix(n, seed=2)
+    inj = syn.inj_array(TWO_IN_A_COLUMN)
+    ref = oracle.potrf(A, nb, inj=inj, mode=mode)
+    st, rep, L = run_gpu(P, A, nb, inj=inj, opt=P.options(mode=mode))
+    assert st == ref.status
+    assert rep["reruns"] == ref.reruns
+    assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
+    if mode == "enhanced_redo":
+        assert st == 0 and rep["reruns"] == 1
+        assert floor_rel(L, ref.L, A) <= 1e-11

@@ -452,3 +452,34 @@ def test_left_looking_verifies_more_than_right_looking():
     assert ll.counts["bytes_check"] > rl.counts["bytes_check"]
     ll3 = oracle.potrf(A, nb, order="left", K=3)
     assert ll3.counts["bytes_check"] < ll.counts["bytes_check"]
+
+
+# ---- NEXT-4: more errors in a block column than two checksums locate ("m+1 checksums
+# ... up to m errors per column"; reading A11) -> Enhanced + re-do (the paper's re-do) ----
+TWO_IN_A_COLUMN = [dict(k=1, hook="REST", row=300, col=150, bit=55),
+                   dict(k=1, hook="REST", row=310, col=150, bit=56)]   # same tile (2,1), same column
+
+
+def test_enhanced_two_errors_in_a_column_uncorrectable_without_redo():
+    n, nb = 512, 64
+    A = syn.spd_matrix(n, seed=2)
+    r = oracle.potrf(A, nb, inj=syn.inj_array(TWO_IN_A_COLUMN))
+    assert r.status == 1 and r.reruns == 0
+    assert any(e[6] == KIND["UNCORRECTABLE"] for e in r.event_tuples())
+
+
+def test_enhanced_redo_recovers_and_matches_lapack():
+    """With re-do the call ends with status 0, one re-run, the UNCORRECTABLE event of the first
+    run in the report, and the factor of the fault-free run (bit-identical: the re-run starts
+    from the saved input without faults) = LAPACK within P4 tolerances."""
+    n, nb = 512, 64
+    A = syn.spd_matrix(n, seed=2)
+    r = oracle.potrf(A, nb, inj=syn.inj_array(TWO_IN_A_COLUMN), mode="enhanced_redo")
+    clean = oracle.potrf(A, nb)
+    assert r.status == 0 and r.reruns == 1
+    assert any(e[6] == KIND["UNCORRECTABLE"] for e in r.event_tuples())
+    assert np.array_equal(np.tril(r.L), np.tril(clean.L))
+    assert floor_rel(r.L, scipy.linalg.cholesky(A, lower=True), A) <= 1e-11
+    # single errors are corrected in place: no re-run
+    one = oracle.potrf(A, nb, inj=syn.inj_array(TWO_IN_A_COLUMN[:1]), mode="enhanced_redo")
+    assert one.status == 0 and one.reruns == 0 and len(one.events) == 1
