@@ -216,6 +216,13 @@ int abft_dev_gemm_nt(int64_t M, int64_t N, int64_t K, const double* A, int64_t l
  * non-positive pivot. Synchronises `stream`. */
 int abft_dev_chol_inv(int64_t nb, double* A, int64_t lda, double* Li, abft_stream_t stream);
 
+/* Diagnostics: abft_dev_chol_inv through the one-launch task-graph path with a per-task trace:
+ * trace_host (cap >= 4 x tasks, host) receives per task {type | i<<8 | j<<16 | b<<24 | smid<<32 |
+ * cta<<48, fetch ns, start ns (dependencies met), end ns} (%globaltimer). Returns the number of
+ * tasks, -1 if nb does not take the task path or cap is too small, -2 if the factorisation failed. */
+int abft_dev_chol_trace(int64_t nb, double* A, int64_t lda, double* Li, uint64_t* trace_host, int64_t cap,
+                        abft_stream_t stream);
+
 /* Diagnostics: kernel launches issued by the last call on this thread, a static version string,
  * and the text of the last CUDA error seen on this thread (empty if none). */
 int64_t abft_last_launch_count(void);

@@ -80,6 +80,8 @@ _lib.abft_potrf_dist_sim.argtypes = [_i64, _i64, _i32, _vp, _i64, _vp, _vp, _vp,
 _lib.abft_potrf_dist_sim.restype = _i32
 _lib.abft_dev_chol_inv.argtypes = [_i64, _vp, _i64, _vp, _vp]
 _lib.abft_dev_chol_inv.restype = _i32
+_lib.abft_dev_chol_trace.argtypes = [_i64, _vp, _i64, _vp, _vp, _i64, _vp]
+_lib.abft_dev_chol_trace.restype = _i32
 _lib.abft_dev_gemm_nt.argtypes = [_i64, _i64, _i64, _vp, _i64, _vp, _i64, _vp, _i64, _dbl, _dbl, _i32, _vp]
 _lib.abft_dev_gemm_nt.restype = _i32
 _lib.abft_last_launch_count.restype = _i64
@@ -95,7 +97,7 @@ for _f in ("abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_po
 EXPORTS = ["abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
            "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist",
            "abft_last_launch_count", "abft_version", "abft_last_error", "abft_last_profile", "abft_dev_gemm_nt", "abft_dev_chol_inv",
-           "abft_potrf_dist_sim",
+           "abft_dev_chol_trace", "abft_potrf_dist_sim",
            "abft_phase_name"]
 
 
@@ -322,6 +324,25 @@ def abft_dev_chol_inv(nb, A, Li, stream=None):
     pa, la = _dev(A)
     pl, _ = _dev(Li)
     return _lib.abft_dev_chol_inv(nb, pa, la or nb, pl, _stream(stream))
+
+
+def abft_dev_chol_trace(nb, A, Li, stream=None):
+    """Diagnostics: the task-graph diagonal block with a per-task trace; returns (ntasks, rows) with
+    rows = (type, i, j, b, smid, cta, fetch_ns, start_ns, end_ns), or (status, [])."""
+    import numpy as np
+    pa, la = _dev(A)
+    pl, _ = _dev(Li)
+    cap = 4 * 4096
+    buf = np.zeros(cap, dtype=np.uint64)
+    nt = _lib.abft_dev_chol_trace(nb, pa, la or nb, pl, buf.ctypes.data, cap, _stream(stream))
+    if nt <= 0:
+        return nt, []
+    rows = []
+    for t in range(nt):
+        w = int(buf[4 * t])
+        rows.append((w & 255, (w >> 8) & 255, (w >> 16) & 255, (w >> 24) & 255, (w >> 32) & 0xFFFF, w >> 48,
+                     int(buf[4 * t + 1]), int(buf[4 * t + 2]), int(buf[4 * t + 3])))
+    return nt, rows
 
 
 def abft_last_launch_count():

@@ -29,6 +29,7 @@ int launch_scales(int64_t n, int64_t nb, const double* A, int64_t lda, double* s
 int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,
                 const int32_t* abort_flag, cudaStream_t s);
 int launch_zero(int64_t rows, int64_t cols, double* dst, int64_t ldd, cudaStream_t s);
+size_t chol_sync_bytes(int64_t nb);
 int launch_chol_inv(double* T, int64_t ldt, double* Li, int64_t B, int64_t info_off, double* tmp,
                     DevState* st, cudaStream_t s);
 int launch_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, cudaStream_t s);
@@ -123,6 +124,7 @@ static int work_alloc(Work& w, int64_t n, int64_t nb, int64_t ncols_local, int64
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.W, sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb), s));
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.Li, sizeof(double) * (size_t)(nb * nb), s));
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.tmp, sizeof(double) * (size_t)(((nb + 1) / 2 + 64) * ((nb + 1) / 2 + 64)), s));
+    ABFT_CUDA_TRY(cudaMemsetAsync(w.tmp, 0, chol_sync_bytes(nb), s));   // task-graph POTRF sync words
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.st, sizeof(DevState), s));
     ABFT_CUDA_TRY(cudaMemsetAsync(w.st, 0, sizeof(DevState), s));
     w.ev_cap = std::max<int64_t>(ev_cap, 1);
@@ -1240,12 +1242,32 @@ extern "C" int abft_dev_chol_inv(int64_t nb, double* A, int64_t lda, double* Li,
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&st, sizeof(DevState), s));
     ABFT_CUDA_TRY(cudaMemsetAsync(st, 0, offsetof(DevState, fl), s));
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&tmp, sizeof(double) * (size_t)(((nb + 1) / 2 + 64) * ((nb + 1) / 2 + 64)), s));
+    ABFT_CUDA_TRY(cudaMemsetAsync(tmp, 0, chol_sync_bytes(nb), s));
     launch_chol_inv(A, lda, Li, nb, 0, tmp, st, s);
     int32_t status = 0;
     ABFT_CUDA_TRY(cudaMemcpyAsync(&status, &st->status, sizeof status, cudaMemcpyDeviceToHost, s));
     cudaFreeAsync(tmp, s); cudaFreeAsync(st, s);
     ABFT_CUDA_TRY(cudaStreamSynchronize(s));
     return status;
+}
+
+void chol_set_trace(unsigned long long* t);
+int chol_task_count(int64_t nb);
+extern "C" int abft_dev_chol_trace(int64_t nb, double* A, int64_t lda, double* Li, uint64_t* trace_host, int64_t cap,
+                                   abft_stream_t stream) {
+    const int nt = chol_task_count(nb);
+    if (nt <= 0 || cap < 4 * (int64_t)nt) return -1;
+    cudaStream_t s = (cudaStream_t)stream;
+    unsigned long long* d = nullptr;
+    ABFT_CUDA_TRY(cudaMalloc((void**)&d, sizeof(uint64_t) * 4 * (size_t)nt));
+    ABFT_CUDA_TRY(cudaMemset(d, 0, sizeof(uint64_t) * 4 * (size_t)nt));
+    chol_set_trace(d);
+    const int st = abft_dev_chol_inv(nb, A, lda, Li, stream);
+    chol_set_trace(nullptr);
+    ABFT_CUDA_TRY(cudaMemcpy(trace_host, d, sizeof(uint64_t) * 4 * (size_t)nt, cudaMemcpyDeviceToHost));
+    cudaFree(d);
+    (void)s;
+    return st == 0 ? nt : -2;
 }
 
 extern "C" int abft_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, abft_stream_t stream) {

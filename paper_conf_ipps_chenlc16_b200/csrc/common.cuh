@@ -174,6 +174,13 @@ __device__ __forceinline__ void thresholds(const StageArgs& a, int64_t I, int64_
 
 __device__ __forceinline__ bool dfinite(double x) { return isfinite(x); }
 
+// One FP64 tensor-core MMA (SASS DMMA.8x8x4): C(8x8) += A(8x4) B(4x8). Fragments: lane holds
+// A[lane/4][lane%4], B[k = lane%4][n = lane/4], C[lane/4][2 (lane%4) + {0, 1}].
+__device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b) {
+    asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                 : "+d"(c0), "+d"(c1) : "d"(a), "d"(b));
+}
+
 }  // namespace abft
 
 // Per-column partial checksums of an updated trailing tile, written by the GEMM epilogue

@@ -10,6 +10,8 @@
 #include "common.cuh"
 
 #include <algorithm>
+#include <cstdlib>
+#include <cstring>
 
 
 namespace abft {
@@ -105,9 +107,395 @@ __global__ void k_zero_block(int64_t rows, int64_t cols, double* dst, int64_t ld
     }
 }
 
+// ---------------------------------------------------------------------------------------------
+// Task-graph diagonal block (nb % 64 == 0, nb >= 128): ONE launch factors the nb x nb block and
+// inverts it. The block is cut into T x T tiles of 64; the tile algorithm is the paper's blocked
+// POTRF/TRSM/SYRK recursion one level down plus a right-looking blocked
+// inverse X = inv(L):
+//   P(b)      [b >= 1: L_{b,b-1} = A_{b,b-1} inv(L_{b-1})^T, A_bb -= L_{b,b-1} L_{b,b-1}^T — the
+//             critical path, fused into the CTA that then factors] L_bb = chol(A_bb), X_bb = inv(L_bb)
+//   S(i,b)    L_ib = A_ib X_bb^T                                       i >= b + 2       (DMMA)
+//   U(i,j,b)  A_ij -= L_ib L_jb^T  (lower half when i == j)           i >= j > b       (DMMA)
+//   Z(i,j,b)  Y_ij (+)= L_ib X_bj  (Y_ij accumulates in X's tile)      i > b >= j       (DMMA)
+//   F(i,j)    X_ij = -X_ii Y_ij  (= -inv(L_ii) sum_{c=j}^{i-1} L_ic X_cj), zero tile (j,i) i > j (DMMA)
+// Tasks are numbered in a topological order (step b: P(b+1), S(., b), U(., ., b), F(b, .),
+// Z(., ., b)); CTAs fetch them with an atomic counter and wait on per-tile completion flags
+// (acquire/release at gpu scope), so no co-residency is needed: every dependency of a fetched
+// task was fetched earlier by a running CTA. This replaces the ~50 dependent launches of the
+// recursive path (each ~7 us of launch latency) on the look-ahead stream's critical path. The
+// last CTA to exit zeroes the flags for the next launch (the sync area is zeroed once when it is
+// allocated).
+constexpr int kTT = 64;                 // tile
+constexpr int kTP = kTT + 4;            // smem pitch: 4 mod 16 8-byte banks, conflict-free fragments
+constexpr int kTaskThreads = 256;       // 8 warps: 2 x 4 grid of 32 x 16 warp tiles
+constexpr size_t kTaskSmem = 2 * (size_t)kTT * kTP * sizeof(double);
+enum { TK_P = 0, TK_S = 1, TK_U = 2, TK_Z = 3, TK_F = 4 };
+
+// tasks of step b (m = T - 1 - b tiles below the diagonal tile b)
+__host__ __device__ __forceinline__ int task_step_count(int T, int b) {
+    const int m = T - 1 - b;
+    return (m >= 1 ? 1 : 0) + (m >= 2 ? m - 1 : 0) + m * (m + 1) / 2 - (m >= 1 ? 1 : 0) + b + m * (b + 1);
+}
+__host__ __device__ __forceinline__ int task_count(int T) {
+    int s = 1;   // P(0)
+    for (int b = 0; b < T; ++b) s += task_step_count(T, b);
+    return s;
+}
+// [next task, exited CTAs, P flags (T), S flags (T x T), U flags (T x T), Z counts (T x T), F flags (T x T)]
+__host__ __device__ __forceinline__ int task_sync_words(int T) { return 2 + T + 4 * T * T; }
+
+__device__ __forceinline__ void decode_task(int T, int t, int& type, int& i, int& j, int& b) {
+    if (t == 0) { type = TK_P; i = j = b = 0; return; }
+    t -= 1;
+    for (b = 0; b < T - 1; ++b) {
+        const int cnt = task_step_count(T, b);
+        if (t < cnt) break;
+        t -= cnt;
+    }
+    const int m = T - 1 - b;
+    if (m >= 1) {
+        if (t == 0) { type = TK_P; i = j = b = b + 1; return; }
+        t -= 1;
+        if (t < m - 1) { type = TK_S; i = b + 2 + t; j = b; return; }
+        t -= m - 1;
+        const int nu = m * (m + 1) / 2 - 1;
+        if (t < nu) {   // column-major over (j, i), b < j <= i, skipping (b+1, b+1)
+            int e = t + 1, jj = b + 1;
+            while (e >= T - jj) { e -= T - jj; ++jj; }
+            type = TK_U; j = jj; i = jj + e; return;
+        }
+        t -= nu;
+    }
+    if (t < b) { type = TK_F; i = b; j = t; return; }
+    t -= b;
+    type = TK_Z; i = b + 1 + t / (b + 1); j = t % (b + 1);   // Z(i, j, b), i > b >= j
+}
+
+__device__ __forceinline__ void cpa16(double* smem, const double* gmem) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cpa_wait_all() {
+    asm volatile("cp.async.commit_group;\ncp.async.wait_group 0;\n" ::: "memory");
+}
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];\n" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;\n" ::"l"(p), "r"(v) : "memory");
+}
+// spin until *f >= v; false if the run aborted meanwhile
+__device__ __forceinline__ bool wait_ge(const uint32_t* f, uint32_t v, const int32_t* abort) {
+    for (;;) {
+        if (ld_acquire(f) >= v) return true;
+        if (*(volatile const int32_t*)abort) return false;
+        __nanosleep(32);
+    }
+}
+
+// s[k][m] = X(m, k) of a 64 x 64 column-major tile (16-byte cp.async, L2 only)
+__device__ __forceinline__ void tile_load_T(double* s, const double* X, int64_t ld) {
+    for (int e = threadIdx.x; e < kTT * kTT / 2; e += kTaskThreads) {
+        const int k = e >> 5, m2 = (e & 31) * 2;
+        cpa16(s + k * kTP + m2, X + k * ld + m2);
+    }
+}
+// s[k][n] = X(k, n) (the NN operand): 16-byte loads down a column, two 8-byte shared stores
+__device__ __forceinline__ void tile_load_N(double* s, const double* X, int64_t ld) {
+    for (int e = threadIdx.x; e < kTT * kTT / 2; e += kTaskThreads) {
+        const int n = e & 63, k2 = (e >> 6) * 2;
+        const double2 v = __ldcg(reinterpret_cast<const double2*>(X + n * ld + k2));
+        s[k2 * kTP + n] = v.x;
+        s[(k2 + 1) * kTP + n] = v.y;
+    }
+}
+// acc (warp tile 32 x 16 at (wm, wn)) += A (64 x 64, staged s[k][m]) * op(B) (staged s[k][n])
+__device__ __forceinline__ void tile_mma(double (&acc)[4][2][2], const double* sA, const double* sB, int wm, int wn,
+                                         int fr, int fc) {
+#pragma unroll 4
+    for (int kk = 0; kk < kTT; kk += 4) {
+        double af[4], bf[2];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) af[i] = sA[(kk + fc) * kTP + wm * 32 + i * 8 + fr];
+#pragma unroll
+        for (int j = 0; j < 2; ++j) bf[j] = sB[(kk + fc) * kTP + wn * 16 + j * 8 + fr];
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int j = 0; j < 2; ++j) dmma(acc[i][j][0], acc[i][j][1], af[i], bf[j]);
+    }
+}
+__device__ __forceinline__ void zero_acc(double (&acc)[4][2][2]) {
+#pragma unroll
+    for (int x = 0; x < 4; ++x)
+#pragma unroll
+        for (int y = 0; y < 2; ++y) acc[x][y][0] = acc[x][y][1] = 0.0;
+}
+// fragment element (x, y, h) of warp (wm, wn), lane (fr, fc) -> tile row m, column n
+#define ABFT_FRAG_MN const int m = wm * 32 + x * 8 + fr, n = wn * 16 + y * 8 + fc * 2 + h
+#define ABFT_FRAG_LOOP _Pragma("unroll") for (int x = 0; x < 4; ++x) _Pragma("unroll") for (int y = 0; y < 2; ++y) \
+    _Pragma("unroll") for (int h = 0; h < 2; ++h)
+
+// P(b) leaf: Cholesky of the 64 x 64 lower tile src (ld lds; shared or global) and its inverse,
+// one CTA. Thread (r = tid % 64, q = tid / 64) keeps row r's elements of columns c = 16 q + u
+// (u < 16) in registers, for the factor (unscaled right-looking: a_rc -= (a_rj / d_j) a_cj) and
+// for the elimination Y = (unit lower)^-1 (Y(r, c) -= (a_rj / d_j) Y(j, c)). A column of a is
+// final after step c-1 and is then published into the shared tile Ls (column-major), a row of Y
+// into Ys (row-major); steps read only published values, so the register updates need no
+// per-element predicate (finished and upper elements take harmless garbage: their final values
+// live in Ls / Ys). Warps with no live element skip that half of the step; one barrier per
+// column. At the end l_rc = a_rc / sqrt(d_c) -> Lb, inv(L)_rc = Y(r, c) / sqrt(d_r) -> Xb (zero
+// above the diagonal). Ls may alias src. Returns false on a non-positive pivot (NOT_SPD raised,
+// LAPACK info).
+__device__ bool leaf_tile(const double* src, int64_t lds, double* Lb, int64_t lda, double* Xb, int64_t ldi, double* Ls,
+                          double* Ys, int64_t info0, DevState* st) {
+    const int tid = threadIdx.x, r = tid & 63, q = tid >> 6, c0 = 16 * q;
+    const int rmax = (tid & 32) + 31;   // warp-uniform: largest row of this warp
+    double a[16], y[16];
+#pragma unroll
+    for (int u = 0; u < 16; ++u) {
+        const int c = c0 + u;
+        a[u] = (c <= r) ? src[c * lds + r] : 0.0;
+        y[u] = (c == r) ? 1.0 : 0.0;
+    }
+    __syncthreads();   // Ls may alias src
+    if (q == 0) Ls[r] = a[0];                                                          // column 0
+    if (r == 0) {
+#pragma unroll
+        for (int u = 0; u < 16; u += 2) *reinterpret_cast<double2*>(Ys + c0 + u) = make_double2(y[u], y[u + 1]);   // row 0
+    }
+    for (int jj = 0; jj < kTT; ++jj) {
+        __syncthreads();
+        const double* cj = Ls + jj * kTP;
+        const double d = cj[jj];
+        if (!(d > 0.0)) {
+            if (tid == 0 && atomicCAS(&st->abort, 0, 1) == 0) { st->status = ABFT_NOT_SPD; st->info = info0 + jj + 1; }
+            return false;
+        }
+        const double f = cj[r] * __drcp_rn(d);
+        if (c0 + 15 > jj && c0 <= rmax) {   // factor: live columns c in (jj, r]
+            double cv[16];
+#pragma unroll
+            for (int u = 0; u < 16; u += 2) {
+                const double2 v = *reinterpret_cast<const double2*>(cj + c0 + u);
+                cv[u] = v.x; cv[u + 1] = v.y;
+            }
+#pragma unroll
+            for (int u = 0; u < 16; ++u) a[u] = fma(-f, cv[u], a[u]);
+            if (((jj + 1) >> 4) == q) {      // this warp owns column jj+1: publish rows r > jj
+                const int u1 = (jj + 1) & 15;
+                double nv = a[0];
+#pragma unroll
+                for (int u = 1; u < 16; ++u) nv = (u == u1) ? a[u] : nv;
+                if (r > jj) Ls[(jj + 1) * kTP + r] = nv;
+            }
+        }
+        if (c0 <= jj && rmax > jj) {        // elimination: rows r > jj (row jj of Y is zero right of jj)
+            const double* yj = Ys + jj * kTP;
+            double yv[16];
+#pragma unroll
+            for (int u = 0; u < 16; u += 2) {
+                const double2 v = *reinterpret_cast<const double2*>(yj + c0 + u);
+                yv[u] = v.x; yv[u + 1] = v.y;
+            }
+#pragma unroll
+            for (int u = 0; u < 16; ++u) y[u] = fma(-f, yv[u], y[u]);
+        }
+        if (r == jj + 1) {   // row jj+1 of Y is final
+#pragma unroll
+            for (int u = 0; u < 16; u += 2) *reinterpret_cast<double2*>(Ys + r * kTP + c0 + u) = make_double2(y[u], y[u + 1]);
+        }
+    }
+    __syncthreads();
+    for (int e = tid; e < kTT * kTT; e += kTaskThreads) {
+        const int c = e >> 6, rr = e & 63;
+        const double sc = sqrt(Ls[c * kTP + c]), sr = sqrt(Ls[rr * kTP + rr]);
+        if (c <= rr) Lb[c * lda + rr] = (c == rr) ? sc : Ls[c * kTP + rr] / sc;
+        Xb[c * ldi + rr] = (c <= rr) ? Ys[rr * kTP + c] / sr : 0.0;
+    }
+    return true;
+}
+
+__global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int64_t lda, double* Li, int64_t ldi, int T,
+                                                                int ntasks, int64_t info_off, uint32_t* sync,
+                                                                DevState* st, unsigned long long* trace) {
+    extern __shared__ __align__(16) double tsm[];
+    double* sA = tsm;
+    double* sB = tsm + kTT * kTP;
+    __shared__ int s_task, s_go;
+    const int32_t* abort_flag = &st->abort;
+    if (*(volatile const int32_t*)abort_flag) return;
+    uint32_t* next = sync;
+    uint32_t* exited = sync + 1;
+    uint32_t* fP = sync + 2;
+    uint32_t* fS = fP + T;
+    uint32_t* fU = fS + T * T;
+    uint32_t* fZ = fU + T * T;
+    uint32_t* fF = fZ + T * T;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int wm = warp >> 2, wn = warp & 3, fr = lane >> 2, fc = lane & 3;
+    auto At = [&](int I, int J) { return A + (int64_t)J * kTT * lda + I * kTT; };     // tile (I, J) of the block
+    auto Xt = [&](int I, int J) { return Li + (int64_t)J * kTT * ldi + I * kTT; };    // tile (I, J) of inv(L)
+    for (;;) {
+        __syncthreads();
+        if (tid == 0) s_task = (int)atomicAdd(next, 1u);
+        __syncthreads();
+        const int t = s_task;
+        if (t >= ntasks) break;
+        int type, i, j, b;
+        decode_task(T, t, type, i, j, b);
+        unsigned long long t0 = 0, t1 = 0;
+        if (trace && tid == 0) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        if (tid == 0) {
+            bool ok = true;
+            switch (type) {
+                case TK_P:   // needs X_{b-1}, and tiles (b, b-1), (b, b) updated through step b-2
+                    if (b > 0) ok = wait_ge(&fP[b - 1], 1u, abort_flag);
+                    if (ok && b > 1) ok = wait_ge(&fU[b * T + b - 1], (uint32_t)(b - 1), abort_flag) &&
+                                         wait_ge(&fU[b * T + b], (uint32_t)(b - 1), abort_flag);
+                    break;
+                case TK_S:
+                    ok = wait_ge(&fP[j], 1u, abort_flag);
+                    if (ok && j > 0) ok = wait_ge(&fU[i * T + j], (uint32_t)j, abort_flag);
+                    break;
+                case TK_U:
+                    ok = wait_ge(&fS[i * T + b], 1u, abort_flag) && wait_ge(&fS[j * T + b], 1u, abort_flag);
+                    if (ok && b > 0) ok = wait_ge(&fU[i * T + j], (uint32_t)b, abort_flag);
+                    break;
+                case TK_Z:
+                    ok = wait_ge(&fS[i * T + b], 1u, abort_flag) &&
+                         wait_ge(b == j ? &fP[b] : &fF[b * T + j], 1u, abort_flag);
+                    if (ok && b > j) ok = wait_ge(&fZ[i * T + j], (uint32_t)(b - j), abort_flag);
+                    break;
+                default:   // F(i, j)
+                    ok = wait_ge(&fP[i], 1u, abort_flag) && wait_ge(&fZ[i * T + j], (uint32_t)(i - j), abort_flag);
+                    break;
+            }
+            s_go = ok;
+            if (trace) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t1));
+        }
+        __syncthreads();
+        if (!s_go) break;
+        uint32_t* flag = nullptr;
+        uint32_t fval = 1;
+        double acc[4][2][2], cv[4][2][2];
+        zero_acc(acc);
+        if (type == TK_P) {
+            const double* src = At(b, b);
+            int64_t lds = lda;
+            if (b > 0) {
+                // L_{b,b-1} = A_{b,b-1} X_{b-1,b-1}^T  (published for the other tasks of step b-1)
+                double* Cs = At(b, b - 1);
+                tile_load_T(sA, Cs, lda);
+                tile_load_T(sB, Xt(b - 1, b - 1), ldi);
+                ABFT_FRAG_LOOP { ABFT_FRAG_MN; cv[x][y][h] = (m >= n) ? __ldcg(At(b, b) + (int64_t)n * lda + m) : 0.0; }
+                cpa_wait_all();
+                __syncthreads();
+                tile_mma(acc, sA, sB, wm, wn, fr, fc);
+                __syncthreads();
+                ABFT_FRAG_LOOP { ABFT_FRAG_MN; Cs[(int64_t)n * lda + m] = acc[x][y][h]; sA[n * kTP + m] = acc[x][y][h]; }
+                __syncthreads();
+                if (tid == 0) { __threadfence(); st_release(&fS[b * T + b - 1], 1u); }
+                // A_bb -= L_{b,b-1} L_{b,b-1}^T into shared memory (the leaf's input)
+                zero_acc(acc);
+                tile_mma(acc, sA, sA, wm, wn, fr, fc);
+                ABFT_FRAG_LOOP { ABFT_FRAG_MN; sB[n * kTP + m] = cv[x][y][h] - acc[x][y][h]; }
+                __syncthreads();
+                src = sB; lds = kTP;
+            }
+            if (!leaf_tile(src, lds, At(b, b), lda, Xt(b, b), ldi, sB, sA, info_off + b * kTT, st)) break;
+            flag = &fP[b];
+        } else if (type == TK_S || type == TK_U || type == TK_Z) {
+            double* C;
+            bool add = true, lower = false;
+            if (type == TK_S) {          // L_ib = A_ib X_bb^T, in place (the tile is staged first)
+                C = At(i, j);
+                tile_load_T(sA, C, lda);
+                tile_load_T(sB, Xt(j, j), ldi);
+                flag = &fS[i * T + j];
+                add = false;
+            } else if (type == TK_U) {   // A_ij -= L_ib L_jb^T
+                C = At(i, j);
+                tile_load_T(sA, At(i, b), lda);
+                tile_load_T(sB, At(j, b), lda);
+                flag = &fU[i * T + j];
+                fval = (uint32_t)(b + 1);
+                lower = (i == j);
+            } else {                     // Y_ij (+)= L_ib X_bj
+                C = Xt(i, j);
+                tile_load_T(sA, At(i, b), lda);
+                tile_load_N(sB, Xt(b, j), ldi);
+                flag = &fZ[i * T + j];
+                fval = (uint32_t)(b - j + 1);
+                add = (b > j);
+            }
+            const int64_t ldc = (type == TK_Z) ? ldi : lda;
+            if (add) { ABFT_FRAG_LOOP { ABFT_FRAG_MN; cv[x][y][h] = (!lower || m >= n) ? __ldcg(C + (int64_t)n * ldc + m) : 0.0; } }
+            cpa_wait_all();
+            __syncthreads();
+            tile_mma(acc, sA, sB, wm, wn, fr, fc);
+            ABFT_FRAG_LOOP {
+                ABFT_FRAG_MN;
+                if (type == TK_U) { if (!lower || m >= n) C[(int64_t)n * ldc + m] = cv[x][y][h] - acc[x][y][h]; }
+                else C[(int64_t)n * ldc + m] = add ? cv[x][y][h] + acc[x][y][h] : acc[x][y][h];
+            }
+        } else {   // F(i, j): X_ij = -X_ii Y_ij, and the zero tile (j, i) of inv(L)
+            tile_load_T(sA, Xt(i, i), ldi);
+            tile_load_N(sB, Xt(i, j), ldi);
+            cpa_wait_all();
+            __syncthreads();
+            tile_mma(acc, sA, sB, wm, wn, fr, fc);
+            double* Xij = Xt(i, j);
+            double* Xji = Xt(j, i);
+            ABFT_FRAG_LOOP { ABFT_FRAG_MN; Xij[(int64_t)n * ldi + m] = -acc[x][y][h]; Xji[(int64_t)n * ldi + m] = 0.0; }
+            flag = &fF[i * T + j];
+        }
+        __syncthreads();
+        if (tid == 0) { __threadfence(); st_release(flag, fval); }
+        if (trace && tid == 0) {   // diagnostics (abft_dev_chol_trace): who ran what, when
+            unsigned long long t2, smid;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t2));
+            asm volatile("{ .reg .u32 r; mov.u32 r, %%smid; cvt.u64.u32 %0, r; }" : "=l"(smid));
+            trace[4 * t + 0] = (unsigned long long)type | ((unsigned long long)i << 8) | ((unsigned long long)j << 16) |
+                               ((unsigned long long)b << 24) | (smid << 32) | ((unsigned long long)blockIdx.x << 48);
+            trace[4 * t + 1] = t0; trace[4 * t + 2] = t1; trace[4 * t + 3] = t2;
+        }
+    }
+    // exit: the last CTA out resets the sync area for the next launch
+    __syncthreads();
+    if (tid == 0) {
+        __threadfence();
+        s_go = (atomicAdd(exited, 1u) == gridDim.x - 1);
+    }
+    __syncthreads();
+    if (s_go) {
+        __threadfence();
+        for (int e = tid; e < task_sync_words(T); e += kTaskThreads) sync[e] = 0u;
+    }
+}
+
 }  // namespace abft
 
 using namespace abft;
+
+size_t chol_sync_bytes(int64_t nb) {   // <= the scratch `tmp` callers allocate ((nb/2 + 64)^2 doubles)
+    const int64_t T = std::max<int64_t>(1, std::min<int64_t>(nb / kTT, 32));
+    return sizeof(uint32_t) * (size_t)task_sync_words((int)T);
+}
+
+// Path choice: the one-launch task graph when the block tiles by 64 (nb % 64 == 0, nb >= 128,
+// 16-byte aligned with an even leading dimension); the recursive multi-launch path otherwise or
+// with ABFT_CHOL=rec (kept for comparison).
+static thread_local unsigned long long* g_chol_trace = nullptr;   // abft_dev_chol_trace only
+void chol_set_trace(unsigned long long* t) { g_chol_trace = t; }
+int chol_task_count(int64_t nb) { return (nb % kTT == 0 && nb / kTT <= 32) ? task_count((int)(nb / kTT)) : 0; }
+
+static bool use_tasks(const double* T, int64_t ldt, int64_t B) {
+    const char* e = getenv("ABFT_CHOL");   // read per call (tests switch paths inside one process)
+    return !(e && !strcmp(e, "rec")) && B % kTT == 0 && B >= 2 * kTT && B / kTT <= 32 && ((uintptr_t)T & 15) == 0 && ldt % 2 == 0;
+}
 
 int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,
                 const int32_t* abort_flag, cudaStream_t s) {
@@ -167,6 +555,21 @@ static void chol_inv_rec(double* T, int64_t ldt, double* Li, int64_t ldi, int64_
 // Factor the B x B diagonal tile at T and produce inv(L) in Li (B x B, ld B, upper zeroed).
 int launch_chol_inv(double* T, int64_t ldt, double* Li, int64_t B, int64_t info_off, double* tmp,
                     DevState* st, cudaStream_t s) {
+    if (use_tasks(T, ldt, B)) {
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k_chol_inv_tasks, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTaskSmem);
+            attr = true;
+        }
+        static int gmax = -1;
+        if (gmax < 0) { const char* e = getenv("ABFT_CHOL_G"); gmax = e ? std::max(1, atoi(e)) : 32; }
+        const int Tt = (int)(B / kTT), nt = task_count(Tt);
+        const int grid = std::min(nt, gmax);
+        k_chol_inv_tasks<<<grid, kTaskThreads, kTaskSmem, s>>>(T, ldt, Li, B, Tt, nt, info_off,
+                                                               reinterpret_cast<uint32_t*>(tmp), st, g_chol_trace);
+        abft_count_launch();
+        return 0;
+    }
     launch_zero(B, B, Li, B, s);
     chol_inv_rec(T, ldt, Li, B, 0, B, info_off, tmp, st, s);
     return 0;

@@ -30,8 +30,19 @@ def run_block(P, A):
     return st, P.to_numpy_colmajor(At), P.to_numpy_colmajor(Li)
 
 
+@pytest.fixture(params=["tasks", "rec"])
+def chol_path(request, monkeypatch):
+    """Both diagonal-block paths: the one-launch task graph (nb % 64 == 0, nb >= 128) and the
+    recursive multi-launch path (ABFT_CHOL=rec, read by the library per call)."""
+    if request.param == "rec":
+        monkeypatch.setenv("ABFT_CHOL", "rec")
+    else:
+        monkeypatch.delenv("ABFT_CHOL", raising=False)
+    return request.param
+
+
 @pytest.mark.parametrize("nb", [29, 64, 96, 128, 192, 512, 1024])
-def test_chol_inv_matches_oracle(P, nb):
+def test_chol_inv_matches_oracle(P, nb, chol_path):
     A = syn.spd_matrix(nb, seed=nb + 7)
     st, L, Li = run_block(P, A)
     assert st == 0
@@ -50,7 +61,7 @@ def test_chol_inv_matches_oracle(P, nb):
 
 
 @pytest.mark.parametrize("bad", [0, 63, 64, 200, 511])
-def test_chol_inv_not_spd_info(P, bad):
+def test_chol_inv_not_spd_info(P, bad, chol_path):
     """A leading minor of order bad+1 that is not positive: LAPACK info = bad + 1."""
     import torch
     nb = 512
