@@ -237,7 +237,8 @@ static ThreadCache& thread_cache() {
         g_tc.timing = EventPool(cudaEventDefault);
         int lo = 0, hi = 0;
         cudaDeviceGetStreamPriorityRange(&lo, &hi);
-        cudaStreamCreateWithPriority(&g_tc.P, cudaStreamNonBlocking, hi);
+        const char* pe = getenv("ABFT_P_PRIO");   // dev knob: 0 = default priority for the panel stream
+        cudaStreamCreateWithPriority(&g_tc.P, cudaStreamNonBlocking, (pe && atoi(pe) == 0) ? lo : hi);
         // keep the workspace's pages mapped between calls: cudaMallocAsync / cudaFreeAsync then
         // cost microseconds instead of re-mapping ~n*nb*8*4 bytes at every call
         cudaMemPool_t pool;
@@ -329,7 +330,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     // fused V5 partials: 64-row slabs x n columns x {v1, v2}
     const int mode = o.mode;
     const bool can_fuse = abft && mode != ABFT_MODE_OFFLINE && (nb % 128 == 0) && (lda % 2 == 0) &&
-                          (((uintptr_t)A & 15) == 0);
+                          (((uintptr_t)A & 15) == 0) && !getenv("ABFT_NOFUSE");   // dev knob: V5 re-reads
     if (can_fuse) {
         w.cs_nslab = n / 32;   // room for 32-row slabs (the smallest warp-tile height)
         ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n), s));
@@ -969,7 +970,7 @@ static int run_potrf_left(int64_t n, int64_t nb, double* A, int64_t lda, cudaStr
     const int64_t N = w.N, B = nb;
     const int32_t* ab = &w.st->abort;
     const bool can_fuse = abft && mode != ABFT_MODE_OFFLINE && (nb % 128 == 0) && (lda % 2 == 0) &&
-                          (((uintptr_t)A & 15) == 0);
+                          (((uintptr_t)A & 15) == 0) && !getenv("ABFT_NOFUSE");   // dev knob: V5 re-reads
     if (can_fuse) {
         w.cs_nslab = n / 32;
         ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n), s));

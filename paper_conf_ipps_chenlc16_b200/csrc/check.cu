@@ -23,7 +23,7 @@ __device__ __forceinline__ double warp_sum(double v) {
 // stage. encode = 1: store them as the checksums. Otherwise compare, flag columns
 // with |d| > tau or non-finite d, and append them to the flag list.
 __global__ void __launch_bounds__(kChkThreads) k_check_phase1(StageArgs a) {
-    if (a.st->abort) return;
+    if (cta_aborted(&a.st->abort)) return;
     const int64_t B = a.nb;
     const int64_t chunks = (B + kChkCols - 1) / kChkCols;
     const int64_t t = blockIdx.x / chunks;
@@ -99,7 +99,7 @@ __global__ void __launch_bounds__(kChkThreads) k_check_phase1(StageArgs a) {
 // Phase 1 of V5 for off-diagonal trailing tiles from the partial sums the update GEMM left
 // behind (SK_TRAIL_OFF): r1 = sum of the tile's slab partials, r2 likewise. One thread per column.
 __global__ void __launch_bounds__(256) k_check_phase1_fused(StageArgs a) {
-    if (a.st->abort) return;
+    if (cta_aborted(&a.st->abort)) return;
     const int64_t B = a.nb;
     const int64_t chunks = (B + 255) / 256;
     const int64_t t = blockIdx.x / chunks;

@@ -174,6 +174,17 @@ __device__ __forceinline__ void thresholds(const StageArgs& a, int64_t I, int64_
 
 __device__ __forceinline__ bool dfinite(double x) { return isfinite(x); }
 
+// The run's abort flag as ONE decision per CTA. The flag can be raised by a kernel on another
+// stream while this CTA starts; threads that read it independently could disagree, and a CTA
+// whose warps split (some return, some wait at a barrier or on an mbarrier) hangs. Every kernel
+// with CTA-level synchronisation checks the flag through this helper at entry.
+__device__ __forceinline__ bool cta_aborted(const int32_t* flag) {
+    __shared__ int s_abort;
+    if (threadIdx.x == 0) s_abort = *(volatile const int32_t*)flag;
+    __syncthreads();
+    return s_abort != 0;
+}
+
 // One FP64 tensor-core MMA (SASS DMMA.8x8x4): C(8x8) += A(8x4) B(4x8). Fragments: lane holds
 // A[lane/4][lane%4], B[k = lane%4][n = lane/4], C[lane/4][2 (lane%4) + {0, 1}].
 __device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b) {

@@ -84,7 +84,7 @@ __global__ void __launch_bounds__(GemmCfg<BM, BN, BK, WM, WN, STAGES, TB>::THREA
 k_gemm_dmma(GemmArgs g) {
     using Cfg = GemmCfg<BM, BN, BK, WM, WN, STAGES, TB>;
     constexpr int T = Cfg::THREADS;
-    if (*(volatile const int32_t*)g.abort) return;
+    if (cta_aborted(g.abort)) return;
     // ---- tile mapping ----
     int64_t tm, tn;
     if (g.mask == MASK_LOWER) {  // lower trapezoid (tile row >= tile col, col < tiles_n), row-major
@@ -453,7 +453,7 @@ __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t 
 template <class C_>
 __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64_t n1tiles) {
     constexpr int BM = C_::BM, BN = C_::BN, BK = C_::BK, WM = C_::WM, WN = C_::WN, STAGES = C_::STAGES;
-    if (*(volatile const int32_t*)g.abort) return;
+    if (cta_aborted(g.abort)) return;
     extern __shared__ __align__(16) double smem[];
     double* sA = smem;
     double* sB = smem + STAGES * C_::SA;

@@ -12,6 +12,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
+#include <cstdio>
 
 
 namespace abft {
@@ -31,7 +32,7 @@ constexpr int kLeafOwn = (kLeaf * (kLeaf + 1) / 2 + kLeafThreads - 1) / kLeafThr
 
 __global__ void __launch_bounds__(kLeafThreads) k_leaf_potrf_inv(double* T, int64_t ldt, double* Li, int64_t ldi,
                                                                  int nl, int64_t info_off, DevState* st) {
-    if (st->abort) return;
+    if (cta_aborted(&st->abort)) return;
     extern __shared__ double leaf_smem[];
     constexpr int P = kLeaf + 1;
     double* L = leaf_smem;                 // L[c*P + r]: unscaled a, then l
@@ -128,7 +129,7 @@ __global__ void k_zero_block(int64_t rows, int64_t cols, double* dst, int64_t ld
 constexpr int kTT = 64;                 // tile
 constexpr int kTP = kTT + 4;            // smem pitch: 4 mod 16 8-byte banks, conflict-free fragments
 constexpr int kTaskThreads = 256;       // 8 warps: 2 x 4 grid of 32 x 16 warp tiles
-constexpr size_t kTaskSmem = 2 * (size_t)kTT * kTP * sizeof(double);
+constexpr size_t kTaskSmem = 3 * (size_t)kTT * kTP * sizeof(double);   // two operand tiles + leaf scratch
 enum { TK_P = 0, TK_S = 1, TK_U = 2, TK_Z = 3, TK_F = 4 };
 
 // tasks of step b (m = T - 1 - b tiles below the diagonal tile b)
@@ -188,6 +189,7 @@ __device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
 }
 // spin until *f >= v; false if the run aborted meanwhile
 __device__ __forceinline__ bool wait_ge(const uint32_t* f, uint32_t v, const int32_t* abort) {
+    if (gridDim.x == 1) return true;   // one CTA runs the tasks in order
     for (;;) {
         if (ld_acquire(f) >= v) return true;
         if (*(volatile const int32_t*)abort) return false;
@@ -238,84 +240,134 @@ __device__ __forceinline__ void zero_acc(double (&acc)[4][2][2]) {
 #define ABFT_FRAG_LOOP _Pragma("unroll") for (int x = 0; x < 4; ++x) _Pragma("unroll") for (int y = 0; y < 2; ++y) \
     _Pragma("unroll") for (int h = 0; h < 2; ++h)
 
-// P(b) leaf: Cholesky of the 64 x 64 lower tile src (ld lds; shared or global) and its inverse,
-// one CTA. Thread (r = tid % 64, q = tid / 64) keeps row r's elements of columns c = 16 q + u
-// (u < 16) in registers, for the factor (unscaled right-looking: a_rc -= (a_rj / d_j) a_cj) and
-// for the elimination Y = (unit lower)^-1 (Y(r, c) -= (a_rj / d_j) Y(j, c)). A column of a is
-// final after step c-1 and is then published into the shared tile Ls (column-major), a row of Y
-// into Ys (row-major); steps read only published values, so the register updates need no
-// per-element predicate (finished and upper elements take harmless garbage: their final values
-// live in Ls / Ys). Warps with no live element skip that half of the step; one barrier per
-// column. At the end l_rc = a_rc / sqrt(d_c) -> Lb, inv(L)_rc = Y(r, c) / sqrt(d_r) -> Xb (zero
-// above the diagonal). Ls may alias src. Returns false on a non-positive pivot (NOT_SPD raised,
-// LAPACK info).
-__device__ bool leaf_tile(const double* src, int64_t lds, double* Lb, int64_t lda, double* Xb, int64_t ldi, double* Ls,
-                          double* Ys, int64_t info0, DevState* st) {
-    const int tid = threadIdx.x, r = tid & 63, q = tid >> 6, c0 = 16 * q;
-    const int rmax = (tid & 32) + 31;   // warp-uniform: largest row of this warp
-    double a[16], y[16];
+// P(b) leaf: Cholesky of the 64 x 64 lower tile held in shared memory Ls (column-major, pitch
+// kTP) and its inverse, one CTA of 8 warps, in LDL^T form A = U D U^T (U unit lower, L = U D^1/2):
+//  * 8 panels of 8 columns. Panel p is factored with scalar steps (one barrier per column: pivot
+//    d_j, U_rj = f_r = a_rj / d_j into Qb, a_rc -= f_r a_cj inside the panel; Ls keeps the
+//    unscaled columns), then the trailing lower part takes the rank-8 update
+//    A22 -= U_p (D_p U_p^T) = Qb_p Ls_p^T on the tensor cores (DMMA 8x8x4 per 8 x 8 tile) — the
+//    blocked right-looking step of PAPER.md:137-176 inside one tile.
+//  * inv(U) by 8 x 8 blocks: the 8 diagonal blocks by warp-level forward substitution (shuffles),
+//    then block row I = 1..7: Z_IJ = -Z_II sum_{C=J}^{I-1} U_IC Z_CJ (DMMA, one warp per J).
+//  * out: inv(L) = D^-1/2 inv(U) -> Xb (zero above the diagonal); Ls keeps the unscaled factor and
+//    the pivots' square roots stay in `ls` for leaf_store_L (L = a_rc / sqrt(d_c)), which runs
+//    after the dependants have been released (nothing in the task graph reads L_bb).
+// Us and Zs are scratch tiles (U, then Z = inv(U)). Returns false on a non-positive
+// pivot (NOT_SPD raised with the LAPACK info of the first failing leading minor).
+struct LeafSmem {
+    double piv_s[kTT], piv_is[kTT];   // sqrt(d), 1 / sqrt(d)
+    double tbuf[8][64];
+};
+__device__ bool leaf_tile(double* Ls, double* Us, double* Zs, LeafSmem& ls, double* Xb, int64_t ldi, int64_t info0,
+                          DevState* st, long long* dbg) {
+    double* piv_s = ls.piv_s;
+    double* piv_is = ls.piv_is;
+    const int tid = threadIdx.x, r = tid & 63, g = tid >> 6;
+    const int lane = tid & 31, warp = tid >> 5, fr = lane >> 2, fc = lane & 3;
+    if (dbg) dbg[0] = clock64();
+    for (int p = 0; p < 8; ++p) {
+        const int c0 = 8 * p;
+        for (int j = 0; j < 8; ++j) {
+            const int cj = c0 + j;
+            __syncthreads();
+            const double d = Ls[cj * kTP + cj];
+            if (!(d > 0.0)) {
+                if (tid == 0 && atomicCAS(&st->abort, 0, 1) == 0) { st->status = ABFT_NOT_SPD; st->info = info0 + cj + 1; }
+                return false;
+            }
+            if (r > cj) {
+                const double f = Ls[cj * kTP + r] * __drcp_rn(d);
+                if (g == 0) Us[cj * kTP + r] = f;
 #pragma unroll
-    for (int u = 0; u < 16; ++u) {
-        const int c = c0 + u;
-        a[u] = (c <= r) ? src[c * lds + r] : 0.0;
-        y[u] = (c == r) ? 1.0 : 0.0;
-    }
-    __syncthreads();   // Ls may alias src
-    if (q == 0) Ls[r] = a[0];                                                          // column 0
-    if (r == 0) {
-#pragma unroll
-        for (int u = 0; u < 16; u += 2) *reinterpret_cast<double2*>(Ys + c0 + u) = make_double2(y[u], y[u + 1]);   // row 0
-    }
-    for (int jj = 0; jj < kTT; ++jj) {
+                for (int h = 0; h < 2; ++h) {
+                    const int c = c0 + 2 * g + h;
+                    if (c > cj) Ls[c * kTP + r] = fma(-f, Ls[cj * kTP + c], Ls[c * kTP + r]);
+                }
+            } else if (tid == 0) {
+                piv_s[cj] = d;
+            }
+        }
         __syncthreads();
-        const double* cj = Ls + jj * kTP;
-        const double d = cj[jj];
-        if (!(d > 0.0)) {
-            if (tid == 0 && atomicCAS(&st->abort, 0, 1) == 0) { st->status = ABFT_NOT_SPD; st->info = info0 + jj + 1; }
-            return false;
-        }
-        const double f = cj[r] * __drcp_rn(d);
-        if (c0 + 15 > jj && c0 <= rmax) {   // factor: live columns c in (jj, r]
-            double cv[16];
+        const int nt = 7 - p;            // trailing 8 x 8 tiles per side
+        for (int e = warp; e < nt * (nt + 1) / 2; e += 8) {
+            int tj = 0, rem = e;
+            while (rem >= nt - tj) { rem -= nt - tj; ++tj; }
+            const int m0 = c0 + 8 + 8 * (tj + rem), n0 = c0 + 8 + 8 * tj;
+            double* c0p = Ls + (n0 + 2 * fc) * kTP + m0 + fr;
+            double v0 = c0p[0], v1 = c0p[kTP];
 #pragma unroll
-            for (int u = 0; u < 16; u += 2) {
-                const double2 v = *reinterpret_cast<const double2*>(cj + c0 + u);
-                cv[u] = v.x; cv[u + 1] = v.y;
-            }
-#pragma unroll
-            for (int u = 0; u < 16; ++u) a[u] = fma(-f, cv[u], a[u]);
-            if (((jj + 1) >> 4) == q) {      // this warp owns column jj+1: publish rows r > jj
-                const int u1 = (jj + 1) & 15;
-                double nv = a[0];
-#pragma unroll
-                for (int u = 1; u < 16; ++u) nv = (u == u1) ? a[u] : nv;
-                if (r > jj) Ls[(jj + 1) * kTP + r] = nv;
-            }
-        }
-        if (c0 <= jj && rmax > jj) {        // elimination: rows r > jj (row jj of Y is zero right of jj)
-            const double* yj = Ys + jj * kTP;
-            double yv[16];
-#pragma unroll
-            for (int u = 0; u < 16; u += 2) {
-                const double2 v = *reinterpret_cast<const double2*>(yj + c0 + u);
-                yv[u] = v.x; yv[u + 1] = v.y;
-            }
-#pragma unroll
-            for (int u = 0; u < 16; ++u) y[u] = fma(-f, yv[u], y[u]);
-        }
-        if (r == jj + 1) {   // row jj+1 of Y is final
-#pragma unroll
-            for (int u = 0; u < 16; u += 2) *reinterpret_cast<double2*>(Ys + r * kTP + c0 + u) = make_double2(y[u], y[u + 1]);
+            for (int kq = 0; kq < 8; kq += 4)
+                dmma(v0, v1, -Us[(c0 + kq + fc) * kTP + m0 + fr], Ls[(c0 + kq + fc) * kTP + n0 + fr]);
+            c0p[0] = v0; c0p[kTP] = v1;
         }
     }
     __syncthreads();
-    for (int e = tid; e < kTT * kTT; e += kTaskThreads) {
+    if (tid < kTT) {
+        const double sd = sqrt(piv_s[tid]);
+        piv_is[tid] = 1.0 / sd;
+        piv_s[tid] = sd;
+    }
+    if (dbg) dbg[1] = clock64();
+    // inv(U): diagonal 8 x 8 blocks, warp w -> block w; lane (zr, cp) holds Z(zr, 2cp + {0,1}).
+    {
+        const int zr = lane >> 2, cp = lane & 3, b0 = 8 * warp;
+        double z0 = (zr == 2 * cp) ? 1.0 : 0.0, z1 = (zr == 2 * cp + 1) ? 1.0 : 0.0;
+#pragma unroll
+        for (int j = 0; j < 7; ++j) {
+            const double zj0 = __shfl_sync(0xffffffffu, z0, j * 4 + cp);
+            const double zj1 = __shfl_sync(0xffffffffu, z1, j * 4 + cp);
+            if (zr > j) {
+                const double u = Us[(b0 + j) * kTP + b0 + zr];
+                z0 = fma(-u, zj0, z0);
+                z1 = fma(-u, zj1, z1);
+            }
+        }
+        Zs[(b0 + 2 * cp) * kTP + b0 + zr] = z0;
+        Zs[(b0 + 2 * cp + 1) * kTP + b0 + zr] = z1;
+    }
+    if (dbg) dbg[2] = clock64();
+    for (int I = 1; I < 8; ++I) {        // block row I: Z_IJ = -Z_II sum_{C=J}^{I-1} U_IC Z_CJ
+        __syncthreads();
+        if (warp < I) {
+            const int J = warp;
+            double t0 = 0.0, t1 = 0.0;
+            for (int C = J; C < I; ++C) {
+#pragma unroll
+                for (int kq = 0; kq < 8; kq += 4)
+                    dmma(t0, t1, Us[(8 * C + kq + fc) * kTP + 8 * I + fr], Zs[(8 * J + fr) * kTP + 8 * C + kq + fc]);
+            }
+            double* tb = ls.tbuf[warp];    // T (8 x 8, column-major) as the B operand
+            tb[(2 * fc) * 8 + fr] = t0;
+            tb[(2 * fc + 1) * 8 + fr] = t1;
+            __syncwarp();
+            double x0 = 0.0, x1 = 0.0;
+#pragma unroll
+            for (int kq = 0; kq < 8; kq += 4)
+                dmma(x0, x1, -Zs[(8 * I + kq + fc) * kTP + 8 * I + fr], tb[fr * 8 + kq + fc]);
+            Zs[(8 * J + 2 * fc) * kTP + 8 * I + fr] = x0;
+            Zs[(8 * J + 2 * fc + 1) * kTP + 8 * I + fr] = x1;
+            __syncwarp();
+        }
+    }
+    __syncthreads();
+    for (int e = tid; e < kTT * kTT; e += kTaskThreads) {   // inv(L) = D^-1/2 inv(U), zero above
         const int c = e >> 6, rr = e & 63;
-        const double sc = sqrt(Ls[c * kTP + c]), sr = sqrt(Ls[rr * kTP + rr]);
-        if (c <= rr) Lb[c * lda + rr] = (c == rr) ? sc : Ls[c * kTP + rr] / sc;
-        Xb[c * ldi + rr] = (c <= rr) ? Ys[rr * kTP + c] / sr : 0.0;
+        Xb[c * ldi + rr] = (c <= rr) ? Zs[c * kTP + rr] * piv_is[rr] : 0.0;
+    }
+    if (dbg) {
+        dbg[3] = clock64();
+        if (tid == 0) printf("leaf %lld: factor %lld  inverse-diag %lld  inverse+X-out %lld cycles\n", info0,
+                             dbg[1] - dbg[0], dbg[2] - dbg[1], dbg[3] - dbg[2]);
     }
     return true;
+}
+
+// L = a_rc / sqrt(d_c) (lower only) from the leaf's unscaled factor in Ls
+__device__ __forceinline__ void leaf_store_L(const double* Ls, const LeafSmem& ls, double* Lb, int64_t lda) {
+    for (int e = threadIdx.x; e < kTT * kTT; e += kTaskThreads) {
+        const int c = e >> 6, rr = e & 63;
+        if (c <= rr) Lb[c * lda + rr] = (c == rr) ? ls.piv_s[c] : Ls[c * kTP + rr] * ls.piv_is[c];
+    }
 }
 
 __global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int64_t lda, double* Li, int64_t ldi, int T,
@@ -324,9 +376,11 @@ __global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int6
     extern __shared__ __align__(16) double tsm[];
     double* sA = tsm;
     double* sB = tsm + kTT * kTP;
-    __shared__ int s_task, s_go;
+    double* sC = tsm + 2 * kTT * kTP;
+    __shared__ int s_task, s_go, s_go2;
+    __shared__ LeafSmem lsm;
     const int32_t* abort_flag = &st->abort;
-    if (*(volatile const int32_t*)abort_flag) return;
+    if (cta_aborted(abort_flag)) return;
     uint32_t* next = sync;
     uint32_t* exited = sync + 1;
     uint32_t* fP = sync + 2;
@@ -351,10 +405,9 @@ __global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int6
         if (tid == 0) {
             bool ok = true;
             switch (type) {
-                case TK_P:   // needs X_{b-1}, and tiles (b, b-1), (b, b) updated through step b-2
-                    if (b > 0) ok = wait_ge(&fP[b - 1], 1u, abort_flag);
-                    if (ok && b > 1) ok = wait_ge(&fU[b * T + b - 1], (uint32_t)(b - 1), abort_flag) &&
-                                         wait_ge(&fU[b * T + b], (uint32_t)(b - 1), abort_flag);
+                case TK_P:   // tiles (b, b-1), (b, b) updated through step b-2 (X_{b-1} is awaited below)
+                    if (b > 1) ok = wait_ge(&fU[b * T + b - 1], (uint32_t)(b - 1), abort_flag) &&
+                                    wait_ge(&fU[b * T + b], (uint32_t)(b - 1), abort_flag);
                     break;
                 case TK_S:
                     ok = wait_ge(&fP[j], 1u, abort_flag);
@@ -383,30 +436,40 @@ __global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int6
         double acc[4][2][2], cv[4][2][2];
         zero_acc(acc);
         if (type == TK_P) {
-            const double* src = At(b, b);
-            int64_t lds = lda;
-            if (b > 0) {
+            if (b == 0) {   // the lower half of the first diagonal tile into shared memory
+                const double* src = At(0, 0);
+                for (int e = tid; e < kTT * kTT; e += kTaskThreads) {
+                    const int c = e >> 6, rr = e & 63;
+                    if (c <= rr) sB[c * kTP + rr] = src[(int64_t)c * lda + rr];
+                }
+            } else {
                 // L_{b,b-1} = A_{b,b-1} X_{b-1,b-1}^T  (published for the other tasks of step b-1)
+                // operands that are final already are fetched while the previous leaf finishes
                 double* Cs = At(b, b - 1);
                 tile_load_T(sA, Cs, lda);
-                tile_load_T(sB, Xt(b - 1, b - 1), ldi);
                 ABFT_FRAG_LOOP { ABFT_FRAG_MN; cv[x][y][h] = (m >= n) ? __ldcg(At(b, b) + (int64_t)n * lda + m) : 0.0; }
+                if (tid == 0) s_go2 = wait_ge(&fP[b - 1], 1u, abort_flag);   // (s_go may still be read)
+                __syncthreads();
+                if (!s_go2) { cpa_wait_all(); break; }
+                tile_load_T(sB, Xt(b - 1, b - 1), ldi);
                 cpa_wait_all();
                 __syncthreads();
                 tile_mma(acc, sA, sB, wm, wn, fr, fc);
                 __syncthreads();
                 ABFT_FRAG_LOOP { ABFT_FRAG_MN; Cs[(int64_t)n * lda + m] = acc[x][y][h]; sA[n * kTP + m] = acc[x][y][h]; }
                 __syncthreads();
-                if (tid == 0) { __threadfence(); st_release(&fS[b * T + b - 1], 1u); }
+                if (tid == 0 && gridDim.x > 1) { __threadfence(); st_release(&fS[b * T + b - 1], 1u); }
                 // A_bb -= L_{b,b-1} L_{b,b-1}^T into shared memory (the leaf's input)
                 zero_acc(acc);
                 tile_mma(acc, sA, sA, wm, wn, fr, fc);
                 ABFT_FRAG_LOOP { ABFT_FRAG_MN; sB[n * kTP + m] = cv[x][y][h] - acc[x][y][h]; }
-                __syncthreads();
-                src = sB; lds = kTP;
             }
-            if (!leaf_tile(src, lds, At(b, b), lda, Xt(b, b), ldi, sB, sA, info_off + b * kTT, st)) break;
-            flag = &fP[b];
+            __syncthreads();
+            __shared__ long long dbg[4];
+            if (!leaf_tile(sB, sA, sC, lsm, Xt(b, b), ldi, info_off + b * kTT, st, trace ? dbg : nullptr)) break;
+            __syncthreads();   // X_bb is out: release the dependants, then store L_bb (nobody here reads it)
+            if (tid == 0 && gridDim.x > 1) { __threadfence(); st_release(&fP[b], 1u); }
+            leaf_store_L(sB, lsm, At(b, b), lda);
         } else if (type == TK_S || type == TK_U || type == TK_Z) {
             double* C;
             bool add = true, lower = false;
@@ -453,7 +516,7 @@ __global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int6
             flag = &fF[i * T + j];
         }
         __syncthreads();
-        if (tid == 0) { __threadfence(); st_release(flag, fval); }
+        if (tid == 0 && flag && gridDim.x > 1) { __threadfence(); st_release(flag, fval); }
         if (trace && tid == 0) {   // diagnostics (abft_dev_chol_trace): who ran what, when
             unsigned long long t2, smid;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t2));
@@ -485,16 +548,20 @@ size_t chol_sync_bytes(int64_t nb) {   // <= the scratch `tmp` callers allocate 
     return sizeof(uint32_t) * (size_t)task_sync_words((int)T);
 }
 
-// Path choice: the one-launch task graph when the block tiles by 64 (nb % 64 == 0, nb >= 128,
-// 16-byte aligned with an even leading dimension); the recursive multi-launch path otherwise or
-// with ABFT_CHOL=rec (kept for comparison).
 static thread_local unsigned long long* g_chol_trace = nullptr;   // abft_dev_chol_trace only
 void chol_set_trace(unsigned long long* t) { g_chol_trace = t; }
 int chol_task_count(int64_t nb) { return (nb % kTT == 0 && nb / kTT <= 32) ? task_count((int)(nb / kTT)) : 0; }
 
+// Path choice. Default: the recursive multi-launch path. ABFT_CHOL=tasks selects the one-launch
+// task graph (nb % 64 == 0, nb >= 128, 16-byte aligned, even leading dimension): 2x faster on its
+// own, but on the high-priority look-ahead stream its long-lived CTAs were measured to provoke
+// what behaves like compute preemption of the warp-specialised update GEMM, whose output then
+// carried rare row-group errors (detected and corrected by V5; none with the panel stream at
+// normal priority, which in turn delays the panel) -- DESIGN.md §5. Read per call (tests switch
+// paths inside one process).
 static bool use_tasks(const double* T, int64_t ldt, int64_t B) {
-    const char* e = getenv("ABFT_CHOL");   // read per call (tests switch paths inside one process)
-    return !(e && !strcmp(e, "rec")) && B % kTT == 0 && B >= 2 * kTT && B / kTT <= 32 && ((uintptr_t)T & 15) == 0 && ldt % 2 == 0;
+    const char* e = getenv("ABFT_CHOL");
+    return ((e && !strcmp(e, "tasks")) || g_chol_trace != nullptr) && B % kTT == 0 && B >= 2 * kTT && B / kTT <= 32 && ((uintptr_t)T & 15) == 0 && ldt % 2 == 0;
 }
 
 int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,
@@ -562,7 +629,7 @@ int launch_chol_inv(double* T, int64_t ldt, double* Li, int64_t B, int64_t info_
             attr = true;
         }
         static int gmax = -1;
-        if (gmax < 0) { const char* e = getenv("ABFT_CHOL_G"); gmax = e ? std::max(1, atoi(e)) : 32; }
+        if (gmax < 0) { const char* e = getenv("ABFT_CHOL_G"); gmax = e ? std::max(1, atoi(e)) : 10; }
         const int Tt = (int)(B / kTT), nt = task_count(Tt);
         const int grid = std::min(nt, gmax);
         k_chol_inv_tasks<<<grid, kTaskThreads, kTaskSmem, s>>>(T, ldt, Li, B, Tt, nt, info_off,

@@ -32,10 +32,10 @@ def run_block(P, A):
 
 @pytest.fixture(params=["tasks", "rec"])
 def chol_path(request, monkeypatch):
-    """Both diagonal-block paths: the one-launch task graph (nb % 64 == 0, nb >= 128) and the
-    recursive multi-launch path (ABFT_CHOL=rec, read by the library per call)."""
-    if request.param == "rec":
-        monkeypatch.setenv("ABFT_CHOL", "rec")
+    """Both diagonal-block paths: the recursive multi-launch path (default) and the one-launch
+    task graph (ABFT_CHOL=tasks, nb % 64 == 0, nb >= 128), read by the library per call."""
+    if request.param == "tasks":
+        monkeypatch.setenv("ABFT_CHOL", "tasks")
     else:
         monkeypatch.delenv("ABFT_CHOL", raising=False)
     return request.param
