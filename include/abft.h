@@ -223,6 +223,15 @@ int abft_dev_chol_inv(int64_t nb, double* A, int64_t lda, double* Li, abft_strea
 int abft_dev_chol_trace(int64_t nb, double* A, int64_t lda, double* Li, uint64_t* trace_host, int64_t cap,
                         abft_stream_t stream);
 
+/* Graph mode. A fault-free Enhanced (or ABFT-off) right-looking abft_potrf / abft_potrf_ex call
+ * without the per-phase profiler is captured once into a CUDA graph (both streams) and replayed
+ * on later calls with the same device, n, nb, A, lda, options and report capacity: no host launch
+ * cost, shorter dependent-launch gaps on the panel chain. The graph and its workspace are cached
+ * per host thread (one entry) and stay allocated until the key changes or this call releases
+ * them. Default for n <= 12288 (measured faster there, slower above); ABFT_GRAPH=0 / 1 in the
+ * environment forces direct launches / graph mode. Returns 0. */
+int abft_graph_release(void);
+
 /* Diagnostics: kernel launches issued by the last call on this thread, a static version string,
  * and the text of the last CUDA error seen on this thread (empty if none). */
 int64_t abft_last_launch_count(void);

@@ -97,7 +97,7 @@ for _f in ("abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_po
 EXPORTS = ["abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
            "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist",
            "abft_last_launch_count", "abft_version", "abft_last_error", "abft_last_profile", "abft_dev_gemm_nt", "abft_dev_chol_inv",
-           "abft_dev_chol_trace", "abft_potrf_dist_sim",
+           "abft_dev_chol_trace", "abft_potrf_dist_sim", "abft_graph_release",
            "abft_phase_name"]
 
 
@@ -343,6 +343,11 @@ def abft_dev_chol_trace(nb, A, Li, stream=None):
         rows.append((w & 255, (w >> 8) & 255, (w >> 16) & 255, (w >> 24) & 255, (w >> 32) & 0xFFFF, w >> 48,
                      int(buf[4 * t + 1]), int(buf[4 * t + 2]), int(buf[4 * t + 3])))
     return nt, rows
+
+
+def abft_graph_release():
+    """Free the cached graph-mode factorisation (graph + workspace) of this thread."""
+    return int(_lib.abft_graph_release())
 
 
 def abft_last_launch_count():

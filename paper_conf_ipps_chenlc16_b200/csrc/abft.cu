@@ -99,6 +99,8 @@ static int collect_inj(const abft_inject_spec_t* inj, int64_t n, int64_t nb, std
     return 0;
 }
 
+namespace abft { bool is_update_kernel(const void* f); }
+
 // ---- workspace -------------------------------------------------------------------------------
 struct Work {
     int64_t n, nb, N;
@@ -317,13 +319,29 @@ static void do_inject_if(const std::vector<abft_inject_spec_t>& list, int64_t k,
 // the rest of update k and V5 to the trailing matrix. Hook timing and the set of events are
 // those of the sequential schedule: injections and checks are split by block column exactly
 // where the two streams split the work.
+// Buffers owned by a captured graph (graph mode, see run_graph): run_potrf then only enqueues the
+// work (resets, kernels, cross-stream events) and leaves the report to the caller.
+struct Persist {
+    Work w;
+    double* W1 = nullptr;
+};
+
 static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t s,
-                     const std::vector<abft_inject_spec_t>& inj, abft_report_t* rep, const abft_options_t& o) {
+                     const std::vector<abft_inject_spec_t>& inj, abft_report_t* rep, const abft_options_t& o,
+                     Persist* ps = nullptr) {
     const bool abft = o.abft_enabled != 0;
     const int K = std::max(1, o.K);
     Work w;
-    int rc = work_alloc(w, n, nb, n, rep ? std::max<int64_t>(rep->cap, 1) : 1024, abft, s);
-    if (rc) return rc;
+    int rc = 0;
+    if (ps) {
+        w = ps->w;
+        ABFT_CUDA_TRY(cudaMemsetAsync(w.st, 0, sizeof(DevState), s));
+        ABFT_CUDA_TRY(cudaMemsetAsync(w.tmp, 0, chol_sync_bytes(nb), s));
+        rep = nullptr;
+    } else {
+        rc = work_alloc(w, n, nb, n, rep ? std::max<int64_t>(rep->cap, 1) : 1024, abft, s);
+        if (rc) return rc;
+    }
     const int64_t N = w.N, B = nb;
     const double Bd = (double)B;
     const int32_t* ab = &w.st->abort;
@@ -331,20 +349,22 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     const int mode = o.mode;
     const bool can_fuse = abft && mode != ABFT_MODE_OFFLINE && (nb % 128 == 0) && (lda % 2 == 0) &&
                           (((uintptr_t)A & 15) == 0) && !getenv("ABFT_NOFUSE");   // dev knob: V5 re-reads
-    if (can_fuse) {
+    if (can_fuse && !ps) {
         w.cs_nslab = n / 32;   // room for 32-row slabs (the smallest warp-tile height)
         ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n), s));
     }
+    if (ps && can_fuse && !w.cs) return ABFT_ERR_CUDA;
     // second panel buffer for the look-ahead
-    double* Wbuf[2] = {w.W, nullptr};
+    double* Wbuf[2] = {w.W, ps ? ps->W1 : nullptr};
     const int64_t wrows = (N - 1) * nb + 2 * N + 2;
-    ABFT_CUDA_TRY(cudaMallocAsync((void**)&Wbuf[1], sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb), s));
+    if (!ps)
+        ABFT_CUDA_TRY(cudaMallocAsync((void**)&Wbuf[1], sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb), s));
     ThreadCache& tc = thread_cache();
     cudaStream_t P = tc.P;
     auto new_event = [&]() { return tc.sync.get(); };
     cudaEvent_t e0 = nullptr, e1 = nullptr;
     if (rep) { e0 = tc.timing.get(); e1 = tc.timing.get(); cudaEventRecord(e0, s); }
-    Profiler prof; prof.on = o.profile != 0; prof.pool = &tc.timing;
+    Profiler prof; prof.on = o.profile != 0 && !ps; prof.pool = &tc.timing;
     const double lowerB = Bd * (Bd + 1) / 2;                 // elements of a tril tile
     launch_zero(B, B, w.Li, B, s);
     if (abft) {   // encode
@@ -516,6 +536,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         prof.end(t, PH_V6, s, 4.0 * el, 8.0 * el);
     }
     ABFT_CUDA_TRY(cudaGetLastError());
+    if (ps) return 0;   // graph mode: the caller launches, reports and keeps the buffers
     int status = 0;
     if (rep) {
         cudaEventRecord(e1, s);
@@ -529,6 +550,152 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     if (rc) return rc;
     ABFT_CUDA_TRY(cudaGetLastError());
     return status;
+}
+
+static int run_potrf_direct(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t s,
+                            const std::vector<abft_inject_spec_t>& inj, abft_report_t* rep, const abft_options_t& o) {
+    return run_potrf(n, nb, A, lda, s, inj, rep, o, nullptr);
+}
+
+// ---- graph mode ------------------------------------------------------------------------------
+// The whole right-looking factorisation (both streams, ~12k kernels at n = 32768) captured once
+// into a CUDA graph and replayed: no host launch overhead and shorter dependent-launch gaps on
+// the look-ahead stream's panel chain. One cached graph per thread, keyed by every argument that
+// shapes the work (device, n, nb, A, lda, options, event capacity); its workspace stays allocated
+// until the key changes or abft_graph_release() is called. Used for fault-free calls only
+// (injection lists change the hook sequence) and without the per-phase profiler.
+struct GraphEntry {
+    bool valid = false;
+    int dev = -1;
+    int64_t n = 0, nb = 0, lda = 0, cap = 0;
+    double* A = nullptr;
+    abft_options_t o{};
+    cudaGraphExec_t exec = nullptr;
+    cudaStream_t cs = nullptr;   // private capture / launch stream (the caller's may be the legacy one)
+    Persist ps;
+    int64_t launches = 0;
+};
+static thread_local GraphEntry g_graph;
+
+static void graph_release(GraphEntry& g) {
+    if (g.exec) cudaGraphExecDestroy(g.exec);
+    Work& w = g.ps.w;
+    for (void* p : {(void*)w.chk, (void*)w.scl, (void*)w.W, (void*)w.Li, (void*)w.tmp, (void*)w.st, (void*)w.ev,
+                    (void*)w.cs, (void*)g.ps.W1})
+        if (p) cudaFree(p);
+    cudaStream_t cs = g.cs;
+    g = GraphEntry();
+    g.cs = cs;
+}
+
+// Default: graph mode for n <= 12288, where launch gaps are a visible share of the step (C2,
+// n = 4096 nb = 256: 7.3 -> 6.2 ms; n = 8192 nb = 1024: 17.5 -> 16.5 ms). Above it the replayed
+// graph was measured slower than direct launches (n = 16384: 59.9 vs 67.4 ms, n = 32768: 375.6 vs
+// 397.9 ms, with or without per-node priorities), so large problems launch directly.
+// ABFT_GRAPH=0 / 1 forces it off / on.
+static bool graph_mode_enabled(int64_t n) {
+    const char* e = getenv("ABFT_GRAPH");
+    if (e) return atoi(e) != 0;
+    return n <= 12288;
+}
+
+static int run_graph(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t s, abft_report_t* rep,
+                     const abft_options_t& o) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    GraphEntry& g = g_graph;
+    const int64_t cap = rep ? std::max<int64_t>(rep->cap, 1) : 1024;
+    const bool hit = g.valid && g.dev == dev && g.n == n && g.nb == nb && g.A == A && g.lda == lda && g.cap == cap &&
+                     !memcmp(&g.o, &o, sizeof o);
+    if (!hit) {
+        if (g.valid || g.exec) { cudaStreamSynchronize(g.cs); graph_release(g); }
+        if (!g.cs || g.dev != dev) ABFT_CUDA_TRY(cudaStreamCreateWithFlags(&g.cs, cudaStreamNonBlocking));
+        const int64_t N = n / nb;
+        Work& w = g.ps.w;
+        w.n = n; w.nb = nb; w.N = N; w.ldc = std::max<int64_t>(1, 2 * N);
+        const bool abft = o.abft_enabled != 0;
+        const int64_t wrows = std::max<int64_t>((N - 1) * nb + 2 * N + 2, 1);
+        const size_t tmpn = (size_t)(((nb + 1) / 2 + 64) * ((nb + 1) / 2 + 64));
+        if (abft) {
+            ABFT_CUDA_TRY(cudaMalloc((void**)&w.chk, sizeof(double) * (size_t)(w.ldc * n)));
+            ABFT_CUDA_TRY(cudaMalloc((void**)&w.scl, sizeof(double) * (size_t)(n + 2 * N + 1)));
+            w.cs_nslab = n / 32;
+            ABFT_CUDA_TRY(cudaMalloc((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n)));
+        }
+        ABFT_CUDA_TRY(cudaMalloc((void**)&w.W, sizeof(double) * (size_t)(wrows * nb)));
+        ABFT_CUDA_TRY(cudaMalloc((void**)&g.ps.W1, sizeof(double) * (size_t)(wrows * nb)));
+        ABFT_CUDA_TRY(cudaMalloc((void**)&w.Li, sizeof(double) * (size_t)(nb * nb)));
+        ABFT_CUDA_TRY(cudaMalloc((void**)&w.tmp, sizeof(double) * tmpn));
+        ABFT_CUDA_TRY(cudaMalloc((void**)&w.st, sizeof(DevState)));
+        w.ev_cap = cap;
+        ABFT_CUDA_TRY(cudaMalloc((void**)&w.ev, sizeof(abft_event_t) * (size_t)cap));
+        g.dev = dev;
+        // capture: everything run_potrf enqueues on cs and on the look-ahead stream it forks
+        const std::vector<abft_inject_spec_t> none;
+        ABFT_CUDA_TRY(cudaStreamBeginCapture(g.cs, cudaStreamCaptureModeRelaxed));
+        g_launches = 0;
+        const int rc = run_potrf(n, nb, A, lda, g.cs, none, nullptr, o, &g.ps);
+        cudaGraph_t graph = nullptr;
+        const cudaError_t ce = cudaStreamEndCapture(g.cs, &graph);
+        if (rc || ce != cudaSuccess || !graph) {
+            if (graph) cudaGraphDestroy(graph);
+            cudaGetLastError();
+            graph_release(g);
+            return rc ? rc : ABFT_ERR_CUDA;
+        }
+        {   // stream priorities are not kept by capture: restore the panel chain's precedence by
+            // giving every kernel node except the trailing updates the high priority
+            size_t nn = 0;
+            cudaGraphGetNodes(graph, nullptr, &nn);
+            std::vector<cudaGraphNode_t> nodes(nn);
+            if (nn) cudaGraphGetNodes(graph, nodes.data(), &nn);
+            int lo = 0, hi = 0;
+            cudaDeviceGetStreamPriorityRange(&lo, &hi);
+            for (cudaGraphNode_t nd : nodes) {
+                cudaGraphNodeType t;
+                if (cudaGraphNodeGetType(nd, &t) != cudaSuccess || t != cudaGraphNodeTypeKernel) continue;
+                cudaKernelNodeParams kp;
+                if (cudaGraphKernelNodeGetParams(nd, &kp) != cudaSuccess) continue;
+                if (abft::is_update_kernel(kp.func)) continue;
+                cudaKernelNodeAttrValue v;
+                memset(&v, 0, sizeof v);
+                v.priority = hi;
+                cudaGraphKernelNodeSetAttribute(nd, cudaLaunchAttributePriority, &v);
+            }
+            cudaGetLastError();
+        }
+        const cudaError_t ie = cudaGraphInstantiate(&g.exec, graph, 0);
+        cudaGraphDestroy(graph);
+        if (ie != cudaSuccess) { cudaGetLastError(); graph_release(g); return ABFT_ERR_CUDA; }
+        g.launches = g_launches;
+        g.n = n; g.nb = nb; g.A = A; g.lda = lda; g.cap = cap; g.o = o; g.valid = true;
+    }
+    // stream semantics of the caller's s: cs waits for s, s waits for the graph
+    ThreadCache& tc = thread_cache();
+    cudaEvent_t fork = tc.sync.get(), join = tc.sync.get();
+    cudaEvent_t e0 = tc.timing.get(), e1 = tc.timing.get();
+    cudaEventRecord(fork, s);
+    cudaStreamWaitEvent(g.cs, fork, 0);
+    cudaEventRecord(e0, g.cs);
+    ABFT_CUDA_TRY(cudaGraphLaunch(g.exec, g.cs));
+    cudaEventRecord(e1, g.cs);
+    cudaEventRecord(join, g.cs);
+    cudaStreamWaitEvent(s, join, 0);
+    g_launches = g.launches;
+    int status = 0;
+    ABFT_CUDA_TRY(cudaGetLastError());
+    const int rc = finish_report(g.ps.w, rep, g.cs, &status);
+    if (rc) return rc;
+    if (rep) { float ms = 0; cudaEventElapsedTime(&ms, e0, e1); rep->seconds = ms * 1e-3; }
+    return status;
+}
+
+extern "C" int abft_graph_release(void) {
+    if (g_graph.valid || g_graph.exec) {
+        if (g_graph.cs) cudaStreamSynchronize(g_graph.cs);
+        graph_release(g_graph);
+    }
+    return 0;
 }
 
 
@@ -1091,10 +1258,13 @@ extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft
     const bool redo = o.mode == ABFT_MODE_ENHANCED_REDO;   // NEXT-4: Enhanced + re-do on UNCORRECTABLE
     if (redo) o.mode = ABFT_MODE_ENHANCED;
     if (o.order != ABFT_ORDER_RIGHT && o.order != ABFT_ORDER_LEFT) return -8;
-    const RunFn run = o.order == ABFT_ORDER_LEFT ? run_potrf_left : run_potrf;
+    const RunFn run = o.order == ABFT_ORDER_LEFT ? run_potrf_left : run_potrf_direct;
     if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; rep->reruns = 0; }
     if (n == 0) return 0;
     cudaStream_t s = (cudaStream_t)stream;
+    if (((o.mode == ABFT_MODE_ENHANCED && !redo) || !o.abft_enabled) && o.order == ABFT_ORDER_RIGHT && list.empty() &&
+        !o.profile && graph_mode_enabled(n))
+        return run_graph(n, nb, A, lda, s, rep, o);
     if ((o.mode == ABFT_MODE_ENHANCED && !redo) || !o.abft_enabled) return run(n, nb, A, lda, s, list, rep, o);
     // Online / Offline: keep the input; an uncorrectable outcome or a detection by the final
     // sweep means an error propagated -> re-do the factorisation once, without the faults.

@@ -655,6 +655,13 @@ static int run_ws(GemmArgs g, cudaStream_t s, bool update) {
     return 0;
 }
 
+// The trailing-update entry points (graph mode gives every other kernel node the panel stream's
+// high priority, these keep the default one).
+bool is_update_kernel(const void* f) {
+    return f == (const void*)k_update_ws<WsCfg> || f == (const void*)k_update_ws<WsCfg16> ||
+           f == (const void*)k_update_ws<WsCfg2a> || f == (const void*)k_update_ws<WsCfg2b>;
+}
+
 static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CTA/SM), 16, 2a
     static int v = -1;
     if (v < 0) {
