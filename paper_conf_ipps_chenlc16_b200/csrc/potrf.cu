@@ -539,6 +539,26 @@ __global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int6
     }
 }
 
+// The recursive path's 64 x 64 leaf with the blocked DMMA leaf routine (one short launch, 8
+// warps): lower half of T -> shared memory, factor + inverse (leaf_tile), L back into T.
+__global__ void __launch_bounds__(kTaskThreads) k_leaf64_blocked(double* T, int64_t ldt, double* Li, int64_t ldi,
+                                                                 int64_t info_off, DevState* st) {
+    if (cta_aborted(&st->abort)) return;
+    extern __shared__ __align__(16) double lsm_dyn[];
+    double* Ls = lsm_dyn;
+    double* Us = lsm_dyn + kTT * kTP;
+    double* Zs = lsm_dyn + 2 * kTT * kTP;
+    __shared__ LeafSmem lsm;
+    for (int e = threadIdx.x; e < kTT * kTT; e += kTaskThreads) {
+        const int c = e >> 6, rr = e & 63;
+        if (c <= rr) Ls[c * kTP + rr] = T[(int64_t)c * ldt + rr];
+    }
+    __syncthreads();
+    if (!leaf_tile(Ls, Us, Zs, lsm, Li, ldi, info_off, st, nullptr)) return;
+    __syncthreads();
+    leaf_store_L(Ls, lsm, T, ldt);
+}
+
 }  // namespace abft
 
 using namespace abft;
@@ -583,11 +603,29 @@ int launch_zero(int64_t rows, int64_t cols, double* dst, int64_t ldd, cudaStream
     return 0;
 }
 
+// 64 x 64 leaves of the recursive path: the blocked DMMA leaf (default) or the one-barrier-per-
+// column shared-memory leaf (ABFT_LEAF=scalar; also every leaf narrower than 64).
+static bool blocked_leaf() {
+    const char* e = getenv("ABFT_LEAF");
+    return !(e && !strcmp(e, "scalar"));
+}
+
 // Recursive factorisation of the diagonal block [off, off+sz) of the B x B tile T (ldt) with
 // its inverse into Li (ld = B). tmp: >= (B/2)^2 doubles of scratch.
 static void chol_inv_rec(double* T, int64_t ldt, double* Li, int64_t ldi, int64_t off, int64_t sz,
                          int64_t info_off, double* tmp, DevState* st, cudaStream_t s) {
     const int32_t* ab = &st->abort;
+    if (sz == kTT && blocked_leaf()) {
+        static bool attr64 = false;
+        if (!attr64) {
+            cudaFuncSetAttribute(k_leaf64_blocked, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTaskSmem);
+            attr64 = true;
+        }
+        k_leaf64_blocked<<<1, kTaskThreads, kTaskSmem, s>>>(T + off * ldt + off, ldt, Li + off * ldi + off, ldi,
+                                                          info_off + off, st);
+        abft_count_launch();
+        return;
+    }
     if (sz <= kLeaf) {
         static bool attr = false;
         const int smem = 2 * kLeaf * (kLeaf + 1) * (int)sizeof(double);
