@@ -90,13 +90,24 @@ __global__ void __launch_bounds__(kLeafThreads) k_leaf_potrf_inv(double* T, int6
     }
 }
 
+// Column-major block copy (the W -> A / chk write-back, L21 in the recursion): blockIdx.y walks
+// columns, threads walk rows two at a time (16-byte accesses when both sides allow), no division.
 __global__ void k_copy_block(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst,
-                             int64_t ldd, const int32_t* abort_flag) {
+                             int64_t ldd, const int32_t* abort_flag, int vec) {
     if (*abort_flag) return;
-    const int64_t total = rows * cols;
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t c = i / rows, r = i % rows;
-        dst[c * ldd + r] = src[c * lds + r];
+    for (int64_t c = blockIdx.y; c < cols; c += gridDim.y) {
+        const double* sc = src + c * lds;
+        double* dc = dst + c * ldd;
+        if (vec) {
+            for (int64_t r = 2 * (blockIdx.x * (int64_t)blockDim.x + threadIdx.x); r < rows;
+                 r += 2 * (int64_t)gridDim.x * blockDim.x) {
+                if (r + 1 < rows) *reinterpret_cast<double2*>(dc + r) = *reinterpret_cast<const double2*>(sc + r);
+                else dc[r] = sc[r];
+            }
+        } else {
+            for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < rows; r += (int64_t)gridDim.x * blockDim.x)
+                dc[r] = sc[r];
+        }
     }
 }
 
@@ -587,9 +598,11 @@ static bool use_tasks(const double* T, int64_t ldt, int64_t B) {
 int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,
                 const int32_t* abort_flag, cudaStream_t s) {
     if (rows <= 0 || cols <= 0) return 0;
-    const int64_t total = rows * cols;
-    const int64_t blocks = std::min<int64_t>((total + 255) / 256, 148 * 16);
-    k_copy_block<<<(unsigned)blocks, 256, 0, s>>>(rows, cols, src, lds, dst, ldd, abort_flag);
+    const int vec = (((uintptr_t)src | (uintptr_t)dst) & 15) == 0 && lds % 2 == 0 && ldd % 2 == 0;
+    const int64_t per = vec ? 512 : 256;                       // rows one CTA covers per pass
+    const int64_t bx = std::min<int64_t>((rows + per - 1) / per, 64);
+    const int64_t by = std::min<int64_t>(cols, std::max<int64_t>(1, 148 * 8 / bx));
+    k_copy_block<<<dim3((unsigned)bx, (unsigned)by), 256, 0, s>>>(rows, cols, src, lds, dst, ldd, abort_flag, vec);
     abft_count_launch();
     return 0;
 }
