@@ -228,6 +228,7 @@ struct EventPool {
 struct ThreadCache {
     int device = -1;
     cudaStream_t P = nullptr;
+    cudaStream_t P2 = nullptr;   // panel side stream: V2 runs here while P factors the diagonal block
     EventPool sync{cudaEventDisableTiming};
     EventPool timing{cudaEventDefault};
 };
@@ -241,6 +242,7 @@ static ThreadCache& thread_cache() {
         cudaDeviceGetStreamPriorityRange(&lo, &hi);
         const char* pe = getenv("ABFT_P_PRIO");   // dev knob: 0 = default priority for the panel stream
         cudaStreamCreateWithPriority(&g_tc.P, cudaStreamNonBlocking, (pe && atoi(pe) == 0) ? lo : hi);
+        cudaStreamCreateWithPriority(&g_tc.P2, cudaStreamNonBlocking, (pe && atoi(pe) == 0) ? lo : hi);
         // keep the workspace's pages mapped between calls: cudaMallocAsync / cudaFreeAsync then
         // cost microseconds instead of re-mapping ~n*nb*8*4 bytes at every call
         cudaMemPool_t pool;
@@ -390,16 +392,33 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         const double md = (double)m, mBd = (double)mB;
         Work wk = w; wk.W = W;
         if (abft) do_inject_if(inj, k, ABFT_HOOK_REST, B, L, ab, P, k, k + 1, true);   // REST(k) into column k
+        cudaEvent_t v2done = nullptr;
         if (abft && mode == ABFT_MODE_ENHANCED) {
-            StageArgs a = stage_base(wk, A, lda, o.c_tau, SK_COLUMN, ABFT_V2, (int)k);
-            a.flist = 1;
+            // V1 (tile k,k) gates POTRF; V2 (the tiles below) only has to precede the TRSM, so it
+            // runs on the side stream P2 while P factors the diagonal block (same checks, same
+            // events: both are labelled V2 as one column stage; separate flag lists)
+            StageArgs a1 = stage_base(wk, A, lda, o.c_tau, m > 0 ? SK_COL_DIAG : SK_COLUMN, ABFT_V2, (int)k);
+            a1.flist = 1;
             cudaEvent_t t = prof.begin(P);
-            launch_check(a, P);                                                  // V1, V2
-            prof.end(t, PH_V12, P, 4.0 * (lowerB + mBd * Bd), 8.0 * (lowerB + mBd * Bd));
+            launch_check(a1, P);                                                 // V1
+            prof.end(t, PH_V12, P, 4.0 * lowerB, 8.0 * lowerB);
+            if (m > 0) {
+                cudaEvent_t f = new_event();
+                cudaEventRecord(f, P);
+                cudaStreamWaitEvent(tc.P2, f, 0);
+                StageArgs a2 = stage_base(wk, A, lda, o.c_tau, SK_COL_BELOW, ABFT_V2, (int)k);
+                a2.flist = 2;
+                t = prof.begin(tc.P2);
+                launch_check(a2, tc.P2);                                         // V2
+                prof.end(t, PH_V12, tc.P2, 4.0 * mBd * Bd, 8.0 * mBd * Bd);
+                v2done = new_event();
+                cudaEventRecord(v2done, tc.P2);
+            }
         }
         cudaEvent_t t = prof.begin(P);
         launch_chol_inv(Akk, lda, w.Li, B, k * B, w.tmp, w.st, P);
         prof.end(t, PH_POTRF, P, 2.0 * Bd * Bd * Bd / 3.0, 0);
+        if (v2done) cudaStreamWaitEvent(P, v2done, 0);                          // V2 before the TRSM reads
         // TRSM (+ Alg. 2 on the checksum rows of tile (k,k)): one GEMM per row segment
         t = prof.begin(P);
         launch_gemm(mB, B, B, Akk + B, lda, w.Li, B, W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, P);

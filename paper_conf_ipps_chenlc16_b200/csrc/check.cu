@@ -259,7 +259,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
                     const long long ev_i = (long long)atomicAdd(&st->nev, 1ull);
                     if (ev_i < a.ev_cap) {
                         abft_event_t& ev = a.ev[ev_i];
-                        ev.k = a.k; ev.check = (a.kind == SK_COLUMN && f.I == a.k) ? ABFT_V1 : a.V;
+                        ev.k = a.k; ev.check = ((a.kind == SK_COLUMN || a.kind == SK_COL_DIAG) && f.I == a.k) ? ABFT_V1 : a.V;
                         ev.tile_i = f.I; ev.tile_j = f.J;
                         ev.row = (int32_t)sr; ev.col = (int32_t)sc; ev.kind = kind; ev.rank = a.rank;
                         ev.delta1 = f.d1; ev.delta2 = f.d2;
@@ -272,7 +272,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
                 const long long ev_i = (long long)atomicAdd(&st->nev, 1ull);
                 if (ev_i < a.ev_cap) {
                     abft_event_t& ev = a.ev[ev_i];
-                    ev.k = a.k; ev.check = (a.kind == SK_COLUMN && f.I == a.k) ? ABFT_V1 : a.V;
+                    ev.k = a.k; ev.check = ((a.kind == SK_COLUMN || a.kind == SK_COL_DIAG) && f.I == a.k) ? ABFT_V1 : a.V;
                     ev.tile_i = f.I; ev.tile_j = f.J;
                     ev.row = kind == ABFT_KIND_CHK1 ? -1 : kind == ABFT_KIND_CHK2 ? -2 : -3;
                     ev.col = (int32_t)c; ev.kind = kind; ev.rank = a.rank;

@@ -32,7 +32,7 @@ struct DevState {
     unsigned long long nev;        // events raised
     unsigned long long n_checks;   // tile checks run
     long long n_detected, n_data, n_nonfinite, n_chk1, n_chk2, n_unc;
-    FlagList fl[2];       // [0]: main stream, [1]: look-ahead panel stream
+    FlagList fl[3];       // [0]: main stream, [1]: look-ahead panel stream, [2]: panel side stream (V2)
 };
 
 // Where the tiles of a check stage live (DESIGN.md §5 "data layout").
@@ -45,6 +45,8 @@ enum StageKind : int32_t {
     SK_TRAIL_OFF = 5,  // V5, off-diagonal trailing tiles, recalculation from the GEMM's fused partials
     SK_TRAIL_DIAG = 6, // V5, diagonal trailing tiles (J, J), J in [j_lo, j_hi), re-read as sym(tril)
     SK_LEFT_L = 7,     // V7 (left-looking): L tiles (I, J), J < k, I in [k, k + j_hi), factored
+    SK_COL_DIAG = 8,   // V1 alone: tile (k, k) in A, unfactored (the part POTRF reads)
+    SK_COL_BELOW = 9,  // V2 alone: tiles (k+1..N-1, k) in A, unfactored (runs concurrently with POTRF)
 };
 
 struct StageArgs {
@@ -76,6 +78,8 @@ __host__ __device__ __forceinline__ int64_t stage_count(const StageArgs& a) {
     const int64_t N = a.N, k = a.k;
     switch (a.kind) {
         case SK_COLUMN: return N - k;
+        case SK_COL_DIAG: return 1;
+        case SK_COL_BELOW: return N - k - 1;
         case SK_DIAG_FACT: return 1;
         case SK_PANEL: return N - k - 1;
         case SK_TRAIL: {
@@ -97,6 +101,8 @@ __device__ __forceinline__ void stage_tile(const StageArgs& a, int64_t t, int64_
     const int64_t N = a.N, k = a.k;
     switch (a.kind) {
         case SK_COLUMN: I = k + t; J = k; return;
+        case SK_COL_DIAG: I = k; J = k; return;
+        case SK_COL_BELOW: I = k + 1 + t; J = k; return;
         case SK_DIAG_FACT: I = k; J = k; return;
         case SK_PANEL: I = k + 1 + t; J = k; return;
         case SK_TRAIL_DIAG: I = J = a.j_lo + t; return;
@@ -135,6 +141,8 @@ __device__ __forceinline__ TileView stage_view(const StageArgs& a, int64_t I, in
             v.c1 = a.W + a.mB + 2 + 2 * (I - a.k - 1); v.c2 = v.c1 + 1; v.ldc = a.ldw;
             v.diag = false; v.factored = true; break;
         case SK_COLUMN:
+        case SK_COL_DIAG:
+        case SK_COL_BELOW:
         case SK_TRAIL:
         case SK_TRAIL_OFF:
         case SK_TRAIL_DIAG:
