@@ -51,6 +51,9 @@ struct GemmArgs {
     // column-block stride (ws kernel, MASK_LOWER + checksum segment): column block t of C and of
     // the B operand's rows is global block t * cstride (1D block-cyclic local columns; 1 = dense)
     int64_t cstride;
+    // ws kernel: prefetch into L2 the C tile of tile index t + pf_ahead (0 = off; the launcher
+    // sets it to the number of CTAs resident at once)
+    int64_t pf_ahead;
 };
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
@@ -470,6 +473,7 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
         // ------------------------------- producer -------------------------------
         asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;\n" ::"n"(C_::REG_PROD) : "memory");
         if (warp != C_::CONSUMERS) return;
+        const int64_t pf_ahead = g.pf_ahead;
         uint32_t it = 0;
         for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
             WsTile T;
@@ -483,11 +487,22 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
             const int64_t ldcp = T.seg2 ? g.ldc2 : g.ldc;
             const uint32_t rowsA = (uint32_t)(Ms - m0 < BM ? Ms - m0 : BM), rowsB = (uint32_t)(g.N - n0 < BN ? g.N - n0 : BN);
             const int64_t bn0 = n0 + (g.cstride > 1 ? (n0 / g.nb) * g.nb * (g.cstride - 1) : 0);   // B row of column n0
-            // warm L2 with the C columns of this tile (they are read at the tile's start)
-            if (g.beta != 0.0) {
-                for (int c = lane; c < (int)rowsB; c += 32) prefetch_l2(Cp + (n0 + c) * ldcp + m0, rowsA * 8);
-            }
             for (int kt = 0; kt < kt_n; ++kt, ++it) {
+                if (kt == 1 && g.beta != 0.0 && pf_ahead > 0) {
+                    // warm L2 with the C tile of the CTA that will start about one residency wave
+                    // later (tiles are dispatched in index order), so its accumulator preload
+                    // hits L2 instead of HBM
+                    WsTile Tn;
+                    const int64_t tn = t + pf_ahead;
+                    if (tn < ntiles && ws_tile<BM, BN>(g, tn, n1tiles, Tn)) {
+                        const int64_t Msn = Tn.seg2 ? g.M2 : g.M;
+                        double* Cn = Tn.seg2 ? g.C2 : g.C;
+                        const int64_t ldn = Tn.seg2 ? g.ldc2 : g.ldc;
+                        const uint32_t rA = (uint32_t)(Msn - Tn.m0 < BM ? Msn - Tn.m0 : BM);
+                        const int cB = (int)(g.N - Tn.n0 < BN ? g.N - Tn.n0 : BN);
+                        for (int c = lane; c < cB; c += 32) prefetch_l2(Cn + (Tn.n0 + c) * ldn + Tn.m0, rA * 8);
+                    }
+                }
                 const int st = it % STAGES;
                 const uint32_t ph = (it / STAGES) & 1;
                 if (lane == 0) {
@@ -649,6 +664,15 @@ static int run_ws(GemmArgs g, cudaStream_t s, bool update) {
     static int64_t tpc = -1;
     if (tpc < 0) { const char* e = getenv("ABFT_WS_TPC"); tpc = e ? std::max(1, atoi(e)) : 1; }
     const int64_t grid = std::max<int64_t>(1, (ntiles + tpc - 1) / tpc);
+    static int64_t ahead = -1;
+    if (ahead < 0) {
+        int dev = 0, nsm = 148;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        const char* e = getenv("ABFT_WS_PF");
+        ahead = e ? atoi(e) : (int64_t)nsm * C_::MINB;
+    }
+    g.pf_ahead = (tpc == 1) ? ahead : 0;
     if (update) k_update_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
     else k_gemm_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
     abft_count_launch();
