@@ -229,6 +229,7 @@ struct ThreadCache {
     int device = -1;
     cudaStream_t P = nullptr;
     cudaStream_t P2 = nullptr;   // panel side stream: V2 runs here while P factors the diagonal block
+    cudaStream_t C = nullptr;    // copy stream of abft_potrf_host's overlapped write-back
     EventPool sync{cudaEventDisableTiming};
     EventPool timing{cudaEventDefault};
 };
@@ -321,6 +322,16 @@ static void do_inject_if(const std::vector<abft_inject_spec_t>& list, int64_t k,
 // the rest of update k and V5 to the trailing matrix. Hook timing and the set of events are
 // those of the sequential schedule: injections and checks are split by block column exactly
 // where the two streams split the work.
+// abft_potrf_host's write-back of L overlapped with the factorisation: block column k of L is
+// final once panel k is written back (only V6 can still correct it, which the host path checks),
+// so it is copied to the host on a copy stream while the trailing updates continue.
+struct HostSink {
+    double* host = nullptr;
+    int64_t ldh = 0;
+    cudaStream_t cs = nullptr;
+};
+static thread_local HostSink g_sink;
+
 // Buffers owned by a captured graph (graph mode, see run_graph): run_potrf then only enqueues the
 // work (resets, kernels, cross-stream events) and leaves the report to the caller.
 struct Persist {
@@ -510,7 +521,16 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         const Loc L0{A, lda, w.chk, w.ldc, Wbuf[0], 1, 0};
         do_inject_if(inj, 0, ABFT_HOOK_REST, B, L0, ab, s, 0, 1, false);
     }
+    const bool sink = g_sink.host != nullptr && !ps;
+    auto sink_col = [&](int64_t k) {   // L(kB:n, block column k) -> host, after panel k's write-back
+        if (!sink) return;
+        cudaStreamWaitEvent(g_sink.cs, pan[k], 0);
+        cudaMemcpy2DAsync(g_sink.host + k * B * g_sink.ldh + k * B, g_sink.ldh * sizeof(double), A + k * B * lda + k * B,
+                          lda * sizeof(double), (size_t)(n - k * B) * sizeof(double), (size_t)B,
+                          cudaMemcpyDeviceToHost, g_sink.cs);
+    };
     pan[0] = panel(0);
+    sink_col(0);
     for (int64_t k = 0; k < N; ++k) {
         {
             cudaEvent_t t = prof.begin(s);
@@ -531,6 +551,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         cudaEvent_t ec = new_event(); cudaEventRecord(ec, s);
         cudaStreamWaitEvent(P, ec, 0);
         pan[k + 1] = panel(k + 1);
+        sink_col(k + 1);
         // (b) the rest of the trailing matrix
         if (m > 1) {
             const bool fb = update_cols(k, k + 2, N);
@@ -1344,8 +1365,36 @@ extern "C" int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t ld
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&dA, sizeof(double) * (size_t)(n * n), s));
     ABFT_CUDA_TRY(cudaMemcpy2DAsync(dA, n * sizeof(double), A_host, lda * sizeof(double), n * sizeof(double), n,
                                     cudaMemcpyHostToDevice, s));
-    rc = abft_potrf_ex(n, nb, dA, n, stream, inj, rep, opt);
-    if (rc >= 0 && rc != ABFT_ERR_CUDA)
+    // Overlapped write-back (HostSink) on the direct right-looking Enhanced / ABFT-off path without
+    // injections; anything else (or a V6 event, i.e. a correction of finished L) copies L back
+    // after the factorisation as before.
+    const abft_options_t o = opt ? *opt : default_options();
+    bool has_inj = false;
+    for (const abft_inject_spec_t* q = inj; q && q->k >= 0; ++q) has_inj = true;
+    const bool overlap = !has_inj && o.order == ABFT_ORDER_RIGHT && (o.mode == ABFT_MODE_ENHANCED || !o.abft_enabled) &&
+                         !graph_mode_enabled(n) && getenv("ABFT_HOST_OVERLAP") == nullptr;
+    abft_report_t lrep;
+    std::vector<abft_event_t> lev;
+    abft_report_t* r = rep;
+    if (overlap && !r) {   // the V6 test needs the events
+        memset(&lrep, 0, sizeof lrep);
+        lev.resize(4096); lrep.cap = (int64_t)lev.size(); lrep.events = lev.data();
+        r = &lrep;
+    }
+    if (overlap) {
+        ThreadCache& tc = thread_cache();
+        if (!tc.C) ABFT_CUDA_TRY(cudaStreamCreateWithFlags(&tc.C, cudaStreamNonBlocking));
+        g_sink.host = A_host; g_sink.ldh = lda; g_sink.cs = tc.C;
+    }
+    rc = abft_potrf_ex(n, nb, dA, n, stream, inj, r, opt);
+    bool recopy = !overlap;
+    if (overlap) {
+        g_sink = HostSink();
+        ABFT_CUDA_TRY(cudaStreamSynchronize(thread_cache().C));
+        for (int64_t e = 0; e < std::min<int64_t>(r->n_events, r->cap); ++e) recopy |= (r->events[e].check == ABFT_V6);
+        recopy |= r->n_events > r->cap || rc != 0;
+    }
+    if (recopy && rc >= 0 && rc != ABFT_ERR_CUDA)
         ABFT_CUDA_TRY(cudaMemcpy2DAsync(A_host, lda * sizeof(double), dA, n * sizeof(double), n * sizeof(double), n,
                                         cudaMemcpyDeviceToHost, s));
     cudaFreeAsync(dA, s);

@@ -372,3 +372,22 @@ def test_two_errors_in_a_column_redo_matches_oracle(P, mode):
     if mode == "enhanced_redo":
         assert st == 0 and rep["reruns"] == 1
         assert floor_rel(L, ref.L, A) <= 1e-11
+
+
+@pytest.mark.parametrize("n,nb", [(2048, 256), (3072, 512)])
+def test_host_entry_overlapped_writeback(P, n, nb, monkeypatch):
+    """abft_potrf_host copies each finished block column of L to the host while the factorisation
+    continues (fault-free direct path; ABFT_GRAPH=0 forces direct launches at this size): the host
+    result equals the device path bit for bit and the strict upper triangle keeps the input."""
+    import torch
+    monkeypatch.setenv("ABFT_GRAPH", "0")
+    A = syn.spd_matrix(n)
+    Ah = A.copy(order="F")
+    st, rep = P.abft_potrf_host(n, nb, Ah)
+    assert st == 0 and rep["n_events"] == 0
+    Ad = P.colmajor(A)
+    st2, _ = P.abft_potrf(n, nb, Ad)
+    torch.cuda.synchronize()
+    Ld = P.to_numpy_colmajor(Ad)
+    assert np.array_equal(np.tril(Ah), np.tril(Ld))
+    assert np.array_equal(np.triu(Ah, 1), np.triu(A, 1))
