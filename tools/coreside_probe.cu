@@ -7,10 +7,13 @@
 #include <cstring>
 #include <vector>
 #include <cuda_runtime.h>
+#include <unistd.h>
+#include <cstdlib>
 extern "C" int abft_dev_chol_inv(int64_t, double*, int64_t, double*, void*);
 extern "C" int abft_gen_spd(int64_t, uint64_t, double*, int64_t, void*);
 extern "C" int abft_dev_gemm_nt(int64_t, int64_t, int64_t, const double*, int64_t, const double*, int64_t, double*,
                                 int64_t, double, double, int, void*);
+static int late_smem(int argc) { return argc > 1 ? 120 * 1024 : 104448; }
 __global__ void guest(int mode, long long cycles, double* sink) {
     extern __shared__ double sm[];
     long long t0 = clock64();
@@ -25,8 +28,9 @@ __global__ void guest(int mode, long long cycles, double* sink) {
     }
     if (acc0 == 12345.0) sink[0] = acc0 + acc1;
 }
-int main() {
-    const int64_t M = 16384, K = 512;
+int main(int argc, char** argv) {
+    const bool late = argc > 1;
+    const int64_t M = argc > 2 ? atoll(argv[2]) : 16384, K = argc > 3 ? atoll(argv[3]) : 512;
     std::vector<double> hW(M * K), hC(M * M);
     uint64_t x = 12345;
     for (auto& v : hW) { x = x * 6364136223846793005ull + 1442695040888963407ull; v = (double)(x >> 11) * 0x1p-53 - 0.5; }
@@ -38,7 +42,7 @@ int main() {
     int lo, hi; cudaDeviceGetStreamPriorityRange(&lo, &hi);
     cudaStreamCreateWithPriority(&s2, cudaStreamNonBlocking, hi);
     std::vector<double> ref(M * M), got(M * M);
-    const int gsm = 104448;
+    const int gsm = late_smem(argc);
     cudaFuncSetAttribute(guest, cudaFuncAttributeMaxDynamicSharedMemorySize, gsm);
     double *Ad, *Lid;
     const int64_t nbc = 1024;
@@ -47,8 +51,12 @@ int main() {
         for (int rep = 0; rep < 3; ++rep) {
             cudaMemcpy(C, hC.data(), 8 * M * M, cudaMemcpyHostToDevice);
             cudaDeviceSynchronize();
-            if (mode >= 0 && mode < 4) guest<<<8, 256, gsm, s2>>>(mode, 40000000LL, sink);   // ~20 ms on 8 SMs
+            if (mode >= 0 && mode < 4 && !late) guest<<<8, 256, gsm, s2>>>(mode, 40000000LL, sink);   // ~20 ms on 8 SMs
             abft_dev_gemm_nt(M, M, K, W, M, W, M, C, M, -1.0, 1.0, 1, s1);
+            if (mode >= 0 && mode < 4 && late) {   // arrive while the GEMM fills the GPU (needs whole SMs)
+                usleep(500);
+                for (int q = 0; q < 20; ++q) guest<<<1, 256, gsm, s2>>>(mode, 400000LL, sink);
+            }
             if (mode == 4)   // the task-graph diagonal block as the guest, repeatedly while the GEMM runs
                 for (int q = 0; q < 6; ++q) { abft_gen_spd(nbc, 7 + q, Ad, nbc, s2); abft_dev_chol_inv(nbc, Ad, nbc, Lid, s2); }
             cudaDeviceSynchronize();
