@@ -167,8 +167,10 @@ int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft_stream_t s
 /* End-to-end variant on HOST memory (A_host: n x n column-major, lda >= n; pinned memory
  * recommended): copies A to the device, factors with abft_potrf_ex, copies L back, then
  * synchronises. On the direct fault-free right-looking path (no injections, n above the graph-
- * mode threshold) each block column of L is copied back (rows from its diagonal down) on a
- * copy stream as soon as its panel is written back, overlapped with the remaining updates; if
+ * mode threshold) only the block columns from their diagonal blocks down go to the device (the
+ * strict upper triangle outside the diagonal blocks is never read, as in LAPACK uplo = 'L'), and
+ * each block column of L is copied back on a copy stream as soon as its panel is written back,
+ * overlapped with the remaining updates; if
  * the final sweep V6 corrected anything, or the call failed, the whole matrix is copied again
  * after the factorisation (ABFT_HOST_OVERLAP set in the environment disables the overlap).
  * Same errors as abft_potrf_ex. */

@@ -1363,8 +1363,6 @@ extern "C" int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t ld
     cudaStream_t s = (cudaStream_t)stream;
     double* dA = nullptr;
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&dA, sizeof(double) * (size_t)(n * n), s));
-    ABFT_CUDA_TRY(cudaMemcpy2DAsync(dA, n * sizeof(double), A_host, lda * sizeof(double), n * sizeof(double), n,
-                                    cudaMemcpyHostToDevice, s));
     // Overlapped write-back (HostSink) on the direct right-looking Enhanced / ABFT-off path without
     // injections; anything else (or a V6 event, i.e. a correction of finished L) copies L back
     // after the factorisation as before.
@@ -1373,6 +1371,17 @@ extern "C" int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t ld
     for (const abft_inject_spec_t* q = inj; q && q->k >= 0; ++q) has_inj = true;
     const bool overlap = !has_inj && o.order == ABFT_ORDER_RIGHT && (o.mode == ABFT_MODE_ENHANCED || !o.abft_enabled) &&
                          !graph_mode_enabled(n) && getenv("ABFT_HOST_OVERLAP") == nullptr;
+    if (overlap) {
+        // only what the factorisation reads goes over PCIe: each block column from its diagonal
+        // block down (the strict upper triangle outside the diagonal blocks is never read)
+        for (int64_t k = 0; k < n / nb; ++k)
+            ABFT_CUDA_TRY(cudaMemcpy2DAsync(dA + k * nb * n + k * nb, n * sizeof(double), A_host + k * nb * lda + k * nb,
+                                            lda * sizeof(double), (size_t)(n - k * nb) * sizeof(double), (size_t)nb,
+                                            cudaMemcpyHostToDevice, s));
+    } else {
+        ABFT_CUDA_TRY(cudaMemcpy2DAsync(dA, n * sizeof(double), A_host, lda * sizeof(double), n * sizeof(double), n,
+                                        cudaMemcpyHostToDevice, s));
+    }
     abft_report_t lrep;
     std::vector<abft_event_t> lev;
     abft_report_t* r = rep;
@@ -1394,9 +1403,17 @@ extern "C" int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t ld
         for (int64_t e = 0; e < std::min<int64_t>(r->n_events, r->cap); ++e) recopy |= (r->events[e].check == ABFT_V6);
         recopy |= r->n_events > r->cap || rc != 0;
     }
-    if (recopy && rc >= 0 && rc != ABFT_ERR_CUDA)
-        ABFT_CUDA_TRY(cudaMemcpy2DAsync(A_host, lda * sizeof(double), dA, n * sizeof(double), n * sizeof(double), n,
-                                        cudaMemcpyDeviceToHost, s));
+    if (recopy && rc >= 0 && rc != ABFT_ERR_CUDA) {
+        if (overlap) {   // the device holds only the block columns from their diagonal blocks down
+            for (int64_t k = 0; k < n / nb; ++k)
+                ABFT_CUDA_TRY(cudaMemcpy2DAsync(A_host + k * nb * lda + k * nb, lda * sizeof(double), dA + k * nb * n + k * nb,
+                                                n * sizeof(double), (size_t)(n - k * nb) * sizeof(double), (size_t)nb,
+                                                cudaMemcpyDeviceToHost, s));
+        } else {
+            ABFT_CUDA_TRY(cudaMemcpy2DAsync(A_host, lda * sizeof(double), dA, n * sizeof(double), n * sizeof(double), n,
+                                            cudaMemcpyDeviceToHost, s));
+        }
+    }
     cudaFreeAsync(dA, s);
     ABFT_CUDA_TRY(cudaStreamSynchronize(s));
     return rc;
