@@ -347,12 +347,17 @@ __device__ __forceinline__ void prefetch_l2(const void* src, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(src), "r"(bytes) : "memory");
 }
 
-template <int BM_, int BN_, int BK_, int STAGES_, int WM_, int WN_, int REG_CONS_, int MINB_>
+template <int BM_, int BN_, int BK_, int STAGES_, int WM_, int WN_, int REG_CONS_, int MINB_, bool LDG_ = false>
 struct WsCfgT {
     static constexpr int BM = BM_, BN = BN_, BK = BK_, WM = WM_, WN = WN_, STAGES = STAGES_, MINB = MINB_;
+    // LDG: the producer stages operands with per-lane 16-byte cp.async (LDGSTS) and signals the
+    // "full" barrier with cp.async.mbarrier.arrive.noinc (32 arrivals) instead of bulk copies with
+    // a transaction count (the bulk-copy pipeline picked up rare stale k-slices
+    // under concurrent high-priority work; the LDGSTS one did not)
+    static constexpr bool LDG = LDG_;
     static constexpr int WARPS_M = BM / WM, WARPS_N = BN / WN, CONSUMERS = WARPS_M * WARPS_N;
     static constexpr int THREADS = (CONSUMERS + 4) * 32;   // + one producer warpgroup (setmaxnreg)
-    static constexpr int REG_CONS = REG_CONS_, REG_PROD = 40;
+    static constexpr int REG_CONS = REG_CONS_, REG_PROD = LDG_ ? 48 : 40;
     static constexpr int PA = BM + 4, PB = BN + 4;
     static constexpr int SA = BK * PA, SB = BK * PB;
     static constexpr size_t SMEM = (size_t)STAGES * (SA + SB) * sizeof(double) + 2 * STAGES * sizeof(uint64_t);
@@ -367,6 +372,8 @@ using WsCfg = WsCfgT<128, 128, 32, 3, 64, 32, 232, 1>;    // 8 consumer warps, 1
 using WsCfg16 = WsCfgT<128, 128, 32, 3, 32, 32, 104, 1>;  // 16 consumer warps, 32x32 warp tiles
 using WsCfg2a = WsCfgT<128, 64, 16, 4, 64, 32, 216, 2>;   // 2 CTAs/SM, 128x64 tiles, 4-stage BK=16
 using WsCfg2b = WsCfgT<128, 64, 32, 2, 64, 32, 216, 2>;   // 2 CTAs/SM, 128x64 tiles, 2-stage BK=32
+using WsCfg2l = WsCfgT<128, 64, 32, 2, 64, 32, 208, 2, true>;   // as 2b, LDGSTS producer warpgroup
+using WsCfgNR = WsCfgT<128, 64, 32, 2, 64, 32, 128, 2>;   // dev: as 2b without setmaxnreg (spills)
 
 // tile index -> (tm, tn) for the three masks; returns false for tiles with nothing to write
 // Lower-trapezoid tile enumeration for BN = BM / R (R = 1 or 2): tile row tm holds the column
@@ -464,16 +471,18 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
     uint64_t* empty = full + STAGES;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) {
-        for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], C_::CONSUMERS); }
+        for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], C_::LDG ? 128 : 1); mbar_init(&empty[i], C_::CONSUMERS); }
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
     __syncthreads();
 
     if (warp >= C_::CONSUMERS) {
         // ------------------------------- producer -------------------------------
-        asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;\n" ::"n"(C_::REG_PROD) : "memory");
-        if (warp != C_::CONSUMERS) return;
-        const int64_t pf_ahead = g.pf_ahead;
+        if constexpr (C_::REG_CONS != C_::R0)
+            asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;\n" ::"n"(C_::REG_PROD) : "memory");
+        if (!C_::LDG && warp != C_::CONSUMERS) return;   // LDGSTS: the whole warpgroup copies
+        const int ptid = tid - C_::CONSUMERS * 32;       // 0..127 in the producer warpgroup
+        const int64_t pf_ahead = (C_::LDG && warp != C_::CONSUMERS) ? 0 : g.pf_ahead;
         uint32_t it = 0;
         for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
             WsTile T;
@@ -505,6 +514,29 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
                 }
                 const int st = it % STAGES;
                 const uint32_t ph = (it / STAGES) & 1;
+                if constexpr (C_::LDG) {
+                    if (lane == 0) mbar_wait(&empty[st], ph ^ 1);
+                    __syncwarp();
+                    const int64_t k0 = (int64_t)kt * BK;
+                    const int64_t ldA = T.seg2 ? g.lda2 : g.lda;
+                    constexpr int CA = BM / 2, CB = BN / 2;      // 16-byte chunks per k-row of A / B
+                    const double* a0 = Ap + k0 * ldA + m0;
+                    const double* b0 = g.B + k0 * g.ldb + bn0;
+                    double* sa = sA + st * C_::SA;
+                    double* sb = sB + st * C_::SB;
+#pragma unroll 4
+                    for (int q = ptid; q < BK * CA; q += 128) {
+                        const int kk = q / CA, r = q % CA;
+                        if (2 * r < (int)rowsA) cp_async16(sa + kk * C_::PA + 2 * r, a0 + kk * ldA + 2 * r, 16);
+                    }
+#pragma unroll 4
+                    for (int q = ptid; q < BK * CB; q += 128) {
+                        const int kk = q / CB, r = q % CB;
+                        if (2 * r < (int)rowsB) cp_async16(sb + kk * C_::PB + 2 * r, b0 + kk * g.ldb + 2 * r, 16);
+                    }
+                    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(&full[st])) : "memory");
+                    continue;
+                }
                 if (lane == 0) {
                     mbar_wait(&empty[st], ph ^ 1);
                     mbar_expect_tx(&full[st], (uint32_t)BK * (rowsA + rowsB) * 8);
@@ -520,7 +552,8 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
         return;
     }
     // ------------------------------- consumers -------------------------------
-    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;\n" ::"n"(C_::REG_CONS) : "memory");
+    if constexpr (C_::REG_CONS != C_::R0)
+        asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;\n" ::"n"(C_::REG_CONS) : "memory");
     const int wm = warp / C_::WARPS_N, wn = warp % C_::WARPS_N;
     const int fr = lane >> 2, fc = lane & 3;
     const double ab = g.alpha * g.beta, alpha = g.alpha;
@@ -683,7 +716,8 @@ static int run_ws(GemmArgs g, cudaStream_t s, bool update) {
 // high priority, these keep the default one).
 bool is_update_kernel(const void* f) {
     return f == (const void*)k_update_ws<WsCfg> || f == (const void*)k_update_ws<WsCfg16> ||
-           f == (const void*)k_update_ws<WsCfg2a> || f == (const void*)k_update_ws<WsCfg2b>;
+           f == (const void*)k_update_ws<WsCfg2a> || f == (const void*)k_update_ws<WsCfg2b> ||
+           f == (const void*)k_update_ws<WsCfgNR> || f == (const void*)k_update_ws<WsCfg2l>;
 }
 
 static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CTA/SM), 16, 2a
@@ -695,6 +729,8 @@ static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CT
         if (e && !strcmp(e, "16")) v = 16;
         if (e && !strcmp(e, "2a")) v = 21;
         if (e && !strcmp(e, "2b")) v = 22;
+        if (e && !strcmp(e, "2l")) v = 25;
+        if (e && !strcmp(e, "nr")) v = 24;
     }
     return v;
 }
@@ -706,6 +742,8 @@ static int run_ws_any(GemmArgs g, cudaStream_t s) {
         case 16: return run_ws<WsCfg16>(g, s, upd);
         case 21: return run_ws<WsCfg2a>(g, s, upd);
         case 22: return run_ws<WsCfg2b>(g, s, upd);
+        case 25: return run_ws<WsCfg2l>(g, s, upd);
+        case 24: return run_ws<WsCfgNR>(g, s, upd);
         default: return run_ws<WsCfg>(g, s, upd);
     }
 }
