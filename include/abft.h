@@ -91,6 +91,9 @@ typedef struct abft_report {
     abft_event_t* events; /* HOST array owned by the caller, sorted by (k, check, J, I, col, row) */
     double seconds;     /* device time of the call (CUDA events on `stream`)                 */
     int64_t reruns;     /* Online / Offline schemes: re-executions after an uncorrectable error */
+    double max_noise_ratio; /* max over every column that PASSED a check of max(|d1|/tau1, |d2|/tau2):
+                               the fault-free rounding noise relative to the threshold of reading A4
+                               (how much margin C_tau = 64 leaves; the oracle's max_ratio)          */
 } abft_report_t;
 
 typedef struct abft_options {

@@ -72,6 +72,8 @@ def lib():
                                        vp, i64, ctypes.POINTER(i64), vp]
         _lib.oracle_verify.restype = i32
         _lib.oracle_num_threads.restype = i32
+        _lib.oracle_potrf_prefix.argtypes = [i64, i64, vp, i64, i64, vp]
+        _lib.oracle_potrf_prefix.restype = i32
     return _lib
 
 
@@ -165,6 +167,18 @@ def verify(A, nb, chk, scl, factored=False, correct=True, c_tau=64.0, cap=1 << 1
     if st < 0:
         raise ValueError(f"oracle_verify: invalid argument {-st}")
     return st, ev[: min(nev.value, cap)], cnt[0]
+
+
+def potrf_prefix(A, nb, kstop):
+    """Timing sample (bench.py only): the Enhanced factorisation of A (modified in place, must be
+    Fortran-ordered float64) stopped after kstop iterations. Returns (status, counts); counts'
+    flops_* fields are the work those iterations did."""
+    assert A.flags.f_contiguous and A.dtype == np.float64
+    cnt = np.zeros(1, dtype=COUNT_DTYPE)
+    st = lib().oracle_potrf_prefix(A.shape[0], nb, _ptr(A), max(A.shape[0], 1), int(kstop), _ptr(cnt))
+    if st < 0:
+        raise ValueError(f"oracle_potrf_prefix: invalid argument {-st}")
+    return st, cnt[0]
 
 
 def num_threads() -> int:

@@ -380,6 +380,10 @@ static int run_checks_column(octx_t* x, int64_t k, int factored, int V_diag, int
  *   mode 0 Enhanced Online-ABFT: V1..V6 (verify before every read)
  *   mode 1 Online-ABFT: verify each operation's result after it: V3, V4, V5, + final V6
  *   mode 2 Offline-ABFT: checksums carried, verified once at the end: V6 only        */
+/* kstop (timing only, bench.py's bounded CPU baseline): run iterations 0..kstop-1 and stop
+ * there (no V6); kstop >= N is the whole factorisation. The arithmetic is unchanged. */
+static int64_t g_kstop = INT64_MAX;
+
 static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
                       int nranks, int K, double c_tau, int abft, int mode, oevent_t* ev, int64_t cap,
                       int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out) {
@@ -404,7 +408,7 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
     panel_t* pan = (panel_t*)malloc(sizeof(panel_t) * (size_t)nranks);
 
     if (abft) { scales(x); encode(x); }
-    for (int64_t k = 0; k < N && x->status == O_OK; ++k) {
+    for (int64_t k = 0; k < N && k < g_kstop && x->status == O_OK; ++k) {
         const int owner = (int)(k % nranks);
         if (abft) {
             inject(x, (int)k, O_HOOK_REST, 0, x->A, lda, x->chk, x->ldc);
@@ -470,7 +474,7 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
             }
         }
     }
-    if (abft && x->status == O_OK) {
+    if (abft && x->status == O_OK && g_kstop >= N) {
         inject(x, (int)N, O_HOOK_REST, 0, x->A, lda, x->chk, x->ldc);
         int stop = 0;
         for (int64_t J = 0; J < N && !stop; ++J)
@@ -705,6 +709,24 @@ int oracle_verify(int64_t n, int64_t nb, double* A, int64_t lda, double* chk, in
 done:
     if (nev) *nev = x->nev;
     return x->status;
+}
+
+/* Bounded sample for timing (bench.py's cpu_baseline / reference arm on large n): the
+ * Enhanced right-looking factorisation stopped after kstop iterations. Returns the status;
+ * cnt receives the work done (flops of the iterations run), so that the caller can extrapolate
+ * the whole factorisation's time by flops. */
+int oracle_potrf_prefix(int64_t n, int64_t nb, double* A, int64_t lda, int64_t kstop, ocount_t* cnt) {
+    if (n < 0) return -1;
+    if (nb < 1 || n % nb) return -2;
+    if (lda < (n > 1 ? n : 1)) return -4;
+    ocount_t dummy;
+    ocount_t* c = cnt ? cnt : &dummy;
+    memset(c, 0, sizeof(ocount_t));
+    int64_t nev = 0, info = 0;
+    g_kstop = kstop < 0 ? 0 : kstop;
+    const int st = potrf_core(n, nb, A, lda, NULL, 0, 1, 1, 64.0, 1, 0, NULL, 0, &nev, &info, c, NULL, NULL);
+    g_kstop = INT64_MAX;
+    return st;
 }
 
 int oracle_num_threads(void) {

@@ -47,7 +47,7 @@ class Report(ctypes.Structure):
                 ("n_data", ctypes.c_int64), ("n_nonfinite", ctypes.c_int64), ("n_chk1", ctypes.c_int64),
                 ("n_chk2", ctypes.c_int64), ("n_uncorrectable", ctypes.c_int64), ("n_events", ctypes.c_int64),
                 ("cap", ctypes.c_int64), ("events", ctypes.c_void_p), ("seconds", ctypes.c_double),
-                ("reruns", ctypes.c_int64)]
+                ("reruns", ctypes.c_int64), ("max_noise_ratio", ctypes.c_double)]
 
 
 class Options(ctypes.Structure):
@@ -150,7 +150,7 @@ def _report_dict(rep, ev):
     return dict(info=rep.info, n_checks=rep.n_checks, n_detected=rep.n_detected, n_data=rep.n_data,
                 n_nonfinite=rep.n_nonfinite, n_chk1=rep.n_chk1, n_chk2=rep.n_chk2,
                 n_uncorrectable=rep.n_uncorrectable, n_events=rep.n_events, events=ev[:n].copy(),
-                seconds=rep.seconds, reruns=rep.reruns)
+                seconds=rep.seconds, reruns=rep.reruns, max_noise_ratio=rep.max_noise_ratio)
 
 
 MODE = {"enhanced": 0, "online": 1, "offline": 2, "enhanced_redo": 3}

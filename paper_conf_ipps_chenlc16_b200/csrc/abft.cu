@@ -25,6 +25,13 @@ using namespace abft;
 
 int launch_check(const StageArgs& a, cudaStream_t s);
 int launch_check_v5_fused(const StageArgs& diag, const StageArgs& off, cudaStream_t s);
+int launch_check2(const StageArgs& a0, const StageArgs& a1, cudaStream_t s);
+
+// Is there an injection at (k, hook)? (A hook between two checks keeps them in separate launches.)
+static bool has_inj(const std::vector<abft_inject_spec_t>& list, int64_t k, int hook) {
+    for (const auto& sp : list) if (sp.k == k && sp.hook == hook) return true;
+    return false;
+}
 int launch_scales(int64_t n, int64_t nb, const double* A, int64_t lda, double* scl, cudaStream_t s);
 int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,
                 const int32_t* abort_flag, cudaStream_t s);
@@ -171,6 +178,7 @@ static int finish_report(const Work& w, abft_report_t* rep, cudaStream_t s, int*
         rep->n_checks = (int64_t)hs.n_checks; rep->n_detected = hs.n_detected; rep->n_data = hs.n_data;
         rep->n_nonfinite = hs.n_nonfinite; rep->n_chk1 = hs.n_chk1; rep->n_chk2 = hs.n_chk2;
         rep->n_uncorrectable = hs.n_unc; rep->n_events = nev;
+        { double q; memcpy(&q, &hs.max_ratio_bits, sizeof q); rep->max_noise_ratio = q; }
         const int64_t ncopy = std::min<int64_t>(std::min<int64_t>(nev, w.ev_cap), std::max<int64_t>(rep->cap, 0));
         if (ncopy > 0 && rep->events) {
             ABFT_CUDA_TRY(cudaMemcpy(rep->events, w.ev, sizeof(abft_event_t) * (size_t)ncopy, cudaMemcpyDeviceToHost));
@@ -339,10 +347,20 @@ struct Persist {
     double* W1 = nullptr;
 };
 
+// Dev knob ABFT_DEV_ABLATE (bit mask; overhead attribution only — results are NOT protected and
+// checks may flag stale checksums, so it is for timing fault-free runs): 1 no checksum rows in the
+// TRSM / update / write-back, 2 no V5, 4 no V1-V4, 8 no fused V5 partials, 16 no encode / V6.
+static int dev_ablate() {
+    static int v = -1;
+    if (v < 0) { const char* e = getenv("ABFT_DEV_ABLATE"); v = e ? atoi(e) : 0; }
+    return v;
+}
+
 static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t s,
                      const std::vector<abft_inject_spec_t>& inj, abft_report_t* rep, const abft_options_t& o,
                      Persist* ps = nullptr) {
     const bool abft = o.abft_enabled != 0;
+    const int abl = abft ? dev_ablate() : 0;
     const int K = std::max(1, o.K);
     Work w;
     int rc = 0;
@@ -361,7 +379,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     // fused V5 partials: 64-row slabs x n columns x {v1, v2}
     const int mode = o.mode;
     const bool can_fuse = abft && mode != ABFT_MODE_OFFLINE && (nb % 128 == 0) && (lda % 2 == 0) &&
-                          (((uintptr_t)A & 15) == 0) && !getenv("ABFT_NOFUSE");   // dev knob: V5 re-reads
+                          (((uintptr_t)A & 15) == 0) && !getenv("ABFT_NOFUSE") && !(abl & 8);   // dev knob: V5 re-reads
     if (can_fuse && !ps) {
         w.cs_nslab = n / 32;   // room for 32-row slabs (the smallest warp-tile height)
         ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n), s));
@@ -380,7 +398,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     Profiler prof; prof.on = o.profile != 0 && !ps; prof.pool = &tc.timing;
     const double lowerB = Bd * (Bd + 1) / 2;                 // elements of a tril tile
     launch_zero(B, B, w.Li, B, s);
-    if (abft) {   // encode
+    if (abft && !(abl & 16)) {   // encode
         cudaEvent_t t = prof.begin(s);
         launch_scales(n, nb, A, lda, w.scl, s);
         StageArgs a = stage_base(w, A, lda, o.c_tau, SK_ALL, 0, -1);
@@ -404,7 +422,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         Work wk = w; wk.W = W;
         if (abft) do_inject_if(inj, k, ABFT_HOOK_REST, B, L, ab, P, k, k + 1, true);   // REST(k) into column k
         cudaEvent_t v2done = nullptr;
-        if (abft && mode == ABFT_MODE_ENHANCED) {
+        if (abft && mode == ABFT_MODE_ENHANCED && !(abl & 4)) {
             // V1 (tile k,k) gates POTRF; V2 (the tiles below) only has to precede the TRSM, so it
             // runs on the side stream P2 while P factors the diagonal block (same checks, same
             // events: both are labelled V2 as one column stage; separate flag lists)
@@ -433,7 +451,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         // TRSM (+ Alg. 2 on the checksum rows of tile (k,k)): one GEMM per row segment
         t = prof.begin(P);
         launch_gemm(mB, B, B, Akk + B, lda, w.Li, B, W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, P);
-        if (abft)
+        if (abft && !(abl & 1))
             launch_gemm(2 * m + 2, B, B, w.chk + k * B * w.ldc + 2 * k, w.ldc, w.Li, B, W + mB, ldw, 1.0, 0.0,
                         true, 0, 1, 0, 0, 0, ab, P);
         prof.end(t, PH_TRSM, P, (mBd + (abft ? 2 * md + 2 : 0)) * Bd * Bd, 0);
@@ -441,23 +459,33 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
             do_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, L, ab, P);
             StageArgs a3 = stage_base(wk, A, lda, o.c_tau, SK_DIAG_FACT, ABFT_V3, (int)k);
             a3.ldw = ldw; a3.mB = mB; a3.flist = 1;
-            if (mode != ABFT_MODE_OFFLINE) {
-                t = prof.begin(P);
-                launch_check(a3, P);                                             // V3
-                prof.end(t, PH_V3, P, 4.0 * lowerB, 8.0 * lowerB);
-            }
-            do_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, L, ab, P);
             StageArgs a4 = stage_base(wk, A, lda, o.c_tau, SK_PANEL, ABFT_V4, (int)k);
             a4.ldw = ldw; a4.mB = mB; a4.flist = 1;
-            if (mode != ABFT_MODE_OFFLINE) {
+            if (abl & 4) {
+            } else if (mode != ABFT_MODE_OFFLINE && !has_inj(inj, k, ABFT_HOOK_TRSM_OUT)) {
+                // V3 and V4 in one launch: V4 reads the solved panel and its checksum rows in W,
+                // never L_kk, so V3's corrections need not precede it; phase 2 resolves tile (k,k)
+                // first, as the sequential schedule does
                 t = prof.begin(P);
-                launch_check(a4, P);                                             // V4
-                prof.end(t, PH_V4, P, 4.0 * mBd * Bd, 8.0 * mBd * Bd);
+                launch_check2(a3, a4, P);                                        // V3 + V4
+                prof.end(t, PH_V4, P, 4.0 * (mBd * Bd + lowerB), 8.0 * (mBd * Bd + lowerB));
+            } else {
+                if (mode != ABFT_MODE_OFFLINE) {
+                    t = prof.begin(P);
+                    launch_check(a3, P);                                         // V3
+                    prof.end(t, PH_V3, P, 4.0 * lowerB, 8.0 * lowerB);
+                }
+                do_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, L, ab, P);
+                if (mode != ABFT_MODE_OFFLINE) {
+                    t = prof.begin(P);
+                    launch_check(a4, P);                                         // V4
+                    prof.end(t, PH_V4, P, 4.0 * mBd * Bd, 8.0 * mBd * Bd);
+                }
             }
         }
         t = prof.begin(P);
         launch_copy(mB, B, W, ldw, Akk + B, lda, ab, P);                        // L panel
-        if (abft) launch_copy(2 * m + 2, B, W + mB, ldw, w.chk + k * B * w.ldc + 2 * k, w.ldc, ab, P);
+        if (abft && !(abl & 1)) launch_copy(2 * m + 2, B, W + mB, ldw, w.chk + k * B * w.ldc + 2 * k, w.ldc, ab, P);
         prof.end(t, PH_WB, P, 0, 16.0 * (mBd + (abft ? 2 * md + 2 : 0)) * Bd);
         cudaEvent_t e = new_event(); cudaEventRecord(e, P);
         return e;
@@ -465,8 +493,9 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
 
     int64_t slab_rows_used = 64;
     // ---- trailing update of iteration k restricted to block columns [jlo, jhi), on S ----
-    // Returns true when the GEMM epilogue produced the fused V5 partials for these columns.
-    auto update_cols = [&](int64_t k, int64_t jlo, int64_t jhi) -> bool {
+    // Returns a bit mask: 1 = the GEMM epilogue produced the fused V5 partials for these columns,
+    // 2 = the epilogue applied the UPDATE_OUT injections of these columns (reading A21).
+    auto update_cols = [&](int64_t k, int64_t jlo, int64_t jhi) -> int {
         const int64_t m = N - k - 1, mB = m * B;
         const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
         double* W = Wbuf[k & 1];
@@ -476,27 +505,36 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         const double r = (double)rows, c = (double)nc;
         cudaEvent_t t = prof.begin(s);
         // C[rows x nc] -= W[c0:, :] W[c0:c0+nc, :]^T, lower (r >= c)
-        bool inj_here = false;
+        EpiInj ei; ei.n = 0;
         for (const auto& sp : inj)
-            if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && sp.col / nb >= jlo && sp.col / nb < jhi) inj_here = true;
+            if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && sp.col / nb >= jlo && sp.col / nb < jhi) {
+                if (ei.n < kMaxEpiInj) {
+                    EpiInjOp& e = ei.op[ei.n];
+                    e.seg = sp.target == ABFT_TGT_DATA ? 0 : 1;
+                    e.r = sp.target == ABFT_TGT_DATA ? sp.row - jlo * B : sp.row - 2 * jlo;
+                    e.c = sp.col - jlo * B; e.mask = sp.xor_mask; e.pad = 0;
+                }
+                ei.n++;
+            }
         ColSumOut cso{w.cs, n, w.cs_nslab, jlo * B, jlo * B, B, 64, jlo * B};
         int fused;
         if (abft) {
             // checksum rows of tiles I >= jlo: chk[2I+t, cols] -= W_chk(I) W[c0:c0+nc]^T, I >= J,
             // appended to the same launch as a second row segment
             const int64_t q0 = 2 * (jlo - k - 1);                       // first chk row of tile jlo in W
-            const int64_t nq = 2 * (N - jlo);
+            const int64_t nq = (abl & 1) ? 0 : 2 * (N - jlo);
             fused = launch_update_with_chk(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, nq, W + mB + 2 + q0,
                                            w.chk + jlo * B * w.ldc + 2 * jlo, w.ldc, B, ab, s,
-                                           (can_fuse && !inj_here) ? &cso : nullptr);
+                                           can_fuse ? &cso : nullptr, 0, 1, &ei);
             const double mm = (double)(N - jlo), jj = (double)(jhi - jlo);
             prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd + 4.0 * Bd * Bd * (jj * mm - jj * (jj - 1) / 2), 0);
         } else {
             fused = launch_gemm(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
+            fused = 0;
             prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd, 0);
         }
-        if (fused == 1) slab_rows_used = cso.slab_rows;
-        return fused == 1;
+        if (fused & 1) slab_rows_used = cso.slab_rows;
+        return fused;
     };
     auto v5_cols = [&](int64_t k, int64_t jlo, int64_t jhi, bool fused) {
         StageArgs a = stage_base(w, A, lda, o.c_tau, SK_TRAIL, ABFT_V5, (int)k);
@@ -543,10 +581,10 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         const Loc L{A, lda, w.chk, w.ldc, Wbuf[k & 1], ldw, mB};
         const bool gated = (((k + 1) % K == 0) || k == N - 2) && mode != ABFT_MODE_OFFLINE;
         // (a) block column k+1 first: update, UPDATE_OUT hook, V5 -> hand it to the panel stream
-        const bool fa = update_cols(k, k + 1, k + 2);
+        const int fa = update_cols(k, k + 1, k + 2);
         if (abft) {
-            do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 1, k + 2, true);
-            if (gated) v5_cols(k, k + 1, k + 2, fa);
+            if (!(fa & 2)) do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 1, k + 2, true);
+            if (gated && !(abl & 2)) v5_cols(k, k + 1, k + 2, (fa & 1) != 0);
         }
         cudaEvent_t ec = new_event(); cudaEventRecord(ec, s);
         cudaStreamWaitEvent(P, ec, 0);
@@ -554,10 +592,10 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         sink_col(k + 1);
         // (b) the rest of the trailing matrix
         if (m > 1) {
-            const bool fb = update_cols(k, k + 2, N);
+            const int fb = update_cols(k, k + 2, N);
             if (abft) {
-                do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 2, N, true);
-                if (gated) v5_cols(k, k + 2, N, fb);
+                if (!(fb & 2)) do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 2, N, true);
+                if (gated && !(abl & 2)) v5_cols(k, k + 2, N, (fb & 1) != 0);
             }
         }
         if (abft) {   // REST(k+1) outside block column k+1 (that one was applied on P)
@@ -565,7 +603,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
             do_inject_if(inj, k + 1, ABFT_HOOK_REST, B, L1, ab, s, k + 1, k + 2, false);
         }
     }
-    if (abft) {
+    if (abft && !(abl & 16)) {
         const Loc L{A, lda, w.chk, w.ldc, w.W, 1, 0};
         do_inject(inj, N, ABFT_HOOK_REST, B, L, ab, s);
         StageArgs a6 = stage_base(w, A, lda, o.c_tau, SK_ALL, ABFT_V6, (int)N);
@@ -901,11 +939,15 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             dist_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, P, q, ldw, mB, PS);
             StageArgs a3 = stage(q, SK_DIAG_FACT, ABFT_V3, (int)k);
             a3.ldw = ldw; a3.mB = mB; a3.flist = 1;
-            launch_check(a3, PS);                                                    // V3
-            dist_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, P, q, ldw, mB, PS);
             StageArgs a4 = stage(q, SK_PANEL, ABFT_V4, (int)k);
             a4.ldw = ldw; a4.mB = mB; a4.flist = 1;
-            launch_check(a4, PS);                                                    // V4
+            if (!has_inj(inj, k, ABFT_HOOK_TRSM_OUT)) {
+                launch_check2(a3, a4, PS);                                           // V3 + V4
+            } else {
+                launch_check(a3, PS);                                                // V3
+                dist_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, P, q, ldw, mB, PS);
+                launch_check(a4, PS);                                                // V4
+            }
         }
         launch_copy(mB, B, q.w.W, ldw, Akk + B, q.lda, ab, PS);
         if (abft) launch_copy(2 * m + 2, B, q.w.W + mB, ldw, ckk + 2 * k, q.w.ldc, ab, PS);
@@ -953,14 +995,10 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         int64_t m, mB, ldw; geom(k, m, mB, ldw);
         double* W = q.Wb[k & 1];
         const int32_t* ab = &q.w.st->abort;
-        bool any = false, inj_here = false;
+        bool any = false;
         for (int64_t J = jlo; J < jhi; ++J) any = any || (J % P == q.r);
         if (!any) return;
-        for (const auto& sp : inj)
-            if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && (sp.col / B) % P == q.r && sp.col / B >= jlo &&
-                sp.col / B < jhi)
-                inj_here = true;
-        bool all_fused = q.w.cs != nullptr && !inj_here;
+        bool all_fused = q.w.cs != nullptr;
         // the owned block columns J in [jlo, jhi) are J0, J0 + P, ...: one launch whose column
         // block t is global block J0 + t P (cstride), checksum rows appended as its second segment
         int64_t J0 = jlo;
@@ -968,13 +1006,28 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         const int64_t nt = (jhi - 1 - J0) / P + 1, t0 = J0 / P;
         double* W0 = W + (J0 - k - 1) * B;
         double* C = q.A + t0 * B * q.lda + J0 * B;
+        // this rank's UPDATE_OUT injections in [jlo, jhi), in the launch's local coordinates
+        EpiInj ei; ei.n = 0;
+        for (const auto& sp : inj)
+            if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && (sp.col / B) % P == q.r && sp.col / B >= jlo &&
+                sp.col / B < jhi) {
+                if (ei.n < kMaxEpiInj) {
+                    EpiInjOp& e = ei.op[ei.n];
+                    e.seg = sp.target == ABFT_TGT_DATA ? 0 : 1;
+                    e.r = sp.target == ABFT_TGT_DATA ? sp.row - J0 * B : sp.row - 2 * J0;
+                    e.c = ((sp.col / B) / P - t0) * B + sp.col % B; e.mask = sp.xor_mask; e.pad = 0;
+                }
+                ei.n++;
+            }
+        bool applied = false;
         ColSumOut cso{q.w.cs, q.ncl, q.w.cs_nslab, J0 * B, t0 * B, B, 64, J0 * B};
         const int f = abft ? launch_update_with_chk((N - J0) * B, nt * B, B, W0, ldw, W0, ldw, C, q.lda, 2 * (N - J0),
                                                     W + mB + 2 + 2 * (J0 - k - 1), q.w.chk + t0 * B * q.w.ldc + 2 * J0,
-                                                    q.w.ldc, B, ab, s, all_fused ? &cso : nullptr, 0, P)
+                                                    q.w.ldc, B, ab, s, all_fused ? &cso : nullptr, 0, P, &ei)
                            : launch_update_with_chk((N - J0) * B, nt * B, B, W0, ldw, W0, ldw, C, q.lda, 0, W0, C,
                                                     q.lda, B, ab, s, nullptr, 0, P);
         if (f < 0) {   // shapes the strided launch cannot take (or ABFT off): one launch per block column
+            if (ei.n > 0) all_fused = false;   // the hook is applied after the launches
             for (int64_t J = J0; J < jhi; J += P) {
                 const int64_t t = J / P;
                 double* Wj = W + (J - k - 1) * B;
@@ -987,15 +1040,16 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
                                                 q.w.ldc, B, ab, s, all_fused ? &csj : nullptr);
                 else
                     fj = launch_gemm((N - J) * B, B, B, Wj, ldw, Wj, ldw, Cj, q.lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
-                if (fj != 1) all_fused = false;
-                if (fj == 1) dist_slab_rows = csj.slab_rows;
+                if (!(fj & 1)) all_fused = false;
+                if (fj & 1) dist_slab_rows = csj.slab_rows;
             }
         } else {
-            if (f != 1) all_fused = false;
-            if (f == 1) dist_slab_rows = cso.slab_rows;
+            applied = (f & 2) != 0;
+            if (!(f & 1)) all_fused = false;
+            if (f & 1) dist_slab_rows = cso.slab_rows;
         }
         if (!abft) return;
-        {   // UPDATE_OUT injections of this rank inside [jlo, jhi)
+        if (!applied) {   // UPDATE_OUT injections of this rank inside [jlo, jhi)
             std::vector<abft_inject_spec_t> sub;
             for (const auto& sp : inj)
                 if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && sp.col / B >= jlo && sp.col / B < jhi) sub.push_back(sp);
@@ -1062,54 +1116,55 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         const int nc = 8;
         std::vector<double> cnt(nc * nlocal, 0.0), mx(2 * nlocal, 0.0);
         std::vector<abft_event_t> evs;
-        constexpr int64_t CAPG = 2048;
         double* dbuf = nullptr;     // device staging for the collectives
         abft_event_t* evg = nullptr;
         const int nr = tp ? tp->nranks : 1;
-        if (tp) {
-            ABFT_CUDA_TRY(cudaMallocAsync((void**)&dbuf, sizeof(double) * 16, s));
-            ABFT_CUDA_TRY(cudaMallocAsync((void**)&evg, sizeof(abft_event_t) * (size_t)(CAPG * (nr + 1)), s));
-        }
+        if (tp) ABFT_CUDA_TRY(cudaMallocAsync((void**)&dbuf, sizeof(double) * 16, s));
         std::vector<char> hbuf(sizeof(DevState));
         DevState& hs = *reinterpret_cast<DevState*>(hbuf.data());
-        double tot[8] = {0}, smax[2] = {0, 0};
+        double tot[8] = {0}, smax[4] = {0, 0, 0, 0};   // status, info, noise ratio, local event count
         for (auto& q : R) {
             ABFT_CUDA_TRY(cudaMemcpyAsync(&hs, q.w.st, offsetof(DevState, fl), cudaMemcpyDeviceToHost, s));
             ABFT_CUDA_TRY(cudaStreamSynchronize(s));
             const double v[8] = {(double)hs.n_checks, (double)hs.n_detected, (double)hs.n_data, (double)hs.n_nonfinite,
                                  (double)hs.n_chk1, (double)hs.n_chk2, (double)hs.n_unc, (double)hs.nev};
             for (int i = 0; i < 8; ++i) tot[i] += v[i];
+            double q_ratio; memcpy(&q_ratio, &hs.max_ratio_bits, sizeof q_ratio);
             smax[0] = std::max(smax[0], (double)hs.status); smax[1] = std::max(smax[1], (double)hs.info);
+            smax[2] = std::max(smax[2], q_ratio);
             const int64_t ne = std::min<int64_t>((int64_t)hs.nev, q.w.ev_cap);
             std::vector<abft_event_t> tmp(ne);
             if (ne > 0) ABFT_CUDA_TRY(cudaMemcpy(tmp.data(), q.w.ev, sizeof(abft_event_t) * (size_t)ne, cudaMemcpyDeviceToHost));
             evs.insert(evs.end(), tmp.begin(), tmp.end());
         }
+        smax[3] = (double)evs.size();
         if (tp) {
             double hb[16] = {0};
             for (int i = 0; i < 8; ++i) hb[i] = tot[i];
             ABFT_CUDA_TRY(cudaMemcpyAsync(dbuf, hb, sizeof(double) * 8, cudaMemcpyHostToDevice, s));
             if (tp->allreduce_sum(dbuf, 8, s)) return ABFT_ERR_NCCL;
             ABFT_CUDA_TRY(cudaMemcpyAsync(hb, dbuf, sizeof(double) * 8, cudaMemcpyDeviceToHost, s));
-            double hm[2] = {smax[0], smax[1]};
-            ABFT_CUDA_TRY(cudaMemcpyAsync(dbuf + 8, hm, sizeof(double) * 2, cudaMemcpyHostToDevice, s));
-            if (tp->allreduce_max(dbuf + 8, 2, s)) return ABFT_ERR_NCCL;
-            ABFT_CUDA_TRY(cudaMemcpyAsync(hm, dbuf + 8, sizeof(double) * 2, cudaMemcpyDeviceToHost, s));
-            // events: fixed CAPG block per rank
-            std::vector<abft_event_t> mine(CAPG);
-            memset(mine.data(), 0, sizeof(abft_event_t) * CAPG);
-            const int64_t nm = std::min<int64_t>((int64_t)evs.size(), CAPG);
-            for (int64_t i = 0; i < nm; ++i) mine[i] = evs[i];
-            for (int64_t i = nm; i < CAPG; ++i) mine[i].k = -2;   // padding marker
-            ABFT_CUDA_TRY(cudaMemcpyAsync(evg + CAPG * nr, mine.data(), sizeof(abft_event_t) * CAPG, cudaMemcpyHostToDevice, s));
-            if (tp->allgather(evg + CAPG * nr, evg, sizeof(abft_event_t) * CAPG, s)) return ABFT_ERR_NCCL;
-            std::vector<abft_event_t> all((size_t)(CAPG * nr));
-            ABFT_CUDA_TRY(cudaMemcpyAsync(all.data(), evg, sizeof(abft_event_t) * (size_t)(CAPG * nr), cudaMemcpyDeviceToHost, s));
+            double hm[4] = {smax[0], smax[1], smax[2], smax[3]};
+            ABFT_CUDA_TRY(cudaMemcpyAsync(dbuf + 8, hm, sizeof(double) * 4, cudaMemcpyHostToDevice, s));
+            if (tp->allreduce_max(dbuf + 8, 4, s)) return ABFT_ERR_NCCL;
+            ABFT_CUDA_TRY(cudaMemcpyAsync(hm, dbuf + 8, sizeof(double) * 4, cudaMemcpyDeviceToHost, s));
+            ABFT_CUDA_TRY(cudaStreamSynchronize(s));
+            // events: every rank contributes a block as large as the largest rank's list (no cap)
+            const int64_t capg = std::max<int64_t>(1, (int64_t)hm[3]);
+            ABFT_CUDA_TRY(cudaMallocAsync((void**)&evg, sizeof(abft_event_t) * (size_t)(capg * (nr + 1)), s));
+            std::vector<abft_event_t> mine((size_t)capg);
+            memset(mine.data(), 0, sizeof(abft_event_t) * (size_t)capg);
+            for (size_t i = 0; i < evs.size(); ++i) mine[i] = evs[i];
+            for (int64_t i = (int64_t)evs.size(); i < capg; ++i) mine[i].k = -2;   // padding marker
+            ABFT_CUDA_TRY(cudaMemcpyAsync(evg + capg * nr, mine.data(), sizeof(abft_event_t) * (size_t)capg, cudaMemcpyHostToDevice, s));
+            if (tp->allgather(evg + capg * nr, evg, sizeof(abft_event_t) * (size_t)capg, s)) return ABFT_ERR_NCCL;
+            std::vector<abft_event_t> all((size_t)(capg * nr));
+            ABFT_CUDA_TRY(cudaMemcpyAsync(all.data(), evg, sizeof(abft_event_t) * (size_t)(capg * nr), cudaMemcpyDeviceToHost, s));
             ABFT_CUDA_TRY(cudaStreamSynchronize(s));
             evs.clear();
             for (auto& e : all) if (e.k != -2) evs.push_back(e);
             for (int i = 0; i < 8; ++i) tot[i] = hb[i];
-            smax[0] = hm[0]; smax[1] = hm[1];
+            for (int i = 0; i < 4; ++i) smax[i] = hm[i];
             cudaFreeAsync(dbuf, s); cudaFreeAsync(evg, s);
         }
         status = (int)smax[0];
@@ -1118,6 +1173,7 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             rep->n_checks = (int64_t)tot[0]; rep->n_detected = (int64_t)tot[1]; rep->n_data = (int64_t)tot[2];
             rep->n_nonfinite = (int64_t)tot[3]; rep->n_chk1 = (int64_t)tot[4]; rep->n_chk2 = (int64_t)tot[5];
             rep->n_uncorrectable = (int64_t)tot[6]; rep->n_events = (int64_t)tot[7];
+            rep->max_noise_ratio = smax[2];
             std::sort(evs.begin(), evs.end(), [](const abft_event_t& x, const abft_event_t& y) {
                 if (x.k != y.k) return x.k < y.k;
                 if (x.check != y.check) return x.check < y.check;
@@ -1208,17 +1264,28 @@ static int run_potrf_left(int64_t n, int64_t nb, double* A, int64_t lda, cudaStr
             launch_check(stage_base(w, A, lda, o.c_tau, SK_COLUMN, ABFT_V2, (int)j), s);   // V1, V2
         bool fused = false;
         if (j > 0) {   // SYRK + GEMM of block column j, checksum rows as a second row segment
-            bool inj_here = false;
-            for (const auto& sp : inj) if (sp.k == j && sp.hook == ABFT_HOOK_UPDATE_OUT) inj_here = true;
+            EpiInj ei; ei.n = 0;
+            for (const auto& sp : inj)
+                if (sp.k == j && sp.hook == ABFT_HOOK_UPDATE_OUT) {
+                    if (ei.n < kMaxEpiInj) {
+                        EpiInjOp& e = ei.op[ei.n];
+                        e.seg = sp.target == ABFT_TGT_DATA ? 0 : 1;
+                        e.r = sp.target == ABFT_TGT_DATA ? sp.row - j * B : sp.row - 2 * j;
+                        e.c = sp.col - j * B; e.mask = sp.xor_mask; e.pad = 0;
+                    }
+                    ei.n++;
+                }
             ColSumOut cso{w.cs, n, w.cs_nslab, j * B, j * B, B, 64, j * B};
+            int f = 0;
             if (abft)
-                fused = launch_update_with_chk((N - j) * B, B, j * B, A + j * B, lda, A + j * B, lda, Ajj, lda,
-                                               2 * (N - j), w.chk + 2 * j, w.chk + j * B * w.ldc + 2 * j, w.ldc, B,
-                                               ab, s, (can_fuse && !inj_here) ? &cso : nullptr, w.ldc) == 1;
+                f = launch_update_with_chk((N - j) * B, B, j * B, A + j * B, lda, A + j * B, lda, Ajj, lda,
+                                           2 * (N - j), w.chk + 2 * j, w.chk + j * B * w.ldc + 2 * j, w.ldc, B,
+                                           ab, s, can_fuse ? &cso : nullptr, w.ldc, 1, &ei);
             else
                 launch_gemm((N - j) * B, B, j * B, A + j * B, lda, A + j * B, lda, Ajj, lda, -1.0, 1.0, true, 1, 0,
                             0, 0, 0, ab, s);
-            if (abft) do_inject(inj, j, ABFT_HOOK_UPDATE_OUT, B, L, ab, s);
+            fused = (f & 1) != 0;
+            if (abft && !(f & 2)) do_inject(inj, j, ABFT_HOOK_UPDATE_OUT, B, L, ab, s);
             if (abft && mode != ABFT_MODE_OFFLINE) {                              // V5: column j
                 StageArgs a = stage_base(w, A, lda, o.c_tau, SK_TRAIL, ABFT_V5, (int)j);
                 a.j_lo = j; a.j_hi = j + 1;
@@ -1343,6 +1410,7 @@ extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft
         rep->n_events = r1.n_events + r2.n_events;
         rep->seconds = r1.seconds + r2.seconds;
         rep->reruns = reruns;
+        rep->max_noise_ratio = std::max(r1.max_noise_ratio, r2.max_noise_ratio);
         int64_t w = 0;
         for (int64_t e = 0; e < std::min<int64_t>(r1.n_events, r1.cap) && w < rep->cap; ++e) rep->events[w++] = ev1[e];
         for (int64_t e = 0; e < std::min<int64_t>(r2.n_events, r2.cap) && w < rep->cap; ++e) rep->events[w++] = ev2[e];

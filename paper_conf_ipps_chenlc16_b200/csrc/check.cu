@@ -19,43 +19,92 @@ __device__ __forceinline__ double warp_sum(double v) {
     return v;
 }
 
-// Phase 1: recompute r1 = v1^T X[:,c], r2 = v2^T X[:,c] for every column of every tile of the
-// stage. encode = 1: store them as the checksums. Otherwise compare, flag columns
-// with |d| > tau or non-finite d, and append them to the flag list.
-__global__ void __launch_bounds__(kChkThreads) k_check_phase1(StageArgs a) {
-    if (cta_aborted(&a.st->abort)) return;
+// Noise bookkeeping: the largest |d|/tau of a passing column (positive doubles order as their
+// bit patterns, so an integer atomicMax keeps the maximum).
+__device__ __forceinline__ void note_ratio(DevState* st, double q) {
+    q = fmax(q, __shfl_xor_sync(0xffffffffu, q, 16));
+    q = fmax(q, __shfl_xor_sync(0xffffffffu, q, 8));
+    q = fmax(q, __shfl_xor_sync(0xffffffffu, q, 4));
+    q = fmax(q, __shfl_xor_sync(0xffffffffu, q, 2));
+    q = fmax(q, __shfl_xor_sync(0xffffffffu, q, 1));
+    if ((threadIdx.x & 31) == 0 && q > 0.0) atomicMax(&st->max_ratio_bits, (unsigned long long)__double_as_longlong(q));
+}
+
+// Compare a recalculated column with its stored checksums, flag it if |d| > tau or d is
+// non-finite (P:195 + A5). Called by every thread of the CTA (inactive threads pass ok = false).
+__device__ __forceinline__ void compare_column(const StageArgs& a, int part, const TileView& v, int64_t I, int64_t J,
+                                               int64_t c, double r1, double r2, bool ok) {
+    double q = 0.0;
+    if (ok) {
+        const double d1 = __dsub_rn(r1, v.c1[c * v.ldc]);
+        const double d2 = __dsub_rn(r2, v.c2[c * v.ldc]);
+        double tau1, tau2;
+        thresholds(a, I, J * a.nb + c, v.factored, tau1, tau2);
+        const bool f1 = !dfinite(d1) || fabs(d1) > tau1;
+        const bool f2 = !dfinite(d2) || fabs(d2) > tau2;
+        if (f1 || f2) {
+            FlagList& FL = a.st->fl[a.flist];
+            const int slot = atomicAdd(&FL.nflag, 1);
+            if (slot >= kFlagCap) FL.overflow = 1;
+            else {
+                Flag& f = FL.flags[slot];
+                f.I = (int32_t)I; f.J = (int32_t)J; f.c = (int32_t)c; f.part = part;
+                f.d1 = d1; f.d2 = d2; f.r1 = r1; f.r2 = r2;
+            }
+        } else {
+            q = fmax(fabs(d1) / tau1, fabs(d2) / tau2);
+        }
+    }
+    note_ratio(a.st, q);
+}
+
+// Phase 1, re-read: recompute r1 = v1^T X[:,c], r2 = v2^T X[:,c] for kChkCols columns of one tile
+// of the stage (block `bid` of this part). encode = 1: store them as the checksums. One warp per
+// column: coalesced loads (16-byte when the column is 16-byte aligned), shuffle reductions; the
+// mirrored half of an unfactored diagonal tile is read row-wise (also coalesced).
+__device__ void phase1_reread(const StageArgs& a, int part, int64_t bid) {
     const int64_t B = a.nb;
     const int64_t chunks = (B + kChkCols - 1) / kChkCols;
-    const int64_t t = blockIdx.x / chunks;
-    const int64_t c0 = (blockIdx.x % chunks) * kChkCols;
+    const int64_t t = bid / chunks;
+    const int64_t c0 = (bid % chunks) * kChkCols;
     int64_t I, J;
     stage_tile(a, t, I, J);
-    if (J % a.col_owner_mod != a.col_owner_rank) return;  // dist: not this rank's column
+    const bool mine = (J % a.col_owner_mod == a.col_owner_rank);   // dist: this rank's column
     const TileView v = stage_view(a, I, J);
     const int cw = (int)((B - c0) < kChkCols ? (B - c0) : kChkCols);
     __shared__ double s_r1[kChkCols], s_r2[kChkCols];
     __shared__ double s_m1[kChkThreads], s_m2[kChkThreads];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-
-    // column part: rows r >= c for diagonal tiles, all rows otherwise
-    for (int cc = warp; cc < cw; cc += kChkThreads / 32) {
-        const int64_t c = c0 + cc;
-        const double* col = v.T + c * v.ldt;
-        const int64_t rbeg = v.diag ? c : 0;
-        double r1 = 0.0, r2 = 0.0;
-        int64_t r = rbeg + lane;
+    if (mine) {
+        for (int cc = warp; cc < cw; cc += kChkThreads / 32) {
+            const int64_t c = c0 + cc;
+            const double* col = v.T + c * v.ldt;
+            const int64_t rbeg = v.diag ? c : 0;
+            double r1 = 0.0, r2 = 0.0;
+            if (!v.diag && ((((uintptr_t)col) & 15) == 0) && (B % 2 == 0)) {
+                const double2* col2 = reinterpret_cast<const double2*>(col);
 #pragma unroll 4
-        for (; r < B; r += 32) {
-            const double x = col[r];
-            r1 += x;
-            r2 = fma((double)(r + 1), x, r2);
+                for (int64_t h = lane; h < B / 2; h += 32) {
+                    const double2 x = col2[h];
+                    r1 += x.x; r1 += x.y;
+                    r2 = fma((double)(2 * h + 1), x.x, r2);
+                    r2 = fma((double)(2 * h + 2), x.y, r2);
+                }
+            } else {
+#pragma unroll 4
+                for (int64_t r = rbeg + lane; r < B; r += 32) {
+                    const double x = col[r];
+                    r1 += x;
+                    r2 = fma((double)(r + 1), x, r2);
+                }
+            }
+            r1 = warp_sum(r1);
+            r2 = warp_sum(r2);
+            if (lane == 0) { s_r1[cc] = r1; s_r2[cc] = r2; }
         }
-        r1 = warp_sum(r1);
-        r2 = warp_sum(r2);
-        if (lane == 0) { s_r1[cc] = r1; s_r2[cc] = r2; }
     }
     // mirrored part of an unfactored diagonal tile: X[r,c] = T[c,r] for r < c (row c of T)
-    if (v.diag && !v.factored) {
+    if (mine && v.diag && !v.factored) {
         const int ngroups = kChkThreads / kChkCols;
         const int cc = threadIdx.x % kChkCols, grp = threadIdx.x / kChkCols;
         double m1 = 0.0, m2 = 0.0;
@@ -76,62 +125,40 @@ __global__ void __launch_bounds__(kChkThreads) k_check_phase1(StageArgs a) {
         }
     }
     __syncthreads();
+    if (!mine) return;   // CTA-uniform
     if (threadIdx.x == 0 && c0 == 0 && !a.encode) atomicAdd(&a.st->n_checks, 1ull);
-    if (threadIdx.x >= cw) return;
+    const bool act = threadIdx.x < cw;
     const int64_t c = c0 + threadIdx.x;
-    const double r1 = s_r1[threadIdx.x], r2 = s_r2[threadIdx.x];
-    if (a.encode) { v.c1[c * v.ldc] = r1; v.c2[c * v.ldc] = r2; return; }
-    const double d1 = __dsub_rn(r1, v.c1[c * v.ldc]);
-    const double d2 = __dsub_rn(r2, v.c2[c * v.ldc]);
-    double tau1, tau2;
-    thresholds(a, I, J * B + c, v.factored, tau1, tau2);
-    const bool f1 = !dfinite(d1) || fabs(d1) > tau1;        // P:195 + A5
-    const bool f2 = !dfinite(d2) || fabs(d2) > tau2;
-    if (!(f1 || f2)) return;
-    FlagList& FL = a.st->fl[a.flist];
-    const int slot = atomicAdd(&FL.nflag, 1);
-    if (slot >= kFlagCap) { FL.overflow = 1; return; }
-    Flag& f = FL.flags[slot];
-    f.I = (int32_t)I; f.J = (int32_t)J; f.c = (int32_t)c;
-    f.d1 = d1; f.d2 = d2; f.r1 = r1; f.r2 = r2;
+    const double r1 = act ? s_r1[threadIdx.x] : 0.0, r2 = act ? s_r2[threadIdx.x] : 0.0;
+    if (a.encode) { if (act) { v.c1[c * v.ldc] = r1; v.c2[c * v.ldc] = r2; } return; }
+    compare_column(a, part, v, I, J, c, r1, r2, act);
 }
 
 // Phase 1 of V5 for off-diagonal trailing tiles from the partial sums the update GEMM left
 // behind (SK_TRAIL_OFF): r1 = sum of the tile's slab partials, r2 likewise. One thread per column.
-__global__ void __launch_bounds__(256) k_check_phase1_fused(StageArgs a) {
-    if (cta_aborted(&a.st->abort)) return;
+__device__ void phase1_fused(const StageArgs& a, int part, int64_t bid) {
     const int64_t B = a.nb;
-    const int64_t chunks = (B + 255) / 256;
-    const int64_t t = blockIdx.x / chunks;
-    const int64_t c = (blockIdx.x % chunks) * 256 + threadIdx.x;
+    const int64_t chunks = (B + kChkThreads - 1) / kChkThreads;
+    const int64_t t = bid / chunks;
+    const int64_t c = (bid % chunks) * kChkThreads + threadIdx.x;
     int64_t I, J;
     stage_tile(a, t, I, J);
-    if (J % a.col_owner_mod != a.col_owner_rank) return;
+    if (J % a.col_owner_mod != a.col_owner_rank) return;   // CTA-uniform
     if (threadIdx.x == 0 && c == 0) atomicAdd(&a.st->n_checks, 1ull);
-    if (c >= B) return;
+    const bool act = c < B;
     const TileView v = stage_view(a, I, J);
-    const int64_t g = local_col(a, J) + c, s0 = I * B / a.cs_slab_rows, ns = B / a.cs_slab_rows;
     double r1 = 0.0, r2 = 0.0;
-    for (int64_t q = 0; q < ns; ++q) {
-        r1 += a.cs[(s0 + q) * a.cs_ld + g];
-        r2 += a.cs[(a.cs_nslab + s0 + q) * a.cs_ld + g];
+    if (act) {
+        const int64_t g = local_col(a, J) + c, s0 = I * B / a.cs_slab_rows, ns = B / a.cs_slab_rows;
+        for (int64_t q = 0; q < ns; ++q) {
+            r1 += a.cs[(s0 + q) * a.cs_ld + g];
+            r2 += a.cs[(a.cs_nslab + s0 + q) * a.cs_ld + g];
+        }
     }
-    const double d1 = __dsub_rn(r1, v.c1[c * v.ldc]);
-    const double d2 = __dsub_rn(r2, v.c2[c * v.ldc]);
-    double tau1, tau2;
-    thresholds(a, I, J * B + c, false, tau1, tau2);
-    const bool f1 = !dfinite(d1) || fabs(d1) > tau1;
-    const bool f2 = !dfinite(d2) || fabs(d2) > tau2;
-    if (!(f1 || f2)) return;
-    FlagList& FL = a.st->fl[a.flist];
-    const int slot = atomicAdd(&FL.nflag, 1);
-    if (slot >= kFlagCap) { FL.overflow = 1; return; }
-    Flag& f = FL.flags[slot];
-    f.I = (int32_t)I; f.J = (int32_t)J; f.c = (int32_t)c;
-    f.d1 = d1; f.d2 = d2; f.r1 = r1; f.r2 = r2;
+    compare_column(a, part, v, I, J, c, r1, r2, act);
 }
 
-// Block-wide reductions used by phase 2 (one CTA).
+// Block-wide reductions used by phase 2.
 __device__ double block_sum(double v, double* red) {
     v = warp_sum(v);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
@@ -171,32 +198,46 @@ struct Fix { double* p; double* p2; double val; };
 // is reported UNCORRECTABLE
 constexpr int kMaxFix = 1024;
 
+// Flags were written by other CTAs of this launch: read them from L2 (they are never in this
+// SM's L1 for a reason this CTA could vouch for).
+__device__ __forceinline__ Flag load_flag(const Flag* p) {
+    Flag f;
+    const int2 h0 = __ldcg(reinterpret_cast<const int2*>(p));       // Flag is 8-byte aligned
+    const int2 h1 = __ldcg(reinterpret_cast<const int2*>(p) + 1);
+    f.I = h0.x; f.J = h0.y; f.c = h1.x; f.part = h1.y;
+    f.d1 = __ldcg(&p->d1); f.d2 = __ldcg(&p->d2); f.r1 = __ldcg(&p->r1); f.r2 = __ldcg(&p->r2);
+    return f;
+}
+
 // Phase 2: resolve the flagged columns in the oracle's order (tile, then column): decide
 // DATA / NONFINITE / CHK1 / CHK2 / UNCORRECTABLE, dedupe diagonal-tile mirrors, compute the
-// corrections from the pre-correction tile, apply them per tile, log events. One CTA.
-__global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
-    DevState* st = a.st;
-    FlagList& FL = st->fl[a.flist];
+// corrections from the pre-correction tile, apply them per tile, log events. Run by one CTA: the
+// last CTA of the check launch to finish its phase 1 (no separate launch).
+__device__ void phase2_body(const StageArgs& a0, const StageArgs& a1, int flist) {
+    DevState* st = a0.st;
+    FlagList& FL = st->fl[flist];
     __shared__ int s_n;
     __shared__ Fix s_fix[kMaxFix];
     __shared__ int s_nfix, s_unc, s_stop;
-    __shared__ double redv[256];
-    __shared__ long long redi[256];
+    __shared__ double redv[kChkThreads];
+    __shared__ long long redi[kChkThreads];
+    __shared__ Flag s_flag;
     if (threadIdx.x == 0) {
-        s_n = min(FL.nflag, kFlagCap);
-        if (st->abort) s_n = 0;
-        if (FL.overflow && !st->abort) {   // more flagged columns than we can resolve
+        s_n = min(__ldcg(&FL.nflag), kFlagCap);
+        if (__ldcg(&st->abort)) s_n = 0;
+        if (__ldcg(&FL.overflow) && !__ldcg(&st->abort)) {   // more flagged columns than we can resolve
             st->status = ABFT_UNCORRECTABLE; st->abort = 1; s_n = 0;
             const long long e = (long long)atomicAdd(&st->nev, 1ull);
-            if (e < a.ev_cap) {
-                abft_event_t& ev = a.ev[e];
-                ev.k = a.k; ev.check = a.V; ev.tile_i = -1; ev.tile_j = -1; ev.row = -3; ev.col = -1;
-                ev.kind = ABFT_KIND_UNCORRECTABLE; ev.rank = a.rank; ev.delta1 = 0; ev.delta2 = 0;
+            if (e < a0.ev_cap) {
+                abft_event_t& ev = a0.ev[e];
+                ev.k = a0.k; ev.check = a0.V; ev.tile_i = -1; ev.tile_j = -1; ev.row = -3; ev.col = -1;
+                ev.kind = ABFT_KIND_UNCORRECTABLE; ev.rank = a0.rank; ev.delta1 = 0; ev.delta2 = 0;
             }
             st->n_unc++;
         }
         // insertion sort by (J, I, c): the oracle's check order
         Flag* F = FL.flags;
+        for (int i = 0; i < s_n; ++i) F[i] = load_flag(&F[i]);
         for (int i = 1; i < s_n; ++i) {
             Flag x = F[i]; int j = i - 1;
             auto key = [](const Flag& f) { return ((long long)f.J << 40) | ((long long)f.I << 20) | f.c; };
@@ -207,13 +248,16 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
     }
     __syncthreads();
     const int n = s_n;
-    const int64_t B = a.nb;
     int i0 = 0;
     while (i0 < n && !s_stop) {
-        // entries [i0, i1) belong to one tile
-        const Flag first = FL.flags[i0];
+        // entries [i0, i1) belong to one tile (of one part)
+        if (threadIdx.x == 0) s_flag = FL.flags[i0];
+        __syncthreads();
+        const Flag first = s_flag;
+        const StageArgs& a = first.part ? a1 : a0;
+        const int64_t B = a.nb;
         int i1 = i0;
-        while (i1 < n && FL.flags[i1].I == first.I && FL.flags[i1].J == first.J) ++i1;
+        while (i1 < n && FL.flags[i1].I == first.I && FL.flags[i1].J == first.J && FL.flags[i1].part == first.part) ++i1;
         const TileView v = stage_view(a, first.I, first.J);
         if (threadIdx.x == 0) { s_nfix = 0; s_unc = 0; }
         __syncthreads();
@@ -241,6 +285,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
             } else {
                 kind = ABFT_KIND_CHK2;
             }
+            const int vcode = ((a.kind == SK_COLUMN || a.kind == SK_COL_DIAG) && f.I == a.k) ? ABFT_V1 : a.V;
             if (kind == ABFT_KIND_DATA || kind == ABFT_KIND_NONFINITE) {
                 double* p = view_store(v, row, c);
                 bool dup = false;
@@ -259,7 +304,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
                     const long long ev_i = (long long)atomicAdd(&st->nev, 1ull);
                     if (ev_i < a.ev_cap) {
                         abft_event_t& ev = a.ev[ev_i];
-                        ev.k = a.k; ev.check = ((a.kind == SK_COLUMN || a.kind == SK_COL_DIAG) && f.I == a.k) ? ABFT_V1 : a.V;
+                        ev.k = a.k; ev.check = vcode;
                         ev.tile_i = f.I; ev.tile_j = f.J;
                         ev.row = (int32_t)sr; ev.col = (int32_t)sc; ev.kind = kind; ev.rank = a.rank;
                         ev.delta1 = f.d1; ev.delta2 = f.d2;
@@ -272,7 +317,7 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
                 const long long ev_i = (long long)atomicAdd(&st->nev, 1ull);
                 if (ev_i < a.ev_cap) {
                     abft_event_t& ev = a.ev[ev_i];
-                    ev.k = a.k; ev.check = ((a.kind == SK_COLUMN || a.kind == SK_COL_DIAG) && f.I == a.k) ? ABFT_V1 : a.V;
+                    ev.k = a.k; ev.check = vcode;
                     ev.tile_i = f.I; ev.tile_j = f.J;
                     ev.row = kind == ABFT_KIND_CHK1 ? -1 : kind == ABFT_KIND_CHK2 ? -2 : -3;
                     ev.col = (int32_t)c; ev.kind = kind; ev.rank = a.rank;
@@ -306,6 +351,33 @@ __global__ void __launch_bounds__(256) k_check_phase2(StageArgs a) {
     if (threadIdx.x == 0) { FL.nflag = 0; FL.overflow = 0; }
 }
 
+// One check launch: phase 1 over the tiles of one or two stage parts (blocks [0, nblk0) run part
+// 0, the rest part 1; kind SK_TRAIL_OFF reads the GEMM's fused partials, every other kind re-reads
+// the tiles), then the last CTA to finish resolves the flags of both parts (phase 2) in the
+// oracle's order. Every CTA reaches the completion counter (also when the run is aborted), and
+// the last one resets it, so the counter is zero again for the next launch on this flag list.
+__global__ void __launch_bounds__(kChkThreads) k_check(StageArgs a0, StageArgs a1, int64_t nblk0) {
+    __shared__ int s_last;
+    const bool aborted = cta_aborted(&a0.st->abort);
+    if (!aborted) {
+        const bool p1 = (int64_t)blockIdx.x >= nblk0;
+        const StageArgs& a = p1 ? a1 : a0;
+        const int64_t bid = p1 ? (int64_t)blockIdx.x - nblk0 : (int64_t)blockIdx.x;
+        if (a.kind == SK_TRAIL_OFF) phase1_fused(a, p1 ? 1 : 0, bid);
+        else phase1_reread(a, p1 ? 1 : 0, bid);
+    }
+    if (a0.encode) return;   // encode launches resolve nothing (no counter use)
+    __threadfence();
+    __syncthreads();
+    const int fl = a0.flist;
+    if (threadIdx.x == 0) s_last = atomicAdd(&a0.st->done[fl], 1u) == gridDim.x - 1;
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    if (threadIdx.x == 0) a0.st->done[fl] = 0u;
+    if (__ldcg(&a0.st->fl[fl].nflag) > 0 || __ldcg(&a0.st->fl[fl].overflow)) phase2_body(a0, a1, fl);
+}
+
 // Threshold scales of reading A4: s_i = sqrt(A_ii); S1_I = sum s_i, S2_I = sum (i+1) s_i over
 // block I, summed sequentially in ascending order with explicit round-to-nearest operations.
 __global__ void k_scales_diag(int64_t n, const double* A, int64_t lda, double* s) {
@@ -328,43 +400,36 @@ __global__ void k_scales_block(int64_t N, int64_t B, const double* s, double* S1
 // ---- host launchers ---------------------------------------------------------------------
 using namespace abft;
 
-int launch_check(const StageArgs& a, cudaStream_t s) {
+static int64_t check_blocks(const StageArgs& a) {
     const int64_t count = stage_count(a);
     if (count <= 0) return 0;
-    if (a.kind == SK_TRAIL_OFF) {
-        const int64_t chunks = (a.nb + 255) / 256;
-        k_check_phase1_fused<<<(unsigned)(count * chunks), 256, 0, s>>>(a);
-    } else {
-        const int64_t chunks = (a.nb + kChkCols - 1) / kChkCols;
-        k_check_phase1<<<(unsigned)(count * chunks), kChkThreads, 0, s>>>(a);
-    }
+    const int64_t per = a.kind == SK_TRAIL_OFF ? kChkThreads : kChkCols;
+    return count * ((a.nb + per - 1) / per);
+}
+
+int launch_check(const StageArgs& a, cudaStream_t s) {
+    const int64_t nb0 = check_blocks(a);
+    if (nb0 <= 0) return 0;
+    k_check<<<(unsigned)nb0, kChkThreads, 0, s>>>(a, a, nb0);
     abft_count_launch();
-    if (a.encode) return 0;
-    k_check_phase2<<<1, 256, 0, s>>>(a);
+    return 0;
+}
+
+// Two stages of one flag list in one launch, resolved together in the oracle's tile order
+// (part 0's tiles precede part 1's in (J, I) order: V5 diagonal + off-diagonal tiles of the same
+// block columns are interleaved by that sort; V3 (tile k,k) + V4 (tiles i>k, k)).
+int launch_check2(const StageArgs& a0, const StageArgs& a1, cudaStream_t s) {
+    const int64_t nb0 = check_blocks(a0), nb1 = check_blocks(a1);
+    if (nb0 + nb1 <= 0) return 0;
+    k_check<<<(unsigned)(nb0 + nb1), kChkThreads, 0, s>>>(a0, a1, nb0);
     abft_count_launch();
     return 0;
 }
 
 // V5 with the fused recalculation: diagonal tiles re-read (sym), off-diagonal tiles from the
-// update GEMM's partials; both phase-1 kernels feed one flag list resolved by one phase 2 in
-// the oracle's tile order.
+// update GEMM's partials; one launch, one flag list.
 int launch_check_v5_fused(const StageArgs& diag, const StageArgs& off, cudaStream_t s) {
-    const int64_t nd = stage_count(diag), no = stage_count(off);
-    if (nd > 0) {
-        const int64_t chunks = (diag.nb + kChkCols - 1) / kChkCols;
-        k_check_phase1<<<(unsigned)(nd * chunks), kChkThreads, 0, s>>>(diag);
-        abft_count_launch();
-    }
-    if (no > 0) {
-        const int64_t chunks = (off.nb + 255) / 256;
-        k_check_phase1_fused<<<(unsigned)(no * chunks), 256, 0, s>>>(off);
-        abft_count_launch();
-    }
-    StageArgs r = diag;
-    r.kind = SK_TRAIL;
-    k_check_phase2<<<1, 256, 0, s>>>(r);
-    abft_count_launch();
-    return 0;
+    return launch_check2(diag, off, s);
 }
 
 int launch_scales_diag(int64_t nrows, const double* Adiag, int64_t lda, double* s_out, cudaStream_t s) {

@@ -12,7 +12,7 @@ namespace abft {
 
 // A flagged column produced by a check's recalculation pass (phase 1), resolved by phase 2.
 struct Flag {
-    int32_t I, J, c, pad;
+    int32_t I, J, c, part;   // part: which StageArgs of a two-part check launch raised it
     double d1, d2, r1, r2;
 };
 
@@ -32,6 +32,10 @@ struct DevState {
     unsigned long long nev;        // events raised
     unsigned long long n_checks;   // tile checks run
     long long n_detected, n_data, n_nonfinite, n_chk1, n_chk2, n_unc;
+    unsigned long long max_ratio_bits;   // max over passing columns of max(|d1|/tau1, |d2|/tau2)
+                                         // (fault-free noise margin, as the oracle's max_ratio)
+    unsigned int done[4];                // per flag list: CTAs of the running check launch that
+                                         // finished phase 1 (the last one resolves the flags)
     FlagList fl[3];       // [0]: main stream, [1]: look-ahead panel stream, [2]: panel side stream (V2)
 };
 
@@ -216,6 +220,15 @@ struct ColSumOut {
 };
 }  // namespace abft
 
+// UPDATE_OUT injections applied inside the update GEMM's epilogue (reading A21: after the
+// update, before the fused V5 partials and the store). Coordinates are relative to the launch's
+// C (seg 0, data rows) or C2 (seg 1, checksum rows), in its local columns.
+namespace abft {
+struct EpiInjOp { int64_t r, c; uint64_t mask; int32_t seg, pad; };
+constexpr int kMaxEpiInj = 4;
+struct EpiInj { int32_t n, pad; EpiInjOp op[kMaxEpiInj]; };
+}  // namespace abft
+
 // Host helpers
 #define ABFT_CUDA_TRY(expr)                                   \
     do {                                                      \
@@ -251,7 +264,10 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
 // The trailing update with the checksum rows as a second row segment of the same launch.
 // cstride > 1: C's column block t (and the B operand's row block t) is global block t * cstride
 // (a rank's 1D block-cyclic local columns in one launch); returns -1 if the shapes do not allow it.
+// Returns a bit mask: 1 = the fused V5 partials were written, 2 = the epilogue applied `inj`
+// (the caller applies the hook itself otherwise); -1 if cstride > 1 and the shapes do not allow it.
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s,
-                           abft::ColSumOut* cs, int64_t lda2 = 0, int64_t cstride = 1);
+                           abft::ColSumOut* cs, int64_t lda2 = 0, int64_t cstride = 1,
+                           const abft::EpiInj* inj = nullptr);

@@ -54,6 +54,7 @@ struct GemmArgs {
     // ws kernel: prefetch into L2 the C tile of tile index t + pf_ahead (0 = off; the launcher
     // sets it to the number of CTAs resident at once)
     int64_t pf_ahead;
+    EpiInj inj;   // UPDATE_OUT hook in the epilogue (ws kernel; inj.n == 0: none)
 };
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
@@ -621,6 +622,27 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
         }
         // epilogue: C = alpha * acc, masked stores only
 #pragma unroll
+        for (int i = 0; i < C_::FM; ++i)
+#pragma unroll
+            for (int j = 0; j < C_::FN; ++j)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) acc[i][j][h] = alpha * acc[i][j][h];
+        // UPDATE_OUT hook (reading A21): XOR the injected bits into the updated value before it is
+        // stored and before the fused V5 partials see it (warp-uniform test, off the common path)
+        for (int q = 0; q < g.inj.n; ++q) {
+            const EpiInjOp e = g.inj.op[q];
+            const int64_t lr = e.r - (m0 + wm * WM), lc = e.c - (n0 + wn * WN);
+            if (e.seg != (seg2 ? 1 : 0) || lr < 0 || lr >= WM || lc < 0 || lc >= WN) continue;
+#pragma unroll
+            for (int i = 0; i < C_::FM; ++i)
+#pragma unroll
+                for (int j = 0; j < C_::FN; ++j)
+#pragma unroll
+                    for (int h = 0; h < 2; ++h)
+                        if (i * 8 + fr == lr && j * 8 + fc * 2 + h == lc)
+                            acc[i][j][h] = __longlong_as_double(__double_as_longlong(acc[i][j][h]) ^ (long long)e.mask);
+        }
+#pragma unroll
         for (int i = 0; i < C_::FM; ++i) {
             const int64_t r = m0 + wm * WM + i * 8 + fr;
 #pragma unroll
@@ -628,7 +650,6 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
 #pragma unroll
                 for (int h = 0; h < 2; ++h) {
                     const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
-                    acc[i][j][h] = alpha * acc[i][j][h];
                     if (owns(r, j, h)) Cp[c * ldcp + r] = acc[i][j][h];
                 }
         }
@@ -767,6 +788,7 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
     g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
     g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
     g.M2 = 0; g.A2 = nullptr; g.C2 = nullptr; g.ldc2 = 1; g.lda2 = 1; g.cstride = 1;
+    g.inj.n = 0;
     g.vecA = aligned16(A) && (lda % 2 == 0);
     g.vecB = aligned16(B) && (ldb % 2 == 0);
     auto tiles = [&](int64_t t) {
@@ -810,7 +832,7 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s, ColSumOut* cs,
-                           int64_t lda2, int64_t cstride) {
+                           int64_t lda2, int64_t cstride, const EpiInj* inj) {
     if (lda2 <= 0) lda2 = lda;
     if (cstride < 1) cstride = 1;
     const bool ok = M > 0 && N > 0 && (M % 2 == 0) && (N % 2 == 0) && (M2 % 2 == 0) && (K % WsCfg::BK == 0) &&
@@ -818,24 +840,27 @@ int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int
                     lda2 % 2 == 0 && M % WsCfg::BM == 0 && getenv("ABFT_GEMM_VARIANT") == nullptr &&
                     (cstride == 1 || nb % WsCfg::BN == 0);
     if (!ok && cstride > 1) return -1;   // strided columns need the warp-specialised kernel
-    if (!ok) {
+    if (!ok) {   // fallback (two generic launches): the caller applies the hook, no fused partials
         const int f = launch_gemm(M, N, K, A, lda, B, ldb, C, ldc, -1.0, 1.0, true, MASK_LOWER, KR_FULL, 0, 0, 0,
-                                  abort_flag, s, 0, cs);
+                                  abort_flag, s, 0, (inj && inj->n > 0) ? nullptr : cs);
         if (M2 > 0)
             launch_gemm(M2, N, K, A2, lda2, B, ldb, C2, ldc2, -1.0, 1.0, true, MASK_CHK, KR_FULL, nb, 0, 0, abort_flag, s);
-        return f;
+        return f == 1 ? 1 : 0;
     }
     GemmArgs g;
     g.M = M; g.N = N; g.K = K; g.A = A; g.lda = lda; g.B = B; g.ldb = ldb; g.C = C; g.ldc = ldc;
     g.alpha = -1.0; g.beta = 1.0; g.mask = MASK_LOWER; g.krange = KR_FULL; g.nb = nb;
     g.q_tile0 = 0; g.c_tile0 = 0; g.tiles_n = 1; g.abort = abort_flag; g.vecA = 1; g.vecB = 1;
     g.cs = ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
-    int fused = 0;
-    if (cs && cs->nb % WsCfg::BM == 0 && cs->row0 % WsCfg::BM == 0 && cs->colg0 % WsCfg::BN == 0) {
-        g.cs = *cs; fused = 1;
+    g.inj.n = 0;
+    int ret = 0;
+    if (inj && inj->n > 0 && inj->n <= kMaxEpiInj) { g.inj = *inj; ret |= 2; }
+    const bool inj_left = inj && inj->n > kMaxEpiInj;   // too many for the epilogue: caller's hook
+    if (cs && !inj_left && cs->nb % WsCfg::BM == 0 && cs->row0 % WsCfg::BM == 0 && cs->colg0 % WsCfg::BN == 0) {
+        g.cs = *cs; ret |= 1;
     }
     g.M2 = M2; g.A2 = A2; g.C2 = C2; g.ldc2 = ldc2; g.lda2 = lda2; g.cstride = cstride;
     run_ws_any(g, s);
-    if (fused) cs->slab_rows = ws_slab_rows();
-    return fused;
+    if (ret & 1) cs->slab_rows = ws_slab_rows();
+    return ret;
 }

@@ -39,7 +39,7 @@ def test_struct_layouts_match_header():
     import synthetic as syn
     assert ctypes.sizeof(p.Event) == 48 == p.EVENT_DTYPE.itemsize
     assert p.INJ_DTYPE.itemsize == 48 == syn.INJ_DTYPE.itemsize
-    assert ctypes.sizeof(p.Report) == 13 * 8
+    assert ctypes.sizeof(p.Report) == 14 * 8
     assert ctypes.sizeof(p.Options) == 32
 
 
