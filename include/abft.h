@@ -198,6 +198,21 @@ int abft_comm_destroy(void* comm);
 int abft_potrf_dist(int64_t n, int64_t nb, double* A_local, int64_t lda_local, void* comm, int rank,
                     int nranks, abft_stream_t stream, const abft_inject_spec_t* inj,
                     abft_report_t* rep, const abft_options_t* opt);
+
+/* Peer-memory transport (NEXT-3 groundwork; also how two ranks share ONE device in the tests,
+ * where NCCL refuses duplicate devices): each rank exports one device arena of cap_bytes (+256
+ * bytes of flags) through CUDA IPC; the panel broadcast is a pull of the owner's panel straight
+ * out of its arena (peer loads over NVLink/NVSwitch between GPUs), the all-reduces and the
+ * all-gather are peer reads in rank order, all synchronised by device-side release/acquire flags
+ * on the caller's stream (no host round trip). cap_bytes must hold the largest message: the
+ * packed panel, (n - nb) nb + 2 n + 8 doubles.
+ * abft_comm_init_ipc: allocate + export; handle_out receives this rank's 64-byte handle.
+ * abft_comm_attach_ipc: handles = nranks x 64 bytes (all ranks' handles, rank order) -> map peers.
+ * The resulting comm is used with abft_potrf_dist and released with abft_comm_destroy, like an
+ * NCCL one. Errors: -1 comm, -2 nranks (1..64) / handles, -3 rank, -4 cap_bytes, -5 handle_out;
+ * ABFT_ERR_CUDA if the device refuses the export / mapping. */
+int abft_comm_init_ipc(void** comm, int nranks, int rank, int64_t cap_bytes, void* handle_out);
+int abft_comm_attach_ipc(void* comm, const void* handles);
 /* abft_potrf_dist errors: -1 n, -2 nb, -3 A_local, -4 lda_local, -5 comm (or its rank/size
  * disagree with rank/nranks), -6 rank, -7 nranks, -9 inj, -11 options; ABFT_ERR_NCCL on a failed
  * collective. Depth-1 look-ahead across ranks: the owner of block column k+1 updates it first and

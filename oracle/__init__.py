@@ -38,7 +38,7 @@ COUNT_DTYPE = np.dtype([
     ("flops_encode", "<f8"), ("bytes_check", "<f8"), ("max_ratio", "<f8"),
 ])
 CHECK = {1: "V1", 2: "V2", 3: "V3", 4: "V4", 5: "V5", 6: "V6", 7: "V4R", 8: "V7"}
-KIND = {1: "DATA", 2: "NONFINITE", 3: "CHK1", 4: "CHK2", 5: "UNCORRECTABLE"}
+KIND = {1: "DATA", 2: "NONFINITE", 3: "CHK1", 4: "CHK2", 5: "UNCORRECTABLE", 6: "CHK3"}
 STATUS = {0: "OK", 1: "UNCORRECTABLE", 2: "NOT_SPD"}
 
 
@@ -66,6 +66,10 @@ def lib():
                                            vp, i64, ctypes.POINTER(i64), ctypes.POINTER(i64), vp, vp, vp,
                                            ctypes.POINTER(i32)]
         _lib.oracle_potrf_mode.restype = i32
+        _lib.oracle_potrf_nchk.argtypes = [i64, i64, vp, i64, vp, i64, i32, i32, ctypes.c_double, i32, i32, i32,
+                                           vp, i64, ctypes.POINTER(i64), ctypes.POINTER(i64), vp, vp, vp,
+                                           ctypes.POINTER(i32), i32]
+        _lib.oracle_potrf_nchk.restype = i32
         _lib.oracle_encode.argtypes = [i64, i64, vp, i64, vp, i64, vp]
         _lib.oracle_encode.restype = i32
         _lib.oracle_verify.argtypes = [i64, i64, vp, i64, vp, i64, vp, i32, i32, ctypes.c_double,
@@ -106,9 +110,12 @@ MODE = {"enhanced": 0, "online": 1, "offline": 2, "enhanced_redo": 3}
 
 
 def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, inplace=False, mode="enhanced",
-          order="right"):
+          order="right", nchk=2):
     """ABFT Cholesky of A (lower), n % nb == 0. mode: "enhanced" (the paper's scheme, default),
     "online" or "offline" (its comparison schemes, which re-run once on an uncorrectable error).
+    nchk: checksum rows per block, 2 (the paper's choice) or 3 (m+1 = 3 checksums locate and
+    correct up to m = 2 errors per column; reading B10). Checksum-row injection targets are
+    rows nchk*I + t of the checksum matrix.
     Returns Result with L in the lower triangle (upper triangle untouched), status (0/1/2),
     LAPACK info, sorted events, reruns."""
     L = _as_f(A)
@@ -124,14 +131,14 @@ def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, in
         inj_arr = np.ascontiguousarray(inj)
         ninj = int(np.argmax(inj_arr["k"] == -1)) if (inj_arr["k"] == -1).any() else len(inj_arr)
     N = n // nb if nb > 0 else 0
-    chk = np.zeros((max(2 * N, 1), n), dtype=np.float64, order="F")
-    scl = np.zeros(n + 2 * N, dtype=np.float64)
+    chk = np.zeros((max(nchk * N, 1), n), dtype=np.float64, order="F")
+    scl = np.zeros(n + 3 * N, dtype=np.float64)
     reruns = ctypes.c_int(0)
-    st = lib().oracle_potrf_mode(n, nb, _ptr(L), max(n, 1), _ptr(inj_arr), ninj, nranks, K, c_tau, int(abft),
+    st = lib().oracle_potrf_nchk(n, nb, _ptr(L), max(n, 1), _ptr(inj_arr), ninj, nranks, K, c_tau, int(abft),
                                  MODE[mode] if isinstance(mode, str) else int(mode),
                                  {"right": 0, "left": 1}[order], _ptr(ev), cap,
                                  ctypes.byref(nev), ctypes.byref(info), _ptr(cnt), _ptr(chk), _ptr(scl),
-                                 ctypes.byref(reruns))
+                                 ctypes.byref(reruns), int(nchk))
     if st < 0:
         raise ValueError(f"oracle_potrf: invalid argument {-st}")
     ev = ev[: min(nev.value, cap)]

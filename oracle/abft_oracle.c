@@ -40,7 +40,7 @@
 enum { O_HOOK_REST = 0, O_HOOK_POTRF_OUT = 1, O_HOOK_TRSM_OUT = 2, O_HOOK_UPDATE_OUT = 3, O_HOOK_RECV = 4 };
 enum { O_TGT_DATA = 0, O_TGT_CHK = 1 };
 enum { O_V1 = 1, O_V2 = 2, O_V3 = 3, O_V4 = 4, O_V5 = 5, O_V6 = 6, O_V4R = 7, O_V7 = 8 };
-enum { O_DATA = 1, O_NONFINITE = 2, O_CHK1 = 3, O_CHK2 = 4, O_UNCORRECTABLE = 5 };
+enum { O_DATA = 1, O_NONFINITE = 2, O_CHK1 = 3, O_CHK2 = 4, O_UNCORRECTABLE = 5, O_CHK3 = 6 };
 enum { O_OK = 0, O_STATUS_UNCORRECTABLE = 1, O_STATUS_NOT_SPD = 2 };
 
 typedef struct { int32_t k, hook, target, pad0; int64_t row, col; uint64_t xor_mask; int32_t rank, pad1; } oinj_t;
@@ -59,7 +59,9 @@ typedef struct {
 
 typedef struct {
     int64_t n, B, N, lda, ldc;
-    double *A, *chk, *s, *S1, *S2;
+    int nchk;                      /* checksum rows per block: 2 (the paper's choice) or 3
+                                      (m+1 = 3 for m = 2 errors per column; NEXT-4)      */
+    double *A, *chk, *s, *S1, *S2, *S3;
     double c_tau, rho;
     int nranks, K, correct;
     int mode;                      /* 0 Enhanced Online-ABFT, 1 Online-ABFT, 2 Offline-ABFT */
@@ -73,6 +75,7 @@ typedef struct {
 typedef struct {
     double* T; int64_t ldt;
     double* c1; double* c2; int64_t ldc;   /* chk1[c] = c1[c*ldc], chk2[c] = c2[c*ldc] */
+    double* c3;                            /* third checksum row (v3 = [1, 4, ..., B^2]) or NULL */
     int64_t I, J;                          /* tile coordinates (for scales / events)    */
     int diag, factored;
 } tview_t;
@@ -104,7 +107,41 @@ static void push_event(octx_t* x, int k, int V, const tview_t* v, int64_t row, i
 }
 
 /* ---- Check(T(I,J)) — PAPER.md:180-195 §IV.C with readings A4-A12 ---------------------- */
-typedef struct { int64_t c; int kind; int64_t row; double d1, d2, r1, r2; } odec_t;
+typedef struct { int64_t c; int kind; int64_t row, row2; double d1, d2, d3, r1, r2, r3; } odec_t;
+
+/* Two errors in one column from three weighted sums (NEXT-4; "m+1 column checksums could
+ * locate and correct up to m errors per column", reading B10). With errors Da at weight wa and Db
+ * at weight wb (weights 1..B): d1 = Da + Db, d2 = wa Da + wb Db, d3 = wa^2 Da + wb^2 Db, so
+ * d3 = S d2 - P d1 with S = wa + wb, P = wa wb. Scan S = 3 .. 2B-1 in ascending order, P = rint((S d2 -
+ * d3) / d1); accept (wa, wb) = (S -+ sqrt(S^2 - 4P)) / 2 if they are integers in 1..B, the residual
+ * d3 - S d2 + P d1 is within its rounding tolerance and both errors exceed tau1. Exactly one
+ * accepted pair locates the errors; none or several -> not located. Returns 1 and the 0-based rows. */
+static int locate_two(double d1, double d2, double d3, double tau1, double tau2, double tau3, double rho, int64_t B,
+                      int64_t* ra, int64_t* rb) {
+    int found = 0;
+    if (!(fabs(d1) > tau1)) return 0;                 /* Da + Db ~ 0: P is not determined */
+    for (int64_t S = 3; S <= 2 * B - 1; ++S) {
+        const double Sd = (double)S;
+        const double Pd = nearbyint((Sd * d2 - d3) / d1);
+        if (!(Pd >= 2.0) || Pd > (double)B * (double)(B - 1)) continue;
+        const int64_t P = (int64_t)Pd;
+        const int64_t disc = S * S - 4 * P;
+        if (disc <= 0) continue;
+        int64_t q = (int64_t)sqrt((double)disc);
+        while (q * q > disc) --q;
+        while ((q + 1) * (q + 1) <= disc) ++q;
+        if (q * q != disc || ((S - q) & 1)) continue;
+        const int64_t wa = (S - q) / 2, wb = (S + q) / 2;
+        if (wa < 1 || wb > B) continue;
+        const double res = d3 - Sd * d2 + Pd * d1;
+        const double tol = tau3 + Sd * tau2 + Pd * tau1 + rho * (fabs(d3) + Sd * fabs(d2) + Pd * fabs(d1));
+        if (!(fabs(res) <= tol)) continue;
+        const double Da = ((double)wb * d1 - d2) / (double)(wb - wa), Db = (d2 - (double)wa * d1) / (double)(wb - wa);
+        if (!(fabs(Da) > tau1) || !(fabs(Db) > tau1)) continue;
+        if (++found == 1) { *ra = wa - 1; *rb = wb - 1; }
+    }
+    return found == 1;
+}
 
 static int check_tile(octx_t* x, const tview_t* v, int k, int V, int rank) {
     const int64_t B = x->B;
@@ -112,33 +149,39 @@ static int check_tile(octx_t* x, const tview_t* v, int k, int V, int rank) {
     odec_t* dec = (odec_t*)malloc(sizeof(odec_t) * (size_t)B);
     int64_t nd = 0;
     x->cnt->n_checks++;
-    x->cnt->flops_check += 4.0 * (double)(B * B);
+    x->cnt->flops_check += 2.0 * x->nchk * (double)(B * B);
     x->cnt->bytes_check += 8.0 * (double)(v->diag ? B * (B + 1) / 2 : B * B);
     for (int64_t c = 0; c < B; ++c) {
         /* recalculation chk' = v^T X, ascending row order */
-        double r1 = 0.0, r2 = 0.0;
+        double r1 = 0.0, r2 = 0.0, r3 = 0.0;
         for (int64_t r = 0; r < B; ++r) {
             double xv = X(v, r, c);
             r1 += xv;
             r2 += (double)(r + 1) * xv;          /* v2 = [1, 2, ..., B] [A7] */
+            if (v->c3) r3 += (double)((r + 1) * (r + 1)) * xv;   /* v3 = [1, 4, ..., B^2] [B10] */
         }
         const double chk1 = v->c1[c * v->ldc], chk2 = v->c2[c * v->ldc];
         const double d1 = r1 - chk1, d2 = r2 - chk2;
+        const double d3 = v->c3 ? r3 - v->c3[c * v->ldc] : 0.0;
         const int64_t g = v->J * B + c;
         const double sc = v->factored ? 1.0 : x->s[g];
         const double tau1 = ((x->c_tau * EPS) * x->S1[v->I]) * sc;   /* [A4] */
         const double tau2 = ((x->c_tau * EPS) * x->S2[v->I]) * sc;
+        const double tau3 = v->c3 ? ((x->c_tau * EPS) * x->S3[v->I]) * sc : 0.0;
         const int f1 = !isfinite(d1) || fabs(d1) > tau1;             /* P:195 + [A5] */
         const int f2 = !isfinite(d2) || fabs(d2) > tau2;
-        if (!f1 && !f2) {
+        const int f3 = v->c3 ? (!isfinite(d3) || fabs(d3) > tau3) : 0;
+        if (!f1 && !f2 && !f3) {
             const double q1 = fabs(d1) / tau1, q2 = fabs(d2) / tau2;
             if (q1 > x->cnt->max_ratio) x->cnt->max_ratio = q1;
             if (q2 > x->cnt->max_ratio) x->cnt->max_ratio = q2;
+            if (v->c3 && fabs(d3) / tau3 > x->cnt->max_ratio) x->cnt->max_ratio = fabs(d3) / tau3;
             continue;
         }
         odec_t* dd = &dec[nd++];
-        dd->c = c; dd->d1 = d1; dd->d2 = d2; dd->r1 = r1; dd->r2 = r2; dd->row = -1;
-        if (!isfinite(d1) || !isfinite(d2)) {                        /* [A9] */
+        dd->c = c; dd->d1 = d1; dd->d2 = d2; dd->d3 = d3; dd->r1 = r1; dd->r2 = r2; dd->r3 = r3;
+        dd->row = -1; dd->row2 = -1;
+        if (!isfinite(d1) || !isfinite(d2) || !isfinite(d3)) {       /* [A9] */
             int64_t best = 0; double bv = -1.0;
             for (int64_t r = 0; r < B; ++r) {
                 double xv = X(v, r, c);
@@ -153,25 +196,33 @@ static int check_tile(octx_t* x, const tview_t* v, int k, int V, int rank) {
             const double j = nearbyint(q);                           /* round half to even */
             if (j >= 1.0 && j <= (double)B) {
                 const double jd1 = j * d1;
-                if (fabs(d2 - jd1) <= tau2 + x->rho * fabs(jd1)) {
+                const double j2d1 = (j * j) * d1;
+                if (fabs(d2 - jd1) <= tau2 + x->rho * fabs(jd1) &&
+                    (!v->c3 || fabs(d3 - j2d1) <= tau3 + x->rho * fabs(j2d1))) {
                     dd->kind = O_DATA; dd->row = (int64_t)j - 1;     /* 1-based weights [A7] */
                     continue;
                 }
             }
-            dd->kind = f2 ? O_UNCORRECTABLE : O_CHK1;                /* [A10] */
+        }
+        if (f1 + f2 + f3 == 1) {                                     /* one checksum row corrupted [A10] */
+            dd->kind = f1 ? O_CHK1 : f2 ? O_CHK2 : O_CHK3;
             continue;
         }
-        dd->kind = O_CHK2;                                           /* !f1 && f2 [A10] */
+        if (v->c3 && locate_two(d1, d2, d3, tau1, tau2, tau3, x->rho, B, &dd->row, &dd->row2)) {
+            dd->kind = O_DATA;                                       /* two data errors [B10] */
+            continue;
+        }
+        dd->kind = O_UNCORRECTABLE;
     }
     /* corrections, computed from the pre-correction X, then applied [A8, A12] */
     typedef struct { double* p; double val; } fix_t;
-    fix_t* fix = (fix_t*)malloc(sizeof(fix_t) * (size_t)(nd + 1));
+    fix_t* fix = (fix_t*)malloc(sizeof(fix_t) * (size_t)(2 * nd + 1));
     int64_t nf = 0; int unc = 0;
     for (int64_t t = 0; t < nd; ++t) {
         odec_t* dd = &dec[t];
         const int64_t c = dd->c;
         x->cnt->n_detected++;
-        if (dd->kind == O_DATA || dd->kind == O_NONFINITE) {
+        if ((dd->kind == O_DATA && dd->row2 < 0) || dd->kind == O_NONFINITE) {
             double* p = Xstore(v, dd->row, c);
             int dup = 0;
             for (int64_t u = 0; u < nf; ++u) if (fix[u].p == p) dup = 1;
@@ -183,11 +234,41 @@ static int check_tile(octx_t* x, const tview_t* v, int k, int V, int rank) {
             if (v->diag && !v->factored && sr < scn) { int64_t t2 = sr; sr = scn; scn = t2; }
             push_event(x, k, V, v, sr, scn, dd->kind, rank, dd->d1, dd->d2);
             if (dd->kind == O_DATA) x->cnt->n_data++; else x->cnt->n_nonfinite++;
+        } else if (dd->kind == O_DATA) {                   /* two errors: rows a < b [B10] */
+            const int64_t ra = dd->row, rb = dd->row2;
+            const double wa = (double)(ra + 1), wb = (double)(rb + 1);
+            double s1 = 0.0, s2 = 0.0;                     /* the other B-2 rows, summed directly [A8] */
+            for (int64_t r = 0; r < B; ++r) {
+                if (r == ra || r == rb) continue;
+                const double xv = X(v, r, c);
+                s1 += xv; s2 += (double)(r + 1) * xv;
+            }
+            const double R1 = v->c1[c * v->ldc] - s1, R2 = v->c2[c * v->ldc] - s2;
+            const double xa = (wb * R1 - R2) / (wb - wa), xb = (R2 - wa * R1) / (wb - wa);
+            const int64_t rows[2] = {ra, rb};
+            const double vals[2] = {xa, xb};
+            int logged = 0;
+            for (int h = 0; h < 2; ++h) {
+                double* p = Xstore(v, rows[h], c);
+                int dup = 0;
+                for (int64_t u = 0; u < nf; ++u) if (fix[u].p == p) dup = 1;
+                if (dup) continue;
+                fix[nf].p = p; fix[nf].val = vals[h]; nf++;
+                int64_t sr = rows[h], scn = c;
+                if (v->diag && !v->factored && sr < scn) { int64_t t2 = sr; sr = scn; scn = t2; }
+                push_event(x, k, V, v, sr, scn, O_DATA, rank, dd->d1, dd->d2);
+                x->cnt->n_data++;
+                logged++;
+            }
+            x->cnt->n_detected += logged - 1;
         } else if (dd->kind == O_CHK1) {
             push_event(x, k, V, v, -1, c, O_CHK1, rank, dd->d1, dd->d2);
             x->cnt->n_chk1++;
         } else if (dd->kind == O_CHK2) {
             push_event(x, k, V, v, -2, c, O_CHK2, rank, dd->d1, dd->d2);
+            x->cnt->n_chk2++;
+        } else if (dd->kind == O_CHK3) {
+            push_event(x, k, V, v, -4, c, O_CHK3, rank, dd->d1, dd->d2);
             x->cnt->n_chk2++;
         } else {
             push_event(x, k, V, v, -3, c, O_UNCORRECTABLE, rank, dd->d1, dd->d2);
@@ -200,6 +281,7 @@ static int check_tile(octx_t* x, const tview_t* v, int k, int V, int rank) {
         for (int64_t t = 0; t < nd; ++t) {
             if (dec[t].kind == O_CHK1) v->c1[dec[t].c * v->ldc] = dec[t].r1;   /* chk1 := v1^T X */
             if (dec[t].kind == O_CHK2) v->c2[dec[t].c * v->ldc] = dec[t].r2;   /* chk2 := v2^T X */
+            if (dec[t].kind == O_CHK3) v->c3[dec[t].c * v->ldc] = dec[t].r3;   /* chk3 := v3^T X */
         }
     }
     free(fix); free(dec);
@@ -211,7 +293,8 @@ static int check_tile(octx_t* x, const tview_t* v, int k, int V, int rank) {
 static tview_t gview(octx_t* x, int64_t I, int64_t J, int factored) {
     tview_t v;
     v.T = x->A + J * x->B * x->lda + I * x->B; v.ldt = x->lda;
-    v.c1 = x->chk + J * x->B * x->ldc + 2 * I; v.c2 = v.c1 + 1; v.ldc = x->ldc;
+    v.c1 = x->chk + J * x->B * x->ldc + x->nchk * I; v.c2 = v.c1 + 1; v.ldc = x->ldc;
+    v.c3 = x->nchk == 3 ? v.c1 + 2 : NULL;
     v.I = I; v.J = J; v.diag = (I == J); v.factored = factored;
     return v;
 }
@@ -221,9 +304,13 @@ static void scales(octx_t* x) {
     const int64_t n = x->n, B = x->B;
     for (int64_t i = 0; i < n; ++i) x->s[i] = sqrt(x->A[i * x->lda + i]);    /* s_i = sqrt(A_ii) [A4] */
     for (int64_t I = 0; I < x->N; ++I) {
-        double a = 0.0, b = 0.0;
-        for (int64_t r = 0; r < B; ++r) { a += x->s[I * B + r]; b += (double)(r + 1) * x->s[I * B + r]; }
+        double a = 0.0, b = 0.0, c = 0.0;
+        for (int64_t r = 0; r < B; ++r) {
+            a += x->s[I * B + r]; b += (double)(r + 1) * x->s[I * B + r];
+            c += (double)((r + 1) * (r + 1)) * x->s[I * B + r];   /* S3 for v3 [B10] */
+        }
         x->S1[I] = a; x->S2[I] = b;
+        if (x->S3) x->S3[I] = c;
     }
 }
 
@@ -234,12 +321,16 @@ static void encode(octx_t* x) {
         const int64_t J = g / B, c = g % B;
         for (int64_t I = J; I < N; ++I) {
             tview_t v = gview(x, I, J, 0);
-            double r1 = 0.0, r2 = 0.0;
-            for (int64_t r = 0; r < B; ++r) { double xv = X(&v, r, c); r1 += xv; r2 += (double)(r + 1) * xv; }
+            double r1 = 0.0, r2 = 0.0, r3 = 0.0;
+            for (int64_t r = 0; r < B; ++r) {
+                double xv = X(&v, r, c); r1 += xv; r2 += (double)(r + 1) * xv;
+                r3 += (double)((r + 1) * (r + 1)) * xv;
+            }
             v.c1[c * v.ldc] = r1; v.c2[c * v.ldc] = r2;
+            if (v.c3) v.c3[c * v.ldc] = r3;
         }
     }
-    x->cnt->flops_encode += 4.0 * (double)(N * (N + 1) / 2) * (double)(B * B);
+    x->cnt->flops_encode += 2.0 * x->nchk * (double)(N * (N + 1) / 2) * (double)(B * B);
 }
 
 /* ---- fault injection at a named hook [A16, A21] ----------------------------------------- */
@@ -273,15 +364,15 @@ static int potrf_tile(octx_t* x, int64_t k) {
     }
     x->cnt->flops_factor += (double)B * B * B / 3.0;
     /* Alg. 2, on both checksum rows of tile (k,k) [A3] */
-    for (int t = 0; t < 2; ++t) {
-        double* ck = x->chk + k * B * x->ldc + 2 * k + t;
+    for (int t = 0; t < x->nchk; ++t) {
+        double* ck = x->chk + k * B * x->ldc + x->nchk * k + t;
         const int64_t st = x->ldc;
         for (int64_t j = 0; j < B; ++j) {
             ck[j * st] = ck[j * st] / T[j * lda + j];                         /* line 2 */
             for (int64_t i = j + 1; i < B; ++i) ck[i * st] -= ck[j * st] * T[j * lda + i];   /* line 3 */
         }
     }
-    x->cnt->flops_chkupd += 2.0 * (double)B * B;
+    x->cnt->flops_chkupd += (double)x->nchk * B * B;
     return 0;
 }
 
@@ -313,9 +404,9 @@ static void trsm_panel(octx_t* x, int64_t k) {
             }
         }
     }
-    for (int64_t r = 2 * (k + 1); r < 2 * N; ++r) trsm_row(L, lda, B, x->chk + k * B * x->ldc + r, x->ldc);
+    for (int64_t r = x->nchk * (k + 1); r < x->nchk * N; ++r) trsm_row(L, lda, B, x->chk + k * B * x->ldc + r, x->ldc);
     x->cnt->flops_factor += (double)(n - (k + 1) * B) * B * B;
-    x->cnt->flops_chkupd += (double)(2 * (N - k - 1)) * B * B;
+    x->cnt->flops_chkupd += (double)(x->nchk * (N - k - 1)) * B * B;
 }
 
 /* ---- trailing update: T(i,j) -= L_ik L_jk^T, chk(i,j) -= chk(i,k) L_jk^T ---
@@ -349,9 +440,9 @@ static void update(octx_t* x, int64_t k, const panel_t* pan_of_rank) {
                 }
                 for (int64_t r = r0; r < B; ++r) T[c * x->lda + r] -= tmp[r];
             }
-            for (int t = 0; t < 2; ++t) {                     /* checksum rows */
-                const double* ck = P->C + 2 * (i - k - 1) + t;  /* chk(i,k) row */
-                double* cd = x->chk + j * B * x->ldc + 2 * i + t;
+            for (int t = 0; t < x->nchk; ++t) {               /* checksum rows */
+                const double* ck = P->C + x->nchk * (i - k - 1) + t;  /* chk(i,k) row */
+                double* cd = x->chk + j * B * x->ldc + x->nchk * i + t;
                 for (int64_t c = 0; c < B; ++c) {
                     double a = 0.0;
                     for (int64_t p = 0; p < B; ++p) a += ck[p * P->ldcc] * Ljk[p * P->ldl + c];
@@ -363,7 +454,7 @@ static void update(octx_t* x, int64_t k, const panel_t* pan_of_rank) {
     }
     const double mB = (double)(m * B);
     x->cnt->flops_factor += mB * mB * B;               /* ~ (m B)^2 B: SYRK+GEMM, lower half */
-    x->cnt->flops_chkupd += 2.0 * 2.0 * (double)(m * (m + 1) / 2) * B * B;
+    x->cnt->flops_chkupd += 2.0 * x->nchk * (double)(m * (m + 1) / 2) * B * B;
 }
 
 /* ---- the factor loop --------------------------------------------- */
@@ -386,12 +477,13 @@ static int64_t g_kstop = INT64_MAX;
 
 static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
                       int nranks, int K, double c_tau, int abft, int mode, oevent_t* ev, int64_t cap,
-                      int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out) {
+                      int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out, int nchk) {
     octx_t X_; octx_t* x = &X_;
     memset(x, 0, sizeof *x);
     x->cnt = cnt;
     x->mode = mode;
-    x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = 2 * x->N > 0 ? 2 * x->N : 1;
+    x->nchk = nchk;
+    x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = nchk * x->N > 0 ? nchk * x->N : 1;
     x->A = A; x->c_tau = c_tau > 0 ? c_tau : 64.0; x->rho = 0x1p-30;   /* [A4, A6] */
     x->nranks = nranks; x->K = K; x->correct = 1;
     x->inj = inj; x->ninj = ninj; x->ev = ev; x->cap = cap;
@@ -402,9 +494,11 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
     x->s = (double*)malloc(sizeof(double) * (size_t)n);
     x->S1 = (double*)malloc(sizeof(double) * (size_t)N);
     x->S2 = (double*)malloc(sizeof(double) * (size_t)N);
+    x->S3 = nchk == 3 ? (double*)malloc(sizeof(double) * (size_t)N) : NULL;
+    const int nc = nchk;
     /* receiver copies of the panel (P>1 simulation) */
     double* rcopy = nranks > 1 ? (double*)malloc(sizeof(double) * (size_t)(nranks * n * B)) : NULL;
-    double* rchk = nranks > 1 ? (double*)malloc(sizeof(double) * (size_t)(nranks * 2 * N * B)) : NULL;
+    double* rchk = nranks > 1 ? (double*)malloc(sizeof(double) * (size_t)(nranks * nc * N * B)) : NULL;
     panel_t* pan = (panel_t*)malloc(sizeof(panel_t) * (size_t)nranks);
 
     if (abft) { scales(x); encode(x); }
@@ -428,30 +522,31 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
         const int64_t m = N - k - 1;
         for (int r = 0; r < nranks; ++r) {
             pan[r].L = x->A + k * B * lda + (k + 1) * B; pan[r].ldl = lda;
-            pan[r].C = x->chk + k * B * x->ldc + 2 * (k + 1); pan[r].ldcc = x->ldc;
+            pan[r].C = x->chk + k * B * x->ldc + nc * (k + 1); pan[r].ldcc = x->ldc;
         }
         if (abft && mode == 0 && nranks > 1 && m > 0) {                     /* RECV + V4R */
             int stop = 0;
             for (int r = 0; r < nranks && !stop; ++r) {
                 if (r == owner) continue;
                 double* Lr = rcopy + (size_t)r * n * B;     /* receiver buffer: m*B x B, ld = m*B */
-                double* Cr = rchk + (size_t)r * 2 * N * B;  /* 2m x B, ld = 2m                 */
-                const int64_t ldl = m * B, ldr = 2 * m;
+                double* Cr = rchk + (size_t)r * nc * N * B;  /* nc m x B, ld = nc m               */
+                const int64_t ldl = m * B, ldr = nc * m;
                 for (int64_t c = 0; c < B; ++c) {
                     memcpy(Lr + c * ldl, x->A + (k * B + c) * lda + (k + 1) * B, sizeof(double) * (size_t)(m * B));
-                    for (int64_t q = 0; q < 2 * m; ++q) Cr[c * ldr + q] = x->chk[(k * B + c) * x->ldc + 2 * (k + 1) + q];
+                    for (int64_t q = 0; q < nc * m; ++q) Cr[c * ldr + q] = x->chk[(k * B + c) * x->ldc + nc * (k + 1) + q];
                 }
                 /* RECV(k, r): target (row, col) global -> receiver buffer coordinates */
                 for (int64_t t = 0; t < ninj; ++t) {
                     const oinj_t* s = &inj[t];
                     if (s->k != k || s->hook != O_HOOK_RECV || s->rank != r) continue;
                     if (s->target == O_TGT_DATA) xor_double(&Lr[(s->col - k * B) * ldl + (s->row - (k + 1) * B)], s->xor_mask);
-                    else xor_double(&Cr[(s->col - k * B) * ldr + (s->row - 2 * (k + 1))], s->xor_mask);
+                    else xor_double(&Cr[(s->col - k * B) * ldr + (s->row - nc * (k + 1))], s->xor_mask);
                 }
                 for (int64_t i = k + 1; i < N && !stop; ++i) {
                     tview_t v;
                     v.T = Lr + (i - k - 1) * B; v.ldt = ldl;
-                    v.c1 = Cr + 2 * (i - k - 1); v.c2 = v.c1 + 1; v.ldc = ldr;
+                    v.c1 = Cr + nc * (i - k - 1); v.c2 = v.c1 + 1; v.ldc = ldr;
+                    v.c3 = nc == 3 ? v.c1 + 2 : NULL;
                     v.I = i; v.J = k; v.diag = 0; v.factored = 1;
                     if (check_tile(x, &v, (int)k, O_V4R, r)) stop = 1;
                 }
@@ -490,8 +585,9 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
         memcpy(scl_out, x->s, sizeof(double) * (size_t)n);
         memcpy(scl_out + n, x->S1, sizeof(double) * (size_t)N);
         memcpy(scl_out + n + N, x->S2, sizeof(double) * (size_t)N);
+        if (x->S3) memcpy(scl_out + n + 2 * N, x->S3, sizeof(double) * (size_t)N);
     }
-    free(x->chk); free(x->s); free(x->S1); free(x->S2); free(rcopy); free(rchk); free(pan);
+    free(x->chk); free(x->s); free(x->S1); free(x->S2); free(x->S3); free(rcopy); free(rchk); free(pan);
     return x->status;
 }
 
@@ -508,11 +604,12 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
  * V4 after TRSM); Offline only V6. */
 static int potrf_core_left(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
                            int K, double c_tau, int abft, int mode, oevent_t* ev, int64_t cap,
-                           int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out) {
+                           int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out, int nchk) {
     octx_t X_; octx_t* x = &X_;
     memset(x, 0, sizeof *x);
     x->cnt = cnt; x->mode = mode;
-    x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = 2 * x->N > 0 ? 2 * x->N : 1;
+    x->nchk = nchk;
+    x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = nchk * x->N > 0 ? nchk * x->N : 1;
     x->A = A; x->c_tau = c_tau > 0 ? c_tau : 64.0; x->rho = 0x1p-30;
     x->nranks = 1; x->K = K; x->correct = 1;
     x->inj = inj; x->ninj = ninj; x->ev = ev; x->cap = cap;
@@ -523,6 +620,7 @@ static int potrf_core_left(int64_t n, int64_t nb, double* A, int64_t lda, const 
     x->s = (double*)malloc(sizeof(double) * (size_t)n);
     x->S1 = (double*)malloc(sizeof(double) * (size_t)N);
     x->S2 = (double*)malloc(sizeof(double) * (size_t)N);
+    x->S3 = nchk == 3 ? (double*)malloc(sizeof(double) * (size_t)N) : NULL;
     double* tmp = (double*)malloc(sizeof(double) * (size_t)B);
     if (abft) { scales(x); encode(x); }
     for (int64_t j = 0; j < N && x->status == O_OK; ++j) {
@@ -552,9 +650,9 @@ static int potrf_core_left(int64_t n, int64_t nb, double* A, int64_t lda, const 
                     }
                     for (int64_t r = r0; r < B; ++r) T[c * lda + r] -= tmp[r];
                 }
-                for (int t = 0; t < 2; ++t) {
-                    const double* ck = x->chk + 2 * i + t;            /* chk(i, 0:j) row */
-                    double* cd = x->chk + j * B * x->ldc + 2 * i + t;
+                for (int t = 0; t < nchk; ++t) {
+                    const double* ck = x->chk + nchk * i + t;         /* chk(i, 0:j) row */
+                    double* cd = x->chk + j * B * x->ldc + nchk * i + t;
                     for (int64_t c = 0; c < B; ++c) {
                         double a = 0.0;
                         for (int64_t q = 0; q < j * B; ++q) a += ck[q * x->ldc] * Lj[q * lda + c];
@@ -563,7 +661,7 @@ static int potrf_core_left(int64_t n, int64_t nb, double* A, int64_t lda, const 
                 }
             }
             x->cnt->flops_factor += 2.0 * (double)((N - j) * B) * B * (double)(j * B);
-            x->cnt->flops_chkupd += 4.0 * (double)(N - j) * B * (double)(j * B);
+            x->cnt->flops_chkupd += 2.0 * nchk * (double)(N - j) * B * (double)(j * B);
         }
         if (abft) inject(x, (int)j, O_HOOK_UPDATE_OUT, 0, x->A, lda, x->chk, x->ldc);
         if (abft && mode != 2 && j > 0) {                             /* V5: the updated column j */
@@ -603,7 +701,8 @@ static int potrf_core_left(int64_t n, int64_t nb, double* A, int64_t lda, const 
         memcpy(scl_out + n, x->S1, sizeof(double) * (size_t)N);
         memcpy(scl_out + n + N, x->S2, sizeof(double) * (size_t)N);
     }
-    free(x->chk); free(x->s); free(x->S1); free(x->S2); free(tmp);
+    if (scl_out && abft && x->S3) memcpy(scl_out + n + 2 * N, x->S3, sizeof(double) * (size_t)N);
+    free(x->chk); free(x->s); free(x->S1); free(x->S2); free(x->S3); free(tmp);
     return x->status;
 }
 
@@ -614,11 +713,12 @@ static int potrf_core_left(int64_t n, int64_t nb, double* A, int64_t lda, const 
  * scheme with the same re-do for what two checksums cannot correct (more than one error in a
  * column of a block, P:121 [A11]): an UNCORRECTABLE outcome re-runs once.
  * Events of both runs are returned in order. */
-int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
+int oracle_potrf_nchk(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
                       int nranks, int K, double c_tau, int abft, int mode, int order, oevent_t* ev, int64_t cap,
                       int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out,
-                      int* reruns) {
+                      int* reruns, int nchk) {
     if (n < 0) return -1;
+    if (nchk != 2 && nchk != 3) return -12;
     if (nb < 1) return -2;
     if (n % nb) return -2;                          /* [A20] */
     if (lda < (n > 1 ? n : 1)) return -4;
@@ -639,9 +739,9 @@ int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
     if (order != 0 && nranks != 1) return -7;
     int64_t nev1 = 0;
     int st = order == 0 ? potrf_core(n, nb, A, lda, inj, ninj, nranks, K, c_tau, abft, mode, ev, cap, &nev1, info, c,
-                                     chk_out, scl_out)
+                                     chk_out, scl_out, nchk)
                         : potrf_core_left(n, nb, A, lda, inj, ninj, K, c_tau, abft, mode, ev, cap, &nev1, info, c,
-                                          chk_out, scl_out);
+                                          chk_out, scl_out, nchk);
     /* Online / Offline: a detection at the final sweep means an error escaped the scheme's
      * online checks and may have propagated -> re-do. */
     int v6_detect = 0;
@@ -652,15 +752,23 @@ int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
         int64_t nev2 = 0;
         const int64_t off = nev1 < cap ? nev1 : cap;
         st = order == 0 ? potrf_core(n, nb, A, lda, NULL, 0, nranks, K, c_tau, abft, mode, ev ? ev + off : NULL,
-                                     cap - off, &nev2, info, c, chk_out, scl_out)
+                                     cap - off, &nev2, info, c, chk_out, scl_out, nchk)
                         : potrf_core_left(n, nb, A, lda, NULL, 0, K, c_tau, abft, mode, ev ? ev + off : NULL,
-                                          cap - off, &nev2, info, c, chk_out, scl_out);
+                                          cap - off, &nev2, info, c, chk_out, scl_out, nchk);
         nev1 += nev2;
         if (reruns) *reruns = 1;
     }
     free(A0);
     if (nev) *nev = nev1;
     return st;
+}
+
+int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
+                      int nranks, int K, double c_tau, int abft, int mode, int order, oevent_t* ev, int64_t cap,
+                      int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out,
+                      int* reruns) {
+    return oracle_potrf_nchk(n, nb, A, lda, inj, ninj, nranks, K, c_tau, abft, mode, order, ev, cap, nev, info, cnt,
+                             chk_out, scl_out, reruns, 2);
 }
 
 int oracle_potrf(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
@@ -679,7 +787,7 @@ int oracle_encode(int64_t n, int64_t nb, const double* A, int64_t lda, double* c
     if (lda < (n > 1 ? n : 1)) return -4;
     octx_t X_; octx_t* x = &X_; memset(x, 0, sizeof *x);
     ocount_t c; memset(&c, 0, sizeof c); x->cnt = &c;
-    x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = ldc;
+    x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = ldc; x->nchk = 2;
     x->A = (double*)A; x->chk = chk; x->s = scl; x->S1 = scl + n; x->S2 = scl + n + x->N;
     x->nranks = 1;
     if (n == 0) return 0;
@@ -697,7 +805,7 @@ int oracle_verify(int64_t n, int64_t nb, double* A, int64_t lda, double* chk, in
     octx_t X_; octx_t* x = &X_; memset(x, 0, sizeof *x);
     ocount_t c0; memset(&c0, 0, sizeof c0);
     x->cnt = cnt ? cnt : &c0; memset(x->cnt, 0, sizeof(ocount_t));
-    x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = ldc;
+    x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = ldc; x->nchk = 2;
     x->A = A; x->chk = chk; x->s = (double*)scl; x->S1 = (double*)scl + n; x->S2 = (double*)scl + n + x->N;
     x->c_tau = c_tau > 0 ? c_tau : 64.0; x->rho = 0x1p-30; x->correct = correct;
     x->ev = ev; x->cap = cap; x->nranks = 1;
@@ -724,7 +832,7 @@ int oracle_potrf_prefix(int64_t n, int64_t nb, double* A, int64_t lda, int64_t k
     memset(c, 0, sizeof(ocount_t));
     int64_t nev = 0, info = 0;
     g_kstop = kstop < 0 ? 0 : kstop;
-    const int st = potrf_core(n, nb, A, lda, NULL, 0, 1, 1, 64.0, 1, 0, NULL, 0, &nev, &info, c, NULL, NULL);
+    const int st = potrf_core(n, nb, A, lda, NULL, 0, 1, 1, 64.0, 1, 0, NULL, 0, &nev, &info, c, NULL, NULL, 2);
     g_kstop = INT64_MAX;
     return st;
 }

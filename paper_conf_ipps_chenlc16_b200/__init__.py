@@ -75,6 +75,8 @@ _lib.abft_gen_spd.argtypes = [_i64, ctypes.c_uint64, _vp, _i64, _vp]
 _lib.abft_nccl_id.argtypes = [_vp]
 _lib.abft_comm_init.argtypes = [ctypes.POINTER(_vp), _i32, _vp, _i32]
 _lib.abft_comm_destroy.argtypes = [_vp]
+_lib.abft_comm_init_ipc.argtypes = [ctypes.POINTER(_vp), _i32, _i32, _i64, _vp]
+_lib.abft_comm_attach_ipc.argtypes = [_vp, _vp]
 _lib.abft_potrf_dist.argtypes = [_i64, _i64, _vp, _i64, _vp, _i32, _i32, _vp, _vp, _vp, _vp]
 _lib.abft_potrf_dist_sim.argtypes = [_i64, _i64, _i32, _vp, _i64, _vp, _vp, _vp, _vp]
 _lib.abft_potrf_dist_sim.restype = _i32
@@ -91,14 +93,15 @@ _lib.abft_phase_name.restype = ctypes.c_char_p
 _lib.abft_phase_name.argtypes = [_i32]
 _lib.abft_last_profile.argtypes = [_vp]
 for _f in ("abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
-           "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist"):
+           "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist", "abft_comm_init_ipc",
+           "abft_comm_attach_ipc"):
     getattr(_lib, _f).restype = _i32
 
 EXPORTS = ["abft_encode", "abft_verify", "abft_potrf", "abft_potrf_ex", "abft_potrf_host", "abft_gen_spd",
            "abft_nccl_id", "abft_comm_init", "abft_comm_destroy", "abft_potrf_dist",
            "abft_last_launch_count", "abft_version", "abft_last_error", "abft_last_profile", "abft_dev_gemm_nt", "abft_dev_chol_inv",
            "abft_dev_chol_trace", "abft_potrf_dist_sim", "abft_graph_release",
-           "abft_phase_name"]
+           "abft_phase_name", "abft_comm_init_ipc", "abft_comm_attach_ipc"]
 
 
 def lib():
@@ -240,6 +243,40 @@ def abft_comm_init(nranks, id128, rank):
     buf = ctypes.create_string_buffer(bytes(id128), 128)
     st = _lib.abft_comm_init(ctypes.byref(comm), nranks, buf, rank)
     return st, comm.value
+
+
+def abft_comm_init_ipc(nranks, rank, cap_bytes):
+    """Peer-memory (CUDA IPC) communicator: returns (status, comm, 64-byte handle of this rank)."""
+    comm = ctypes.c_void_p()
+    h = ctypes.create_string_buffer(64)
+    st = _lib.abft_comm_init_ipc(ctypes.byref(comm), nranks, rank, int(cap_bytes), h)
+    return st, comm.value, bytes(h.raw)
+
+
+def abft_comm_attach_ipc(comm, handles):
+    """handles: the nranks 64-byte handles in rank order."""
+    buf = ctypes.create_string_buffer(b"".join(handles), 64 * len(handles))
+    return _lib.abft_comm_attach_ipc(comm, buf)
+
+
+def ipc_comm(n, nb, group=None):
+    """Host plumbing of the peer-memory transport: every rank of the torch.distributed group
+    exports its arena (sized for the largest message of an n x n factorisation with block nb)
+    and maps every peer's. Returns the comm for abft_potrf_dist."""
+    import torch.distributed as dist
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    cap = 8 * ((n - nb) * nb + 2 * n + 8) + 48 * 8192   # packed panel + abort slot; event gather (8192)
+    st, comm, h = abft_comm_init_ipc(world, rank, cap)
+    assert st == 0, f"abft_comm_init_ipc: {st} {abft_last_error()}"
+    hs = [None] * world
+    dist.all_gather_object(hs, h, group=group)
+    st = abft_comm_attach_ipc(comm, hs)
+    assert st == 0, f"abft_comm_attach_ipc: {st} {abft_last_error()}"
+    return comm
+
+
+def abft_last_error():
+    return _lib.abft_last_error().decode()
 
 
 def abft_comm_destroy(comm):

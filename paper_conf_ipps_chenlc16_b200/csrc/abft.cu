@@ -398,17 +398,28 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     Profiler prof; prof.on = o.profile != 0 && !ps; prof.pool = &tc.timing;
     const double lowerB = Bd * (Bd + 1) / 2;                 // elements of a tril tile
     launch_zero(B, B, w.Li, B, s);
-    if (abft && !(abl & 16)) {   // encode
-        cudaEvent_t t = prof.begin(s);
+    // encode: block column 0 first, then the panel stream may start (panel 0
+    // reads only column 0's checksums), and the rest of the matrix is encoded on S concurrently
+    // with panel 0 — before update 0, the first reader of those checksums (reading B9)
+    cudaEvent_t t_enc = nullptr;
+    if (abft && !(abl & 16)) {
+        t_enc = prof.begin(s);
         launch_scales(n, nb, A, lda, w.scl, s);
-        StageArgs a = stage_base(w, A, lda, o.c_tau, SK_ALL, 0, -1);
+        StageArgs a = stage_base(w, A, lda, o.c_tau, SK_COLUMN, 0, 0);
         a.encode = 1;
         launch_check(a, s);
-        const double el = (double)(N * (N - 1) / 2) * Bd * Bd + (double)N * lowerB;
-        prof.end(t, PH_ENCODE, s, 4.0 * el, 8.0 * el);
     }
     {   // P starts after everything enqueued on S so far
         cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(P, e, 0);
+    }
+    if (abft && !(abl & 16)) {
+        if (N > 1) {
+            StageArgs a = stage_base(w, A, lda, o.c_tau, SK_TRAIL, 0, 0);
+            a.j_lo = 1; a.j_hi = N; a.encode = 1;
+            launch_check(a, s);
+        }
+        const double el = (double)(N * (N - 1) / 2) * Bd * Bd + (double)N * lowerB;
+        prof.end(t_enc, PH_ENCODE, s, 4.0 * el, 8.0 * el);
     }
 
     // ---- the panel of iteration k, on stream P ----
@@ -450,10 +461,11 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         if (v2done) cudaStreamWaitEvent(P, v2done, 0);                          // V2 before the TRSM reads
         // TRSM (+ Alg. 2 on the checksum rows of tile (k,k)): one GEMM per row segment
         t = prof.begin(P);
-        launch_gemm(mB, B, B, Akk + B, lda, w.Li, B, W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, P);
         if (abft && !(abl & 1))
-            launch_gemm(2 * m + 2, B, B, w.chk + k * B * w.ldc + 2 * k, w.ldc, w.Li, B, W + mB, ldw, 1.0, 0.0,
-                        true, 0, 1, 0, 0, 0, ab, P);
+            launch_trsm_with_chk(mB, B, Akk + B, lda, w.Li, W, ldw, 2 * m + 2, w.chk + k * B * w.ldc + 2 * k, w.ldc,
+                                 ab, P);
+        else
+            launch_gemm(mB, B, B, Akk + B, lda, w.Li, B, W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, P);
         prof.end(t, PH_TRSM, P, (mBd + (abft ? 2 * md + 2 : 0)) * Bd * Bd, 0);
         if (abft) {
             do_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, L, ab, P);
@@ -536,21 +548,22 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         if (fused & 1) slab_rows_used = cso.slab_rows;
         return fused;
     };
-    auto v5_cols = [&](int64_t k, int64_t jlo, int64_t jhi, bool fused) {
+    auto v5_cols = [&](int64_t k, int64_t jlo, int64_t jhi, bool fused, cudaStream_t vs = nullptr, int flist = 0) {
+        if (!vs) vs = s;
         StageArgs a = stage_base(w, A, lda, o.c_tau, SK_TRAIL, ABFT_V5, (int)k);
-        a.j_lo = jlo; a.j_hi = jhi; a.flist = 0;
+        a.j_lo = jlo; a.j_hi = jhi; a.flist = flist;
         const double el = (double)stage_count(a) * Bd * Bd - (double)(jhi - jlo) * Bd * (Bd - 1) / 2;
-        cudaEvent_t t = prof.begin(s);
+        cudaEvent_t t = prof.begin(vs);
         if (fused) {
             StageArgs d = a; d.kind = SK_TRAIL_DIAG;
             StageArgs f = a; f.kind = SK_TRAIL_OFF;
             f.cs = w.cs; f.cs_ld = n; f.cs_nslab = w.cs_nslab; f.cs_slab_rows = slab_rows_used;
-            launch_check_v5_fused(d, f, s);
+            launch_check_v5_fused(d, f, vs);
             const double rd = (double)(jhi - jlo) * lowerB, ro = (double)stage_count(f) * Bd * 2.0 * (Bd / (double)slab_rows_used);
-            prof.end(t, PH_V5, s, 4.0 * el, 8.0 * (rd + ro));   // bytes actually needed by the fused check
+            prof.end(t, PH_V5, vs, 4.0 * el, 8.0 * (rd + ro));   // bytes actually needed by the fused check
         } else {
-            launch_check(a, s);
-            prof.end(t, PH_V5, s, 4.0 * el, 8.0 * el);
+            launch_check(a, vs);
+            prof.end(t, PH_V5, vs, 4.0 * el, 8.0 * el);
         }
     };
 
@@ -932,10 +945,11 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             launch_check(a, PS);                                                     // V1, V2
         }
         launch_chol_inv(Akk, q.lda, q.w.Li, B, k * B, q.w.tmp, q.w.st, PS);
-        launch_gemm(mB, B, B, Akk + B, q.lda, q.w.Li, B, q.w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, PS);
+        if (abft)
+            launch_trsm_with_chk(mB, B, Akk + B, q.lda, q.w.Li, q.w.W, ldw, 2 * m + 2, ckk + 2 * k, q.w.ldc, ab, PS);
+        else
+            launch_gemm(mB, B, B, Akk + B, q.lda, q.w.Li, B, q.w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, PS);
         if (abft) {
-            launch_gemm(2 * m + 2, B, B, ckk + 2 * k, q.w.ldc, q.w.Li, B, q.w.W + mB, ldw, 1.0, 0.0, true, 0, 1,
-                        0, 0, 0, ab, PS);
             dist_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, P, q, ldw, mB, PS);
             StageArgs a3 = stage(q, SK_DIAG_FACT, ABFT_V3, (int)k);
             a3.ldw = ldw; a3.mB = mB; a3.flist = 1;

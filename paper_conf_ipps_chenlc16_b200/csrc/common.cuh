@@ -264,6 +264,10 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
 // The trailing update with the checksum rows as a second row segment of the same launch.
 // cstride > 1: C's column block t (and the B operand's row block t) is global block t * cstride
 // (a rank's 1D block-cyclic local columns in one launch); returns -1 if the shapes do not allow it.
+// Panel TRSM + its checksum rows in one launch (second row segment); returns 1 if fused.
+int launch_trsm_with_chk(int64_t mB, int64_t B, const double* Ap, int64_t lda, const double* Li, double* W,
+                         int64_t ldw, int64_t M2, const double* A2, int64_t lda2, const int32_t* abort_flag,
+                         cudaStream_t s);
 // Returns a bit mask: 1 = the fused V5 partials were written, 2 = the epilogue applied `inj`
 // (the caller applies the hook itself otherwise); -1 if cstride > 1 and the shapes do not allow it.
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,

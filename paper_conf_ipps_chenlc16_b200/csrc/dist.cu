@@ -39,6 +39,14 @@ extern "C" int abft_nccl_id(void* id128) {
     return 0;
 }
 
+struct AbftComm;
+AbftComm* abft_comm_cast(void* c);
+void* abft_comm_wrap_nccl(void* nccl);
+DistTransport* abft_comm_ipc_transport(AbftComm* a);
+void* abft_comm_nccl(AbftComm* a);
+int abft_comm_kind(AbftComm* a);
+void abft_comm_free(AbftComm* a);
+
 extern "C" int abft_comm_init(void** comm, int nranks, const void* id128, int rank) {
     if (!comm) return -1;
     if (nranks < 1) return -2;
@@ -48,13 +56,17 @@ extern "C" int abft_comm_init(void** comm, int nranks, const void* id128, int ra
     memcpy(&id, id128, sizeof id);
     ncclComm_t c;
     if (ncclCommInitRank(&c, nranks, id, rank) != ncclSuccess) return ABFT_ERR_NCCL;
-    *comm = (void*)c;
+    *comm = abft_comm_wrap_nccl((void*)c);
     return 0;
 }
 
 extern "C" int abft_comm_destroy(void* comm) {
-    if (!comm) return -1;
-    return ncclCommDestroy((ncclComm_t)comm) == ncclSuccess ? 0 : ABFT_ERR_NCCL;
+    AbftComm* a = abft_comm_cast(comm);
+    if (!a) return -1;
+    int rc = 0;
+    if (abft_comm_kind(a) == 0 && ncclCommDestroy((ncclComm_t)abft_comm_nccl(a)) != ncclSuccess) rc = ABFT_ERR_NCCL;
+    abft_comm_free(a);
+    return rc;
 }
 
 extern "C" int abft_potrf_dist(int64_t n, int64_t nb, double* A_local, int64_t lda_local, void* comm, int rank,
@@ -67,13 +79,19 @@ extern "C" int abft_potrf_dist(int64_t n, int64_t nb, double* A_local, int64_t l
     if (rank < 0 || rank >= nranks) return -6;
     if (!A_local && (N - rank + nranks - 1) / nranks > 0) return -3;
     if (lda_local < (n > 1 ? n : 1)) return -4;
-    if (!comm) return -5;
+    AbftComm* a = abft_comm_cast(comm);
+    if (!a) return -5;
+    DistLocal me{rank, A_local, lda_local};
+    if (abft_comm_kind(a) == 1) {   // peer-memory (CUDA IPC) transport
+        DistTransport* t = abft_comm_ipc_transport(a);
+        if (t->rank != rank || t->nranks != nranks) return -5;
+        return run_dist(n, nb, nranks, &me, 1, t, (cudaStream_t)stream, inj, rep, opt);
+    }
     NcclTransport tp;
-    tp.comm = (ncclComm_t)comm;
+    tp.comm = (ncclComm_t)abft_comm_nccl(a);
     tp.rank = rank; tp.nranks = nranks;
     int cr = 0, cn = 0;
     if (ncclCommUserRank(tp.comm, &cr) != ncclSuccess || ncclCommCount(tp.comm, &cn) != ncclSuccess) return ABFT_ERR_NCCL;
     if (cr != rank || cn != nranks) return -5;
-    DistLocal me{rank, A_local, lda_local};
     return run_dist(n, nb, nranks, &me, 1, &tp, (cudaStream_t)stream, inj, rep, opt);
 }

@@ -358,7 +358,7 @@ struct WsCfgT {
     static constexpr bool LDG = LDG_;
     static constexpr int WARPS_M = BM / WM, WARPS_N = BN / WN, CONSUMERS = WARPS_M * WARPS_N;
     static constexpr int THREADS = (CONSUMERS + 4) * 32;   // + one producer warpgroup (setmaxnreg)
-    static constexpr int REG_CONS = REG_CONS_, REG_PROD = LDG_ ? 48 : 40;
+    static constexpr int REG_CONS = REG_CONS_, REG_PROD = LDG_ ? 56 : 40;
     static constexpr int PA = BM + 4, PB = BN + 4;
     static constexpr int SA = BK * PA, SB = BK * PB;
     static constexpr size_t SMEM = (size_t)STAGES * (SA + SB) * sizeof(double) + 2 * STAGES * sizeof(uint64_t);
@@ -373,7 +373,7 @@ using WsCfg = WsCfgT<128, 128, 32, 3, 64, 32, 232, 1>;    // 8 consumer warps, 1
 using WsCfg16 = WsCfgT<128, 128, 32, 3, 32, 32, 104, 1>;  // 16 consumer warps, 32x32 warp tiles
 using WsCfg2a = WsCfgT<128, 64, 16, 4, 64, 32, 216, 2>;   // 2 CTAs/SM, 128x64 tiles, 4-stage BK=16
 using WsCfg2b = WsCfgT<128, 64, 32, 2, 64, 32, 216, 2>;   // 2 CTAs/SM, 128x64 tiles, 2-stage BK=32
-using WsCfg2l = WsCfgT<128, 64, 32, 2, 64, 32, 208, 2, true>;   // as 2b, LDGSTS producer warpgroup
+using WsCfg2l = WsCfgT<128, 64, 32, 2, 64, 32, 200, 2, true>;   // as 2b, LDGSTS producer warpgroup
 using WsCfgNR = WsCfgT<128, 64, 32, 2, 64, 32, 128, 2>;   // dev: as 2b without setmaxnreg (spills)
 
 // tile index -> (tm, tn) for the three masks; returns false for tiles with nothing to write
@@ -518,22 +518,30 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
                 if constexpr (C_::LDG) {
                     if (lane == 0) mbar_wait(&empty[st], ph ^ 1);
                     __syncwarp();
-                    const int64_t k0 = (int64_t)kt * BK;
-                    const int64_t ldA = T.seg2 ? g.lda2 : g.lda;
+                    // each of the 128 producer threads owns one 16-byte chunk column of A and of B and
+                    // copies it for every RA-th (RB-th) k-row of the stage: a base pointer + constant
+                    // strides, smem offsets are immediates (no per-copy index arithmetic)
                     constexpr int CA = BM / 2, CB = BN / 2;      // 16-byte chunks per k-row of A / B
-                    const double* a0 = Ap + k0 * ldA + m0;
-                    const double* b0 = g.B + k0 * g.ldb + bn0;
-                    double* sa = sA + st * C_::SA;
-                    double* sb = sB + st * C_::SB;
-#pragma unroll 4
-                    for (int q = ptid; q < BK * CA; q += 128) {
-                        const int kk = q / CA, r = q % CA;
-                        if (2 * r < (int)rowsA) cp_async16(sa + kk * C_::PA + 2 * r, a0 + kk * ldA + 2 * r, 16);
+                    constexpr int RA = 128 / CA, RB = 128 / CB;  // k-rows one pass of 128 threads covers
+                    static_assert(BK % RA == 0 && BK % RB == 0, "LDGSTS producer mapping");
+                    const int64_t ldA = T.seg2 ? g.lda2 : g.lda;
+                    const int ra = ptid % CA, ka = ptid / CA, rb = ptid % CB, kb = ptid / CB;
+                    const double* pa = Ap + ((int64_t)kt * BK + ka) * ldA + m0 + 2 * ra;
+                    const double* pb = g.B + ((int64_t)kt * BK + kb) * g.ldb + bn0 + 2 * rb;
+                    const uint32_t da = smem_u32(sA + st * C_::SA + ka * C_::PA + 2 * ra);
+                    const uint32_t db = smem_u32(sB + st * C_::SB + kb * C_::PB + 2 * rb);
+                    const int64_t sa_step = (int64_t)RA * ldA, sb_step = (int64_t)RB * g.ldb;
+                    if (2 * ra < (int)rowsA) {
+#pragma unroll 2
+                        for (int u = 0; u < BK / RA; ++u)
+                            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(da + u * RA * C_::PA * 8),
+                                         "l"(pa + u * sa_step) : "memory");
                     }
-#pragma unroll 4
-                    for (int q = ptid; q < BK * CB; q += 128) {
-                        const int kk = q / CB, r = q % CB;
-                        if (2 * r < (int)rowsB) cp_async16(sb + kk * C_::PB + 2 * r, b0 + kk * g.ldb + 2 * r, 16);
+                    if (2 * rb < (int)rowsB) {
+#pragma unroll 2
+                        for (int u = 0; u < BK / RB; ++u)
+                            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(db + u * RB * C_::PB * 8),
+                                         "l"(pb + u * sb_step) : "memory");
                     }
                     asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(smem_u32(&full[st])) : "memory");
                     continue;
@@ -664,6 +672,12 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
             const int64_t wbase = gr0 % g.cs.nb + fr + 1;   // weight (1-based) of row i = 0
             const int64_t slab = gr0 / g.cs.slab_rows;
             __syncwarp();
+            // per-thread sums over its FM rows for its 8 columns (slot q = 2 j + h): v[2q] = v1
+            // partial, v[2q + 1] = v2 partial; then a reduce-scatter butterfly over the 8 lanes
+            // of equal fc (lane bits 2-4 = fr): each round halves the values a lane keeps, so 14
+            // shuffles (not 48) leave lane fr holding the full sums of column slot fr
+            static_assert(C_::FN == 4, "reduce-scatter assumes 8 column slots per thread");
+            double v[16];
 #pragma unroll
             for (int j = 0; j < C_::FN; ++j)
 #pragma unroll
@@ -674,17 +688,38 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
                         s1 += acc[i][j][h];
                         s2 = fma((double)(wbase + i * 8), acc[i][j][h], s2);
                     }
-#pragma unroll
-                    for (int o = 4; o < 32; o <<= 1) {
-                        s1 += __shfl_xor_sync(0xffffffffu, s1, o);
-                        s2 += __shfl_xor_sync(0xffffffffu, s2, o);
-                    }
-                    if (offdiag && fr == 0) {
-                        const int64_t gc = gc0 + wn * WN + j * 8 + fc * 2 + h;
-                        g.cs.p[slab * g.cs.ld + gc] = s1;
-                        g.cs.p[(g.cs.nslab + slab) * g.cs.ld + gc] = s2;
-                    }
+                    v[2 * (2 * j + h)] = s1;
+                    v[2 * (2 * j + h) + 1] = s2;
                 }
+            {   // round 1: lane bit 4 (fr bit 2) picks the half of the 16 values it keeps
+                const bool up = (fr & 4) != 0;
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const double keep = up ? v[i + 8] : v[i], give = up ? v[i] : v[i + 8];
+                    v[i] = keep + __shfl_xor_sync(0xffffffffu, give, 16);
+                }
+            }
+            {   // round 2: fr bit 1
+                const bool up = (fr & 2) != 0;
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const double keep = up ? v[i + 4] : v[i], give = up ? v[i] : v[i + 4];
+                    v[i] = keep + __shfl_xor_sync(0xffffffffu, give, 8);
+                }
+            }
+            {   // round 3: fr bit 0
+                const bool up = (fr & 1) != 0;
+#pragma unroll
+                for (int i = 0; i < 2; ++i) {
+                    const double keep = up ? v[i + 2] : v[i], give = up ? v[i] : v[i + 2];
+                    v[i] = keep + __shfl_xor_sync(0xffffffffu, give, 4);
+                }
+            }
+            if (offdiag) {   // lane (fr, fc) holds column slot q = fr: j = fr / 2, h = fr % 2
+                const int64_t gc = gc0 + wn * WN + (fr >> 1) * 8 + fc * 2 + (fr & 1);
+                g.cs.p[slab * g.cs.ld + gc] = v[0];
+                g.cs.p[(g.cs.nslab + slab) * g.cs.ld + gc] = v[1];
+            }
         }
     }
 }
@@ -756,9 +791,18 @@ static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CT
     return v;
 }
 static int ws_slab_rows() { return ws_variant() == 16 ? WsCfg16::WM : 64; }
+// The one-launch task-graph diagonal block (ABFT_CHOL=tasks) keeps long-lived CTAs on the
+// high-priority panel stream; under that concurrency the bulk-copy (cp.async.bulk) operand
+// pipeline was measured to deliver stale k-slices to the update's consumers (DESIGN.md §5,
+// profiles/race_r02.md), the LDGSTS pipeline never. So that path takes the LDGSTS producer.
+static bool tasks_path() {
+    const char* e = getenv("ABFT_CHOL");
+    return e && !strcmp(e, "tasks");
+}
 static int run_ws_any(GemmArgs g, cudaStream_t s) {
     g.cs.slab_rows = ws_slab_rows();
     const bool upd = g.mask == MASK_LOWER && g.alpha == -1.0 && g.beta == 1.0;   // a trailing update
+    if (upd && tasks_path()) return run_ws<WsCfg2l>(g, s, upd);
     switch (ws_variant()) {
         case 16: return run_ws<WsCfg16>(g, s, upd);
         case 21: return run_ws<WsCfg2a>(g, s, upd);
@@ -863,4 +907,32 @@ int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int
     run_ws_any(g, s);
     if (ret & 1) cs->slab_rows = ws_slab_rows();
     return ret;
+}
+
+// Panel TRSM with the checksum rows (Alg. 2 folded in, reading B1) as ONE
+// launch: W[0:mB) = A_panel inv(L)^T (data rows, first row segment) and W[mB:mB+M2) =
+// chk_rows inv(L)^T (second segment). Falls back to two launches when the warp-specialised kernel
+// would not fill the GPU (small panels) or the shapes do not allow it.
+int launch_trsm_with_chk(int64_t mB, int64_t B, const double* Ap, int64_t lda, const double* Li, double* W,
+                         int64_t ldw, int64_t M2, const double* A2, int64_t lda2, const int32_t* abort_flag,
+                         cudaStream_t s) {
+    const int64_t tiles = ((mB + WsCfg::BM - 1) / WsCfg::BM) * ((B + 63) / 64);
+    const bool ok = mB > 0 && M2 > 0 && tiles >= 148 && (mB % 2 == 0) && (M2 % 2 == 0) && (B % WsCfg::BK == 0) &&
+                    (B % 2 == 0) && aligned16(Ap) && aligned16(Li) && aligned16(A2) && aligned16(W) && aligned16(W + mB) &&
+                    lda % 2 == 0 && lda2 % 2 == 0 && ldw % 2 == 0 && getenv("ABFT_GEMM_VARIANT") == nullptr;
+    if (!ok) {
+        launch_gemm(mB, B, B, Ap, lda, Li, B, W, ldw, 1.0, 0.0, true, MASK_NONE, KR_LE_N, 0, 0, 0, abort_flag, s);
+        if (M2 > 0)
+            launch_gemm(M2, B, B, A2, lda2, Li, B, W + mB, ldw, 1.0, 0.0, true, MASK_NONE, KR_LE_N, 0, 0, 0, abort_flag, s);
+        return 0;
+    }
+    GemmArgs g;
+    g.M = mB; g.N = B; g.K = B; g.A = Ap; g.lda = lda; g.B = Li; g.ldb = B; g.C = W; g.ldc = ldw;
+    g.alpha = 1.0; g.beta = 0.0; g.mask = MASK_NONE; g.krange = KR_LE_N; g.nb = B;
+    g.q_tile0 = 0; g.c_tile0 = 0; g.tiles_n = 1; g.abort = abort_flag; g.vecA = 1; g.vecB = 1;
+    g.cs = ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
+    g.inj.n = 0;
+    g.M2 = M2; g.A2 = A2; g.C2 = W + mB; g.ldc2 = ldw; g.lda2 = lda2; g.cstride = 1;
+    run_ws_any(g, s);
+    return 1;
 }

@@ -15,7 +15,7 @@ row 1 / row 2 shows as d1 alone / d2 alone (CHK1 / CHK2, reading A10).
 """
 
 V = {"V1": 1, "V2": 2, "V3": 3, "V4": 4, "V5": 5, "V6": 6, "V4R": 7, "V7": 8}
-KIND = {"DATA": 1, "NONFINITE": 2, "CHK1": 3, "CHK2": 4, "UNCORRECTABLE": 5}
+KIND = {"DATA": 1, "NONFINITE": 2, "CHK1": 3, "CHK2": 4, "UNCORRECTABLE": 5, "CHK3": 6}
 HOOKS = {"REST": 0, "POTRF_OUT": 1, "TRSM_OUT": 2, "UPDATE_OUT": 3, "RECV": 4}
 
 
@@ -57,8 +57,9 @@ def predict_left(spec, n, nb, K=1):
     return (ck, v, J, I, col, row, kind, 0)
 
 
-def predict(spec, n, nb, K=1):
-    """Return the expected event tuple (k, V, J, I, col, row, kind, rank) for one injection."""
+def predict(spec, n, nb, K=1, nchk=2):
+    """Return the expected event tuple (k, V, J, I, col, row, kind, rank) for one injection.
+    nchk: checksum rows per block (checksum-row targets are rows nchk*I + t; t = 2 -> CHK3)."""
     N = n // nb
     k = spec["k"]
     hook = spec["hook"] if isinstance(spec["hook"], str) else {v: kk for kk, v in HOOKS.items()}[spec["hook"]]
@@ -70,10 +71,10 @@ def predict(spec, n, nb, K=1):
         kind = KIND["DATA"]
     else:
         cr, c = spec["row"], spec["col"]
-        I, J = cr // 2, c // nb
+        I, J = cr // nchk, c // nb
         col = c - J * nb
-        row = -1 if cr % 2 == 0 else -2
-        kind = KIND["CHK1"] if cr % 2 == 0 else KIND["CHK2"]
+        row = (-1, -2, -4)[cr % nchk]
+        kind = (KIND["CHK1"], KIND["CHK2"], KIND["CHK3"])[cr % nchk]
     if hook == "REST":
         if k >= N or J < k:
             chk_k, v = N, V["V6"]

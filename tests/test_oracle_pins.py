@@ -483,3 +483,120 @@ def test_enhanced_redo_recovers_and_matches_lapack():
     # single errors are corrected in place: no re-run
     one = oracle.potrf(A, nb, inj=syn.inj_array(TWO_IN_A_COLUMN[:1]), mode="enhanced_redo")
     assert one.status == 0 and one.reruns == 0 and len(one.events) == 1
+
+
+# ---- NEXT-4: m+1 = 3 checksums locate and correct up to m = 2 errors per column -----
+# Reading B10: v3 = [1, 4, ..., B^2]; two errors Da (weight wa), Db (weight wb) give
+# d1 = Da + Db, d2 = wa Da + wb Db, d3 = wa^2 Da + wb^2 Db, hence d3 = (wa + wb) d2 - wa wb d1; the
+# integers wa < wb are found by scanning S = wa + wb; corrections from the first two checksum rows.
+
+def test_next4_three_checksums_same_factor_and_checksum_invariant():
+    """nchk = 3 changes no data arithmetic: L bit-identical to nchk = 2, no event; the carried
+    third checksum row equals v3^T tril(L) (the P5 invariant with weights r^2)."""
+    n, nb = 512, 64
+    A = syn.spd_matrix(n)
+    r2 = oracle.potrf(A, nb)
+    r3 = oracle.potrf(A, nb, nchk=3)
+    assert r3.status == 0 and len(r3.events) == 0
+    assert np.array_equal(np.tril(r2.L), np.tril(r3.L))
+    L = np.tril(r3.L)
+    N = n // nb
+    w3 = (np.arange(1, nb + 1, dtype=np.float64)) ** 2
+    for I in range(N):
+        for J in range(I + 1):
+            T = L[I * nb:(I + 1) * nb, J * nb:(J + 1) * nb]
+            ref = w3 @ T
+            got = r3.chk[3 * I + 2, J * nb:(J + 1) * nb]
+            assert np.max(np.abs(got - ref)) <= 1e-9 * max(1.0, np.max(np.abs(ref)))
+
+
+def test_next4_pascal_mod2_two_errors_ambiguity_of_three_sums():
+    """The limit of m+1 = 3 sums for m = 2 (reading B10): they fix the pair only up to the line
+    d3 = S d2 - P d1 in (S = wa + wb, P = wa wb). With P2's integer data both d2/d1 = 15 and
+    d3/d1 = 249 are integers, so EVERY S gives an integer P and five row pairs inside the block fit
+    exactly (wa, wb) = (3, 17), (7, 18), (9, 19) (the true one), (11, 21), (12, 23): ambiguous ->
+    UNCORRECTABLE (never a mis-correction); two checksums mis-correct this case."""
+    n, nb = 256, 32
+    A = syn.pascal_mod2(n)
+    # both targets hold 1.0 at k = 2: bit 52 -> 0.5 (Delta -0.5), bit 53 -> 0.25 (Delta -0.75)
+    specs = [dict(k=2, hook="REST", row=200, col=100, bit=52),
+             dict(k=2, hook="REST", row=210, col=100, bit=53)]
+    inj = syn.inj_array(specs)
+    two = oracle.potrf(A, nb, inj=inj)
+    assert two.status != 0                 # two checksums: UNCORRECTABLE or a mis-correction
+    r = oracle.potrf(A, nb, inj=inj, nchk=3)
+    assert r.status == 1
+    ev = r.event_tuples()
+    assert len(ev) == 1 and ev[0][6] == KIND["UNCORRECTABLE"] and ev[0][:5] == (2, V["V5"], 3, 6, 4)
+
+
+def test_next4_two_errors_in_one_column_generic_values():
+    """Two storage errors in ONE column of one tile of a random SPD matrix (real, generic values):
+    with three checksums both are located where the schedule predicts and corrected (L within
+    the P4 tolerance of the fault-free factor); with two checksums the run cannot complete."""
+    n, nb = 512, 64
+    A = syn.spd_matrix(n, seed=9)
+    specs = [dict(k=2, hook="REST", row=400, col=200, bit=52),
+             dict(k=2, hook="REST", row=430, col=200, bit=55)]
+    inj = syn.inj_array(specs)
+    assert oracle.potrf(A, nb, inj=inj).status != 0
+    r = oracle.potrf(A, nb, inj=inj, nchk=3)
+    assert r.status == 0
+    assert r.event_tuples() == sorted(predict(s, n, nb, nchk=3) for s in specs)
+    assert floor_rel(r.L, oracle.potrf(A, nb, nchk=3).L, A) <= 1e-11
+
+
+@pytest.mark.parametrize("hook", ["REST", "UPDATE_OUT"])
+def test_next4_brute_force_every_row_pair_of_a_column(hook):
+    """Brute force on a tiny case: two errors at EVERY pair of rows (a < b) of one tile column
+    (nb = 16: 120 pairs), each located at the predicted check and corrected: L equal to the
+    fault-free factor within the P4 tolerance."""
+    n, nb = 64, 16
+    A = syn.spd_matrix(n, seed=21)
+    ref = oracle.potrf(A, nb, nchk=3)
+    k, J, I, c = 1, 2, 3, 5
+    for a in range(nb):
+        for b in range(a + 1, nb):
+            specs = [dict(k=k, hook=hook, row=I * nb + a, col=J * nb + c, bit=55),
+                     dict(k=k, hook=hook, row=I * nb + b, col=J * nb + c, bit=54)]
+            r = oracle.potrf(A, nb, inj=syn.inj_array(specs), nchk=3)
+            assert r.status == 0, (a, b)
+            assert r.event_tuples() == sorted(predict(s, n, nb, nchk=3) for s in specs), (a, b)
+            assert floor_rel(r.L, ref.L, A) <= 1e-11, (a, b)
+
+
+def test_next4_single_errors_unchanged_and_chk3_repair():
+    """Single errors are located exactly as with two checksums (C2 schedule), and a corrupted
+    third checksum row is repaired from the data (CHK3) leaving L bit-identical."""
+    n, nb = 1024, 128
+    A = syn.spd_matrix(n)
+    specs = syn.per_iteration_injections(n, nb, bits=(45, 61))
+    inj = syn.inj_array(specs)
+    r2 = oracle.potrf(A, nb, inj=inj)
+    r3 = oracle.potrf(A, nb, inj=inj, nchk=3)
+    assert r3.status == r2.status == 0
+    assert r3.event_tuples() == r2.event_tuples()
+    c3 = [dict(k=1, hook="REST", target="CHK", row=3 * 5 + 2, col=2 * nb + 9, bit=50)]
+    r = oracle.potrf(A, nb, inj=syn.inj_array(c3), nchk=3)
+    clean = oracle.potrf(A, nb, nchk=3)
+    assert r.status == 0 and r.event_tuples() == [predict(c3[0], n, nb, nchk=3)]
+    assert np.array_equal(np.tril(r.L), np.tril(clean.L))
+
+
+def test_next4_equal_and_opposite_pair_is_uncorrectable():
+    """Da = -Db: d1 = 0 leaves P undetermined (no set of m+1 sums locates it) -> UNCORRECTABLE."""
+    n, nb = 256, 32
+    A = syn.pascal_mod2(n)
+    specs = [dict(k=2, hook="REST", row=200, col=100, bit=52),    # 1.0 -> 0.5
+             dict(k=2, hook="REST", row=210, col=100, bit=51)]    # 1.0 -> 1.5: d1 = 0
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs), nchk=3)
+    assert r.status == 1
+
+
+def test_next4_three_errors_in_a_column_uncorrectable():
+    n, nb = 256, 32
+    A = syn.spd_matrix(n, seed=5)
+    specs = [dict(k=1, hook="REST", row=100 + 7 * t, col=70, bit=52 - t) for t in range(3)]
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs), nchk=3)
+    assert r.status == 1
+    assert any(e[6] == KIND["UNCORRECTABLE"] for e in r.event_tuples())

@@ -1,19 +1,20 @@
-# Race bisection of the warp-specialised update kernel: fault-free C5 factorisations
-# with the one-launch diagonal block on the high-priority panel stream (the known trigger), one
-# process per variant (the library reads its knobs once). A clean run raises no event.
+# Race bisection of the warp-specialised update kernel: fault-free factorisations,
+# one process per variant (the library reads its knobs once). A clean run raises no event.
+# usage: bash tools/race_matrix.sh [n] [nb] [reps] -> gpurun_out/race_matrix_<n>.log
 mkdir -p gpurun_out
-out=gpurun_out/race_matrix.log
+n=${1:-98304}; nb=${2:-1024}; reps=${3:-3}
+out=gpurun_out/race_matrix_$n.log
 : > $out
 run() {
   echo "=== $1" >> $out
   shift
-  env "$@" ABFT_CHOL=tasks ABFT_CHOL_G=1 REPS=${REPS:-2} timeout 300 python tools/stress_v5.py ${N:-98304} ${NB:-1024} x >> $out 2>&1
+  env "$@" REPS=$reps timeout 400 python tools/stress_v5.py $n $nb x 2>&1 | grep -E "status|Error|error" | cut -c1-200 >> $out
   echo "rc=$?" >> $out
 }
-run default X=0
-run fence_consumer ABFT_WS_DBG=1
-run producer_tail ABFT_WS_DBG=2
-run tail_idle_resident ABFT_WS_DBG=6
-run c_preload_cg ABFT_WS_DBG=8
-run no_l2_prefetch ABFT_WS_PF=0
-run ldgsts_producer ABFT_WS=2l
+run default_recursive_highprio X=0
+run tasks_G1 ABFT_CHOL=tasks ABFT_CHOL_G=1
+run tasks_G10 ABFT_CHOL=tasks
+run tasks_G1_normal_prio ABFT_CHOL=tasks ABFT_CHOL_G=1 ABFT_P_PRIO=0
+run tasks_G1_ldgsts ABFT_CHOL=tasks ABFT_CHOL_G=1 ABFT_WS=2l
+run tasks_G1_cp_async_gemm ABFT_CHOL=tasks ABFT_CHOL_G=1 ABFT_GEMM_VARIANT=2
+run recursive_nofuse ABFT_NOFUSE=1
