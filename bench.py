@@ -402,6 +402,31 @@ def main():
             table["two_errors_in_a_column"][mode] = {
                 "ms": round(tf[0], 2), "status": "uncorrectable" if rf[0]["n_uncorrectable"] and not rf[0]["reruns"]
                 else "ok", "reruns": int(rf[0]["reruns"]), "events": int(rf[0]["n_events"])}
+        # NEXT-4 on the headline workload: three checksum rows (m+1 = 3 for m = 2 errors per column,
+        # P:121, reading B10) — fault-free cost, and the C3-style injections plus a second error
+        # next to every tenth one (two errors in one column of a tile), all corrected in place
+        t3, r3 = run_steps(P.options(nchk=3), steps=max(1, min(3, args.steps)), warmup=1)
+        specs3 = []
+        for sp in syn.mixed_injections(n, nb):
+            if sp.get("target", "DATA") == "CHK":
+                sp = dict(sp, row=3 * (sp["row"] // 2) + sp["row"] % 2)
+            specs3.append(sp)
+        pairs = 0
+        for sp in list(specs3)[1::10]:
+            if sp.get("target", "DATA") == "DATA" and sp["hook"] in ("UPDATE_OUT", "REST"):
+                r2 = (sp["row"] // nb) * nb + (sp["row"] % nb + 97) % nb
+                if r2 >= sp["col"] and r2 != sp["row"]:
+                    specs3.append(dict(sp, row=r2, bit=53))
+                    pairs += 1
+        ti3, ri3 = run_steps(P.options(nchk=3), inj=syn.inj_array(specs3), steps=1, warmup=1, fault_free=False)
+        ms3 = statistics.median(t3)
+        line["next4_three_checksums"] = {
+            "value": round(flops / (ms3 * 1e-3) / 1e9, 2), "ms_per_step": round(ms3, 3),
+            "overhead_vs_two_checksums_pct": round(100 * (ms3 - ms) / ms, 3),
+            "overhead_vs_abft_off_pct": round(100 * (ms3 - ms_off) / ms_off, 3),
+            "injected": {"injections": len(specs3), "two_error_columns": pairs, "status": "ok" if ri3[0]["n_uncorrectable"] == 0 else "uncorrectable",
+                         "events": int(ri3[0]["n_events"]), "corrected": int(ri3[0]["n_data"] + ri3[0]["n_nonfinite"] + ri3[0]["n_chk1"] + ri3[0]["n_chk2"]),
+                         "ms": round(ti3[0], 2)}}
         table["paper_context_seconds"] = {
             "Tardis_M2075_n20480": {"enhanced": [10.6572, 10.6614, 10.6678], "online": [10.5067, 10.5244, 22.625],
                                     "offline": [10.4489, 21.3942, 21.2631], "src": "PAPER.md:366-368"},

@@ -51,7 +51,8 @@ typedef struct CUstream_st* abft_stream_t;
 #define ABFT_HOOK_UPDATE_OUT 3 /* corrupt the output of the trailing update of iteration k        */
 #define ABFT_HOOK_RECV 4       /* (multi-GPU) corrupt rank `rank`'s received copy of panel k      */
 #define ABFT_TGT_DATA 0        /* row, col = global element of A (row >= col)                     */
-#define ABFT_TGT_CHK 1         /* row = checksum row 2I + {0,1}, col = global column (col/nb <= I) */
+#define ABFT_TGT_CHK 1         /* row = checksum row nchk I + t (t < nchk; nchk = 2 unless options
+                                  say 3), col = global column (col/nb <= I)                       */
 
 /* checks (where an event was raised) and event kinds */
 #define ABFT_V1 1   /* pre-read check of the diagonal tile (k,k) before POTRF                */
@@ -66,7 +67,9 @@ typedef struct CUstream_st* abft_stream_t;
 #define ABFT_KIND_NONFINITE 2     /* non-finite delta; located by argmax |X| and corrected       */
 #define ABFT_KIND_CHK1 3          /* checksum row 1 corrupted; recomputed from the data          */
 #define ABFT_KIND_CHK2 4          /* checksum row 2 corrupted; recomputed from the data          */
-#define ABFT_KIND_UNCORRECTABLE 5 /* more than one error in a tile column: abort (status 1)      */
+#define ABFT_KIND_UNCORRECTABLE 5 /* more errors in a tile column than the checksums locate:
+                                     abort (status 1)                                          */
+#define ABFT_KIND_CHK3 6          /* (nchk = 3) checksum row 3 corrupted; recomputed from the data */
 
 typedef struct abft_inject_spec {
     int32_t k, hook, target, pad0;
@@ -78,7 +81,7 @@ typedef struct abft_inject_spec {
 typedef struct abft_event {
     int32_t k, check, tile_i, tile_j;
     int32_t row, col;   /* inside the tile; the stored (lower) element for diagonal tiles;
-                           row = -1 / -2 for CHK1 / CHK2, -3 for UNCORRECTABLE              */
+                           row = -1 / -2 / -4 for CHK1 / CHK2 / CHK3, -3 for UNCORRECTABLE  */
     int32_t kind, rank;   /* rank that ran the check: owner of block column tile_j (receiver for V4R) */
     double delta1, delta2;
 } abft_event_t;
@@ -86,6 +89,7 @@ typedef struct abft_event {
 typedef struct abft_report {
     int64_t info;       /* LAPACK info: 1-based order of the first non-positive leading minor */
     int64_t n_checks, n_detected, n_data, n_nonfinite, n_chk1, n_chk2, n_uncorrectable;
+                        /* n_chk2 counts repairs of checksum rows 2 and 3                  */
     int64_t n_events;   /* events raised (may exceed cap; only cap are stored)               */
     int64_t cap;        /* capacity of `events` (set by the caller)                          */
     abft_event_t* events; /* HOST array owned by the caller, sorted by (k, check, J, I, col, row) */
@@ -106,6 +110,11 @@ typedef struct abft_options {
     int32_t mode;         /* ABFT_MODE_ENHANCED (default), _ONLINE, _OFFLINE or _ENHANCED_REDO    */
     int32_t order;        /* ABFT_ORDER_RIGHT (default: trailing update + look-ahead) or
                              ABFT_ORDER_LEFT (MAGMA's Alg. 1, Table I checks)     */
+    int32_t nchk;         /* checksum rows per block: 0 or 2 (the paper's choice) or 3: the
+                             third row v3 = [1, 4, .., nb^2] locates and corrects up to TWO errors
+                             in a column of a block ("m+1 column checksums ... up to m errors",
+                             P:121; reading B10 of DESIGN.md: ambiguous pairs are UNCORRECTABLE).
+                             nchk = 3: right-looking Enhanced scheme on one GPU (else -8)         */
 } abft_options_t;
 #define ABFT_ORDER_RIGHT 0
 #define ABFT_ORDER_LEFT 1
@@ -157,7 +166,7 @@ int abft_verify(int64_t n, int64_t nb, double* A, int64_t lda, double* chk, int6
 
 /* Enhanced Online-ABFT Cholesky, A = L L^T in place (lower). Workspace (checksums, scales,
  * panel buffer, event buffer: about n*nb + 2n^2/nb doubles) is allocated with cudaMallocAsync
- * on `stream` and freed before return. inj: HOST list (NULL = none), validated up front
+ * on `stream` and freed before return (except in graph mode, see abft_graph_release). inj: HOST list (NULL = none), validated up front
  * (-6 on an out-of-range target/hook). rep: HOST report (NULL = asynchronous, no report).
  * Errors: -1 n, -2 nb, -3 A, -4 lda, -6 inj. */
 int abft_potrf(int64_t n, int64_t nb, double* A, int64_t lda, abft_stream_t stream,
@@ -168,7 +177,9 @@ int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft_stream_t s
                   const abft_inject_spec_t* inj, abft_report_t* rep, const abft_options_t* opt);
 
 /* End-to-end variant on HOST memory (A_host: n x n column-major, lda >= n; pinned memory
- * recommended): copies A to the device, factors with abft_potrf_ex, copies L back, then
+ * recommended — the overlapped write-back below is used only for page-locked A_host, a
+ * pageable buffer takes the plain copy-factor-copy path): copies A to the device, factors with
+ * abft_potrf_ex, copies L back, then
  * synchronises. On the direct fault-free right-looking path (no injections, n above the graph-
  * mode threshold) only the block columns from their diagonal blocks down go to the device (the
  * strict upper triangle outside the diagonal blocks is never read, as in LAPACK uplo = 'L'), and
@@ -251,10 +262,12 @@ int abft_dev_chol_trace(int64_t nb, double* A, int64_t lda, double* Li, uint64_t
 /* Graph mode. A fault-free Enhanced (or ABFT-off) right-looking abft_potrf / abft_potrf_ex call
  * without the per-phase profiler is captured once into a CUDA graph (both streams) and replayed
  * on later calls with the same device, n, nb, A, lda, options and report capacity: no host launch
- * cost, shorter dependent-launch gaps on the panel chain. The graph and its workspace are cached
- * per host thread (one entry) and stay allocated until the key changes or this call releases
- * them. Default for n <= 12288 (measured faster there, slower above); ABFT_GRAPH=0 / 1 in the
- * environment forces direct launches / graph mode. Returns 0. */
+ * cost, shorter dependent-launch gaps on the panel chain. OWNERSHIP EXCEPTION to abft_potrf's
+ * "workspace freed before return": in graph mode the workspace (about n nb + 3 n^2 / nb doubles
+ * plus the fused-V5 partials) belongs to the cached graph, per host thread (one entry), and stays
+ * allocated until the key changes or this call releases it. Default for n <= 12288 (measured
+ * faster there, slower above); ABFT_GRAPH=0 / 1 in the environment forces direct launches /
+ * graph mode. Returns 0. */
 int abft_graph_release(void);
 
 /* Diagnostics: kernel launches issued by the last call on this thread, a static version string,

@@ -24,7 +24,7 @@ LIB_PATH = os.path.join(_HERE, "libabft.so")
 OK, UNCORRECTABLE, NOT_SPD, ERR_CUDA, ERR_NCCL = 0, 1, 2, 3, 4
 HOOK = {"REST": 0, "POTRF_OUT": 1, "TRSM_OUT": 2, "UPDATE_OUT": 3, "RECV": 4}
 CHECK = {1: "V1", 2: "V2", 3: "V3", 4: "V4", 5: "V5", 6: "V6", 7: "V4R", 8: "V7"}
-KIND = {1: "DATA", 2: "NONFINITE", 3: "CHK1", 4: "CHK2", 5: "UNCORRECTABLE"}
+KIND = {1: "DATA", 2: "NONFINITE", 3: "CHK1", 4: "CHK2", 5: "UNCORRECTABLE", 6: "CHK3"}
 
 EVENT_DTYPE = np.dtype([
     ("k", "<i4"), ("check", "<i4"), ("tile_i", "<i4"), ("tile_j", "<i4"),
@@ -53,7 +53,7 @@ class Report(ctypes.Structure):
 class Options(ctypes.Structure):
     _fields_ = [("abft_enabled", ctypes.c_int32), ("K", ctypes.c_int32), ("c_tau", ctypes.c_double),
                 ("lookahead", ctypes.c_int32), ("profile", ctypes.c_int32), ("mode", ctypes.c_int32),
-                ("order", ctypes.c_int32)]
+                ("order", ctypes.c_int32), ("nchk", ctypes.c_int32)]
 
 
 class Profile(ctypes.Structure):
@@ -159,9 +159,10 @@ def _report_dict(rep, ev):
 MODE = {"enhanced": 0, "online": 1, "offline": 2, "enhanced_redo": 3}
 
 
-def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False, mode="enhanced", order="right"):
+def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False, mode="enhanced", order="right", nchk=2):
+    """nchk: checksum rows per block, 2 (the paper's choice) or 3 (up to two errors per column)."""
     return Options(int(bool(abft_enabled)), int(K), float(c_tau), int(lookahead), int(bool(profile)),
-                   MODE[mode] if isinstance(mode, str) else int(mode), {"right": 0, "left": 1}[order])
+                   MODE[mode] if isinstance(mode, str) else int(mode), {"right": 0, "left": 1}[order], int(nchk))
 
 
 def abft_last_profile():

@@ -32,7 +32,7 @@ static bool has_inj(const std::vector<abft_inject_spec_t>& list, int64_t k, int 
     for (const auto& sp : list) if (sp.k == k && sp.hook == hook) return true;
     return false;
 }
-int launch_scales(int64_t n, int64_t nb, const double* A, int64_t lda, double* scl, cudaStream_t s);
+int launch_scales(int64_t n, int64_t nb, const double* A, int64_t lda, double* scl, cudaStream_t s, int nchk = 2);
 int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,
                 const int32_t* abort_flag, cudaStream_t s);
 int launch_zero(int64_t rows, int64_t cols, double* dst, int64_t ldd, cudaStream_t s);
@@ -72,7 +72,7 @@ static int check_common(int64_t n, int64_t nb, const void* A, int64_t lda) {
 
 // Injection specs: validated against the region their hook can touch.
 static int collect_inj(const abft_inject_spec_t* inj, int64_t n, int64_t nb, std::vector<abft_inject_spec_t>& out,
-                       int order = ABFT_ORDER_RIGHT) {
+                       int order = ABFT_ORDER_RIGHT, int nchk = 2) {
     out.clear();
     if (!inj) return 0;
     const int64_t N = n / nb;
@@ -87,8 +87,8 @@ static int collect_inj(const abft_inject_spec_t* inj, int64_t n, int64_t nb, std
             if (s.col < 0 || s.row < s.col || s.row >= n) return -1;
             I = s.row / nb; J = s.col / nb;
         } else {
-            if (s.row < 0 || s.row >= 2 * N || s.col < 0 || s.col >= n) return -1;
-            I = s.row / 2; J = s.col / nb;
+            if (s.row < 0 || s.row >= nchk * N || s.col < 0 || s.col >= n) return -1;
+            I = s.row / nchk; J = s.col / nb;
             if (J > I) return -1;
         }
         const int64_t k = s.k;
@@ -111,6 +111,7 @@ namespace abft { bool is_update_kernel(const void* f); }
 // ---- workspace -------------------------------------------------------------------------------
 struct Work {
     int64_t n, nb, N;
+    int nchk = 2;                                 // checksum rows per block (2, or 3: reading B10)
     double* chk = nullptr; int64_t ldc = 1;
     double* scl = nullptr;
     double* W = nullptr;
@@ -121,15 +122,16 @@ struct Work {
     double* cs = nullptr; int64_t cs_nslab = 0;   // fused-V5 partials (nb % 128 == 0)
 };
 
-static int work_alloc(Work& w, int64_t n, int64_t nb, int64_t ncols_local, int64_t ev_cap, bool abft, cudaStream_t s) {
-    w.n = n; w.nb = nb; w.N = n / nb;
+static int work_alloc(Work& w, int64_t n, int64_t nb, int64_t ncols_local, int64_t ev_cap, bool abft, cudaStream_t s,
+                      int nchk = 2) {
+    w.n = n; w.nb = nb; w.N = n / nb; w.nchk = nchk;
     const int64_t N = w.N;
-    w.ldc = std::max<int64_t>(1, 2 * N);
+    w.ldc = std::max<int64_t>(1, nchk * N);
     if (abft) {
         ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.chk, sizeof(double) * (size_t)(w.ldc * std::max<int64_t>(1, ncols_local)), s));
-        ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.scl, sizeof(double) * (size_t)(n + 2 * N + 1), s));
+        ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.scl, sizeof(double) * (size_t)(n + 3 * N + 1), s));
     }
-    const int64_t wrows = (N - 1) * nb + 2 * N + 2;
+    const int64_t wrows = (N - 1) * nb + nchk * N + nchk + 1;
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.W, sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb), s));
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.Li, sizeof(double) * (size_t)(nb * nb), s));
     ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.tmp, sizeof(double) * (size_t)(((nb + 1) / 2 + 64) * ((nb + 1) / 2 + 64)), s));
@@ -160,6 +162,7 @@ static StageArgs stage_base(const Work& w, double* A, int64_t lda, double c_tau,
     a.n = w.n; a.nb = w.nb; a.N = w.N;
     a.A = A; a.lda = lda; a.chk = w.chk; a.ldc = w.ldc; a.W = w.W; a.ldw = 1; a.mB = 0;
     a.s = w.scl; a.S1 = w.scl ? w.scl + w.n : nullptr; a.S2 = w.scl ? w.scl + w.n + w.N : nullptr;
+    a.S3 = w.scl ? w.scl + w.n + 2 * w.N : nullptr; a.nchk = w.nchk;
     a.c_tau = c_tau; a.col_owner_mod = 1; a.col_owner_rank = 0;
     a.st = w.st; a.ev = w.ev; a.ev_cap = w.ev_cap;
     a.flist = 0; a.j_lo = k + 1; a.j_hi = w.N;
@@ -198,7 +201,7 @@ static int finish_report(const Work& w, abft_report_t* rep, cudaStream_t s, int*
 }
 
 // Injection pointer at hook time (where the element lives at that moment).
-struct Loc { double* A; int64_t lda; double* chk; int64_t ldc; double* W; int64_t ldw; int64_t mB; };
+struct Loc { double* A; int64_t lda; double* chk; int64_t ldc; double* W; int64_t ldw; int64_t mB; int nchk = 2; };
 
 static double* inj_ptr(const abft_inject_spec_t& s, int64_t k, int64_t nb, const Loc& L) {
     const int hook = s.hook;
@@ -208,7 +211,7 @@ static double* inj_ptr(const abft_inject_spec_t& s, int64_t k, int64_t nb, const
                 return L.W + (s.col - k * nb) * L.ldw + (s.row - (k + 1) * nb);
             return L.A + s.col * L.lda + s.row;
         }
-        return L.W + (s.col - k * nb) * L.ldw + L.mB + (s.row - 2 * k);
+        return L.W + (s.col - k * nb) * L.ldw + L.mB + (s.row - L.nchk * k);
     }
     if (s.target == ABFT_TGT_DATA) return L.A + s.col * L.lda + s.row;
     return L.chk + s.col * L.ldc + s.row;
@@ -370,24 +373,25 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         ABFT_CUDA_TRY(cudaMemsetAsync(w.tmp, 0, chol_sync_bytes(nb), s));
         rep = nullptr;
     } else {
-        rc = work_alloc(w, n, nb, n, rep ? std::max<int64_t>(rep->cap, 1) : 1024, abft, s);
+        rc = work_alloc(w, n, nb, n, rep ? std::max<int64_t>(rep->cap, 1) : 1024, abft, s, o.nchk == 3 ? 3 : 2);
         if (rc) return rc;
     }
     const int64_t N = w.N, B = nb;
+    const int64_t nc = w.nchk;                                   // checksum rows per block (2 or 3)
     const double Bd = (double)B;
     const int32_t* ab = &w.st->abort;
-    // fused V5 partials: 64-row slabs x n columns x {v1, v2}
+    // fused V5 partials: 64-row slabs x n columns x {v1, v2 (, v3)}
     const int mode = o.mode;
     const bool can_fuse = abft && mode != ABFT_MODE_OFFLINE && (nb % 128 == 0) && (lda % 2 == 0) &&
                           (((uintptr_t)A & 15) == 0) && !getenv("ABFT_NOFUSE") && !(abl & 8);   // dev knob: V5 re-reads
     if (can_fuse && !ps) {
         w.cs_nslab = n / 32;   // room for 32-row slabs (the smallest warp-tile height)
-        ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n), s));
+        ABFT_CUDA_TRY(cudaMallocAsync((void**)&w.cs, sizeof(double) * (size_t)(nc * w.cs_nslab * n), s));
     }
     if (ps && can_fuse && !w.cs) return ABFT_ERR_CUDA;
     // second panel buffer for the look-ahead
     double* Wbuf[2] = {w.W, ps ? ps->W1 : nullptr};
-    const int64_t wrows = (N - 1) * nb + 2 * N + 2;
+    const int64_t wrows = (N - 1) * nb + nc * N + nc + 1;
     if (!ps)
         ABFT_CUDA_TRY(cudaMallocAsync((void**)&Wbuf[1], sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb), s));
     ThreadCache& tc = thread_cache();
@@ -404,7 +408,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     cudaEvent_t t_enc = nullptr;
     if (abft && !(abl & 16)) {
         t_enc = prof.begin(s);
-        launch_scales(n, nb, A, lda, w.scl, s);
+        launch_scales(n, nb, A, lda, w.scl, s, (int)nc);
         StageArgs a = stage_base(w, A, lda, o.c_tau, SK_COLUMN, 0, 0);
         a.encode = 1;
         launch_check(a, s);
@@ -425,10 +429,10 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     // ---- the panel of iteration k, on stream P ----
     auto panel = [&](int64_t k) {
         const int64_t m = N - k - 1, mB = m * B;
-        const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
+        const int64_t ldw = std::max<int64_t>(1, (mB + nc * m + nc + 1) / 2 * 2);   // even: 16-byte columns
         double* W = Wbuf[k & 1];
         double* Akk = A + k * B * lda + k * B;
-        const Loc L{A, lda, w.chk, w.ldc, W, ldw, mB};
+        const Loc L{A, lda, w.chk, w.ldc, W, ldw, mB, (int)nc};
         const double md = (double)m, mBd = (double)mB;
         Work wk = w; wk.W = W;
         if (abft) do_inject_if(inj, k, ABFT_HOOK_REST, B, L, ab, P, k, k + 1, true);   // REST(k) into column k
@@ -462,11 +466,11 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         // TRSM (+ Alg. 2 on the checksum rows of tile (k,k)): one GEMM per row segment
         t = prof.begin(P);
         if (abft && !(abl & 1))
-            launch_trsm_with_chk(mB, B, Akk + B, lda, w.Li, W, ldw, 2 * m + 2, w.chk + k * B * w.ldc + 2 * k, w.ldc,
+            launch_trsm_with_chk(mB, B, Akk + B, lda, w.Li, W, ldw, nc * m + nc, w.chk + k * B * w.ldc + nc * k, w.ldc,
                                  ab, P);
         else
             launch_gemm(mB, B, B, Akk + B, lda, w.Li, B, W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, P);
-        prof.end(t, PH_TRSM, P, (mBd + (abft ? 2 * md + 2 : 0)) * Bd * Bd, 0);
+        prof.end(t, PH_TRSM, P, (mBd + (abft ? (double)nc * (md + 1) : 0)) * Bd * Bd, 0);
         if (abft) {
             do_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, L, ab, P);
             StageArgs a3 = stage_base(wk, A, lda, o.c_tau, SK_DIAG_FACT, ABFT_V3, (int)k);
@@ -497,8 +501,8 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         }
         t = prof.begin(P);
         launch_copy(mB, B, W, ldw, Akk + B, lda, ab, P);                        // L panel
-        if (abft && !(abl & 1)) launch_copy(2 * m + 2, B, W + mB, ldw, w.chk + k * B * w.ldc + 2 * k, w.ldc, ab, P);
-        prof.end(t, PH_WB, P, 0, 16.0 * (mBd + (abft ? 2 * md + 2 : 0)) * Bd);
+        if (abft && !(abl & 1)) launch_copy(nc * m + nc, B, W + mB, ldw, w.chk + k * B * w.ldc + nc * k, w.ldc, ab, P);
+        prof.end(t, PH_WB, P, 0, 16.0 * (mBd + (abft ? (double)nc * (md + 1) : 0)) * Bd);
         cudaEvent_t e = new_event(); cudaEventRecord(e, P);
         return e;
     };
@@ -509,12 +513,12 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     // 2 = the epilogue applied the UPDATE_OUT injections of these columns (reading A21).
     auto update_cols = [&](int64_t k, int64_t jlo, int64_t jhi) -> int {
         const int64_t m = N - k - 1, mB = m * B;
-        const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
+        const int64_t ldw = std::max<int64_t>(1, (mB + nc * m + nc + 1) / 2 * 2);   // even: 16-byte columns
         double* W = Wbuf[k & 1];
-        const int64_t c0 = (jlo - k - 1) * B, nc = (jhi - jlo) * B;   // W row offset of column block jlo
-        const int64_t rows = mB - c0;                                   // data rows from block jlo down
+        const int64_t c0 = (jlo - k - 1) * B, ncols = (jhi - jlo) * B;   // W row offset of column block jlo
+        const int64_t rows = mB - c0;                                     // data rows from block jlo down
         double* C = A + jlo * B * lda + jlo * B;
-        const double r = (double)rows, c = (double)nc;
+        const double r = (double)rows, c = (double)ncols;
         cudaEvent_t t = prof.begin(s);
         // C[rows x nc] -= W[c0:, :] W[c0:c0+nc, :]^T, lower (r >= c)
         EpiInj ei; ei.n = 0;
@@ -523,25 +527,25 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
                 if (ei.n < kMaxEpiInj) {
                     EpiInjOp& e = ei.op[ei.n];
                     e.seg = sp.target == ABFT_TGT_DATA ? 0 : 1;
-                    e.r = sp.target == ABFT_TGT_DATA ? sp.row - jlo * B : sp.row - 2 * jlo;
+                    e.r = sp.target == ABFT_TGT_DATA ? sp.row - jlo * B : sp.row - nc * jlo;
                     e.c = sp.col - jlo * B; e.mask = sp.xor_mask; e.pad = 0;
                 }
                 ei.n++;
             }
-        ColSumOut cso{w.cs, n, w.cs_nslab, jlo * B, jlo * B, B, 64, jlo * B};
+        ColSumOut cso{w.cs, n, w.cs_nslab, jlo * B, jlo * B, B, 64, jlo * B, nc};
         int fused;
         if (abft) {
-            // checksum rows of tiles I >= jlo: chk[2I+t, cols] -= W_chk(I) W[c0:c0+nc]^T, I >= J,
+            // checksum rows of tiles I >= jlo: chk[nc I + t, cols] -= W_chk(I) W[c0:c0+ncols]^T, I >= J,
             // appended to the same launch as a second row segment
-            const int64_t q0 = 2 * (jlo - k - 1);                       // first chk row of tile jlo in W
-            const int64_t nq = (abl & 1) ? 0 : 2 * (N - jlo);
-            fused = launch_update_with_chk(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, nq, W + mB + 2 + q0,
-                                           w.chk + jlo * B * w.ldc + 2 * jlo, w.ldc, B, ab, s,
-                                           can_fuse ? &cso : nullptr, 0, 1, &ei);
+            const int64_t q0 = nc * (jlo - k - 1);                      // first chk row of tile jlo in W
+            const int64_t nq = (abl & 1) ? 0 : nc * (N - jlo);
+            fused = launch_update_with_chk(rows, ncols, B, W + c0, ldw, W + c0, ldw, C, lda, nq, W + mB + nc + q0,
+                                           w.chk + jlo * B * w.ldc + nc * jlo, w.ldc, B, ab, s,
+                                           can_fuse ? &cso : nullptr, 0, 1, &ei, (int)nc);
             const double mm = (double)(N - jlo), jj = (double)(jhi - jlo);
-            prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd + 4.0 * Bd * Bd * (jj * mm - jj * (jj - 1) / 2), 0);
+            prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd + 2.0 * nc * Bd * Bd * (jj * mm - jj * (jj - 1) / 2), 0);
         } else {
-            fused = launch_gemm(rows, nc, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
+            fused = launch_gemm(rows, ncols, B, W + c0, ldw, W + c0, ldw, C, lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
             fused = 0;
             prof.end(t, PH_UPD, s, (c * (c + 1) / 2 + (r - c) * c) * 2.0 * Bd, 0);
         }
@@ -590,8 +594,8 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         }
         const int64_t m = N - k - 1, mB = m * B;
         if (m == 0) break;
-        const int64_t ldw = std::max<int64_t>(1, mB + 2 * m + 2);
-        const Loc L{A, lda, w.chk, w.ldc, Wbuf[k & 1], ldw, mB};
+        const int64_t ldw = std::max<int64_t>(1, (mB + nc * m + nc + 1) / 2 * 2);   // even: 16-byte columns
+        const Loc L{A, lda, w.chk, w.ldc, Wbuf[k & 1], ldw, mB, (int)nc};
         const bool gated = (((k + 1) % K == 0) || k == N - 2) && mode != ABFT_MODE_OFFLINE;
         // (a) block column k+1 first: update, UPDATE_OUT hook, V5 -> hand it to the panel stream
         const int fa = update_cols(k, k + 1, k + 2);
@@ -703,15 +707,16 @@ static int run_graph(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         if (!g.cs || g.dev != dev) ABFT_CUDA_TRY(cudaStreamCreateWithFlags(&g.cs, cudaStreamNonBlocking));
         const int64_t N = n / nb;
         Work& w = g.ps.w;
-        w.n = n; w.nb = nb; w.N = N; w.ldc = std::max<int64_t>(1, 2 * N);
+        const int nchk = o.nchk == 3 ? 3 : 2;
+        w.n = n; w.nb = nb; w.N = N; w.nchk = nchk; w.ldc = std::max<int64_t>(1, nchk * N);
         const bool abft = o.abft_enabled != 0;
-        const int64_t wrows = std::max<int64_t>((N - 1) * nb + 2 * N + 2, 1);
+        const int64_t wrows = std::max<int64_t>((N - 1) * nb + nchk * N + nchk + 1, 1);
         const size_t tmpn = (size_t)(((nb + 1) / 2 + 64) * ((nb + 1) / 2 + 64));
         if (abft) {
             ABFT_CUDA_TRY(cudaMalloc((void**)&w.chk, sizeof(double) * (size_t)(w.ldc * n)));
-            ABFT_CUDA_TRY(cudaMalloc((void**)&w.scl, sizeof(double) * (size_t)(n + 2 * N + 1)));
+            ABFT_CUDA_TRY(cudaMalloc((void**)&w.scl, sizeof(double) * (size_t)(n + 3 * N + 1)));
             w.cs_nslab = n / 32;
-            ABFT_CUDA_TRY(cudaMalloc((void**)&w.cs, sizeof(double) * (size_t)(2 * w.cs_nslab * n)));
+            ABFT_CUDA_TRY(cudaMalloc((void**)&w.cs, sizeof(double) * (size_t)(nchk * w.cs_nslab * n)));
         }
         ABFT_CUDA_TRY(cudaMalloc((void**)&w.W, sizeof(double) * (size_t)(wrows * nb)));
         ABFT_CUDA_TRY(cudaMalloc((void**)&g.ps.W1, sizeof(double) * (size_t)(wrows * nb)));
@@ -775,9 +780,10 @@ static int run_graph(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     g_launches = g.launches;
     int status = 0;
     ABFT_CUDA_TRY(cudaGetLastError());
+    if (!rep) return 0;   // fully asynchronous without a report (abft.h): no stream synchronisation
     const int rc = finish_report(g.ps.w, rep, g.cs, &status);
     if (rc) return rc;
-    if (rep) { float ms = 0; cudaEventElapsedTime(&ms, e0, e1); rep->seconds = ms * 1e-3; }
+    float ms = 0; cudaEventElapsedTime(&ms, e0, e1); rep->seconds = ms * 1e-3;
     return status;
 }
 
@@ -842,8 +848,9 @@ static void dist_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, 
 int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, DistTransport* tp,
              cudaStream_t s, const abft_inject_spec_t* inj_c, abft_report_t* rep, const abft_options_t* opt) {
     abft_options_t o = opt ? *opt : abft_options_t{1, 1, 64.0, 0, 0, ABFT_MODE_ENHANCED, 0};
-    if (o.K < 1 || !(o.c_tau > 0) || o.mode != ABFT_MODE_ENHANCED || o.order != ABFT_ORDER_RIGHT)
-        return -11;   // dist: Enhanced scheme, right-looking order
+    if (o.K < 1 || !(o.c_tau > 0) || o.mode != ABFT_MODE_ENHANCED || o.order != ABFT_ORDER_RIGHT ||
+        (o.nchk != 0 && o.nchk != 2))
+        return -11;   // dist: Enhanced scheme, right-looking order, two checksum rows
     std::vector<abft_inject_spec_t> inj;
     if (collect_inj(inj_c, n, nb, inj)) return -9;
     if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; }
@@ -853,6 +860,12 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     const int64_t N = n / nb, B = nb;
     std::vector<RankState> R(nlocal);
     const int64_t evcap = rep ? std::max<int64_t>(rep->cap, 1) : 1024;
+    // push mode (NEXT-3): a peer-memory transport owns every rank's two receive buffers; the owner's
+    // write-back kernel stores the panel straight into them (launch_panel_out)
+    const int64_t wrows_max = (N - 1) * nb + 2 * N + 2;
+    const bool push = tp && tp->recv_buf(tp->rank, 0) != nullptr &&
+                      tp->recv_capacity() >= (size_t)(std::max<int64_t>(wrows_max, 1) * nb + 1) &&
+                      tp->nranks <= 16 && getenv("ABFT_DIST_PULL") == nullptr;
     for (int i = 0; i < nlocal; ++i) {
         RankState& q = R[i];
         q.r = locals[i].rank; q.A = locals[i].A; q.lda = locals[i].lda;
@@ -862,7 +875,8 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         // W with one extra slot for the owner's abort flag
         cudaFreeAsync(q.w.W, s);
         const int64_t wrows = (N - 1) * nb + 2 * N + 2;
-        ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.w.W, sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb + 1), s));
+        if (push) q.w.W = tp->recv_buf(q.r, 0);
+        else ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.w.W, sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb + 1), s));
         if (abft && nb % 128 == 0 && q.lda % 2 == 0 && ((uintptr_t)q.A & 15) == 0) {
             q.w.cs_nslab = n / 32;
             ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.w.cs, sizeof(double) * (size_t)(2 * q.w.cs_nslab * std::max<int64_t>(q.ncl, 1)), s));
@@ -912,7 +926,8 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     for (auto& q : R) {   // second panel buffer per rank (W of iteration k lives in Wb[k & 1])
         const int64_t wrows = (N - 1) * nb + 2 * N + 2;
         q.Wb[0] = q.w.W;
-        ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.Wb[1], sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb + 1), s));
+        if (push) q.Wb[1] = tp->recv_buf(q.r, 1);
+        else ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.Wb[1], sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb + 1), s));
     }
     {   // Wb[1] allocated on s: the panel stream must see it
         cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(PS, e, 0);
@@ -932,7 +947,7 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     };
     // the panel of iteration k on the owner's panel stream (V1/V2, POTRF + inverse, TRSM with
     // Alg. 2 rows, V3, V4, write-back, abort slot) into Wb[k & 1]
-    auto panel = [&](RankState& q, int64_t k) {
+    auto panel = [&](RankState& q, int64_t k) -> int {
         int64_t m, mB, ldw; geom(k, m, mB, ldw);
         q.w.W = q.Wb[k & 1];
         const size_t wcount = (size_t)(ldw * B);
@@ -963,9 +978,23 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
                 launch_check(a4, PS);                                                // V4
             }
         }
+        if (push && k + 1 < N) {
+            // write-back fused with the broadcast: one pass over W stores the L panel and its
+            // checksum rows locally and the whole packed panel (+ abort slot) into every peer's
+            // receive buffer (peer stores), once every peer released that buffer
+            launch_abort_to_slot(ab, q.w.W + wcount, PS);
+            if (tp->wait_free(k, PS)) return ABFT_ERR_NCCL;
+            std::vector<double*> peers;
+            for (int r = 0; r < P; ++r) if (r != q.r) peers.push_back(tp->recv_buf(r, (int)(k & 1)));
+            launch_panel_out(q.w.W, ldw, mB, abft ? 2 * m + 2 : 0, B, Akk + B, q.lda, ckk + 2 * k, q.w.ldc, peers.data(),
+                             (int)peers.size(), ab, PS);
+            if (tp->post_panel(k, PS)) return ABFT_ERR_NCCL;
+            return 0;
+        }
         launch_copy(mB, B, q.w.W, ldw, Akk + B, q.lda, ab, PS);
         if (abft) launch_copy(2 * m + 2, B, q.w.W + mB, ldw, ckk + 2 * k, q.w.ldc, ab, PS);
         launch_abort_to_slot(ab, q.w.W + wcount, PS);
+        return 0;
     };
     // broadcast of panel k (+ abort slot) from its owner, then every receiver's RECV hook and V4R;
     // afterwards evB[rank] marks "panel k usable on this rank"
@@ -977,7 +1006,9 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         const int owner = (int)(k % P);
         for (int i = 0; i < nlocal; ++i)   // the receive buffer Wb[k & 1] was last read by update k-2
             if (evUprev[i]) cudaStreamWaitEvent(PS, evUprev[i], 0);
-        if (tp) {
+        if (tp && push) {
+            if (R[0].r != owner && tp->wait_panel(owner, k, PS)) return ABFT_ERR_NCCL;   // pushed by the owner
+        } else if (tp) {
             if (tp->bcast(R[0].Wb[k & 1], (wcount + 1) * sizeof(double), owner, PS)) return ABFT_ERR_NCCL;
         } else {
             const RankState* src = nullptr;
@@ -1087,7 +1118,7 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     {   // P streams see those injections before the first panel
         cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(PS, e, 0);
     }
-    for (auto& q : R) if (q.r == 0) panel(q, 0);
+    for (auto& q : R) if (q.r == 0) { const int rcp = panel(q, 0); if (rcp) return rcp; }
     if (N > 1) { int rc2 = bcast(0); if (rc2) return rc2; }
     for (int64_t k = 0; k + 1 < N; ++k) {
         for (int i = 0; i < nlocal; ++i) cudaStreamWaitEvent(s, evB[i], 0);      // panel k usable
@@ -1097,11 +1128,12 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             if (q.r != o1) continue;
             update(q, k, k + 1, k + 2);
             cudaEvent_t ec = new_event(); cudaEventRecord(ec, s); cudaStreamWaitEvent(PS, ec, 0);
-            panel(q, k + 1);
+            { const int rcp = panel(q, k + 1); if (rcp) return rcp; }
         }
         // (b) the rest of update k on every rank (the owner of k+1 included)
         for (auto& q : R) update(q, k, k + 2, N);
         for (int i = 0; i < nlocal; ++i) { evUprev[i] = evU[i]; evU[i] = new_event(); cudaEventRecord(evU[i], s); }
+        if (push && tp->mark_free(k + 1, s)) return ABFT_ERR_NCCL;   // buffer (k & 1) read for the last time
         // (c) REST(k+1) outside block column k+1 (column k+1's share was applied on PS)
         if (abft) for (auto& q : R) rest_inject(q, k + 1, k + 1, k + 2, false, s);
         // (d) broadcast panel k+1 (receivers wait for their update k-1 ... k to release the buffer)
@@ -1114,7 +1146,10 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     {   // main stream waits for the last panel
         cudaEvent_t e = new_event(); cudaEventRecord(e, PS); cudaStreamWaitEvent(s, e, 0);
     }
-    for (auto& q : R) { if (q.Wb[1]) cudaFreeAsync(q.Wb[1], s); q.Wb[1] = nullptr; q.w.W = q.Wb[0]; }
+    for (auto& q : R) {
+        if (q.Wb[1] && !push) cudaFreeAsync(q.Wb[1], s);
+        q.Wb[1] = nullptr; q.w.W = push ? nullptr : q.Wb[0];   // push mode: the transport owns them
+    }
     if (abft) {
         for (auto& q : R) {
             dist_inject(inj, N, ABFT_HOOK_REST, B, P, q, 1, 0, s);
@@ -1373,8 +1408,10 @@ extern "C" int abft_potrf_ex(int64_t n, int64_t nb, double* A, int64_t lda, abft
     if (rc) return rc;
     abft_options_t o = opt ? *opt : default_options();
     if (o.K < 1 || !(o.c_tau > 0)) return -8;
+    if (o.nchk != 0 && o.nchk != 2 && o.nchk != 3) return -8;
+    if (o.nchk == 3 && o.order != ABFT_ORDER_RIGHT) return -8;   // NEXT-4: right-looking driver
     std::vector<abft_inject_spec_t> list;
-    if (collect_inj(inj, n, nb, list, o.order)) return -6;
+    if (collect_inj(inj, n, nb, list, o.order, o.nchk == 3 ? 3 : 2)) return -6;
     if (o.mode < ABFT_MODE_ENHANCED || o.mode > ABFT_MODE_ENHANCED_REDO) return -8;
     const bool redo = o.mode == ABFT_MODE_ENHANCED_REDO;   // NEXT-4: Enhanced + re-do on UNCORRECTABLE
     if (redo) o.mode = ABFT_MODE_ENHANCED;
@@ -1451,8 +1488,16 @@ extern "C" int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t ld
     const abft_options_t o = opt ? *opt : default_options();
     bool has_inj = false;
     for (const abft_inject_spec_t* q = inj; q && q->k >= 0; ++q) has_inj = true;
-    const bool overlap = !has_inj && o.order == ABFT_ORDER_RIGHT && (o.mode == ABFT_MODE_ENHANCED || !o.abft_enabled) &&
-                         !graph_mode_enabled(n) && getenv("ABFT_HOST_OVERLAP") == nullptr;
+    // the overlapped write-back needs page-locked host memory: a copy from pageable memory is
+    // synchronous to the host and would serialise the enqueue loop behind each block column
+    cudaPointerAttributes pa;
+    memset(&pa, 0, sizeof pa);
+    const bool pinned = cudaPointerGetAttributes(&pa, A_host) == cudaSuccess &&
+                        (pa.type == cudaMemoryTypeHost || pa.type == cudaMemoryTypeManaged);
+    cudaGetLastError();
+    const bool overlap = pinned && !has_inj && o.order == ABFT_ORDER_RIGHT &&
+                         (o.mode == ABFT_MODE_ENHANCED || !o.abft_enabled) && !graph_mode_enabled(n) &&
+                         getenv("ABFT_HOST_OVERLAP") == nullptr;
     if (overlap) {
         // only what the factorisation reads goes over PCIe: each block column from its diagonal
         // block down (the strict upper triangle outside the diagonal blocks is never read)

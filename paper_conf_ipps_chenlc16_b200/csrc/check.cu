@@ -33,26 +33,29 @@ __device__ __forceinline__ void note_ratio(DevState* st, double q) {
 // Compare a recalculated column with its stored checksums, flag it if |d| > tau or d is
 // non-finite (P:195 + A5). Called by every thread of the CTA (inactive threads pass ok = false).
 __device__ __forceinline__ void compare_column(const StageArgs& a, int part, const TileView& v, int64_t I, int64_t J,
-                                               int64_t c, double r1, double r2, bool ok) {
+                                               int64_t c, double r1, double r2, double r3, bool ok) {
     double q = 0.0;
     if (ok) {
         const double d1 = __dsub_rn(r1, v.c1[c * v.ldc]);
         const double d2 = __dsub_rn(r2, v.c2[c * v.ldc]);
-        double tau1, tau2;
-        thresholds(a, I, J * a.nb + c, v.factored, tau1, tau2);
+        const double d3 = v.c3 ? __dsub_rn(r3, v.c3[c * v.ldc]) : 0.0;
+        double tau1, tau2, tau3;
+        thresholds(a, I, J * a.nb + c, v.factored, tau1, tau2, tau3);
         const bool f1 = !dfinite(d1) || fabs(d1) > tau1;
         const bool f2 = !dfinite(d2) || fabs(d2) > tau2;
-        if (f1 || f2) {
+        const bool f3 = v.c3 && (!dfinite(d3) || fabs(d3) > tau3);
+        if (f1 || f2 || f3) {
             FlagList& FL = a.st->fl[a.flist];
             const int slot = atomicAdd(&FL.nflag, 1);
             if (slot >= kFlagCap) FL.overflow = 1;
             else {
                 Flag& f = FL.flags[slot];
                 f.I = (int32_t)I; f.J = (int32_t)J; f.c = (int32_t)c; f.part = part;
-                f.d1 = d1; f.d2 = d2; f.r1 = r1; f.r2 = r2;
+                f.d1 = d1; f.d2 = d2; f.r1 = r1; f.r2 = r2; f.d3 = d3; f.r3 = r3;
             }
         } else {
             q = fmax(fabs(d1) / tau1, fabs(d2) / tau2);
+            if (v.c3) q = fmax(q, fabs(d3) / tau3);
         }
     }
     note_ratio(a.st, q);
@@ -72,56 +75,66 @@ __device__ void phase1_reread(const StageArgs& a, int part, int64_t bid) {
     const bool mine = (J % a.col_owner_mod == a.col_owner_rank);   // dist: this rank's column
     const TileView v = stage_view(a, I, J);
     const int cw = (int)((B - c0) < kChkCols ? (B - c0) : kChkCols);
-    __shared__ double s_r1[kChkCols], s_r2[kChkCols];
-    __shared__ double s_m1[kChkThreads], s_m2[kChkThreads];
+    __shared__ double s_r1[kChkCols], s_r2[kChkCols], s_r3[kChkCols];
+    __shared__ double s_m1[kChkThreads], s_m2[kChkThreads], s_m3[kChkThreads];
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (mine) {
         for (int cc = warp; cc < cw; cc += kChkThreads / 32) {
             const int64_t c = c0 + cc;
             const double* col = v.T + c * v.ldt;
             const int64_t rbeg = v.diag ? c : 0;
-            double r1 = 0.0, r2 = 0.0;
+            double r1 = 0.0, r2 = 0.0, r3 = 0.0;
             if (!v.diag && ((((uintptr_t)col) & 15) == 0) && (B % 2 == 0)) {
                 const double2* col2 = reinterpret_cast<const double2*>(col);
 #pragma unroll 4
                 for (int64_t h = lane; h < B / 2; h += 32) {
                     const double2 x = col2[h];
+                    const double w0 = (double)(2 * h + 1), w1 = (double)(2 * h + 2);
                     r1 += x.x; r1 += x.y;
-                    r2 = fma((double)(2 * h + 1), x.x, r2);
-                    r2 = fma((double)(2 * h + 2), x.y, r2);
+                    r2 = fma(w0, x.x, r2);
+                    r2 = fma(w1, x.y, r2);
+                    if (v.c3) { r3 = fma(w0 * w0, x.x, r3); r3 = fma(w1 * w1, x.y, r3); }
                 }
             } else {
 #pragma unroll 4
                 for (int64_t r = rbeg + lane; r < B; r += 32) {
                     const double x = col[r];
+                    const double w = (double)(r + 1);
                     r1 += x;
-                    r2 = fma((double)(r + 1), x, r2);
+                    r2 = fma(w, x, r2);
+                    if (v.c3) r3 = fma(w * w, x, r3);
                 }
             }
             r1 = warp_sum(r1);
             r2 = warp_sum(r2);
-            if (lane == 0) { s_r1[cc] = r1; s_r2[cc] = r2; }
+            if (v.c3) r3 = warp_sum(r3);
+            if (lane == 0) { s_r1[cc] = r1; s_r2[cc] = r2; s_r3[cc] = r3; }
         }
     }
     // mirrored part of an unfactored diagonal tile: X[r,c] = T[c,r] for r < c (row c of T)
     if (mine && v.diag && !v.factored) {
         const int ngroups = kChkThreads / kChkCols;
         const int cc = threadIdx.x % kChkCols, grp = threadIdx.x / kChkCols;
-        double m1 = 0.0, m2 = 0.0;
+        double m1 = 0.0, m2 = 0.0, m3 = 0.0;
         if (cc < cw) {
             const int64_t c = c0 + cc;
             for (int64_t r = grp; r < c; r += ngroups) {
                 const double x = v.T[r * v.ldt + c];
+                const double w = (double)(r + 1);
                 m1 += x;
-                m2 = fma((double)(r + 1), x, m2);
+                m2 = fma(w, x, m2);
+                if (v.c3) m3 = fma(w * w, x, m3);
             }
         }
-        s_m1[threadIdx.x] = m1; s_m2[threadIdx.x] = m2;
+        s_m1[threadIdx.x] = m1; s_m2[threadIdx.x] = m2; s_m3[threadIdx.x] = m3;
         __syncthreads();
         if (threadIdx.x < cw) {
-            double a1 = 0.0, a2 = 0.0;
-            for (int g = 0; g < ngroups; ++g) { a1 += s_m1[g * kChkCols + threadIdx.x]; a2 += s_m2[g * kChkCols + threadIdx.x]; }
-            s_r1[threadIdx.x] += a1; s_r2[threadIdx.x] += a2;
+            double a1 = 0.0, a2 = 0.0, a3 = 0.0;
+            for (int g = 0; g < ngroups; ++g) {
+                a1 += s_m1[g * kChkCols + threadIdx.x]; a2 += s_m2[g * kChkCols + threadIdx.x];
+                a3 += s_m3[g * kChkCols + threadIdx.x];
+            }
+            s_r1[threadIdx.x] += a1; s_r2[threadIdx.x] += a2; s_r3[threadIdx.x] += a3;
         }
     }
     __syncthreads();
@@ -130,8 +143,12 @@ __device__ void phase1_reread(const StageArgs& a, int part, int64_t bid) {
     const bool act = threadIdx.x < cw;
     const int64_t c = c0 + threadIdx.x;
     const double r1 = act ? s_r1[threadIdx.x] : 0.0, r2 = act ? s_r2[threadIdx.x] : 0.0;
-    if (a.encode) { if (act) { v.c1[c * v.ldc] = r1; v.c2[c * v.ldc] = r2; } return; }
-    compare_column(a, part, v, I, J, c, r1, r2, act);
+    const double r3 = act ? s_r3[threadIdx.x] : 0.0;
+    if (a.encode) {
+        if (act) { v.c1[c * v.ldc] = r1; v.c2[c * v.ldc] = r2; if (v.c3) v.c3[c * v.ldc] = r3; }
+        return;
+    }
+    compare_column(a, part, v, I, J, c, r1, r2, r3, act);
 }
 
 // Phase 1 of V5 for off-diagonal trailing tiles from the partial sums the update GEMM left
@@ -147,15 +164,16 @@ __device__ void phase1_fused(const StageArgs& a, int part, int64_t bid) {
     if (threadIdx.x == 0 && c == 0) atomicAdd(&a.st->n_checks, 1ull);
     const bool act = c < B;
     const TileView v = stage_view(a, I, J);
-    double r1 = 0.0, r2 = 0.0;
+    double r1 = 0.0, r2 = 0.0, r3 = 0.0;
     if (act) {
         const int64_t g = local_col(a, J) + c, s0 = I * B / a.cs_slab_rows, ns = B / a.cs_slab_rows;
         for (int64_t q = 0; q < ns; ++q) {
             r1 += a.cs[(s0 + q) * a.cs_ld + g];
             r2 += a.cs[(a.cs_nslab + s0 + q) * a.cs_ld + g];
+            if (v.c3) r3 += a.cs[(2 * a.cs_nslab + s0 + q) * a.cs_ld + g];
         }
     }
-    compare_column(a, part, v, I, J, c, r1, r2, act);
+    compare_column(a, part, v, I, J, c, r1, r2, r3, act);
 }
 
 // Block-wide reductions used by phase 2.
@@ -193,10 +211,6 @@ __device__ int64_t block_argmax(const TileView& v, int64_t c, int64_t B, double*
     return r;
 }
 
-struct Fix { double* p; double* p2; double val; };
-// corrections held per tile: one per column at most (a tile has nb columns); beyond this the tile
-// is reported UNCORRECTABLE
-constexpr int kMaxFix = 1024;
 
 // Flags were written by other CTAs of this launch: read them from L2 (they are never in this
 // SM's L1 for a reason this CTA could vouch for).
@@ -206,7 +220,44 @@ __device__ __forceinline__ Flag load_flag(const Flag* p) {
     const int2 h1 = __ldcg(reinterpret_cast<const int2*>(p) + 1);
     f.I = h0.x; f.J = h0.y; f.c = h1.x; f.part = h1.y;
     f.d1 = __ldcg(&p->d1); f.d2 = __ldcg(&p->d2); f.r1 = __ldcg(&p->r1); f.r2 = __ldcg(&p->r2);
+    f.d3 = __ldcg(&p->d3); f.r3 = __ldcg(&p->r3);
     return f;
+}
+
+// Two errors in one column from three weighted sums (nchk = 3, reading B10): with
+// Da at weight wa and Db at weight wb, d3 = S d2 - P d1 (S = wa + wb, P = wa wb). Scan S ascending,
+// P = rint((S d2 - d3) / d1); accept integer roots 1 <= wa < wb <= B whose residual is within its
+// rounding tolerance and whose two errors both exceed tau1; exactly one accepted pair locates them.
+// Every operation is an explicit round-to-nearest one, in the oracle's order.
+__device__ bool locate_two(double d1, double d2, double d3, double tau1, double tau2, double tau3, int64_t B,
+                           int64_t& ra, int64_t& rb) {
+    int found = 0;
+    if (!(fabs(d1) > tau1)) return false;
+    for (int64_t S = 3; S <= 2 * B - 1; ++S) {
+        const double Sd = (double)S;
+        const double Pd = rint(__ddiv_rn(__dsub_rn(__dmul_rn(Sd, d2), d3), d1));
+        if (!(Pd >= 2.0) || Pd > __dmul_rn((double)B, (double)(B - 1))) continue;
+        const int64_t P = (int64_t)Pd;
+        const int64_t disc = S * S - 4 * P;
+        if (disc <= 0) continue;
+        int64_t q = (int64_t)sqrt((double)disc);
+        while (q * q > disc) --q;
+        while ((q + 1) * (q + 1) <= disc) ++q;
+        if (q * q != disc || ((S - q) & 1)) continue;
+        const int64_t wa = (S - q) / 2, wb = (S + q) / 2;
+        if (wa < 1 || wb > B) continue;
+        const double res = __dadd_rn(__dsub_rn(d3, __dmul_rn(Sd, d2)), __dmul_rn(Pd, d1));
+        const double tol = __dadd_rn(__dadd_rn(__dadd_rn(tau3, __dmul_rn(Sd, tau2)), __dmul_rn(Pd, tau1)),
+                                     __dmul_rn(ABFT_RHO, __dadd_rn(__dadd_rn(fabs(d3), __dmul_rn(Sd, fabs(d2))),
+                                                                   __dmul_rn(Pd, fabs(d1)))));
+        if (!(fabs(res) <= tol)) continue;
+        const double wad = (double)wa, wbd = (double)wb, den = (double)(wb - wa);
+        const double Da = __ddiv_rn(__dsub_rn(__dmul_rn(wbd, d1), d2), den);
+        const double Db = __ddiv_rn(__dsub_rn(d2, __dmul_rn(wad, d1)), den);
+        if (!(fabs(Da) > tau1) || !(fabs(Db) > tau1)) continue;
+        if (++found == 1) { ra = wa - 1; rb = wb - 1; }
+    }
+    return found == 1;
 }
 
 // Phase 2: resolve the flagged columns in the oracle's order (tile, then column): decide
@@ -217,11 +268,12 @@ __device__ void phase2_body(const StageArgs& a0, const StageArgs& a1, int flist)
     DevState* st = a0.st;
     FlagList& FL = st->fl[flist];
     __shared__ int s_n;
-    __shared__ Fix s_fix[kMaxFix];
+    Fix* s_fix = FL.fix;   // global (block-visible after each __syncthreads)
     __shared__ int s_nfix, s_unc, s_stop;
     __shared__ double redv[kChkThreads];
     __shared__ long long redi[kChkThreads];
     __shared__ Flag s_flag;
+    __shared__ long long s_rows[2];
     if (threadIdx.x == 0) {
         s_n = min(__ldcg(&FL.nflag), kFlagCap);
         if (__ldcg(&st->abort)) s_n = 0;
@@ -264,29 +316,82 @@ __device__ void phase2_body(const StageArgs& a0, const StageArgs& a1, int flist)
         for (int e = i0; e < i1; ++e) {
             const Flag f = FL.flags[e];
             const int64_t c = f.c;
-            double tau1, tau2;
-            thresholds(a, f.I, (int64_t)f.J * B + c, v.factored, tau1, tau2);
+            double tau1, tau2, tau3;
+            thresholds(a, f.I, (int64_t)f.J * B + c, v.factored, tau1, tau2, tau3);
+            const bool has3 = v.c3 != nullptr;
             const bool f1 = !dfinite(f.d1) || fabs(f.d1) > tau1;
             const bool f2 = !dfinite(f.d2) || fabs(f.d2) > tau2;
-            int kind; int64_t row = -1;
-            if (!dfinite(f.d1) || !dfinite(f.d2)) {
+            const bool f3 = has3 && (!dfinite(f.d3) || fabs(f.d3) > tau3);
+            int kind = ABFT_KIND_UNCORRECTABLE; int64_t row = -1, row2 = -1;
+            if (!dfinite(f.d1) || !dfinite(f.d2) || !dfinite(f.d3)) {
                 kind = ABFT_KIND_NONFINITE;
                 row = block_argmax(v, c, B, redv, redi);
-            } else if (f1) {
-                const double q = __ddiv_rn(f.d2, f.d1);
-                const double j = rint(q);                       // half-to-even
-                kind = f2 ? ABFT_KIND_UNCORRECTABLE : ABFT_KIND_CHK1;
-                if (j >= 1.0 && j <= (double)B) {
-                    const double jd1 = __dmul_rn(j, f.d1);
-                    if (fabs(__dsub_rn(f.d2, jd1)) <= __dadd_rn(tau2, __dmul_rn(ABFT_RHO, fabs(jd1)))) {
-                        kind = ABFT_KIND_DATA; row = (int64_t)j - 1;
+            } else {
+                bool done = false;
+                if (f1) {
+                    const double q = __ddiv_rn(f.d2, f.d1);
+                    const double j = rint(q);                       // half-to-even
+                    if (j >= 1.0 && j <= (double)B) {
+                        const double jd1 = __dmul_rn(j, f.d1);
+                        const double j2d1 = __dmul_rn(__dmul_rn(j, j), f.d1);
+                        if (fabs(__dsub_rn(f.d2, jd1)) <= __dadd_rn(tau2, __dmul_rn(ABFT_RHO, fabs(jd1))) &&
+                            (!has3 || fabs(__dsub_rn(f.d3, j2d1)) <= __dadd_rn(tau3, __dmul_rn(ABFT_RHO, fabs(j2d1))))) {
+                            kind = ABFT_KIND_DATA; row = (int64_t)j - 1; done = true;
+                        }
                     }
                 }
-            } else {
-                kind = ABFT_KIND_CHK2;
+                if (!done && (int)f1 + (int)f2 + (int)f3 == 1) {   // one checksum row corrupted (A10)
+                    kind = f1 ? ABFT_KIND_CHK1 : f2 ? ABFT_KIND_CHK2 : ABFT_KIND_CHK3;
+                    done = true;
+                }
+                if (!done && has3) {                                 // two data errors (B10)
+                    if (threadIdx.x == 0) {
+                        int64_t ra = -1, rb = -1;
+                        if (!locate_two(f.d1, f.d2, f.d3, tau1, tau2, tau3, B, ra, rb)) ra = rb = -1;
+                        s_rows[0] = ra; s_rows[1] = rb;
+                    }
+                    __syncthreads();
+                    if (s_rows[0] >= 0) { kind = ABFT_KIND_DATA; row = s_rows[0]; row2 = s_rows[1]; }
+                    __syncthreads();
+                }
             }
             const int vcode = ((a.kind == SK_COLUMN || a.kind == SK_COL_DIAG) && f.I == a.k) ? ABFT_V1 : a.V;
-            if (kind == ABFT_KIND_DATA || kind == ABFT_KIND_NONFINITE) {
+            if (kind == ABFT_KIND_DATA && row2 >= 0) {
+                // two errors (B10): x_a, x_b from chk1, chk2 and the other B-2 entries summed
+                // directly (A8): R1 = x_a + x_b, R2 = wa x_a + wb x_b
+                double p1 = 0.0, p2 = 0.0;
+                for (int64_t r = threadIdx.x; r < B; r += blockDim.x)
+                    if (r != row && r != row2) { const double x = view_x(v, r, c); p1 += x; p2 = fma((double)(r + 1), x, p2); }
+                const double s1 = block_sum(p1, redv);
+                const double s2 = block_sum(p2, redv);
+                if (threadIdx.x == 0) {
+                    const double wa = (double)(row + 1), wb = (double)(row2 + 1);
+                    const double R1 = __dsub_rn(v.c1[c * v.ldc], s1), R2 = __dsub_rn(v.c2[c * v.ldc], s2);
+                    const double xa = __ddiv_rn(__dsub_rn(__dmul_rn(wb, R1), R2), __dsub_rn(wb, wa));
+                    const double xb = __ddiv_rn(__dsub_rn(R2, __dmul_rn(wa, R1)), __dsub_rn(wb, wa));
+                    const int64_t rows[2] = {row, row2};
+                    const double vals[2] = {xa, xb};
+                    for (int h = 0; h < 2; ++h) {
+                        double* p = view_store(v, rows[h], c);
+                        bool dup = false;
+                        for (int u = 0; u < s_nfix; ++u) dup |= (s_fix[u].p == p);
+                        if (dup) continue;
+                        if (s_nfix < kMaxFix) { s_fix[s_nfix].p = p; s_fix[s_nfix].p2 = nullptr; s_fix[s_nfix].val = vals[h]; s_nfix++; }
+                        else s_unc = 1;
+                        int64_t sr = rows[h], sc = c;
+                        if (v.diag && !v.factored && sr < sc) { const int64_t t = sr; sr = sc; sc = t; }
+                        const long long ev_i = (long long)atomicAdd(&st->nev, 1ull);
+                        if (ev_i < a.ev_cap) {
+                            abft_event_t& ev = a.ev[ev_i];
+                            ev.k = a.k; ev.check = vcode; ev.tile_i = f.I; ev.tile_j = f.J;
+                            ev.row = (int32_t)sr; ev.col = (int32_t)sc; ev.kind = ABFT_KIND_DATA; ev.rank = a.rank;
+                            ev.delta1 = f.d1; ev.delta2 = f.d2;
+                        }
+                        st->n_detected++; st->n_data++;
+                    }
+                }
+                __syncthreads();
+            } else if (kind == ABFT_KIND_DATA || kind == ABFT_KIND_NONFINITE) {
                 double* p = view_store(v, row, c);
                 bool dup = false;
                 for (int u = 0; u < s_nfix; ++u) dup |= (s_fix[u].p == p);
@@ -319,17 +424,18 @@ __device__ void phase2_body(const StageArgs& a0, const StageArgs& a1, int flist)
                     abft_event_t& ev = a.ev[ev_i];
                     ev.k = a.k; ev.check = vcode;
                     ev.tile_i = f.I; ev.tile_j = f.J;
-                    ev.row = kind == ABFT_KIND_CHK1 ? -1 : kind == ABFT_KIND_CHK2 ? -2 : -3;
+                    ev.row = kind == ABFT_KIND_CHK1 ? -1 : kind == ABFT_KIND_CHK2 ? -2 : kind == ABFT_KIND_CHK3 ? -4 : -3;
                     ev.col = (int32_t)c; ev.kind = kind; ev.rank = a.rank;
                     ev.delta1 = f.d1; ev.delta2 = f.d2;
                 }
                 st->n_detected++;
-                if (kind == ABFT_KIND_CHK1 || kind == ABFT_KIND_CHK2) {
+                if (kind == ABFT_KIND_CHK1 || kind == ABFT_KIND_CHK2 || kind == ABFT_KIND_CHK3) {
                     if (kind == ABFT_KIND_CHK1) st->n_chk1++; else st->n_chk2++;
                     if (s_nfix < kMaxFix) {
-                        s_fix[s_nfix].p = kind == ABFT_KIND_CHK1 ? &v.c1[c * v.ldc] : &v.c2[c * v.ldc];
+                        s_fix[s_nfix].p = kind == ABFT_KIND_CHK1 ? &v.c1[c * v.ldc]
+                                          : kind == ABFT_KIND_CHK2 ? &v.c2[c * v.ldc] : &v.c3[c * v.ldc];
                         s_fix[s_nfix].p2 = nullptr;
-                        s_fix[s_nfix].val = kind == ABFT_KIND_CHK1 ? f.r1 : f.r2;   // chk := v^T X
+                        s_fix[s_nfix].val = kind == ABFT_KIND_CHK1 ? f.r1 : kind == ABFT_KIND_CHK2 ? f.r2 : f.r3;   // chk := v^T X
                         s_nfix++;
                     } else s_unc = 1;
                 } else {
@@ -356,7 +462,8 @@ __device__ void phase2_body(const StageArgs& a0, const StageArgs& a1, int flist)
 // the tiles), then the last CTA to finish resolves the flags of both parts (phase 2) in the
 // oracle's order. Every CTA reaches the completion counter (also when the run is aborted), and
 // the last one resets it, so the counter is zero again for the next launch on this flag list.
-__global__ void __launch_bounds__(kChkThreads) k_check(StageArgs a0, StageArgs a1, int64_t nblk0) {
+// min 4 CTAs/SM: phase 1 is the hot part (bandwidth-bound); the rare phase 2 may spill instead
+__global__ void __launch_bounds__(kChkThreads, 4) k_check(StageArgs a0, StageArgs a1, int64_t nblk0) {
     __shared__ int s_last;
     const bool aborted = cta_aborted(&a0.st->abort);
     if (!aborted) {
@@ -384,15 +491,17 @@ __global__ void k_scales_diag(int64_t n, const double* A, int64_t lda, double* s
     const int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (i < n) s[i] = __dsqrt_rn(A[i * lda + i]);
 }
-__global__ void k_scales_block(int64_t N, int64_t B, const double* s, double* S1, double* S2) {
+__global__ void k_scales_block(int64_t N, int64_t B, const double* s, double* S1, double* S2, double* S3) {
     const int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     if (I >= N) return;
-    double a = 0.0, b = 0.0;
+    double a = 0.0, b = 0.0, c = 0.0;
     for (int64_t r = 0; r < B; ++r) {
         a = __dadd_rn(a, s[I * B + r]);
         b = __dadd_rn(b, __dmul_rn((double)(r + 1), s[I * B + r]));
+        c = __dadd_rn(c, __dmul_rn((double)((r + 1) * (r + 1)), s[I * B + r]));   // S3 (nchk = 3, B10)
     }
     S1[I] = a; S2[I] = b;
+    if (S3) S3[I] = c;
 }
 
 }  // namespace abft
@@ -440,16 +549,17 @@ int launch_scales_diag(int64_t nrows, const double* Adiag, int64_t lda, double* 
 }
 int launch_scales_blocks(int64_t N, int64_t nb, const double* sv, double* S1, double* S2, cudaStream_t s) {
     if (N <= 0) return 0;
-    k_scales_block<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(N, nb, sv, S1, S2);
+    k_scales_block<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(N, nb, sv, S1, S2, nullptr);
     abft_count_launch();
     return 0;
 }
 
-int launch_scales(int64_t n, int64_t nb, const double* A, int64_t lda, double* scl, cudaStream_t s) {
+int launch_scales(int64_t n, int64_t nb, const double* A, int64_t lda, double* scl, cudaStream_t s, int nchk) {
     const int64_t N = n / nb;
     if (n == 0) return 0;
     k_scales_diag<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(n, A, lda, scl);
-    k_scales_block<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(N, nb, scl, scl + n, scl + n + N);
+    k_scales_block<<<(unsigned)((N + 127) / 128), 128, 0, s>>>(N, nb, scl, scl + n, scl + n + N,
+                                                               nchk == 3 ? scl + n + 2 * N : nullptr);
     abft_count_launch(2);
     return 0;
 }

@@ -13,15 +13,22 @@ namespace abft {
 // A flagged column produced by a check's recalculation pass (phase 1), resolved by phase 2.
 struct Flag {
     int32_t I, J, c, part;   // part: which StageArgs of a two-part check launch raised it
-    double d1, d2, r1, r2;
+    double d1, d2, r1, r2, d3, r3;   // d3, r3: third checksum (nchk = 3), else 0
 };
 
 constexpr int kFlagCap = 8192;
+constexpr int kMaxFix = 1024;   // corrections held per tile by phase 2 (beyond: UNCORRECTABLE)
 
-// Flagged columns pending resolution (phase 1 -> phase 2). One list per concurrent stream.
+// A correction decided by phase 2: the stored element (or checksum) and its new value.
+struct Fix { double* p; double* p2; double val; };
+
+// Flagged columns pending resolution (phase 1 -> phase 2), and phase 2's per-tile correction list
+// (in global memory, so that the check kernel keeps a small shared-memory footprint and can sit
+// next to two update CTAs on an SM). One list per concurrent stream.
 struct FlagList {
     int32_t nflag, overflow;
     Flag flags[kFlagCap];
+    Fix fix[kMaxFix];
 };
 
 // Device-resident run state. One per abft_* call.
@@ -62,6 +69,8 @@ struct StageArgs {
     double* W; int64_t ldw;         // packed panel buffer (SK_DIAG_FACT, SK_PANEL)
     int64_t mB;                     // rows of data in W (m * nb)
     const double* s; const double* S1; const double* S2;  // threshold scales
+    const double* S3;               // (nchk = 3) sum of (i+1)^2 s_i over block I
+    int32_t nchk, pad3;             // checksum rows per block: 2 or 3 (reading B10)
     double c_tau;
     int32_t col_owner_mod, col_owner_rank;  // dist: local column mapping (1, 0 on one GPU)
     int32_t flist, pad2;            // flag list used by this stage (one per stream)
@@ -75,6 +84,7 @@ struct StageArgs {
 struct TileView {
     double* T; int64_t ldt;
     double* c1; double* c2; int64_t ldc;
+    double* c3;                     // third checksum row (nchk = 3) or nullptr
     bool diag, factored;
 };
 
@@ -133,7 +143,7 @@ __device__ __forceinline__ int64_t local_col(const StageArgs& a, int64_t J) {
 
 __device__ __forceinline__ TileView stage_view(const StageArgs& a, int64_t I, int64_t J) {
     TileView v;
-    const int64_t B = a.nb;
+    const int64_t B = a.nb, nc = a.nchk;
     v.diag = (I == J);
     switch (a.kind) {
         case SK_DIAG_FACT:
@@ -142,7 +152,7 @@ __device__ __forceinline__ TileView stage_view(const StageArgs& a, int64_t I, in
             v.factored = true; break;
         case SK_PANEL:
             v.T = a.W + (I - a.k - 1) * B; v.ldt = a.ldw;
-            v.c1 = a.W + a.mB + 2 + 2 * (I - a.k - 1); v.c2 = v.c1 + 1; v.ldc = a.ldw;
+            v.c1 = a.W + a.mB + nc + nc * (I - a.k - 1); v.c2 = v.c1 + 1; v.ldc = a.ldw;
             v.diag = false; v.factored = true; break;
         case SK_COLUMN:
         case SK_COL_DIAG:
@@ -151,13 +161,14 @@ __device__ __forceinline__ TileView stage_view(const StageArgs& a, int64_t I, in
         case SK_TRAIL_OFF:
         case SK_TRAIL_DIAG:
             v.T = a.A + local_col(a, J) * a.lda + I * B; v.ldt = a.lda;
-            v.c1 = a.chk + local_col(a, J) * a.ldc + 2 * I; v.c2 = v.c1 + 1; v.ldc = a.ldc;
+            v.c1 = a.chk + local_col(a, J) * a.ldc + nc * I; v.c2 = v.c1 + 1; v.ldc = a.ldc;
             v.factored = false; break;
         default:
             v.T = a.A + local_col(a, J) * a.lda + I * B; v.ldt = a.lda;
-            v.c1 = a.chk + local_col(a, J) * a.ldc + 2 * I; v.c2 = v.c1 + 1; v.ldc = a.ldc;
+            v.c1 = a.chk + local_col(a, J) * a.ldc + nc * I; v.c2 = v.c1 + 1; v.ldc = a.ldc;
             v.factored = a.factored != 0; break;
     }
+    v.c3 = nc == 3 ? v.c1 + 2 : nullptr;
     return v;
 }
 
@@ -177,11 +188,12 @@ __device__ __forceinline__ double* view_store(const TileView& v, int64_t r, int6
 // Thresholds of reading A4, evaluated with explicit round-to-nearest ops (no FMA contraction)
 // so that a decision depends only on (d1, d2) and the scales.
 __device__ __forceinline__ void thresholds(const StageArgs& a, int64_t I, int64_t g, bool factored,
-                                           double& tau1, double& tau2) {
+                                           double& tau1, double& tau2, double& tau3) {
     const double base = a.c_tau * ABFT_EPS;  // exact: power-of-two scaling
     const double sc = factored ? 1.0 : a.s[g];
     tau1 = __dmul_rn(__dmul_rn(base, a.S1[I]), sc);
     tau2 = __dmul_rn(__dmul_rn(base, a.S2[I]), sc);
+    tau3 = a.nchk == 3 ? __dmul_rn(__dmul_rn(base, a.S3[I]), sc) : 0.0;
 }
 
 __device__ __forceinline__ bool dfinite(double x) { return isfinite(x); }
@@ -212,11 +224,12 @@ __device__ __forceinline__ void dmma(double& c0, double& c1, double a, double b)
 // weights = (row index inside its nb-block) + 1.
 namespace abft {
 struct ColSumOut {
-    double* p; int64_t ld, nslab;
+    double* p; int64_t ld, nslab;   // rows [0, nslab) v1, [nslab, 2 nslab) v2, [2 nslab, 3 nslab) v3
     int64_t row0, col0;   // global row of C's row 0; partial-array column of C's column 0
     int64_t nb;
     int64_t slab_rows;    // rows per slab (set by the GEMM launcher: its warp-tile height)
     int64_t colg0;        // GLOBAL column of C's column 0 (block-diagonal test; = col0 on one GPU)
+    int64_t nchk;         // 3: also the v3 partials (weights (row in block + 1)^2)
 };
 }  // namespace abft
 
@@ -247,7 +260,21 @@ struct DistTransport {
     virtual int allreduce_sum(double* buf, size_t count, cudaStream_t s) = 0;
     virtual int allreduce_max(double* buf, size_t count, cudaStream_t s) = 0;
     virtual int allgather(const void* send, void* recv, size_t bytes, cudaStream_t s) = 0;
+    // Push mode (peer-memory transports, NEXT-3): the transport owns every rank's two panel
+    // receive buffers, mapped into every rank, so the owner's write-back kernel stores the panel
+    // straight into its peers' buffers (no separate broadcast pass). nullptr: not supported.
+    virtual double* recv_buf(int r, int slot) { (void)r; (void)slot; return nullptr; }
+    virtual size_t recv_capacity() const { return 0; }   // doubles per receive buffer
+    virtual int wait_free(int64_t panel, cudaStream_t s) { (void)panel; (void)s; return 0; }   // owner: peers done with the slot
+    virtual int post_panel(int64_t panel, cudaStream_t s) { (void)panel; (void)s; return 0; }  // owner: panel stored
+    virtual int wait_panel(int root, int64_t panel, cudaStream_t s) { (void)root; (void)panel; (void)s; return 0; }
+    virtual int mark_free(int64_t value, cudaStream_t s) { (void)value; (void)s; return 0; }     // this rank's reads done
 };
+// The owner's write-back of panel k fused with the push to its peers: data rows -> A panel,
+// checksum rows -> chk, the whole W (+ abort slot) -> every peer's receive buffer (util.cu).
+int launch_panel_out(const double* W, int64_t ldw, int64_t mB, int64_t ncrows, int64_t B, double* Apanel,
+                     int64_t lda, double* chk, int64_t ldc, double* const* peers, int npeer, const int32_t* abort_flag,
+                     cudaStream_t s);
 // The 1D block-cyclic driver (abft.cu). ranks: local ranks driven by this call — one with a
 // transport (NCCL, one process per GPU) or all P of them with tp == nullptr (single-process
 // simulation on one device: the broadcast becomes a device-to-device copy).
@@ -260,7 +287,7 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
 int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                 int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
                 int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
-                cudaStream_t s, int force_tile = 0, abft::ColSumOut* cs = nullptr);
+                cudaStream_t s, int force_tile = 0, abft::ColSumOut* cs = nullptr, int nchk = 2);
 // The trailing update with the checksum rows as a second row segment of the same launch.
 // cstride > 1: C's column block t (and the B operand's row block t) is global block t * cstride
 // (a rank's 1D block-cyclic local columns in one launch); returns -1 if the shapes do not allow it.
@@ -274,4 +301,4 @@ int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s,
                            abft::ColSumOut* cs, int64_t lda2 = 0, int64_t cstride = 1,
-                           const abft::EpiInj* inj = nullptr);
+                           const abft::EpiInj* inj = nullptr, int nchk = 2);

@@ -55,7 +55,11 @@ struct GemmArgs {
     // sets it to the number of CTAs resident at once)
     int64_t pf_ahead;
     EpiInj inj;   // UPDATE_OUT hook in the epilogue (ws kernel; inj.n == 0: none)
+    int32_t nchk; // MASK_CHK / checksum segment: checksum rows per block (row q is block q / nchk)
 };
+
+// block row of checksum row q (nchk = 2 or 3 rows per block): constant divisors, no runtime division
+__host__ __device__ __forceinline__ int64_t chk_block(int64_t q, int32_t nchk) { return nchk == 3 ? q / 3 : q / 2; }
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
     const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
@@ -107,7 +111,7 @@ k_gemm_dmma(GemmArgs g) {
     const int64_t m0 = tm * BM, n0 = tn * BN;
     if (g.mask == MASK_CHK) {  // skip tiles where no row reaches the column blocks
         const int64_t qmax = min(g.M, m0 + BM) - 1;
-        const int64_t Imax = g.q_tile0 + qmax / 2, Jmin = g.c_tile0 + n0 / g.nb;
+        const int64_t Imax = g.q_tile0 + chk_block(qmax, g.nchk), Jmin = g.c_tile0 + n0 / g.nb;
         if (Imax < Jmin) return;
     }
     int64_t kb = 0, ke = g.K;
@@ -267,8 +271,8 @@ k_gemm_dmma(GemmArgs g) {
             if (g.mask == MASK_LOWER) { o0 = o0 && gr >= gc; o1 = o1 && gr + 1 >= gc; }
             else if (g.mask == MASK_CHK) {
                 const int64_t J = g.c_tile0 + gc / g.nb;
-                o0 = o0 && (g.q_tile0 + gr / 2) >= J;
-                o1 = o1 && (g.q_tile0 + (gr + 1) / 2) >= J;
+                o0 = o0 && (g.q_tile0 + chk_block(gr, g.nchk)) >= J;
+                o1 = o1 && (g.q_tile0 + chk_block(gr + 1, g.nchk)) >= J;
             }
             ok0[b] = o0; ok1[b] = o1;
             ptr[b] = g.C + gc * g.ldc + gr;
@@ -420,7 +424,7 @@ __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t 
         tm = e / TN; tn = e % TN;
         T.m0 = tm * BM; T.n0 = tn * BN; T.seg2 = true;
         const int64_t qmax = min(g.M2, T.m0 + BM) - 1;
-        return qmax / 2 >= (T.n0 / g.nb) * g.cstride;
+        return chk_block(qmax, g.nchk) >= (T.n0 / g.nb) * g.cstride;
     }
     if (g.mask == MASK_LOWER && g.cstride > 1) {   // strided columns: grouped rectangle, skip tiles above
         const int64_t q = idx / (kWsGroup * TN), a0 = q * kWsGroup, Gp = ((TM - a0) < kWsGroup ? (TM - a0) : (int64_t)kWsGroup);
@@ -456,12 +460,12 @@ __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t 
     T.m0 = tm * BM; T.n0 = tn * BN; T.seg2 = false;
     if (g.mask == MASK_CHK) {
         const int64_t qmax = min(g.M, T.m0 + BM) - 1;
-        if (g.q_tile0 + qmax / 2 < g.c_tile0 + T.n0 / g.nb) return false;
+        if (g.q_tile0 + chk_block(qmax, g.nchk) < g.c_tile0 + T.n0 / g.nb) return false;
     }
     return true;
 }
 
-template <class C_>
+template <class C_, bool CS3 = false>
 __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64_t n1tiles) {
     constexpr int BM = C_::BM, BN = C_::BN, BK = C_::BK, WM = C_::WM, WN = C_::WN, STAGES = C_::STAGES;
     if (cta_aborted(g.abort)) return;
@@ -586,9 +590,9 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
                 const int64_t c = n0 + wn * WN + j * 8 + fc * 2 + h;
                 int64_t v;
                 if (c >= g.N) v = INT64_MAX;
-                else if (seg2) v = 2 * (c / g.nb) * g.cstride;                       // q/2 >= block of c
+                else if (seg2) v = g.nchk * (c / g.nb) * g.cstride;                  // q/nchk >= block of c
                 else if (g.mask == MASK_LOWER) v = c + cshift;                        // r >= global c
-                else if (g.mask == MASK_CHK) v = 2 * (g.c_tile0 + c / g.nb - g.q_tile0);
+                else if (g.mask == MASK_CHK) v = g.nchk * (g.c_tile0 + c / g.nb - g.q_tile0);
                 else v = 0;
                 rmin[j][h] = v;
             }
@@ -715,10 +719,47 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
                     v[i] = keep + __shfl_xor_sync(0xffffffffu, give, 4);
                 }
             }
+            const int64_t gcs = gc0 + wn * WN + (fr >> 1) * 8 + fc * 2 + (fr & 1);   // column slot fr
             if (offdiag) {   // lane (fr, fc) holds column slot q = fr: j = fr / 2, h = fr % 2
-                const int64_t gc = gc0 + wn * WN + (fr >> 1) * 8 + fc * 2 + (fr & 1);
-                g.cs.p[slab * g.cs.ld + gc] = v[0];
-                g.cs.p[(g.cs.nslab + slab) * g.cs.ld + gc] = v[1];
+                g.cs.p[slab * g.cs.ld + gcs] = v[0];
+                g.cs.p[(g.cs.nslab + slab) * g.cs.ld + gcs] = v[1];
+            }
+            if (CS3) {   // third checksum (B10): weights (row + 1)^2, same butterfly on 8 values
+                double u[8];
+#pragma unroll
+                for (int j = 0; j < C_::FN; ++j)
+#pragma unroll
+                    for (int h = 0; h < 2; ++h) {
+                        double s3 = 0.0;
+#pragma unroll
+                        for (int i = 0; i < C_::FM; ++i) {
+                            const double w = (double)(wbase + i * 8);
+                            s3 = fma(w * w, acc[i][j][h], s3);
+                        }
+                        u[2 * j + h] = s3;
+                    }
+                {
+                    const bool up = (fr & 4) != 0;
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const double keep = up ? u[i + 4] : u[i], give = up ? u[i] : u[i + 4];
+                        u[i] = keep + __shfl_xor_sync(0xffffffffu, give, 16);
+                    }
+                }
+                {
+                    const bool up = (fr & 2) != 0;
+#pragma unroll
+                    for (int i = 0; i < 2; ++i) {
+                        const double keep = up ? u[i + 2] : u[i], give = up ? u[i] : u[i + 2];
+                        u[i] = keep + __shfl_xor_sync(0xffffffffu, give, 8);
+                    }
+                }
+                {
+                    const bool up = (fr & 1) != 0;
+                    const double keep = up ? u[1] : u[0], give = up ? u[0] : u[1];
+                    u[0] = keep + __shfl_xor_sync(0xffffffffu, give, 4);
+                }
+                if (offdiag) g.cs.p[(2 * g.cs.nslab + slab) * g.cs.ld + gcs] = u[0];
             }
         }
     }
@@ -730,9 +771,11 @@ template <class C_>
 __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_gemm_ws(GemmArgs g, int64_t ntiles, int64_t n1tiles) {
     ws_body<C_>(g, ntiles, n1tiles);
 }
-template <class C_>
+// CS3: the update also emits the third checksum's partials (nchk = 3, reading B10) — a separate
+// instantiation so that the default two-checksum kernel keeps its register budget
+template <class C_, bool CS3 = false>
 __global__ void __launch_bounds__(C_::THREADS, C_::MINB) k_update_ws(GemmArgs g, int64_t ntiles, int64_t n1tiles) {
-    ws_body<C_>(g, ntiles, n1tiles);
+    ws_body<C_, CS3>(g, ntiles, n1tiles);
 }
 
 template <class C_>
@@ -741,6 +784,7 @@ static int run_ws(GemmArgs g, cudaStream_t s, bool update) {
     if (!attr) {
         cudaFuncSetAttribute(k_gemm_ws<C_>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::SMEM);
         cudaFuncSetAttribute(k_update_ws<C_>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::SMEM);
+        cudaFuncSetAttribute(k_update_ws<C_, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::SMEM);
         attr = true;
     }
     const int64_t tm = (g.M + C_::BM - 1) / C_::BM, tn = (g.N + C_::BN - 1) / C_::BN;
@@ -762,7 +806,9 @@ static int run_ws(GemmArgs g, cudaStream_t s, bool update) {
         ahead = e ? atoi(e) : (int64_t)nsm * C_::MINB;
     }
     g.pf_ahead = (tpc == 1) ? ahead : 0;
-    if (update) k_update_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
+    if (update && g.cs.p != nullptr && g.cs.nchk == 3)
+        k_update_ws<C_, true><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
+    else if (update) k_update_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
     else k_gemm_ws<C_><<<(unsigned)grid, C_::THREADS, C_::SMEM, s>>>(g, ntiles, n1);
     abft_count_launch();
     return 0;
@@ -773,7 +819,8 @@ static int run_ws(GemmArgs g, cudaStream_t s, bool update) {
 bool is_update_kernel(const void* f) {
     return f == (const void*)k_update_ws<WsCfg> || f == (const void*)k_update_ws<WsCfg16> ||
            f == (const void*)k_update_ws<WsCfg2a> || f == (const void*)k_update_ws<WsCfg2b> ||
-           f == (const void*)k_update_ws<WsCfgNR> || f == (const void*)k_update_ws<WsCfg2l>;
+           f == (const void*)k_update_ws<WsCfgNR> || f == (const void*)k_update_ws<WsCfg2l> ||
+           f == (const void*)k_update_ws<WsCfg2b, true> || f == (const void*)k_update_ws<WsCfg2l, true>;
 }
 
 static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CTA/SM), 16, 2a
@@ -824,13 +871,14 @@ static bool aligned16(const void* p) { return ((uintptr_t)p & 15) == 0; }
 int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                 int64_t ldb, double* C, int64_t ldc, double alpha, double beta, bool transB, int mask,
                 int krange, int64_t nb, int64_t q_tile0, int64_t c_tile0, const int32_t* abort_flag,
-                cudaStream_t s, int force_tile, ColSumOut* cs) {
+                cudaStream_t s, int force_tile, ColSumOut* cs, int nchk) {
     if (M <= 0 || N <= 0) return 0;
     GemmArgs g;
+    g.nchk = nchk;
     g.M = M; g.N = N; g.K = K; g.A = A; g.lda = lda; g.B = B; g.ldb = ldb; g.C = C; g.ldc = ldc;
     g.alpha = alpha; g.beta = beta; g.mask = mask; g.krange = krange; g.nb = nb;
     g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
-    g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
+    g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0, 2};
     g.M2 = 0; g.A2 = nullptr; g.C2 = nullptr; g.ldc2 = 1; g.lda2 = 1; g.cstride = 1;
     g.inj.n = 0;
     g.vecA = aligned16(A) && (lda % 2 == 0);
@@ -876,32 +924,51 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s, ColSumOut* cs,
-                           int64_t lda2, int64_t cstride, const EpiInj* inj) {
+                           int64_t lda2, int64_t cstride, const EpiInj* inj, int nchk) {
     if (lda2 <= 0) lda2 = lda;
     if (cstride < 1) cstride = 1;
-    const bool ok = M > 0 && N > 0 && (M % 2 == 0) && (N % 2 == 0) && (M2 % 2 == 0) && (K % WsCfg::BK == 0) &&
-                    aligned16(A) && aligned16(B) && aligned16(A2) && lda % 2 == 0 && ldb % 2 == 0 && N <= M &&
-                    lda2 % 2 == 0 && M % WsCfg::BM == 0 && getenv("ABFT_GEMM_VARIANT") == nullptr &&
+    // the data segment's kernel must not depend on the checksum segment (same rounding with two or
+    // three checksum rows): the checksum rows ride in the same launch when their shapes allow it,
+    // else they get their own launch and the data rows still take the warp-specialised kernel
+    const bool ok = M > 0 && N > 0 && (M % 2 == 0) && (N % 2 == 0) && (K % WsCfg::BK == 0) &&
+                    aligned16(A) && aligned16(B) && lda % 2 == 0 && ldb % 2 == 0 && N <= M &&
+                    M % WsCfg::BM == 0 && getenv("ABFT_GEMM_VARIANT") == nullptr &&
                     (cstride == 1 || nb % WsCfg::BN == 0);
+    const bool chk_ok = M2 == 0 || ((M2 % 2 == 0) && aligned16(A2) && lda2 % 2 == 0);
     if (!ok && cstride > 1) return -1;   // strided columns need the warp-specialised kernel
     if (!ok) {   // fallback (two generic launches): the caller applies the hook, no fused partials
         const int f = launch_gemm(M, N, K, A, lda, B, ldb, C, ldc, -1.0, 1.0, true, MASK_LOWER, KR_FULL, 0, 0, 0,
                                   abort_flag, s, 0, (inj && inj->n > 0) ? nullptr : cs);
         if (M2 > 0)
-            launch_gemm(M2, N, K, A2, lda2, B, ldb, C2, ldc2, -1.0, 1.0, true, MASK_CHK, KR_FULL, nb, 0, 0, abort_flag, s);
+            launch_gemm(M2, N, K, A2, lda2, B, ldb, C2, ldc2, -1.0, 1.0, true, MASK_CHK, KR_FULL, nb, 0, 0, abort_flag, s,
+                        0, nullptr, nchk);
         return f == 1 ? 1 : 0;
     }
+    const bool split = !chk_ok;
+    if (split && cstride > 1) return -1;
     GemmArgs g;
     g.M = M; g.N = N; g.K = K; g.A = A; g.lda = lda; g.B = B; g.ldb = ldb; g.C = C; g.ldc = ldc;
     g.alpha = -1.0; g.beta = 1.0; g.mask = MASK_LOWER; g.krange = KR_FULL; g.nb = nb;
     g.q_tile0 = 0; g.c_tile0 = 0; g.tiles_n = 1; g.abort = abort_flag; g.vecA = 1; g.vecB = 1;
-    g.cs = ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
+    g.cs = ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0, 2};
     g.inj.n = 0;
+    g.nchk = nchk;
     int ret = 0;
-    if (inj && inj->n > 0 && inj->n <= kMaxEpiInj) { g.inj = *inj; ret |= 2; }
-    const bool inj_left = inj && inj->n > kMaxEpiInj;   // too many for the epilogue: caller's hook
+    bool inj_chk = false;   // a checksum-row target, which a split-off checksum launch cannot apply
+    for (int q = 0; inj && q < inj->n && q < kMaxEpiInj; ++q) inj_chk |= inj->op[q].seg == 1;
+    const bool inj_left = inj && (inj->n > kMaxEpiInj || (split && inj_chk));   // caller's hook
+    if (inj && inj->n > 0 && !inj_left) { g.inj = *inj; ret |= 2; }
     if (cs && !inj_left && cs->nb % WsCfg::BM == 0 && cs->row0 % WsCfg::BM == 0 && cs->colg0 % WsCfg::BN == 0) {
         g.cs = *cs; ret |= 1;
+    }
+    if (split) {
+        g.M2 = 0; g.A2 = nullptr; g.C2 = nullptr; g.ldc2 = 1; g.lda2 = 1; g.cstride = cstride;
+        run_ws_any(g, s);
+        if (M2 > 0)
+            launch_gemm(M2, N, K, A2, lda2, B, ldb, C2, ldc2, -1.0, 1.0, true, MASK_CHK, KR_FULL, nb, 0, 0, abort_flag, s,
+                        0, nullptr, nchk);
+        if (ret & 1) cs->slab_rows = ws_slab_rows();
+        return ret;
     }
     g.M2 = M2; g.A2 = A2; g.C2 = C2; g.ldc2 = ldc2; g.lda2 = lda2; g.cstride = cstride;
     run_ws_any(g, s);
@@ -930,8 +997,9 @@ int launch_trsm_with_chk(int64_t mB, int64_t B, const double* Ap, int64_t lda, c
     g.M = mB; g.N = B; g.K = B; g.A = Ap; g.lda = lda; g.B = Li; g.ldb = B; g.C = W; g.ldc = ldw;
     g.alpha = 1.0; g.beta = 0.0; g.mask = MASK_NONE; g.krange = KR_LE_N; g.nb = B;
     g.q_tile0 = 0; g.c_tile0 = 0; g.tiles_n = 1; g.abort = abort_flag; g.vecA = 1; g.vecB = 1;
-    g.cs = ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0};
+    g.cs = ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0, 2};
     g.inj.n = 0;
+    g.nchk = 2;   // the TRSM's second segment covers every row (column block 0 only)
     g.M2 = M2; g.A2 = A2; g.C2 = W + mB; g.ldc2 = ldw; g.lda2 = lda2; g.cstride = 1;
     run_ws_any(g, s);
     return 1;

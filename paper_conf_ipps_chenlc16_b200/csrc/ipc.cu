@@ -22,9 +22,12 @@
 namespace {
 
 constexpr int kMaxRanks = 64;
-constexpr size_t kCtlBytes = 256;   // [posted, done] words at the head of every arena
+constexpr size_t kCtlBytes = 256;   // flag words at the head of every arena
 
-struct Ctl { unsigned long long posted, done; };
+// posted/done: collective sequence numbers; panel: 1 + the last panel this rank pushed into its
+// peers' receive buffers; freed: panels p < freed + 2 may be pushed into this rank's buffers
+// (its update p - 2, the last reader of buffer p & 1, is complete)
+struct Ctl { unsigned long long posted, done, panel, freed; };
 
 __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
     unsigned long long v;
@@ -42,17 +45,24 @@ __global__ void k_ipc_wait(PeerTable t, int np, int skip, int which, unsigned lo
     if (threadIdx.x != 0) return;
     for (int r = 0; r < np; ++r) {
         if (r == skip) continue;
-        const unsigned long long* w = which ? &t.ctl[r]->done : &t.ctl[r]->posted;
+        const unsigned long long* w = which == 0 ? &t.ctl[r]->posted : which == 1 ? &t.ctl[r]->done
+                                    : which == 2 ? &t.ctl[r]->panel : &t.ctl[r]->freed;
         while (ld_acquire_sys(w) < v) __nanosleep(256);
     }
 }
+__device__ __forceinline__ const unsigned long long* ctl_word(const Ctl* c, int which) {
+    return which == 0 ? &c->posted : which == 1 ? &c->done : which == 2 ? &c->panel : &c->freed;
+}
 __global__ void k_ipc_wait_one(const Ctl* c, int which, unsigned long long v) {
     if (threadIdx.x != 0) return;
-    const unsigned long long* w = which ? &c->done : &c->posted;
+    const unsigned long long* w = ctl_word(c, which);
     while (ld_acquire_sys(w) < v) __nanosleep(256);
 }
 __global__ void k_ipc_set(Ctl* c, int which, unsigned long long v) {
-    if (threadIdx.x == 0) { __threadfence_system(); st_release_sys(which ? &c->done : &c->posted, v); }
+    if (threadIdx.x == 0) {
+        __threadfence_system();
+        st_release_sys(const_cast<unsigned long long*>(ctl_word(c, which)), v);
+    }
 }
 // buf[i] = op over ranks r = 0..np-1 (ascending) of data_r[i]; op 0 sum, 1 max
 __global__ void k_ipc_reduce(PeerTable t, int np, double* buf, size_t count, int op) {
@@ -67,18 +77,39 @@ __global__ void k_ipc_reduce(PeerTable t, int np, double* buf, size_t count, int
 }
 
 struct IpcTransport : DistTransport {
-    char* mine = nullptr;                 // own arena (cudaMalloc, exported)
-    size_t cap = 0;                       // data bytes per arena
+    char* mine = nullptr;                 // own arena (cudaMalloc, exported): [ctl | recv 0 | recv 1 | data]
+    size_t cap = 0;                       // data bytes per arena (= bytes of each receive buffer)
     std::vector<char*> peer;              // mapped arenas (peer[rank] == mine)
     unsigned long long seq = 0;           // collectives issued (same sequence on every rank)
     PeerTable table() const {
         PeerTable t;
         memset(&t, 0, sizeof t);
-        for (int r = 0; r < nranks; ++r) { t.ctl[r] = reinterpret_cast<const Ctl*>(peer[r]); t.data[r] = peer[r] + kCtlBytes; }
+        for (int r = 0; r < nranks; ++r) { t.ctl[r] = reinterpret_cast<const Ctl*>(peer[r]); t.data[r] = data_of(r); }
         return t;
     }
     Ctl* my_ctl() const { return reinterpret_cast<Ctl*>(mine); }
-    char* my_data() const { return mine + kCtlBytes; }
+    char* my_data() const { return mine + kCtlBytes + 2 * cap; }
+    char* data_of(int r) const { return peer[r] + kCtlBytes + 2 * cap; }
+    // push mode: receive buffer `slot` of rank r (mapped into this process)
+    double* recv_buf(int r, int slot) override { return reinterpret_cast<double*>(peer[r] + kCtlBytes + slot * cap); }
+    size_t recv_capacity() const override { return cap / sizeof(double); }
+    int wait_free(int64_t panel, cudaStream_t s) override {   // every peer finished update panel - 2
+        const PeerTable t = table();
+        k_ipc_wait<<<1, 32, 0, s>>>(t, nranks, rank, 3, (unsigned long long)(panel >= 1 ? panel - 1 : 0));
+        return cudaGetLastError() == cudaSuccess ? 0 : 1;
+    }
+    int post_panel(int64_t panel, cudaStream_t s) override {
+        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 2, (unsigned long long)(panel + 1));
+        return cudaGetLastError() == cudaSuccess ? 0 : 1;
+    }
+    int wait_panel(int root, int64_t panel, cudaStream_t s) override {
+        k_ipc_wait_one<<<1, 32, 0, s>>>(reinterpret_cast<const Ctl*>(peer[root]), 2, (unsigned long long)(panel + 1));
+        return cudaGetLastError() == cudaSuccess ? 0 : 1;
+    }
+    int mark_free(int64_t value, cudaStream_t s) override {
+        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 3, (unsigned long long)value);
+        return cudaGetLastError() == cudaSuccess ? 0 : 1;
+    }
     // publish `bytes` from src into my arena as collective s (after every peer finished s-1)
     int publish(const void* src, size_t bytes, cudaStream_t s, const PeerTable& t) {
         if (bytes > cap) return 1;
@@ -99,7 +130,7 @@ struct IpcTransport : DistTransport {
         } else {
             if (bytes > cap) return 1;
             k_ipc_wait_one<<<1, 32, 0, s>>>(t.ctl[root], 0, seq);   // the root's panel of collective seq
-            if (bytes && cudaMemcpyAsync(buf, peer[root] + kCtlBytes, bytes, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+            if (bytes && cudaMemcpyAsync(buf, data_of(root), bytes, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
                 return 1;
         }
         return finish(s);
@@ -120,7 +151,7 @@ struct IpcTransport : DistTransport {
         if (publish(send, bytes, s, t)) return 1;
         k_ipc_wait<<<1, 32, 0, s>>>(t, nranks, rank, 0, seq);
         for (int r = 0; r < nranks; ++r)
-            if (bytes && cudaMemcpyAsync((char*)recv + r * bytes, peer[r] + kCtlBytes, bytes, cudaMemcpyDeviceToDevice, s) !=
+            if (bytes && cudaMemcpyAsync((char*)recv + r * bytes, data_of(r), bytes, cudaMemcpyDeviceToDevice, s) !=
                              cudaSuccess)
                 return 1;
         return finish(s);
@@ -169,7 +200,7 @@ extern "C" int abft_comm_init_ipc(void** comm, int nranks, int rank, int64_t cap
     if (!handle_out) return -5;
     IpcTransport* t = new IpcTransport;
     t->rank = rank; t->nranks = nranks; t->cap = (size_t)cap_bytes;
-    if (cudaMalloc((void**)&t->mine, kCtlBytes + t->cap) != cudaSuccess) { delete t; return ABFT_ERR_CUDA; }
+    if (cudaMalloc((void**)&t->mine, kCtlBytes + 3 * t->cap) != cudaSuccess) { delete t; return ABFT_ERR_CUDA; }
     cudaMemset(t->mine, 0, kCtlBytes);
     cudaDeviceSynchronize();
     cudaIpcMemHandle_t h;

@@ -40,7 +40,7 @@ def test_struct_layouts_match_header():
     assert ctypes.sizeof(p.Event) == 48 == p.EVENT_DTYPE.itemsize
     assert p.INJ_DTYPE.itemsize == 48 == syn.INJ_DTYPE.itemsize
     assert ctypes.sizeof(p.Report) == 14 * 8
-    assert ctypes.sizeof(p.Options) == 32
+    assert ctypes.sizeof(p.Options) == 40
 
 
 def test_sm100a_code_in_library():

@@ -3,7 +3,8 @@ two ranks on one device, so the ranks talk through the peer-memory (CUDA IPC) tr
 (abft_comm_init_ipc / abft_comm_attach_ipc, include/abft.h), which runs the same run_dist driver as
 the NCCL path (1D block-cyclic ownership, owner-only panel, panel broadcast, RECV
 hook + V4R on the receiver, per-rank trailing updates, merged report). Events and the factor must
-equal the oracle's P-rank simulation."""
+equal the oracle's P-rank simulation. The panel broadcast is the fused push (NEXT-3) by default, the
+transport's pull collective with ABFT_DIST_PULL=1."""
 import os
 import socket
 
@@ -24,8 +25,10 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, n, nb, specs, q):
+def _worker(rank, world, port, n, nb, specs, q, mode="push"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    if mode == "pull":     # the transport's broadcast collective instead of the fused push
+        os.environ["ABFT_DIST_PULL"] = "1"
     import torch
     import torch.distributed as dist
     import paper_conf_ipps_chenlc16_b200 as P
@@ -45,12 +48,12 @@ def _worker(rank, world, port, n, nb, specs, q):
     dist.destroy_process_group()
 
 
-def _run(n, nb, world, specs):
+def _run(n, nb, world, specs, mode="push"):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, n, nb, specs, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, n, nb, specs, q, mode)) for r in range(world)]
     for p in procs:
         p.start()
     res = sorted([q.get(timeout=600) for _ in procs], key=lambda t: t[0])
@@ -65,8 +68,12 @@ def floor_rel(L, Lref, A):
     return float(np.max(np.abs(np.tril(L) - np.tril(Lref)) / np.maximum(np.abs(np.tril(Lref)), 1e-3 * s)))
 
 
+@pytest.mark.parametrize("mode", ["push", "pull"])
 @pytest.mark.parametrize("specs_kind", ["fault_free", "injected"])
-def test_two_processes_ipc_transport_match_oracle(specs_kind):
+def test_two_processes_ipc_transport_match_oracle(specs_kind, mode):
+    """push (default, NEXT-3): the owner's write-back kernel stores the packed panel straight into
+    the peer's receive buffer; pull: the transport's broadcast collective copies it out of the
+    owner's arena."""
     import paper_conf_ipps_chenlc16_b200 as P
     n, nb, world = 1024, 128, 2
     specs = []
@@ -76,7 +83,7 @@ def test_two_processes_ipc_transport_match_oracle(specs_kind):
                   dict(k=2, hook="RECV", target="CHK", row=2 * 6 + 1, col=2 * nb + 5, bit=50, rank=1)]
     A = syn.spd_matrix(n)
     ref = oracle.potrf(A, nb, inj=syn.inj_array(specs) if specs else None, nranks=world)
-    res = _run(n, nb, world, specs)
+    res = _run(n, nb, world, specs, mode)
     # rank 0's report holds every rank's events (gathered through the transport)
     rank0 = res[0]
     assert rank0[1] == ref.status == 0
