@@ -116,8 +116,13 @@ typedef struct { int64_t c; int kind; int64_t row, row2; double d1, d2, d3, r1, 
  * d3) / d1); accept (wa, wb) = (S -+ sqrt(S^2 - 4P)) / 2 if they are integers in 1..B, the residual
  * d3 - S d2 + P d1 is within its rounding tolerance and both errors exceed tau1. Exactly one
  * accepted pair locates the errors; none or several -> not located. Returns 1 and the 0-based rows. */
+#define RHO2 0x1p-40   /* relative slack of the two-error residual [B10]: the single-error 2^-30 [A6]
+                         would let a large error's slack hide a small second error (ambiguity);
+                         2^-40 still exceeds the worst-case relative rounding of the sums, B eps */
 static int locate_two(double d1, double d2, double d3, double tau1, double tau2, double tau3, double rho, int64_t B,
                       int64_t* ra, int64_t* rb) {
+    (void)rho;
+    rho = RHO2;
     int found = 0;
     if (!(fabs(d1) > tau1)) return 0;                 /* Da + Db ~ 0: P is not determined */
     for (int64_t S = 3; S <= 2 * B - 1; ++S) {
@@ -134,7 +139,9 @@ static int locate_two(double d1, double d2, double d3, double tau1, double tau2,
         const int64_t wa = (S - q) / 2, wb = (S + q) / 2;
         if (wa < 1 || wb > B) continue;
         const double res = d3 - Sd * d2 + Pd * d1;
-        const double tol = tau3 + Sd * tau2 + Pd * tau1 + rho * (fabs(d3) + Sd * fabs(d2) + Pd * fabs(d1));
+        /* the thresholds bound each sum's fault-free noise with a wide margin (P9: measured <= 2^-6
+         * of tau); their full combination admits false pairs, so the residual allows 1/16 of it */
+        const double tol = (tau3 + Sd * tau2 + Pd * tau1) * 0.0625 + rho * (fabs(d3) + Sd * fabs(d2) + Pd * fabs(d1));
         if (!(fabs(res) <= tol)) continue;
         const double Da = ((double)wb * d1 - d2) / (double)(wb - wa), Db = (d2 - (double)wa * d1) / (double)(wb - wa);
         if (!(fabs(Da) > tau1) || !(fabs(Db) > tau1)) continue;

@@ -118,6 +118,7 @@ __device__ void phase1_reread(const StageArgs& a, int part, int64_t bid) {
         double m1 = 0.0, m2 = 0.0, m3 = 0.0;
         if (cc < cw) {
             const int64_t c = c0 + cc;
+#pragma unroll 8
             for (int64_t r = grp; r < c; r += ngroups) {
                 const double x = v.T[r * v.ldt + c];
                 const double w = (double)(r + 1);
@@ -166,11 +167,24 @@ __device__ void phase1_fused(const StageArgs& a, int part, int64_t bid) {
     const TileView v = stage_view(a, I, J);
     double r1 = 0.0, r2 = 0.0, r3 = 0.0;
     if (act) {
+        // the slab partials of the column are loaded 8 at a time before they are summed (in slab
+        // order): the loads are independent, so a batch is in flight at once, not one per latency
         const int64_t g = local_col(a, J) + c, s0 = I * B / a.cs_slab_rows, ns = B / a.cs_slab_rows;
-        for (int64_t q = 0; q < ns; ++q) {
-            r1 += a.cs[(s0 + q) * a.cs_ld + g];
-            r2 += a.cs[(a.cs_nslab + s0 + q) * a.cs_ld + g];
-            if (v.c3) r3 += a.cs[(2 * a.cs_nslab + s0 + q) * a.cs_ld + g];
+        const double* b1 = a.cs + s0 * a.cs_ld + g;
+        const double* b2 = a.cs + (a.cs_nslab + s0) * a.cs_ld + g;
+        const double* b3 = a.cs + (2 * a.cs_nslab + s0) * a.cs_ld + g;
+        for (int64_t q0 = 0; q0 < ns; q0 += 8) {
+            double p1[8], p2[8], p3[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                const bool in = q0 + q < ns;
+                p1[q] = in ? b1[(q0 + q) * a.cs_ld] : 0.0;
+                p2[q] = in ? b2[(q0 + q) * a.cs_ld] : 0.0;
+                p3[q] = (in && v.c3) ? b3[(q0 + q) * a.cs_ld] : 0.0;
+            }
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+                if (q0 + q < ns) { r1 += p1[q]; r2 += p2[q]; r3 += p3[q]; }
         }
     }
     compare_column(a, part, v, I, J, c, r1, r2, r3, act);
@@ -247,8 +261,10 @@ __device__ bool locate_two(double d1, double d2, double d3, double tau1, double 
         const int64_t wa = (S - q) / 2, wb = (S + q) / 2;
         if (wa < 1 || wb > B) continue;
         const double res = __dadd_rn(__dsub_rn(d3, __dmul_rn(Sd, d2)), __dmul_rn(Pd, d1));
-        const double tol = __dadd_rn(__dadd_rn(__dadd_rn(tau3, __dmul_rn(Sd, tau2)), __dmul_rn(Pd, tau1)),
-                                     __dmul_rn(ABFT_RHO, __dadd_rn(__dadd_rn(fabs(d3), __dmul_rn(Sd, fabs(d2))),
+        // 1/16 of the thresholds' combination (their full sum admits false pairs; the measured
+        // noise is <= 2^-6 of tau, P9) + the relative slack ABFT_RHO2
+        const double tol = __dadd_rn(__dmul_rn(__dadd_rn(__dadd_rn(tau3, __dmul_rn(Sd, tau2)), __dmul_rn(Pd, tau1)), 0.0625),
+                                     __dmul_rn(ABFT_RHO2, __dadd_rn(__dadd_rn(fabs(d3), __dmul_rn(Sd, fabs(d2))),
                                                                    __dmul_rn(Pd, fabs(d1)))));
         if (!(fabs(res) <= tol)) continue;
         const double wad = (double)wa, wbd = (double)wb, den = (double)(wb - wa);

@@ -7,6 +7,7 @@
 
 #define ABFT_EPS 0x1p-52  /* DBL_EPSILON (reading A17) */
 #define ABFT_RHO 0x1p-30  /* relative slack of the location test (reading A6) */
+#define ABFT_RHO2 0x1p-40 /* relative slack of the two-error residual (reading B10, nchk = 3) */
 
 namespace abft {
 

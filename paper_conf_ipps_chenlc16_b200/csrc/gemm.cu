@@ -562,6 +562,12 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
                 }
             }
         }
+        if constexpr (!C_::LDG) {
+            // producer tail: the copying warp stays resident until the consumers have finished
+            // (named barrier 1: this warp waits, the consumer warps arrive at their end), so it
+            // never exits while bulk copies it issued may still be in flight
+            asm volatile("bar.sync 1, %0;\n" ::"n"((C_::CONSUMERS + 1) * 32) : "memory");
+        }
         return;
     }
     // ------------------------------- consumers -------------------------------
@@ -763,6 +769,8 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
             }
         }
     }
+    // release the copying producer warp (its tail waits on named barrier 1)
+    if constexpr (!C_::LDG) asm volatile("bar.arrive 1, %0;\n" ::"n"((C_::CONSUMERS + 1) * 32) : "memory");
 }
 
 // Two entry points with one body, so that profiles attribute the trailing update (the dominant
@@ -849,7 +857,7 @@ static bool tasks_path() {
 static int run_ws_any(GemmArgs g, cudaStream_t s) {
     g.cs.slab_rows = ws_slab_rows();
     const bool upd = g.mask == MASK_LOWER && g.alpha == -1.0 && g.beta == 1.0;   // a trailing update
-    if (upd && tasks_path()) return run_ws<WsCfg2l>(g, s, upd);
+    if (upd && tasks_path() && getenv("ABFT_WS_FORCE_BULK") == nullptr) return run_ws<WsCfg2l>(g, s, upd);
     switch (ws_variant()) {
         case 16: return run_ws<WsCfg16>(g, s, upd);
         case 21: return run_ws<WsCfg2a>(g, s, upd);

@@ -23,7 +23,7 @@ import numpy as np
 __all__ = [
     "splitmix64", "spd_matrix", "spd_diag", "pascal_mod2", "pascal", "HOOK", "TARGET",
     "inj_array", "INJ_DTYPE", "bit_mask", "c1_injections", "per_iteration_injections",
-    "mixed_injections",
+    "mixed_injections", "next4_injections",
 ]
 
 _GOLDEN = np.uint64(0x9E3779B97F4A7C15)
@@ -217,3 +217,22 @@ def mixed_injections(n: int, nb: int, seed: int | None = None, kmax=None):
             sub["row"], sub["col"] = int(max(a, b)), int(min(a, b))
         out.append(sub)
     return out
+
+
+def next4_injections(n: int, nb: int, seed: int | None = None):
+    """NEXT-4 recipe (three checksum rows per block): the mixed_injections list with its
+    checksum-row targets renumbered for three rows per block (row 2I+t -> 3I+t), plus a second
+    error next to every tenth data error of hook UPDATE_OUT / REST whose bit is <= 58 (no
+    overflow: a non-finite error would mask its partner), 97 rows further down the same block
+    column of the same tile — two errors in one column of a block."""
+    specs = []
+    for sp in mixed_injections(n, nb, seed):
+        if sp.get("target", "DATA") == "CHK":
+            sp = dict(sp, row=3 * (sp["row"] // 2) + sp["row"] % 2)
+        specs.append(sp)
+    for sp in list(specs)[1::10]:
+        if sp.get("target", "DATA") == "DATA" and sp["hook"] in ("UPDATE_OUT", "REST") and sp["bit"] <= 58:
+            r2 = (sp["row"] // nb) * nb + (sp["row"] % nb + 97) % nb
+            if r2 >= sp["col"] and r2 != sp["row"]:
+                specs.append(dict(sp, row=r2, bit=53))
+    return specs

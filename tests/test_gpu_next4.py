@@ -117,17 +117,7 @@ def test_mixed_injections_plus_pairs_at_scale(P):
     fifth computing error, full event list equal to the oracle's."""
     n, nb = 8192, 512
     A = syn.spd_matrix(n)
-    base = []
-    for s in syn.mixed_injections(n, nb):   # checksum-row targets in the three-row numbering
-        if s.get("target", "DATA") == "CHK":
-            s = dict(s, row=3 * (s["row"] // 2) + s["row"] % 2)
-        base.append(s)
-    specs = list(base)
-    for s in base[1::10]:
-        if s.get("target", "DATA") == "DATA" and s["hook"] in ("UPDATE_OUT", "REST"):
-            r2 = (s["row"] // nb) * nb + (s["row"] % nb + 97) % nb
-            if r2 >= s["col"] and r2 != s["row"]:
-                specs.append(dict(s, row=r2, bit=53))
+    specs = syn.next4_injections(n, nb)
     inj = syn.inj_array(specs)
     ref = oracle.potrf(A, nb, inj=inj, nchk=3)
     st, rep, L = run_gpu(P, A, nb, inj=inj)
@@ -135,3 +125,22 @@ def test_mixed_injections_plus_pairs_at_scale(P):
     assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
     if st == 0:
         assert floor_rel(L, ref.L, A) <= 1e-9
+
+
+def test_c4_full_size_events_equal_oracle_golden(P):
+    """C4 (n = 32768, nb = 512) with three checksum rows, the C3-style injections and a second error
+    next to every tenth one: the GPU's full event list equals the oracle's, stored by the committed
+    script tests/golden/make_c4_nchk3_events.py (oracle only)."""
+    import os
+    import torch
+    here = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
+    lines = open(os.path.join(here, "c4_nchk3_events.txt")).read().splitlines()
+    status = int(lines[0].split()[3].rstrip(";"))
+    want = [tuple(int(v) for v in ln.split()) for ln in lines[1:] if ln.strip()]
+    n, nb = 32768, 512
+    A = torch.empty(n, n, dtype=torch.float64, device="cuda").T
+    assert P.abft_gen_spd(n, A) == 0
+    st, rep = P.abft_potrf_ex(n, nb, A, inj=syn.inj_array(syn.next4_injections(n, nb)), opt=P.options(nchk=3))
+    torch.cuda.synchronize()
+    assert st == status == 0
+    assert P.sorted_event_tuples(rep["events"]) == want

@@ -13,7 +13,8 @@ print("gpu", torch.cuda.get_device_properties(0).uuid, flush=True)
 A = torch.empty(n, n, dtype=torch.float64, device="cuda").T
 for it in range(int(os.environ.get("REPS", "2"))):
     P.abft_gen_spd(n, A)
-    st, rep = P.abft_potrf_ex(n, nb, A, inj=syn.inj_array(specs) if specs else None)
+    st, rep = P.abft_potrf_ex(n, nb, A, inj=syn.inj_array(specs) if specs else None,
+                              opt=P.options(nchk=int(os.environ.get("ABFT_NCHK", "2"))))
     torch.cuda.synchronize()
     print(it, "status", st, "n_events", rep["n_events"], P.sorted_event_tuples(rep["events"])[:4], flush=True)
     ev = rep["events"]
