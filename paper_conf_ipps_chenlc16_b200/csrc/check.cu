@@ -11,7 +11,7 @@
 namespace abft {
 
 constexpr int kChkThreads = 256;  // 8 warps
-constexpr int kChkCols = 64;      // tile columns per CTA (8 per warp)
+constexpr int kChkCols = 32;      // tile columns per CTA (4 per warp; the mirrored half of a diagonal tile: 8 row groups)
 
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll

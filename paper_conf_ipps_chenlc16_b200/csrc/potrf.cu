@@ -9,6 +9,8 @@
 // Alg. 2 (chk <- chk L^-T) into one tensor-core GEMM.
 #include "common.cuh"
 
+#include <vector>
+
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
@@ -381,9 +383,12 @@ __device__ __forceinline__ void leaf_store_L(const double* Ls, const LeafSmem& l
     }
 }
 
+// Tasks [t_begin, t_end) of the topological order (one launch = the whole graph, or one chunk of
+// it: the chunked path splits the graph at step boundaries into short launches, see
+// launch_chol_inv); reset_flags: the last chunk's last CTA clears the completion flags.
 __global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int64_t lda, double* Li, int64_t ldi, int T,
-                                                                int ntasks, int64_t info_off, uint32_t* sync,
-                                                                DevState* st, unsigned long long* trace) {
+                                                                int t_begin, int t_end, int reset_flags, int64_t info_off,
+                                                                uint32_t* sync, DevState* st, unsigned long long* trace) {
     extern __shared__ __align__(16) double tsm[];
     double* sA = tsm;
     double* sB = tsm + kTT * kTP;
@@ -405,10 +410,10 @@ __global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int6
     auto Xt = [&](int I, int J) { return Li + (int64_t)J * kTT * ldi + I * kTT; };    // tile (I, J) of inv(L)
     for (;;) {
         __syncthreads();
-        if (tid == 0) s_task = (int)atomicAdd(next, 1u);
+        if (tid == 0) s_task = t_begin + (int)atomicAdd(next, 1u);
         __syncthreads();
         const int t = s_task;
-        if (t >= ntasks) break;
+        if (t >= t_end) break;
         int type, i, j, b;
         decode_task(T, t, type, i, j, b);
         unsigned long long t0 = 0, t1 = 0;
@@ -546,7 +551,8 @@ __global__ void __launch_bounds__(kTaskThreads) k_chol_inv_tasks(double* A, int6
     __syncthreads();
     if (s_go) {
         __threadfence();
-        for (int e = tid; e < task_sync_words(T); e += kTaskThreads) sync[e] = 0u;
+        const int words = reset_flags ? task_sync_words(T) : 2;   // counters always, flags at the end
+        for (int e = tid; e < words; e += kTaskThreads) sync[e] = 0u;
     }
 }
 
@@ -682,10 +688,29 @@ int launch_chol_inv(double* T, int64_t ldt, double* Li, int64_t B, int64_t info_
         static int gmax = -1;
         if (gmax < 0) { const char* e = getenv("ABFT_CHOL_G"); gmax = e ? std::max(1, atoi(e)) : 10; }
         const int Tt = (int)(B / kTT), nt = task_count(Tt);
-        const int grid = std::min(nt, gmax);
-        k_chol_inv_tasks<<<grid, kTaskThreads, kTaskSmem, s>>>(T, ldt, Li, B, Tt, nt, info_off,
-                                                               reinterpret_cast<uint32_t*>(tmp), st, g_chol_trace);
-        abft_count_launch();
+        // ABFT_CHOL_CHUNKS = c > 1: the graph split at step boundaries into c short launches
+        // (long-lived high-priority CTAs are what the bulk-copy update pipeline does not survive,
+        // profiles/r02/race_r02.md); 1 (default): one launch
+        const char* ce = getenv("ABFT_CHOL_CHUNKS");
+        const int chunks = std::max(1, std::min(ce ? atoi(ce) : 1, Tt));
+        std::vector<int> cut(1, 0);
+        {
+            int t = 1;   // after P(0)
+            for (int b = 0; b < Tt; ++b) {
+                t += task_step_count(Tt, b);
+                if ((int)cut.size() < chunks && (b + 1) * chunks / Tt >= (int)cut.size() && t < nt) cut.push_back(t);
+            }
+            cut.push_back(nt);
+        }
+        for (size_t c = 0; c + 1 < cut.size(); ++c) {
+            const int cnt = cut[c + 1] - cut[c];
+            if (cnt <= 0) continue;
+            const int grid = std::min(cnt, gmax);
+            k_chol_inv_tasks<<<grid, kTaskThreads, kTaskSmem, s>>>(T, ldt, Li, B, Tt, cut[c], cut[c + 1],
+                                                                   c + 2 == cut.size() ? 1 : 0, info_off,
+                                                                   reinterpret_cast<uint32_t*>(tmp), st, g_chol_trace);
+            abft_count_launch();
+        }
         return 0;
     }
     launch_zero(B, B, Li, B, s);
