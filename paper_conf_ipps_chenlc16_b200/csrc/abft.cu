@@ -919,6 +919,15 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     // issued on the owner's panel stream.
     ThreadCache& tc = thread_cache();
     cudaStream_t PS = tc.P;
+    // The transport's waiting kernels (NCCL collectives, IPC flag waits) are long-lived CTAs; they
+    // run on a NORMAL-priority comm stream joined to PS by events, because long-lived high-priority
+    // CTAs next to the bulk-copy update are what produced stale operand stages
+    if (tp && !tc.C) ABFT_CUDA_TRY(cudaStreamCreateWithFlags(&tc.C, cudaStreamNonBlocking));
+    cudaStream_t CS = tp ? tc.C : PS;
+    auto hop = [&](cudaStream_t from, cudaStream_t to) {   // `to` waits for everything enqueued on `from`
+        if (from == to) return;
+        cudaEvent_t e = tc.sync.get(); cudaEventRecord(e, from); cudaStreamWaitEvent(to, e, 0);
+    };
     auto new_event = [&]() { return tc.sync.get(); };
     {   // panel stream starts after the encode
         cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(PS, e, 0);
@@ -983,7 +992,9 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             // checksum rows locally and the whole packed panel (+ abort slot) into every peer's
             // receive buffer (peer stores), once every peer released that buffer
             launch_abort_to_slot(ab, q.w.W + wcount, PS);
-            if (tp->wait_free(k, PS)) return ABFT_ERR_NCCL;
+            hop(PS, CS);
+            if (tp->wait_free(k, CS)) return ABFT_ERR_NCCL;
+            hop(CS, PS);
             std::vector<double*> peers;
             for (int r = 0; r < P; ++r) if (r != q.r) peers.push_back(tp->recv_buf(r, (int)(k & 1)));
             launch_panel_out(q.w.W, ldw, mB, abft ? 2 * m + 2 : 0, B, Akk + B, q.lda, ckk + 2 * k, q.w.ldc, peers.data(),
@@ -1007,9 +1018,13 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         for (int i = 0; i < nlocal; ++i)   // the receive buffer Wb[k & 1] was last read by update k-2
             if (evUprev[i]) cudaStreamWaitEvent(PS, evUprev[i], 0);
         if (tp && push) {
-            if (R[0].r != owner && tp->wait_panel(owner, k, PS)) return ABFT_ERR_NCCL;   // pushed by the owner
+            hop(PS, CS);
+            if (R[0].r != owner && tp->wait_panel(owner, k, CS)) return ABFT_ERR_NCCL;   // pushed by the owner
+            hop(CS, PS);
         } else if (tp) {
-            if (tp->bcast(R[0].Wb[k & 1], (wcount + 1) * sizeof(double), owner, PS)) return ABFT_ERR_NCCL;
+            hop(PS, CS);
+            if (tp->bcast(R[0].Wb[k & 1], (wcount + 1) * sizeof(double), owner, CS)) return ABFT_ERR_NCCL;
+            hop(CS, PS);
         } else {
             const RankState* src = nullptr;
             for (auto& q : R) if (q.r == owner) src = &q;

@@ -30,12 +30,16 @@ def run_block(P, A):
     return st, P.to_numpy_colmajor(At), P.to_numpy_colmajor(Li)
 
 
-@pytest.fixture(params=["tasks", "rec"])
+@pytest.fixture(params=["tasks", "tasks_chunked", "rec"])
 def chol_path(request, monkeypatch):
-    """Both diagonal-block paths: the recursive multi-launch path (default) and the one-launch
-    task graph (ABFT_CHOL=tasks, nb % 64 == 0, nb >= 128), read by the library per call."""
-    if request.param == "tasks":
+    """The diagonal-block paths: the recursive multi-launch path (default), the one-launch task
+    graph (ABFT_CHOL=tasks, nb % 64 == 0, nb >= 128) and the same graph split into short launches
+    at its step boundaries (ABFT_CHOL_CHUNKS), all read by the library per call."""
+    monkeypatch.delenv("ABFT_CHOL_CHUNKS", raising=False)
+    if request.param.startswith("tasks"):
         monkeypatch.setenv("ABFT_CHOL", "tasks")
+        if request.param == "tasks_chunked":
+            monkeypatch.setenv("ABFT_CHOL_CHUNKS", "3")
     else:
         monkeypatch.delenv("ABFT_CHOL", raising=False)
     return request.param
