@@ -852,7 +852,7 @@ static int ws_slab_rows() { return ws_variant() == 16 ? WsCfg16::WM : 64; }
 // profiles/race_r02.md), the LDGSTS pipeline never. So that path takes the LDGSTS producer.
 static bool tasks_path() {
     const char* e = getenv("ABFT_CHOL");
-    return e && !strcmp(e, "tasks");
+    return (e && !strcmp(e, "tasks")) || g_fast_diag;
 }
 static int run_ws_any(GemmArgs g, cudaStream_t s) {
     g.cs.slab_rows = ws_slab_rows();

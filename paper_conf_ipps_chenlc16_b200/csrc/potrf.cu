@@ -587,6 +587,10 @@ size_t chol_sync_bytes(int64_t nb) {   // <= the scratch `tmp` callers allocate 
 
 static thread_local unsigned long long* g_chol_trace = nullptr;   // abft_dev_chol_trace only
 void chol_set_trace(unsigned long long* t) { g_chol_trace = t; }
+// set by run_dist for P >= 4 ranks (DESIGN.md §5 P-model): the one-launch task-graph diagonal
+// block shortens the owner's serial panel chain; the update then takes the LDGSTS producer
+// (gemm.cu run_ws_any), the combination that is clean under concurrent high-priority work
+thread_local int g_fast_diag = 0;
 int chol_task_count(int64_t nb) { return (nb % kTT == 0 && nb / kTT <= 32) ? task_count((int)(nb / kTT)) : 0; }
 
 // Path choice. Default: the recursive multi-launch path. ABFT_CHOL=tasks selects the one-launch
@@ -598,7 +602,7 @@ int chol_task_count(int64_t nb) { return (nb % kTT == 0 && nb / kTT <= 32) ? tas
 // paths inside one process).
 static bool use_tasks(const double* T, int64_t ldt, int64_t B) {
     const char* e = getenv("ABFT_CHOL");
-    return ((e && !strcmp(e, "tasks")) || g_chol_trace != nullptr) && B % kTT == 0 && B >= 2 * kTT && B / kTT <= 32 && ((uintptr_t)T & 15) == 0 && ldt % 2 == 0;
+    return ((e && !strcmp(e, "tasks")) || g_chol_trace != nullptr || g_fast_diag) && B % kTT == 0 && B >= 2 * kTT && B / kTT <= 32 && ((uintptr_t)T & 15) == 0 && ldt % 2 == 0;
 }
 
 int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,

@@ -45,7 +45,7 @@ def test_sim_fault_free(P, Pn, n, nb):
     assert rep["n_checks"] == ref.counts["n_checks"]
 
 
-@pytest.mark.parametrize("Pn", [2, 3])
+@pytest.mark.parametrize("Pn", [2, 3, 4])
 def test_sim_injections_including_recv(P, Pn):
     n, nb = 1024, 128
     A = syn.spd_matrix(n)
@@ -55,6 +55,25 @@ def test_sim_injections_including_recv(P, Pn):
     inj = syn.inj_array(specs)
     ref = oracle.potrf(A, nb, inj=inj, nranks=Pn)
     st, rep, L = run_sim(P, A, nb, Pn, inj=inj)
+    assert st == ref.status == 0
+    assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
+    assert floor_rel(L, ref.L, A) <= 1e-11
+
+
+@pytest.mark.parametrize("diag", ["default", "recursive"])
+def test_sim_four_ranks_c4_block_size(P, diag, monkeypatch):
+    """P = 4 at the C4 block size: run_dist selects the task-graph diagonal block + LDGSTS update
+    producer for P >= 4 (DESIGN.md §5 P-model); ABFT_DIST_DIAG=recursive restores the single-GPU
+    configuration. Both: same events as the oracle's 4-rank simulation, factor within 1e-11."""
+    if diag != "default":
+        monkeypatch.setenv("ABFT_DIST_DIAG", diag)
+    n, nb = 4096, 512
+    A = syn.spd_matrix(n, seed=5)
+    specs = syn.per_iteration_injections(n, nb, bits=(45, 61))
+    specs.append(dict(k=2, hook="RECV", row=3000, col=1100, bit=51, rank=3))
+    inj = syn.inj_array(specs)
+    ref = oracle.potrf(A, nb, inj=inj, nranks=4)
+    st, rep, L = run_sim(P, A, nb, 4, inj=inj)
     assert st == ref.status == 0
     assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
     assert floor_rel(L, ref.L, A) <= 1e-11
