@@ -855,20 +855,6 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     if (collect_inj(inj_c, n, nb, inj)) return -9;
     if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; }
     if (n == 0) return 0;
-    // P >= 4: the owner's panel chain bounds most iterations (DESIGN.md §5 P-model), so the diagonal
-    // block runs as the one-launch task graph and the update takes the LDGSTS producer (the pair that
-    // is clean under concurrent high-priority work, profiles/r02/race_r02.md); ABFT_DIST_DIAG =
-    // recursive | tasks overrides
-    struct FastDiag {
-        int prev;
-        explicit FastDiag(int on) : prev(g_fast_diag) { g_fast_diag = on; }
-        ~FastDiag() { g_fast_diag = prev; }
-    } fast_diag([&] {
-        const char* e = getenv("ABFT_DIST_DIAG");
-        if (e && !strcmp(e, "recursive")) return 0;
-        if (e && !strcmp(e, "tasks")) return 1;
-        return P >= 4 ? 1 : 0;
-    }());
     const bool abft = o.abft_enabled != 0;
     const int K = std::max(1, o.K);
     const int64_t N = n / nb, B = nb;

@@ -298,9 +298,6 @@ int launch_trsm_with_chk(int64_t mB, int64_t B, const double* Ap, int64_t lda, c
                          cudaStream_t s);
 // Returns a bit mask: 1 = the fused V5 partials were written, 2 = the epilogue applied `inj`
 // (the caller applies the hook itself otherwise); -1 if cstride > 1 and the shapes do not allow it.
-// potrf.cu: nonzero while run_dist factors with P >= 4 ranks (task-graph diagonal block + LDGSTS
-// update producer)
-extern thread_local int g_fast_diag;
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s,

@@ -352,7 +352,8 @@ __device__ __forceinline__ void prefetch_l2(const void* src, uint32_t bytes) {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(src), "r"(bytes) : "memory");
 }
 
-template <int BM_, int BN_, int BK_, int STAGES_, int WM_, int WN_, int REG_CONS_, int MINB_, bool LDG_ = false>
+template <int BM_, int BN_, int BK_, int STAGES_, int WM_, int WN_, int REG_CONS_, int MINB_, bool LDG_ = false,
+          bool IDLE_EXIT_ = false, bool CFENCE_ = true>
 struct WsCfgT {
     static constexpr int BM = BM_, BN = BN_, BK = BK_, WM = WM_, WN = WN_, STAGES = STAGES_, MINB = MINB_;
     // LDG: the producer stages operands with per-lane 16-byte cp.async (LDGSTS) and signals the
@@ -360,6 +361,14 @@ struct WsCfgT {
     // a transaction count (the bulk-copy pipeline picked up rare stale k-slices
     // under concurrent high-priority work; the LDGSTS one did not)
     static constexpr bool LDG = LDG_;
+    // IDLE_EXIT (dev variant 2x, the round-2 kernel): with bulk copies the three idle producer warps
+    // returned right after setmaxnreg.dec instead of waiting at the tail barrier
+    static constexpr bool IDLE_EXIT = IDLE_EXIT_;
+    // CFENCE (bulk copies): consumers issue fence.proxy.async before releasing a stage, ordering
+    // their generic-proxy fragment loads (LDS) before the producer's next async-proxy (bulk) write
+    // into that stage. Without it a delayed LDS could read the k-slice two stages later (a wrong
+    // row of one warp tile, seen under concurrent high-priority work; profiles/r02/race_r02.md)
+    static constexpr bool CFENCE = CFENCE_;
     static constexpr int WARPS_M = BM / WM, WARPS_N = BN / WN, CONSUMERS = WARPS_M * WARPS_N;
     static constexpr int THREADS = (CONSUMERS + 4) * 32;   // + one producer warpgroup (setmaxnreg)
     static constexpr int REG_CONS = REG_CONS_, REG_PROD = LDG_ ? 56 : 40;
@@ -377,7 +386,9 @@ using WsCfg = WsCfgT<128, 128, 32, 3, 64, 32, 232, 1>;    // 8 consumer warps, 1
 using WsCfg16 = WsCfgT<128, 128, 32, 3, 32, 32, 104, 1>;  // 16 consumer warps, 32x32 warp tiles
 using WsCfg2a = WsCfgT<128, 64, 16, 4, 64, 32, 216, 2>;   // 2 CTAs/SM, 128x64 tiles, 4-stage BK=16
 using WsCfg2b = WsCfgT<128, 64, 32, 2, 64, 32, 216, 2>;   // 2 CTAs/SM, 128x64 tiles, 2-stage BK=32
+using WsCfg2nf = WsCfgT<128, 64, 32, 2, 64, 32, 216, 2, false, false, false>;  // dev: 2b without the consumer proxy fence
 using WsCfg2l = WsCfgT<128, 64, 32, 2, 64, 32, 200, 2, true>;   // as 2b, LDGSTS producer warpgroup
+using WsCfg2x = WsCfgT<128, 64, 32, 2, 64, 32, 216, 2, false, true, false>;   // dev: 2nf + idle producer warps exit (round-2 kernel)
 using WsCfgNR = WsCfgT<128, 64, 32, 2, 64, 32, 128, 2>;   // dev: as 2b without setmaxnreg (spills)
 
 // tile index -> (tm, tn) for the three masks; returns false for tiles with nothing to write
@@ -474,7 +485,7 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
     double* sB = smem + STAGES * C_::SA;
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * (C_::SA + C_::SB));
     uint64_t* empty = full + STAGES;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int tid = threadIdx.x, lane = tid & 31, warp = __shfl_sync(0xffffffffu, tid >> 5, 0);   // warp-uniform
     if (tid == 0) {
         for (int i = 0; i < STAGES; ++i) { mbar_init(&full[i], C_::LDG ? 128 : 1); mbar_init(&empty[i], C_::CONSUMERS); }
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
@@ -485,7 +496,13 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
         // ------------------------------- producer -------------------------------
         if constexpr (C_::REG_CONS != C_::R0)
             asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;\n" ::"n"(C_::REG_PROD) : "memory");
-        if (!C_::LDG && warp != C_::CONSUMERS) return;   // LDGSTS: the whole warpgroup copies
+        // bulk copies: one warp issues them; the other three warps of the producer warpgroup idle
+        // at the tail barrier below instead of exiting (variant 2x restores the early exit for the
+        // race matrix, profiles/r02/race_r02.md)
+        if (!C_::LDG && warp != C_::CONSUMERS) {
+            if constexpr (!C_::IDLE_EXIT) asm volatile("bar.sync 1, %0;\n" ::"n"((C_::CONSUMERS + 4) * 32) : "memory");
+            return;
+        }
         const int ptid = tid - C_::CONSUMERS * 32;       // 0..127 in the producer warpgroup
         const int64_t pf_ahead = (C_::LDG && warp != C_::CONSUMERS) ? 0 : g.pf_ahead;
         uint32_t it = 0;
@@ -563,10 +580,12 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
             }
         }
         if constexpr (!C_::LDG) {
-            // producer tail: the copying warp stays resident until the consumers have finished
-            // (named barrier 1: this warp waits, the consumer warps arrive at their end), so it
-            // never exits while bulk copies it issued may still be in flight
-            asm volatile("bar.sync 1, %0;\n" ::"n"((C_::CONSUMERS + 1) * 32) : "memory");
+            // producer tail: the producer warps stay resident until the consumers have finished
+            // (named barrier 1: these warps wait, the consumer warps arrive at their end), so no
+            // warp of the CTA exits while bulk copies may still be in flight or while the
+            // consumers run on registers the producer warpgroup released with setmaxnreg.dec
+            if constexpr (C_::IDLE_EXIT) asm volatile("bar.sync 1, %0;\n" ::"n"((C_::CONSUMERS + 1) * 32) : "memory");
+            else asm volatile("bar.sync 1, %0;\n" ::"n"((C_::CONSUMERS + 4) * 32) : "memory");
         }
         return;
     }
@@ -635,6 +654,7 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
 #pragma unroll
                     for (int j = 0; j < C_::FN; ++j) dmma(acc[i][j][0], acc[i][j][1], af[i], bf[j]);
             }
+            if constexpr (C_::CFENCE && !C_::LDG) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
             __syncwarp();
             if (lane == 0) mbar_arrive(&empty[st]);
         }
@@ -770,7 +790,10 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
         }
     }
     // release the copying producer warp (its tail waits on named barrier 1)
-    if constexpr (!C_::LDG) asm volatile("bar.arrive 1, %0;\n" ::"n"((C_::CONSUMERS + 1) * 32) : "memory");
+    if constexpr (!C_::LDG) {
+        if constexpr (C_::IDLE_EXIT) asm volatile("bar.arrive 1, %0;\n" ::"n"((C_::CONSUMERS + 1) * 32) : "memory");
+        else asm volatile("bar.arrive 1, %0;\n" ::"n"((C_::CONSUMERS + 4) * 32) : "memory");
+    }
 }
 
 // Two entry points with one body, so that profiles attribute the trailing update (the dominant
@@ -828,10 +851,12 @@ bool is_update_kernel(const void* f) {
     return f == (const void*)k_update_ws<WsCfg> || f == (const void*)k_update_ws<WsCfg16> ||
            f == (const void*)k_update_ws<WsCfg2a> || f == (const void*)k_update_ws<WsCfg2b> ||
            f == (const void*)k_update_ws<WsCfgNR> || f == (const void*)k_update_ws<WsCfg2l> ||
-           f == (const void*)k_update_ws<WsCfg2b, true> || f == (const void*)k_update_ws<WsCfg2l, true>;
+           f == (const void*)k_update_ws<WsCfg2b, true> || f == (const void*)k_update_ws<WsCfg2l, true> ||
+           f == (const void*)k_update_ws<WsCfg2x> || f == (const void*)k_update_ws<WsCfg2x, true> ||
+           f == (const void*)k_update_ws<WsCfg2nf> || f == (const void*)k_update_ws<WsCfg2nf, true>;
 }
 
-static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CTA/SM), 16, 2a
+static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CTA/SM), 16, 2a, 2l, 2nf, 2x, nr
     static int v = -1;
     if (v < 0) {
         const char* e = getenv("ABFT_WS");
@@ -842,26 +867,22 @@ static int ws_variant() {   // dev knob ABFT_WS: 2b (default), 1 (one 128x128 CT
         if (e && !strcmp(e, "2b")) v = 22;
         if (e && !strcmp(e, "2l")) v = 25;
         if (e && !strcmp(e, "nr")) v = 24;
+        if (e && !strcmp(e, "2x")) v = 26;
+        if (e && !strcmp(e, "2nf")) v = 27;
     }
     return v;
 }
 static int ws_slab_rows() { return ws_variant() == 16 ? WsCfg16::WM : 64; }
-// The one-launch task-graph diagonal block (ABFT_CHOL=tasks) keeps long-lived CTAs on the
-// high-priority panel stream; under that concurrency the bulk-copy (cp.async.bulk) operand
-// pipeline was measured to deliver stale k-slices to the update's consumers (DESIGN.md §5,
-// profiles/race_r02.md), the LDGSTS pipeline never. So that path takes the LDGSTS producer.
-static bool tasks_path() {
-    const char* e = getenv("ABFT_CHOL");
-    return (e && !strcmp(e, "tasks")) || g_fast_diag;
-}
+
 static int run_ws_any(GemmArgs g, cudaStream_t s) {
     g.cs.slab_rows = ws_slab_rows();
     const bool upd = g.mask == MASK_LOWER && g.alpha == -1.0 && g.beta == 1.0;   // a trailing update
-    if (upd && tasks_path() && getenv("ABFT_WS_FORCE_BULK") == nullptr) return run_ws<WsCfg2l>(g, s, upd);
     switch (ws_variant()) {
         case 16: return run_ws<WsCfg16>(g, s, upd);
         case 21: return run_ws<WsCfg2a>(g, s, upd);
         case 22: return run_ws<WsCfg2b>(g, s, upd);
+        case 26: return run_ws<WsCfg2x>(g, s, upd);
+        case 27: return run_ws<WsCfg2nf>(g, s, upd);
         case 25: return run_ws<WsCfg2l>(g, s, upd);
         case 24: return run_ws<WsCfgNR>(g, s, upd);
         default: return run_ws<WsCfg>(g, s, upd);

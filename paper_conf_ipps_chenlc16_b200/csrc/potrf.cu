@@ -587,22 +587,17 @@ size_t chol_sync_bytes(int64_t nb) {   // <= the scratch `tmp` callers allocate 
 
 static thread_local unsigned long long* g_chol_trace = nullptr;   // abft_dev_chol_trace only
 void chol_set_trace(unsigned long long* t) { g_chol_trace = t; }
-// set by run_dist for P >= 4 ranks (DESIGN.md §5 P-model): the one-launch task-graph diagonal
-// block shortens the owner's serial panel chain; the update then takes the LDGSTS producer
-// (gemm.cu run_ws_any), the combination that is clean under concurrent high-priority work
-thread_local int g_fast_diag = 0;
 int chol_task_count(int64_t nb) { return (nb % kTT == 0 && nb / kTT <= 32) ? task_count((int)(nb / kTT)) : 0; }
 
-// Path choice. Default: the recursive multi-launch path. ABFT_CHOL=tasks selects the one-launch
-// task graph (nb % 64 == 0, nb >= 128, 16-byte aligned, even leading dimension): 2x faster on its
-// own, but on the high-priority look-ahead stream its long-lived CTAs were measured to provoke
-// what behaves like compute preemption of the warp-specialised update GEMM, whose output then
-// carried rare row-group errors (detected and corrected by V5; none with the panel stream at
-// normal priority, which in turn delays the panel) -- DESIGN.md §5. Read per call (tests switch
+// Path choice. Default: the one-launch task graph (nb % 64 == 0, nb >= 128, 16-byte aligned, even
+// leading dimension; about 3x faster than the recursive path on its own). ABFT_CHOL=recursive
+// selects the recursive multi-launch path. (Until the update kernel's consumer proxy fence, the
+// task graph's long-lived high-priority CTAs exposed a stage-release race in the bulk-copy update
+// pipeline, so it was opt-in: profiles/r02/race_r02.md.) Read per call (tests switch
 // paths inside one process).
 static bool use_tasks(const double* T, int64_t ldt, int64_t B) {
     const char* e = getenv("ABFT_CHOL");
-    return ((e && !strcmp(e, "tasks")) || g_chol_trace != nullptr || g_fast_diag) && B % kTT == 0 && B >= 2 * kTT && B / kTT <= 32 && ((uintptr_t)T & 15) == 0 && ldt % 2 == 0;
+    return (!(e && !strcmp(e, "recursive")) || g_chol_trace != nullptr) && B % kTT == 0 && B >= 2 * kTT && B / kTT <= 32 && ((uintptr_t)T & 15) == 0 && ldt % 2 == 0;
 }
 
 int launch_copy(int64_t rows, int64_t cols, const double* src, int64_t lds, double* dst, int64_t ldd,

@@ -32,16 +32,17 @@ def run_block(P, A):
 
 @pytest.fixture(params=["tasks", "tasks_chunked", "rec"])
 def chol_path(request, monkeypatch):
-    """The diagonal-block paths: the recursive multi-launch path (default), the one-launch task
-    graph (ABFT_CHOL=tasks, nb % 64 == 0, nb >= 128) and the same graph split into short launches
-    at its step boundaries (ABFT_CHOL_CHUNKS), all read by the library per call."""
+    """The diagonal-block paths: the one-launch task graph (default where nb % 64 == 0,
+    nb >= 128), the same graph split into short launches at its step boundaries
+    (ABFT_CHOL_CHUNKS) and the recursive multi-launch path (ABFT_CHOL=recursive), all read by the
+    library per call."""
     monkeypatch.delenv("ABFT_CHOL_CHUNKS", raising=False)
     if request.param.startswith("tasks"):
-        monkeypatch.setenv("ABFT_CHOL", "tasks")
+        monkeypatch.delenv("ABFT_CHOL", raising=False)
         if request.param == "tasks_chunked":
             monkeypatch.setenv("ABFT_CHOL_CHUNKS", "3")
     else:
-        monkeypatch.delenv("ABFT_CHOL", raising=False)
+        monkeypatch.setenv("ABFT_CHOL", "recursive")
     return request.param
 
 

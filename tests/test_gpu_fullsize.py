@@ -192,18 +192,20 @@ def test_c3_whole_factor_vs_oracle_mixed_injections(P, c3_runs):
 @pytest.mark.parametrize("path", ["recursive", "tasks"])
 def test_fault_free_runs_raise_no_event(P, path, monkeypatch):
     """Fault-free factorisations must raise no correction (Tables VII/VIII 'no error' columns,
-    PAPER.md:362-377): 5 back-to-back C4 runs on the default diagonal-block path and on the
-    one-launch task-graph path, each asserting status 0 and zero events, and the noise margin."""
+    PAPER.md:362-377): 10 back-to-back C4 runs on the default (task-graph) diagonal-block path
+    and on the recursive one, each asserting status 0 and zero events, and the noise margin. (The
+    update kernel's stage-release race showed up in about 1-3 % of such runs before the consumer
+    proxy fence, profiles/r02/race_r02.md.)"""
     import torch
     if path == "tasks":
-        monkeypatch.setenv("ABFT_CHOL", "tasks")
+        monkeypatch.delenv("ABFT_CHOL", raising=False)
     else:
         monkeypatch.setenv("ABFT_CHOL", "recursive")
     n, nb = 32768, 512
     A0 = torch.empty(n, n, dtype=torch.float64, device="cuda").T
     assert P.abft_gen_spd(n, A0) == 0
     A = torch.empty_like(A0.T).T
-    for rep_i in range(5):
+    for rep_i in range(10):
         A.copy_(A0)
         st, rep = P.abft_potrf_ex(n, nb, A, cap=64)
         torch.cuda.synchronize()
