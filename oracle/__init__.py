@@ -70,6 +70,10 @@ def lib():
                                            vp, i64, ctypes.POINTER(i64), ctypes.POINTER(i64), vp, vp, vp,
                                            ctypes.POINTER(i32), i32]
         _lib.oracle_potrf_nchk.restype = i32
+        _lib.oracle_potrf_grid.argtypes = [i64, i64, vp, i64, vp, i64, i32, i32, i32, ctypes.c_double, i32, i32,
+                                           i32, vp, i64, ctypes.POINTER(i64), ctypes.POINTER(i64), vp, vp, vp,
+                                           ctypes.POINTER(i32), i32]
+        _lib.oracle_potrf_grid.restype = i32
         _lib.oracle_encode.argtypes = [i64, i64, vp, i64, vp, i64, vp]
         _lib.oracle_encode.restype = i32
         _lib.oracle_verify.argtypes = [i64, i64, vp, i64, vp, i64, vp, i32, i32, ctypes.c_double,
@@ -110,14 +114,18 @@ MODE = {"enhanced": 0, "online": 1, "offline": 2, "enhanced_redo": 3}
 
 
 def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, inplace=False, mode="enhanced",
-          order="right", nchk=2):
+          order="right", nchk=2, prows=1):
     """ABFT Cholesky of A (lower), n % nb == 0. mode: "enhanced" (the paper's scheme, default),
     "online" or "offline" (its comparison schemes, which re-run once on an uncorrectable error).
     nchk: checksum rows per block, 2 (the paper's choice) or 3 (m+1 = 3 checksums locate and
     correct up to m = 2 errors per column; reading B10). Checksum-row injection targets are
     rows nchk*I + t of the checksum matrix.
     Returns Result with L in the lower triangle (upper triangle untouched), status (0/1/2),
-    LAPACK info, sorted events, reruns."""
+    LAPACK info, sorted events, reruns.
+    nranks > 1 simulates the multi-GPU path: process grid prows x (nranks / prows), tile (I, J) owned
+    by rank (I % prows) * (nranks / prows) + J % (nranks / prows) (prows = 1: 1D column-cyclic;
+    prows > 1: 2D block-cyclic); events carry the checking rank, every rank
+    re-checks the panel tiles it receives (V4R) after its RECV hook."""
     L = _as_f(A)
     if not inplace:
         L = L.copy(order="F")
@@ -134,7 +142,7 @@ def potrf(A, nb, inj=None, nranks=1, K=1, c_tau=64.0, abft=True, cap=1 << 16, in
     chk = np.zeros((max(nchk * N, 1), n), dtype=np.float64, order="F")
     scl = np.zeros(n + 3 * N, dtype=np.float64)
     reruns = ctypes.c_int(0)
-    st = lib().oracle_potrf_nchk(n, nb, _ptr(L), max(n, 1), _ptr(inj_arr), ninj, nranks, K, c_tau, int(abft),
+    st = lib().oracle_potrf_grid(n, nb, _ptr(L), max(n, 1), _ptr(inj_arr), ninj, nranks, prows, K, c_tau, int(abft),
                                  MODE[mode] if isinstance(mode, str) else int(mode),
                                  {"right": 0, "left": 1}[order], _ptr(ev), cap,
                                  ctypes.byref(nev), ctypes.byref(info), _ptr(cnt), _ptr(chk), _ptr(scl),

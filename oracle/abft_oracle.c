@@ -64,6 +64,9 @@ typedef struct {
     double *A, *chk, *s, *S1, *S2, *S3;
     double c_tau, rho;
     int nranks, K, correct;
+    int prows;                     /* P>1 simulation: process grid prows x (nranks / prows); tile (I,J)
+                                      belongs to rank (I mod prows) * pcols + (J mod pcols) — 2D
+                                      block-cyclic; prows = 1 is the 1D column cyclic */
     int mode;                      /* 0 Enhanced Online-ABFT, 1 Online-ABFT, 2 Offline-ABFT */
     const oinj_t* inj; int64_t ninj;
     oevent_t* ev; int64_t cap, nev;
@@ -150,9 +153,15 @@ static int locate_two(double d1, double d2, double d3, double tau1, double tau2,
     return found == 1;
 }
 
+/* the rank that owns (stores, updates and checks) tile (I, J) of the P>1 simulation */
+static int tile_owner(const octx_t* x, int64_t I, int64_t J) {
+    const int pr = x->prows > 0 ? x->prows : 1, pc = x->nranks / pr;
+    return (int)((I % pr) * pc + (J % pc));
+}
+
 static int check_tile(octx_t* x, const tview_t* v, int k, int V, int rank) {
     const int64_t B = x->B;
-    if (V != O_V4R) rank = (int)(v->J % x->nranks);    /* the owner of block column J runs the check */
+    if (V != O_V4R) rank = tile_owner(x, v->I, v->J);   /* the owner of tile (I, J) runs the check */
     odec_t* dec = (odec_t*)malloc(sizeof(odec_t) * (size_t)B);
     int64_t nd = 0;
     x->cnt->n_checks++;
@@ -417,8 +426,8 @@ static void trsm_panel(octx_t* x, int64_t k) {
 }
 
 /* ---- trailing update: T(i,j) -= L_ik L_jk^T, chk(i,j) -= chk(i,k) L_jk^T ---
- * Lp(j) gives the panel copy that the owner of column j holds (P>1 simulation); at P=1
- * every Lp is the panel stored in A / chk. */
+ * pan_of_rank[r] is the panel copy rank r holds (P>1 simulation); tile (i, j) is updated by its
+ * owner with that rank's copy. At P=1 every copy is the panel stored in A / chk. */
 typedef struct { const double* L; int64_t ldl; const double* C; int64_t ldcc; } panel_t;
 
 static void update(octx_t* x, int64_t k, const panel_t* pan_of_rank) {
@@ -434,7 +443,7 @@ static void update(octx_t* x, int64_t k, const panel_t* pan_of_rank) {
             int64_t jj = 0, rem = q;
             while (rem >= m - jj) { rem -= m - jj; jj++; }
             const int64_t j = k + 1 + jj, i = j + rem;
-            const panel_t* P = &pan_of_rank[j % x->nranks];
+            const panel_t* P = &pan_of_rank[tile_owner(x, i, j)];   /* that rank's panel copy */
             const double* Lik = P->L + (i - k - 1) * B;      /* rows of L_ik inside the panel */
             const double* Ljk = P->L + (j - k - 1) * B;
             double* T = x->A + j * B * x->lda + i * B;
@@ -484,7 +493,8 @@ static int64_t g_kstop = INT64_MAX;
 
 static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
                       int nranks, int K, double c_tau, int abft, int mode, oevent_t* ev, int64_t cap,
-                      int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out, int nchk) {
+                      int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out, int nchk,
+                      int prows) {
     octx_t X_; octx_t* x = &X_;
     memset(x, 0, sizeof *x);
     x->cnt = cnt;
@@ -492,7 +502,7 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
     x->nchk = nchk;
     x->n = n; x->B = nb; x->N = n / nb; x->lda = lda; x->ldc = nchk * x->N > 0 ? nchk * x->N : 1;
     x->A = A; x->c_tau = c_tau > 0 ? c_tau : 64.0; x->rho = 0x1p-30;   /* [A4, A6] */
-    x->nranks = nranks; x->K = K; x->correct = 1;
+    x->nranks = nranks; x->prows = prows; x->K = K; x->correct = 1;
     x->inj = inj; x->ninj = ninj; x->ev = ev; x->cap = cap;
     if (info) *info = 0;
     if (n == 0) { if (nev) *nev = 0; return 0; }
@@ -510,7 +520,6 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
 
     if (abft) { scales(x); encode(x); }
     for (int64_t k = 0; k < N && k < g_kstop && x->status == O_OK; ++k) {
-        const int owner = (int)(k % nranks);
         if (abft) {
             inject(x, (int)k, O_HOOK_REST, 0, x->A, lda, x->chk, x->ldc);
             if (mode == 0 && run_checks_column(x, k, 0, O_V1, O_V2, 1)) break;   /* V1, V2 */
@@ -532,9 +541,14 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
             pan[r].C = x->chk + k * B * x->ldc + nc * (k + 1); pan[r].ldcc = x->ldc;
         }
         if (abft && mode == 0 && nranks > 1 && m > 0) {                     /* RECV + V4R */
+            /* every rank receives the panel tiles (i, k), i > k, that it does not own (their
+             * owners solved them; at prows = 1 that is the whole panel from the owner of column
+             * k), applies its RECV hook to its copy and re-checks the tiles it received */
             int stop = 0;
             for (int r = 0; r < nranks && !stop; ++r) {
-                if (r == owner) continue;
+                int received = 0;
+                for (int64_t i = k + 1; i < N; ++i) received |= (tile_owner(x, i, k) != r);
+                if (!received) continue;
                 double* Lr = rcopy + (size_t)r * n * B;     /* receiver buffer: m*B x B, ld = m*B */
                 double* Cr = rchk + (size_t)r * nc * N * B;  /* nc m x B, ld = nc m               */
                 const int64_t ldl = m * B, ldr = nc * m;
@@ -542,14 +556,18 @@ static int potrf_core(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
                     memcpy(Lr + c * ldl, x->A + (k * B + c) * lda + (k + 1) * B, sizeof(double) * (size_t)(m * B));
                     for (int64_t q = 0; q < nc * m; ++q) Cr[c * ldr + q] = x->chk[(k * B + c) * x->ldc + nc * (k + 1) + q];
                 }
-                /* RECV(k, r): target (row, col) global -> receiver buffer coordinates */
+                /* RECV(k, r): target (row, col) global -> receiver buffer coordinates; a target in a
+                 * tile rank r owns is not received by it (no effect) */
                 for (int64_t t = 0; t < ninj; ++t) {
                     const oinj_t* s = &inj[t];
                     if (s->k != k || s->hook != O_HOOK_RECV || s->rank != r) continue;
+                    const int64_t ti = s->target == O_TGT_DATA ? s->row / B : s->row / nc;
+                    if (tile_owner(x, ti, k) == r) continue;
                     if (s->target == O_TGT_DATA) xor_double(&Lr[(s->col - k * B) * ldl + (s->row - (k + 1) * B)], s->xor_mask);
                     else xor_double(&Cr[(s->col - k * B) * ldr + (s->row - nc * (k + 1))], s->xor_mask);
                 }
                 for (int64_t i = k + 1; i < N && !stop; ++i) {
+                    if (tile_owner(x, i, k) == r) continue;
                     tview_t v;
                     v.T = Lr + (i - k - 1) * B; v.ldt = ldl;
                     v.c1 = Cr + nc * (i - k - 1); v.c2 = v.c1 + 1; v.ldc = ldr;
@@ -720,11 +738,15 @@ static int potrf_core_left(int64_t n, int64_t nb, double* A, int64_t lda, const 
  * scheme with the same re-do for what two checksums cannot correct (more than one error in a
  * column of a block, P:121 [A11]): an UNCORRECTABLE outcome re-runs once.
  * Events of both runs are returned in order. */
-int oracle_potrf_nchk(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
-                      int nranks, int K, double c_tau, int abft, int mode, int order, oevent_t* ev, int64_t cap,
-                      int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out,
+/* prows (P>1 simulation): 2D block-cyclic process grid prows x (nranks / prows);
+ * 1 = the 1D column-cyclic distribution. The arithmetic of every tile is that of one process; only
+ * which rank checks a tile, and which rank's received panel copy an update reads, depend on it. */
+int oracle_potrf_grid(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
+                      int nranks, int prows, int K, double c_tau, int abft, int mode, int order, oevent_t* ev,
+                      int64_t cap, int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out,
                       int* reruns, int nchk) {
     if (n < 0) return -1;
+    if (prows < 1 || nranks < 1 || nranks % prows) return -13;
     if (nchk != 2 && nchk != 3) return -12;
     if (nb < 1) return -2;
     if (n % nb) return -2;                          /* [A20] */
@@ -746,7 +768,7 @@ int oracle_potrf_nchk(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
     if (order != 0 && nranks != 1) return -7;
     int64_t nev1 = 0;
     int st = order == 0 ? potrf_core(n, nb, A, lda, inj, ninj, nranks, K, c_tau, abft, mode, ev, cap, &nev1, info, c,
-                                     chk_out, scl_out, nchk)
+                                     chk_out, scl_out, nchk, prows)
                         : potrf_core_left(n, nb, A, lda, inj, ninj, K, c_tau, abft, mode, ev, cap, &nev1, info, c,
                                           chk_out, scl_out, nchk);
     /* Online / Offline: a detection at the final sweep means an error escaped the scheme's
@@ -759,7 +781,7 @@ int oracle_potrf_nchk(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
         int64_t nev2 = 0;
         const int64_t off = nev1 < cap ? nev1 : cap;
         st = order == 0 ? potrf_core(n, nb, A, lda, NULL, 0, nranks, K, c_tau, abft, mode, ev ? ev + off : NULL,
-                                     cap - off, &nev2, info, c, chk_out, scl_out, nchk)
+                                     cap - off, &nev2, info, c, chk_out, scl_out, nchk, prows)
                         : potrf_core_left(n, nb, A, lda, NULL, 0, K, c_tau, abft, mode, ev ? ev + off : NULL,
                                           cap - off, &nev2, info, c, chk_out, scl_out, nchk);
         nev1 += nev2;
@@ -768,6 +790,14 @@ int oracle_potrf_nchk(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_
     free(A0);
     if (nev) *nev = nev1;
     return st;
+}
+
+int oracle_potrf_nchk(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
+                      int nranks, int K, double c_tau, int abft, int mode, int order, oevent_t* ev, int64_t cap,
+                      int64_t* nev, int64_t* info, ocount_t* cnt, double* chk_out, double* scl_out,
+                      int* reruns, int nchk) {
+    return oracle_potrf_grid(n, nb, A, lda, inj, ninj, nranks < 1 ? 1 : nranks, 1, K, c_tau, abft, mode, order, ev,
+                             cap, nev, info, cnt, chk_out, scl_out, reruns, nchk);
 }
 
 int oracle_potrf_mode(int64_t n, int64_t nb, double* A, int64_t lda, const oinj_t* inj, int64_t ninj,
@@ -839,7 +869,7 @@ int oracle_potrf_prefix(int64_t n, int64_t nb, double* A, int64_t lda, int64_t k
     memset(c, 0, sizeof(ocount_t));
     int64_t nev = 0, info = 0;
     g_kstop = kstop < 0 ? 0 : kstop;
-    const int st = potrf_core(n, nb, A, lda, NULL, 0, 1, 1, 64.0, 1, 0, NULL, 0, &nev, &info, c, NULL, NULL, 2);
+    const int st = potrf_core(n, nb, A, lda, NULL, 0, 1, 1, 64.0, 1, 0, NULL, 0, &nev, &info, c, NULL, NULL, 2, 1);
     g_kstop = INT64_MAX;
     return st;
 }

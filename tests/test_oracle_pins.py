@@ -312,6 +312,51 @@ def test_recv_injection_caught_by_receiver():
     assert floor_rel(r.L, ref.L, A) <= 1e-12
 
 
+def _grid_owner(I, J, P, prows):
+    pc = P // prows
+    return (I % prows) * pc + J % pc
+
+
+@pytest.mark.parametrize("P,prows", [(2, 2), (4, 2), (6, 2), (6, 3), (8, 4)])
+def test_grid_simulation_matches_single_rank(P, prows):
+    """2D block-cyclic simulation: the arithmetic of every tile is the one-process
+    arithmetic, so L is bit-identical and every decision is the same; the rank field names the
+    owner of the tile that was checked, (I mod prows) * pcols + J mod pcols."""
+    n, nb = 1024, 128
+    A = syn.spd_matrix(n)
+    specs = syn.per_iteration_injections(n, nb, bits=(45, 61))
+    r1 = oracle.potrf(A, nb, inj=syn.inj_array(specs))
+    rP = oracle.potrf(A, nb, inj=syn.inj_array(specs), nranks=P, prows=prows)
+    assert rP.status == 0 and np.array_equal(r1.L, rP.L)
+    assert [e[:7] for e in r1.event_tuples()] == [e[:7] for e in rP.event_tuples() if e[1] != V["V4R"]]
+    assert all(e[7] == _grid_owner(e[3], e[2], P, prows) for e in rP.event_tuples() if e[1] != V["V4R"])
+    # fault-free: the tile checks are the one-rank ones plus one V4R per (rank, received panel tile)
+    f1, fP = oracle.potrf(A, nb), oracle.potrf(A, nb, nranks=P, prows=prows)
+    N = n // nb
+    v4r = sum(1 for k in range(N - 1) for r in range(P) for i in range(k + 1, N) if _grid_owner(i, k, P, prows) != r)
+    assert fP.counts["n_checks"] - f1.counts["n_checks"] == v4r
+    assert np.array_equal(f1.L, fP.L) and len(fP.events) == 0
+
+
+def test_grid_recv_injection_caught_by_receiver_only():
+    """A RECV error lands in the receiving rank's copy of a panel tile it does not own and is
+    corrected there by V4R (event on that rank); a RECV target inside a tile the rank owns is not
+    received by it and has no effect."""
+    n, nb, P, prows = 1024, 128, 4, 2
+    A = syn.spd_matrix(n)
+    ref = oracle.potrf(A, nb)
+    # k = 1: panel tiles (i, 1), owners (i % 2) * 2 + 1 -> tile 5 (rows 640..767) belongs to rank 3
+    assert _grid_owner(5, 1, P, prows) == 3 and _grid_owner(6, 2, P, prows) == 0
+    specs = [dict(k=1, hook="RECV", row=700, col=150, bit=50, rank=0),
+             dict(k=2, hook="RECV", target="CHK", row=2 * 6 + 1, col=2 * nb + 5, bit=50, rank=3)]
+    r = oracle.potrf(A, nb, inj=syn.inj_array(specs), nranks=P, prows=prows)
+    assert r.event_tuples() == sorted(predict(s, n, nb) for s in specs)
+    assert floor_rel(r.L, ref.L, A) <= 1e-12
+    owned = [dict(k=1, hook="RECV", row=700, col=150, bit=50, rank=3)]   # rank 3 owns tile (5, 1)
+    r2 = oracle.potrf(A, nb, inj=syn.inj_array(owned), nranks=P, prows=prows)
+    assert len(r2.events) == 0 and np.array_equal(r2.L, ref.L)
+
+
 @pytest.mark.parametrize("K", [3, 5])
 def test_opt3_verify_every_K(K):
     n, nb = 1024, 64
