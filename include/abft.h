@@ -115,6 +115,10 @@ typedef struct abft_options {
                              in a column of a block ("m+1 column checksums ... up to m errors",
                              P:121; reading B10 of DESIGN.md: ambiguous pairs are UNCORRECTABLE).
                              nchk = 3: right-looking Enhanced scheme on one GPU (else -8)         */
+    int32_t prows;        /* multi-GPU only (abft_potrf_dist / _dist_sim): process-grid rows Pr of a
+                             2D block-cyclic distribution of the nranks = Pr x Pc ranks;
+                             0 or 1 = the 1D column-cyclic distribution. Must divide nranks, <= 15;
+                             Pr > 1 needs the peer-memory transport or the one-device harness (-11) */
 } abft_options_t;
 #define ABFT_ORDER_RIGHT 0
 #define ABFT_ORDER_LEFT 1
@@ -196,13 +200,21 @@ int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t lda, abft_str
  * Writes the full n x n matrix. Errors: -1 n, -3 A, -4 lda. */
 int abft_gen_spd(int64_t n, uint64_t seed, double* A, int64_t lda, abft_stream_t stream);
 
-/* ---- multi-GPU (one process per GPU, 1D block-cyclic block columns, NCCL panel broadcast) ---
+/* ---- multi-GPU (one process per GPU, block-cyclic tiles, panel broadcast) ---------------------
  * abft_nccl_id: fill 128 bytes (ncclUniqueId) on rank 0, share them out of band.
  * abft_comm_init: create the communicator for `rank` of `nranks` on the current device.
- * abft_potrf_dist: rank r owns block columns {j : j mod nranks == r}, stored contiguously in
- * A_local (n x (n_local_cols) column-major, lda_local >= n, local block column t is global
- * block column t*nranks + r). Same semantics and report as abft_potrf; events of all ranks are
- * gathered into rank 0's report (other ranks report their own). Errors as abft_potrf, 4 NCCL. */
+ * abft_potrf_dist: 1D (options.prows <= 1): rank r owns block columns {j : j mod nranks == r},
+ * stored contiguously in A_local (n x (n_local_cols) column-major, lda_local >= n, local block
+ * column t is global block column t*nranks + r). 2D (options.prows = Pr > 1, Pc = nranks / Pr,
+ * rank r = pr * Pc + pc): rank r owns the tiles (I, J) with I mod Pr = pr and J mod Pc = pc; it
+ * stores the block columns {j : j mod Pc == pc} contiguously and full height (global rows, local
+ * block column t = global t*Pc + pc), reads and writes only its own tiles (the other rows are
+ * workspace). Per iteration the diagonal block's owner factors it and pushes inv(L_kk) to the other
+ * ranks of its process column, each of those solves and checks its own panel tiles and pushes them
+ * to every rank; every rank re-checks the tiles it received (V4R). Same semantics and report as
+ * abft_potrf; events of all ranks are gathered into rank 0's report (other ranks report their
+ * own); an event's rank is the owner of the checked tile (the receiver for V4R). Errors as
+ * abft_potrf, 4 NCCL. */
 int abft_nccl_id(void* id128);
 int abft_comm_init(void** comm, int nranks, const void* id128, int rank);
 int abft_comm_destroy(void* comm);
@@ -239,6 +251,8 @@ int abft_comm_attach_ipc(void* comm, const void* handles);
 int abft_potrf_dist_sim(int64_t n, int64_t nb, int nranks, double* const* A_locals, int64_t lda_local,
                         abft_stream_t stream, const abft_inject_spec_t* inj, abft_report_t* rep,
                         const abft_options_t* opt);
+/* (2D, options.prows > 1: A_locals[r] holds the block columns of process column r mod Pc, full
+ * height, as abft_potrf_dist; the owners push their panel rows into the other ranks' buffers.) */
 
 /* Diagnostics: the trailing-update GEMM on its own (for benchmarking the dominant kernel):
  * C = beta C + alpha A B^T over the lower triangle (lower = 1: r >= c, requires N <= M) or all

@@ -53,7 +53,7 @@ class Report(ctypes.Structure):
 class Options(ctypes.Structure):
     _fields_ = [("abft_enabled", ctypes.c_int32), ("K", ctypes.c_int32), ("c_tau", ctypes.c_double),
                 ("lookahead", ctypes.c_int32), ("profile", ctypes.c_int32), ("mode", ctypes.c_int32),
-                ("order", ctypes.c_int32), ("nchk", ctypes.c_int32)]
+                ("order", ctypes.c_int32), ("nchk", ctypes.c_int32), ("prows", ctypes.c_int32)]
 
 
 class Profile(ctypes.Structure):
@@ -159,10 +159,13 @@ def _report_dict(rep, ev):
 MODE = {"enhanced": 0, "online": 1, "offline": 2, "enhanced_redo": 3}
 
 
-def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False, mode="enhanced", order="right", nchk=2):
-    """nchk: checksum rows per block, 2 (the paper's choice) or 3 (up to two errors per column)."""
+def options(abft_enabled=True, K=1, c_tau=64.0, lookahead=0, profile=False, mode="enhanced", order="right", nchk=2,
+            prows=1):
+    """nchk: checksum rows per block, 2 (the paper's choice) or 3 (up to two errors per column).
+    prows: multi-GPU process-grid rows (2D block-cyclic when > 1; 1 = column-cyclic)."""
     return Options(int(bool(abft_enabled)), int(K), float(c_tau), int(lookahead), int(bool(profile)),
-                   MODE[mode] if isinstance(mode, str) else int(mode), {"right": 0, "left": 1}[order], int(nchk))
+                   MODE[mode] if isinstance(mode, str) else int(mode), {"right": 0, "left": 1}[order], int(nchk),
+                   int(prows))
 
 
 def abft_last_profile():
@@ -266,7 +269,8 @@ def ipc_comm(n, nb, group=None):
     and maps every peer's. Returns the comm for abft_potrf_dist."""
     import torch.distributed as dist
     rank, world = dist.get_rank(group), dist.get_world_size(group)
-    cap = 8 * ((n - nb) * nb + 2 * n + 8) + 48 * 8192   # packed panel + abort slot; event gather (8192)
+    # packed panel + 16 abort slots + a received inv(L_kk) (2D) + its slot; event gather (8192)
+    cap = 8 * ((n - nb) * nb + 2 * n + 2 * nb + 16 + nb * nb + 2) + 48 * 8192
     st, comm, h = abft_comm_init_ipc(world, rank, cap)
     assert st == 0, f"abft_comm_init_ipc: {st} {abft_last_error()}"
     hs = [None] * world
@@ -345,6 +349,34 @@ def block_cyclic_split(A, nb, nranks):
         idx = np.concatenate(cols) if cols else np.zeros(0, dtype=np.int64)
         out.append(np.asfortranarray(A[:, idx]))
     return out
+
+
+def grid_owner(I, J, nranks, prows=1):
+    """Rank owning tile (I, J) on the prows x (nranks / prows) process grid (2D block-cyclic)."""
+    pc = nranks // prows
+    return (I % prows) * pc + J % pc
+
+
+def block_cyclic_split_2d(A, nb, nranks, prows):
+    """Per-rank local arrays of the 2D layout: rank r = pr * Pc + pc holds the block columns
+    J = pc (mod Pc), full height (its own tiles are the rows I = pr (mod Pr); the rest is workspace)."""
+    pc_n = nranks // prows
+    cols = block_cyclic_split(A, nb, pc_n)
+    return [cols[r % pc_n].copy(order="F") for r in range(nranks)]
+
+
+def block_cyclic_join_2d(locals_, nb, n, prows):
+    """Inverse of block_cyclic_split_2d: tile (I, J) from its owner's local array."""
+    P = len(locals_)
+    pc_n = P // prows
+    A = np.zeros((n, n), order="F")
+    N = n // nb
+    for J in range(N):
+        t = J // pc_n
+        for I in range(N):
+            L = locals_[grid_owner(I, J, P, prows)]
+            A[I * nb:(I + 1) * nb, J * nb:(J + 1) * nb] = L[I * nb:(I + 1) * nb, t * nb:(t + 1) * nb]
+    return A
 
 
 def block_cyclic_join(locals_, nb, n):

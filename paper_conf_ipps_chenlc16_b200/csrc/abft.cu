@@ -164,6 +164,7 @@ static StageArgs stage_base(const Work& w, double* A, int64_t lda, double c_tau,
     a.s = w.scl; a.S1 = w.scl ? w.scl + w.n : nullptr; a.S2 = w.scl ? w.scl + w.n + w.N : nullptr;
     a.S3 = w.scl ? w.scl + w.n + 2 * w.N : nullptr; a.nchk = w.nchk;
     a.c_tau = c_tau; a.col_owner_mod = 1; a.col_owner_rank = 0;
+    a.row_owner_mod = 1; a.row_owner_rank = 0; a.own_invert = 0;
     a.st = w.st; a.ev = w.ev; a.ev_cap = w.ev_cap;
     a.flist = 0; a.j_lo = k + 1; a.j_hi = w.N;
     return a;
@@ -808,21 +809,35 @@ extern "C" int abft_graph_release(void) {
 // =============================================================================================
 namespace {
 struct RankState {
-    int r;
+    int r, pr, pc;            // rank, its process-grid row and column (2D block-cyclic; pr = 0 in 1D)
     double* A; int64_t lda;
     int64_t nblk, ncl;        // local block columns, local columns
     Work w;
-    double* xslot = nullptr;  // abort flag slot right after the packed panel inside W
     double* Wb[2] = {nullptr, nullptr};   // double-buffered panel (look-ahead)
+    double* Wt = nullptr;     // 2D: this rank's TRSM output (its own panel rows), pushed from here into
+                              // every rank's Wb (its own included), which the other owners fill too
+};
+// Process grid of the dist driver: P = Pr x Pc ranks, rank r = pr * Pc + pc; tile (I, J) is owned by
+// rank (I mod Pr) * Pc + (J mod Pc) (Pr = 1: the 1D column-cyclic distribution). Every rank stores
+// its block columns {J : J mod Pc = pc} contiguously and full height (global rows); it maintains
+// only its own tiles.
+struct Grid {
+    int P, Pr, Pc;
+    int owner(int64_t I, int64_t J) const { return (int)((I % Pr) * Pc + (J % Pc)); }
 };
 }
 
-static int64_t dist_lc(int64_t J, int P, int64_t nb) { return (J / P) * nb; }   // local column of block J
+static int64_t dist_lc(int64_t J, int Pc, int64_t nb) { return (J / Pc) * nb; }   // local column of block J
 
-static double* dist_inj_ptr(const abft_inject_spec_t& sp, int64_t k, int64_t nb, int P, const RankState& R,
+// block row of an injection's target (data row / nb, or checksum row / 2)
+static int64_t inj_row_block(const abft_inject_spec_t& sp, int64_t nb) {
+    return sp.target == ABFT_TGT_DATA ? sp.row / nb : sp.row / 2;
+}
+
+static double* dist_inj_ptr(const abft_inject_spec_t& sp, int64_t k, int64_t nb, const Grid& G, const RankState& R,
                             int64_t ldw, int64_t mB) {
     const int hook = sp.hook;
-    const int64_t Jc = sp.col / nb, lcol = dist_lc(Jc, P, nb) + sp.col % nb;
+    const int64_t Jc = sp.col / nb, lcol = dist_lc(Jc, G.Pc, nb) + sp.col % nb;
     if (hook == ABFT_HOOK_TRSM_OUT || hook == ABFT_HOOK_RECV) {
         if (sp.target == ABFT_TGT_DATA) return R.w.W + (sp.col - k * nb) * ldw + (sp.row - (k + 1) * nb);
         return R.w.W + (sp.col - k * nb) * ldw + mB + (sp.row - 2 * k);
@@ -833,24 +848,30 @@ static double* dist_inj_ptr(const abft_inject_spec_t& sp, int64_t k, int64_t nb,
     return R.w.chk + lcol * R.w.ldc + sp.row;
 }
 
-static void dist_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, int hook, int64_t nb, int P,
+// Apply rank R's share of the injections at (k, hook): targets in the tiles it owns, or for RECV
+// the ones addressed to it that land in a panel tile it received (not one it owns).
+static void dist_inject(const std::vector<abft_inject_spec_t>& list, int64_t k, int hook, int64_t nb, const Grid& G,
                         const RankState& R, int64_t ldw, int64_t mB, cudaStream_t s) {
     std::vector<double*> ptrs; std::vector<uint64_t> masks;
     for (const auto& sp : list) {
         if (sp.k != k || sp.hook != hook) continue;
-        if (hook == ABFT_HOOK_RECV) { if (sp.rank != R.r) continue; }
-        else if ((sp.col / nb) % P != R.r) continue;       // the owner of the target's block column
-        ptrs.push_back(dist_inj_ptr(sp, k, nb, P, R, ldw, mB)); masks.push_back(sp.xor_mask);
+        const int own = G.owner(inj_row_block(sp, nb), sp.col / nb);
+        if (hook == ABFT_HOOK_RECV) { if (sp.rank != R.r || own == R.r) continue; }
+        else if (own != R.r) continue;       // the owner of the target's tile
+        ptrs.push_back(dist_inj_ptr(sp, k, nb, G, R, ldw, mB)); masks.push_back(sp.xor_mask);
     }
     if (!ptrs.empty()) launch_inject((int)ptrs.size(), ptrs.data(), masks.data(), &R.w.st->abort, s);
 }
 
 int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, DistTransport* tp,
              cudaStream_t s, const abft_inject_spec_t* inj_c, abft_report_t* rep, const abft_options_t* opt) {
-    abft_options_t o = opt ? *opt : abft_options_t{1, 1, 64.0, 0, 0, ABFT_MODE_ENHANCED, 0};
+    abft_options_t o = opt ? *opt : abft_options_t{1, 1, 64.0, 0, 0, ABFT_MODE_ENHANCED, 0, 0, 0};
+    const int Pr = o.prows > 0 ? o.prows : 1;
     if (o.K < 1 || !(o.c_tau > 0) || o.mode != ABFT_MODE_ENHANCED || o.order != ABFT_ORDER_RIGHT ||
-        (o.nchk != 0 && o.nchk != 2))
-        return -11;   // dist: Enhanced scheme, right-looking order, two checksum rows
+        (o.nchk != 0 && o.nchk != 2) || P % Pr != 0 || Pr > 15)
+        return -11;   // dist: Enhanced scheme, right-looking order, two checksum rows, Pr | P
+    const Grid G{P, Pr, P / Pr};
+    const int Pc = G.Pc;
     std::vector<abft_inject_spec_t> inj;
     if (collect_inj(inj_c, n, nb, inj)) return -9;
     if (rep) { rep->info = 0; rep->n_events = 0; rep->n_checks = 0; }
@@ -860,23 +881,25 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     const int64_t N = n / nb, B = nb;
     std::vector<RankState> R(nlocal);
     const int64_t evcap = rep ? std::max<int64_t>(rep->cap, 1) : 1024;
+    // W layout: packed panel (ldw x B) + 16 abort slots (one per contributing process row); 2D also
+    // keeps the received inv(L_kk) (+ its abort slot) behind them
+    const int64_t wrows_max = (N - 1) * nb + 2 * N + 2;
+    const size_t wcap = (size_t)(std::max<int64_t>(wrows_max, 1) * nb) + 16;
+    const size_t wbuf = wcap + (Pr > 1 ? (size_t)(B * B) + 2 : 0);
     // push mode (NEXT-3): a peer-memory transport owns every rank's two receive buffers; the owner's
     // write-back kernel stores the panel straight into them (launch_panel_out)
-    const int64_t wrows_max = (N - 1) * nb + 2 * N + 2;
-    const bool push = tp && tp->recv_buf(tp->rank, 0) != nullptr &&
-                      tp->recv_capacity() >= (size_t)(std::max<int64_t>(wrows_max, 1) * nb + 1) &&
+    const bool push = tp && tp->recv_buf(tp->rank, 0) != nullptr && tp->recv_capacity() >= wbuf &&
                       tp->nranks <= 16 && getenv("ABFT_DIST_PULL") == nullptr;
+    if (Pr > 1 && tp && !push) return -11;   // 2D needs peer memory (IPC transport) or the one-device harness
     for (int i = 0; i < nlocal; ++i) {
         RankState& q = R[i];
-        q.r = locals[i].rank; q.A = locals[i].A; q.lda = locals[i].lda;
-        q.nblk = (N - q.r + P - 1) / P; q.ncl = q.nblk * B;
+        q.r = locals[i].rank; q.pr = q.r / Pc; q.pc = q.r % Pc; q.A = locals[i].A; q.lda = locals[i].lda;
+        q.nblk = (N - q.pc + Pc - 1) / Pc; q.ncl = q.nblk * B;
         int rc = work_alloc(q.w, n, nb, std::max<int64_t>(q.ncl, 1), evcap, abft, s);
         if (rc) return rc;
-        // W with one extra slot for the owner's abort flag
         cudaFreeAsync(q.w.W, s);
-        const int64_t wrows = (N - 1) * nb + 2 * N + 2;
         if (push) q.w.W = tp->recv_buf(q.r, 0);
-        else ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.w.W, sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb + 1), s));
+        else ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.w.W, sizeof(double) * wbuf, s));
         if (abft && nb % 128 == 0 && q.lda % 2 == 0 && ((uintptr_t)q.A & 15) == 0) {
             q.w.cs_nslab = n / 32;
             ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.w.cs, sizeof(double) * (size_t)(2 * q.w.cs_nslab * std::max<int64_t>(q.ncl, 1)), s));
@@ -885,7 +908,7 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     }
     auto stage = [&](RankState& q, int kind, int V, int k) {
         StageArgs a = stage_base(q.w, q.A, q.lda, o.c_tau, kind, V, k);
-        a.col_owner_mod = P; a.col_owner_rank = q.r; a.rank = q.r;
+        a.col_owner_mod = Pc; a.col_owner_rank = q.pc; a.row_owner_mod = Pr; a.row_owner_rank = q.pr; a.rank = q.r;
         return a;
     };
     cudaEvent_t e0 = nullptr, e1 = nullptr;
@@ -894,8 +917,9 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     if (abft) {
         for (auto& q : R) {
             cudaMemsetAsync(q.w.scl, 0, sizeof(double) * (size_t)(n + 2 * N), s);
-            for (int64_t J = q.r; J < N; J += P)
-                launch_scales_diag(B, q.A + dist_lc(J, P, B) * q.lda + J * B, q.lda, q.w.scl + J * B, s);
+            for (int64_t J = q.pc; J < N; J += Pc)
+                if (G.owner(J, J) == q.r)
+                    launch_scales_diag(B, q.A + dist_lc(J, Pc, B) * q.lda + J * B, q.lda, q.w.scl + J * B, s);
         }
         if (tp) {
             if (tp->allreduce_sum(R[0].w.scl, (size_t)n, s)) return ABFT_ERR_NCCL;
@@ -911,17 +935,16 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             launch_check(a, s);
         }
     }
-    // ---- look-ahead across ranks: the owner of block column k+1 updates that
-    // column with panel k first, then factors it and broadcasts panel k+1 on its panel stream
-    // while every rank applies the rest of update k on its main stream. Panel + broadcast + V4R
-    // run on the panel stream PS (high priority), updates + V5 on the main stream (the caller's).
+    // ---- look-ahead across ranks: the owners of block column k+1 update that
+    // column with panel k first, then factor it and broadcast panel k+1 on their panel stream while
+    // every rank applies the rest of update k on its main stream. Panel + broadcast + V4R run on the
+    // panel stream PS (high priority), updates + V5 on the main stream (the caller's).
     // Single-process simulation: every rank shares the two streams; the broadcast is a device copy
-    // issued on the owner's panel stream.
+    // (1D) or the owners' push into the other ranks' panel buffers (2D), issued on PS.
     ThreadCache& tc = thread_cache();
     cudaStream_t PS = tc.P;
     // The transport's waiting kernels (NCCL collectives, IPC flag waits) are long-lived CTAs; they
-    // run on a NORMAL-priority comm stream joined to PS by events, because long-lived high-priority
-    // CTAs next to the bulk-copy update are what produced stale operand stages
+    // run on a NORMAL-priority comm stream joined to PS by events
     if (tp && !tc.C) ABFT_CUDA_TRY(cudaStreamCreateWithFlags(&tc.C, cudaStreamNonBlocking));
     cudaStream_t CS = tp ? tc.C : PS;
     auto hop = [&](cudaStream_t from, cudaStream_t to) {   // `to` waits for everything enqueued on `from`
@@ -933,10 +956,10 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(PS, e, 0);
     }
     for (auto& q : R) {   // second panel buffer per rank (W of iteration k lives in Wb[k & 1])
-        const int64_t wrows = (N - 1) * nb + 2 * N + 2;
         q.Wb[0] = q.w.W;
         if (push) q.Wb[1] = tp->recv_buf(q.r, 1);
-        else ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.Wb[1], sizeof(double) * (size_t)(std::max<int64_t>(wrows, 1) * nb + 1), s));
+        else ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.Wb[1], sizeof(double) * wbuf, s));
+        if (Pr > 1) ABFT_CUDA_TRY(cudaMallocAsync((void**)&q.Wt, sizeof(double) * wcap, s));
     }
     {   // Wb[1] allocated on s: the panel stream must see it
         cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(PS, e, 0);
@@ -952,95 +975,152 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             const int64_t J = sp.col / nb;
             if ((J >= jlo && J < jhi) == inside) sub.push_back(sp);
         }
-        if (!sub.empty()) dist_inject(sub, k, ABFT_HOOK_REST, B, P, q, 1, 0, st);
+        if (!sub.empty()) dist_inject(sub, k, ABFT_HOOK_REST, B, G, q, 1, 0, st);
     };
-    // the panel of iteration k on the owner's panel stream (V1/V2, POTRF + inverse, TRSM with
-    // Alg. 2 rows, V3, V4, write-back, abort slot) into Wb[k & 1]
-    auto panel = [&](RankState& q, int64_t k) -> int {
+    // the other ranks' panel buffers Wb[slot] (peer stores of the push)
+    auto peer_bufs = [&](const RankState& q, int slot) {
+        std::vector<double*> peers;
+        if (push) { for (int r = 0; r < P; ++r) if (r != q.r) peers.push_back(tp->recv_buf(r, slot)); }
+        else for (auto& p : R) if (p.r != q.r) peers.push_back(p.Wb[slot]);
+        return peers;
+    };
+    // the panel of iteration k, on the panel stream of the ranks of process column k mod Pc: V1/V2
+    // of their tiles of block column k, POTRF + inverse on the diagonal block's owner (2D: inv(L_kk)
+    // pushed to the column's other ranks), TRSM of each rank's own panel rows (+ Alg. 2 rows), V3,
+    // V4, write-back, abort slot; 2D / peer memory: each rank's rows pushed into every other rank's
+    // panel buffer Wb[k & 1]
+    auto panel = [&](int64_t k) -> int {
         int64_t m, mB, ldw; geom(k, m, mB, ldw);
-        q.w.W = q.Wb[k & 1];
+        const int kc = (int)(k % Pc), d = G.owner(k, k);
         const size_t wcount = (size_t)(ldw * B);
-        const int32_t* ab = &q.w.st->abort;
-        double* Akk = q.A + dist_lc(k, P, B) * q.lda + k * B;
-        double* ckk = q.w.chk + dist_lc(k, P, B) * q.w.ldc;
-        if (abft) {
-            rest_inject(q, k, k, k + 1, true, PS);                                    // REST(k), column k
-            StageArgs a = stage(q, SK_COLUMN, ABFT_V2, (int)k); a.flist = 1;
-            launch_check(a, PS);                                                     // V1, V2
-        }
-        launch_chol_inv(Akk, q.lda, q.w.Li, B, k * B, q.w.tmp, q.w.st, PS);
-        if (abft)
-            launch_trsm_with_chk(mB, B, Akk + B, q.lda, q.w.Li, q.w.W, ldw, 2 * m + 2, ckk + 2 * k, q.w.ldc, ab, PS);
-        else
-            launch_gemm(mB, B, B, Akk + B, q.lda, q.w.Li, B, q.w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, PS);
-        if (abft) {
-            dist_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, P, q, ldw, mB, PS);
-            StageArgs a3 = stage(q, SK_DIAG_FACT, ABFT_V3, (int)k);
-            a3.ldw = ldw; a3.mB = mB; a3.flist = 1;
-            StageArgs a4 = stage(q, SK_PANEL, ABFT_V4, (int)k);
-            a4.ldw = ldw; a4.mB = mB; a4.flist = 1;
-            if (!has_inj(inj, k, ABFT_HOOK_TRSM_OUT)) {
-                launch_check2(a3, a4, PS);                                           // V3 + V4
-            } else {
-                launch_check(a3, PS);                                                // V3
-                dist_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, P, q, ldw, mB, PS);
-                launch_check(a4, PS);                                                // V4
+        std::vector<RankState*> col;
+        for (auto& q : R) if (q.pc == kc) col.push_back(&q);
+        if (col.empty()) return 0;
+        for (RankState* qp : col) {                                                    // REST(k), V1, V2
+            RankState& q = *qp;
+            q.w.W = q.Wb[k & 1];
+            if (abft) {
+                rest_inject(q, k, k, k + 1, true, PS);
+                StageArgs a = stage(q, SK_COLUMN, ABFT_V2, (int)k); a.flist = 1;
+                launch_check(a, PS);
             }
         }
-        if (push && k + 1 < N) {
-            // write-back fused with the broadcast: one pass over W stores the L panel and its
-            // checksum rows locally and the whole packed panel (+ abort slot) into every peer's
-            // receive buffer (peer stores), once every peer released that buffer
-            launch_abort_to_slot(ab, q.w.W + wcount, PS);
-            hop(PS, CS);
-            if (tp->wait_free(k, CS)) return ABFT_ERR_NCCL;
-            hop(CS, PS);
-            std::vector<double*> peers;
-            for (int r = 0; r < P; ++r) if (r != q.r) peers.push_back(tp->recv_buf(r, (int)(k & 1)));
-            launch_panel_out(q.w.W, ldw, mB, abft ? 2 * m + 2 : 0, B, Akk + B, q.lda, ckk + 2 * k, q.w.ldc, peers.data(),
-                             (int)peers.size(), ab, PS);
-            if (tp->post_panel(k, PS)) return ABFT_ERR_NCCL;
-            return 0;
+        for (RankState* qp : col) {                                                    // POTRF + inverse
+            RankState& q = *qp;
+            if (q.r != d) continue;
+            double* Akk = q.A + dist_lc(k, Pc, B) * q.lda + k * B;
+            launch_chol_inv(Akk, q.lda, q.w.Li, B, k * B, q.w.tmp, q.w.st, PS);
+            if (Pr > 1 && m > 0) {   // inv(L_kk) + abort flag to the column's other ranks (their Wb + wcap)
+                for (int pr = 0; pr < Pr; ++pr) {
+                    const int r = pr * Pc + kc;
+                    if (r == d) continue;
+                    double* dst = nullptr;
+                    if (push) dst = tp->recv_buf(r, (int)(k & 1)) + wcap;
+                    else for (auto& p : R) if (p.r == r) dst = p.Wb[k & 1] + wcap;
+                    if (!dst) continue;
+                    cudaMemcpyAsync(dst, q.w.Li, sizeof(double) * (size_t)(B * B), cudaMemcpyDeviceToDevice, PS);
+                    launch_abort_to_slot(&q.w.st->abort, dst + B * B, PS);
+                }
+                if (push && tp->post_li(k, PS)) return ABFT_ERR_NCCL;
+            }
         }
-        launch_copy(mB, B, q.w.W, ldw, Akk + B, q.lda, ab, PS);
-        if (abft) launch_copy(2 * m + 2, B, q.w.W + mB, ldw, ckk + 2 * k, q.w.ldc, ab, PS);
-        launch_abort_to_slot(ab, q.w.W + wcount, PS);
+        for (RankState* qp : col) {
+            RankState& q = *qp;
+            const int32_t* ab = &q.w.st->abort;
+            double* Akk = q.A + dist_lc(k, Pc, B) * q.lda + k * B;
+            double* ckk = q.w.chk + dist_lc(k, Pc, B) * q.w.ldc;
+            if (m == 0 && q.r != d) continue;                     // last panel: the diagonal block only
+            if (Pr > 1) q.w.W = q.Wt;   // 2D: solve into the private buffer (Wb[k & 1] receives the other owners' rows)
+            const double* Li = q.w.Li;
+            if (q.r != d) {                                       // 2D: the column's other ranks
+                double* li_in = q.Wb[k & 1] + wcap;
+                if (push) { hop(PS, CS); if (tp->wait_li(d, k, CS)) return ABFT_ERR_NCCL; hop(CS, PS); }
+                launch_abort_from_slot(li_in + B * B, q.w.st, PS);
+                Li = li_in;
+            }
+            // this rank's panel rows: data blocks k+1+b with (k+1+b) mod Pr = pr
+            const int64_t rfirst = ((q.pr - (k + 1) % Pr) % Pr + Pr) % Pr;
+            if (abft)
+                launch_trsm_with_chk(mB, B, Akk + B, q.lda, Li, q.w.W, ldw, 2 * m + 2, ckk + 2 * k, q.w.ldc, ab, PS, Pr,
+                                     rfirst);
+            else
+                launch_gemm(mB, B, B, Akk + B, q.lda, Li, B, q.w.W, ldw, 1.0, 0.0, true, 0, 1, 0, 0, 0, ab, PS);
+            if (abft) {
+                StageArgs a3 = stage(q, SK_DIAG_FACT, ABFT_V3, (int)k);
+                a3.ldw = ldw; a3.mB = mB; a3.flist = 1;
+                StageArgs a4 = stage(q, SK_PANEL, ABFT_V4, (int)k);
+                a4.ldw = ldw; a4.mB = mB; a4.flist = 1;
+                dist_inject(inj, k, ABFT_HOOK_POTRF_OUT, B, G, q, ldw, mB, PS);
+                if (q.r == d && !has_inj(inj, k, ABFT_HOOK_TRSM_OUT)) {
+                    launch_check2(a3, a4, PS);                                         // V3 + V4
+                } else {
+                    if (q.r == d) launch_check(a3, PS);                                // V3
+                    dist_inject(inj, k, ABFT_HOOK_TRSM_OUT, B, G, q, ldw, mB, PS);
+                    launch_check(a4, PS);                                              // V4
+                }
+            }
+            launch_abort_to_slot(ab, q.w.W + wcount + q.pr, PS);
+            const int64_t ncr = abft ? 2 * m + 2 : 0;
+            if ((push || Pr > 1) && k + 1 < N) {
+                // write-back fused with the broadcast: one pass over this rank's rows of W stores them
+                // locally (L panel, checksum rows) and into every other rank's panel buffer (peer
+                // stores), once every peer released that buffer
+                if (push) { hop(PS, CS); if (tp->wait_free(k, CS)) return ABFT_ERR_NCCL; hop(CS, PS); }
+                std::vector<double*> peers = peer_bufs(q, (int)(k & 1));
+                if (Pr > 1) peers.push_back(q.Wb[k & 1]);   // and its own receive buffer
+                if (launch_panel_out(q.w.W, ldw, mB, ncr, B, Akk + B, q.lda, ckk + 2 * k, q.w.ldc, peers.data(),
+                                     (int)peers.size(), ab, PS, Pr, rfirst, ((q.pr - k % Pr) % Pr + Pr) % Pr, q.pr))
+                    return -11;
+                if (push && tp->post_panel(k, PS)) return ABFT_ERR_NCCL;
+                q.w.W = q.Wb[k & 1];
+                continue;
+            }
+            launch_copy(mB, B, q.w.W, ldw, Akk + B, q.lda, ab, PS);
+            if (abft) launch_copy(ncr, B, q.w.W + mB, ldw, ckk + 2 * k, q.w.ldc, ab, PS);
+            q.w.W = q.Wb[k & 1];
+        }
         return 0;
     };
-    // broadcast of panel k (+ abort slot) from its owner, then every receiver's RECV hook and V4R;
-    // afterwards evB[rank] marks "panel k usable on this rank"
+    // broadcast of panel k (+ abort slots) from its owners, then every receiver's RECV hook and V4R
+    // on the tiles it received; afterwards evB[rank] marks "panel k usable on this rank"
     std::vector<cudaEvent_t> evU(nlocal, nullptr), evUprev(nlocal, nullptr);   // after update k / k-1
     std::vector<cudaEvent_t> evB(nlocal, nullptr);
     auto bcast = [&](int64_t k) -> int {
         int64_t m, mB, ldw; geom(k, m, mB, ldw);
         const size_t wcount = (size_t)(ldw * B);
-        const int owner = (int)(k % P);
+        const int kc = (int)(k % Pc), owner = G.owner(k, k);
         for (int i = 0; i < nlocal; ++i)   // the receive buffer Wb[k & 1] was last read by update k-2
             if (evUprev[i]) cudaStreamWaitEvent(PS, evUprev[i], 0);
         if (tp && push) {
             hop(PS, CS);
-            if (R[0].r != owner && tp->wait_panel(owner, k, CS)) return ABFT_ERR_NCCL;   // pushed by the owner
+            for (int pr = 0; pr < Pr; ++pr) {   // pushed by the panel's owners (the ranks of column kc)
+                const int c = pr * Pc + kc;
+                if (c != R[0].r && tp->wait_panel(c, k, CS)) return ABFT_ERR_NCCL;
+            }
             hop(CS, PS);
         } else if (tp) {
             hop(PS, CS);
             if (tp->bcast(R[0].Wb[k & 1], (wcount + 1) * sizeof(double), owner, CS)) return ABFT_ERR_NCCL;
             hop(CS, PS);
-        } else {
+        } else if (Pr == 1) {
             const RankState* src = nullptr;
             for (auto& q : R) if (q.r == owner) src = &q;
             for (auto& q : R)
                 if (q.r != owner)
                     cudaMemcpyAsync(q.Wb[k & 1], src->Wb[k & 1], (wcount + 1) * sizeof(double), cudaMemcpyDeviceToDevice, PS);
-        }
+        }   // 2D one-device harness: the owners' pushes on PS already filled every buffer
         for (int i = 0; i < nlocal; ++i) {
             RankState& q = R[i];
             q.w.W = q.Wb[k & 1];
-            if (q.r != owner) {
-                launch_abort_from_slot(q.w.W + wcount, q.w.st, PS);
+            bool received = false;
+            for (int64_t I = k + 1; I < N; ++I) received = received || G.owner(I, k) != q.r;
+            if (received) {
+                for (int pr = 0; pr < Pr; ++pr)
+                    if (pr * Pc + kc != q.r) launch_abort_from_slot(q.w.W + wcount + pr, q.w.st, PS);
                 if (abft) {
-                    dist_inject(inj, k, ABFT_HOOK_RECV, B, P, q, ldw, mB, PS);
+                    dist_inject(inj, k, ABFT_HOOK_RECV, B, G, q, ldw, mB, PS);
                     StageArgs a = stage(q, SK_PANEL, ABFT_V4R, (int)k);               // V4R
-                    a.ldw = ldw; a.mB = mB; a.col_owner_mod = 1; a.col_owner_rank = 0; a.flist = 1;
+                    a.ldw = ldw; a.mB = mB; a.own_invert = 1; a.flist = 1;
                     launch_check(a, PS);
                 }
             }
@@ -1049,33 +1129,35 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         return 0;
     };
     int64_t dist_slab_rows = 64;
-    // trailing update of iteration k on rank q's block columns J in [jlo, jhi) (main stream),
-    // UPDATE_OUT hook and V5 of those columns
+    // trailing update of iteration k on rank q's tiles in block columns [jlo, jhi) (main stream),
+    // UPDATE_OUT hook and V5 of those tiles
     auto update = [&](RankState& q, int64_t k, int64_t jlo, int64_t jhi) {
         int64_t m, mB, ldw; geom(k, m, mB, ldw);
         double* W = q.Wb[k & 1];
         const int32_t* ab = &q.w.st->abort;
         bool any = false;
-        for (int64_t J = jlo; J < jhi; ++J) any = any || (J % P == q.r);
+        for (int64_t J = jlo; J < jhi; ++J) any = any || (J % Pc == q.pc);
         if (!any) return;
         bool all_fused = q.w.cs != nullptr;
-        // the owned block columns J in [jlo, jhi) are J0, J0 + P, ...: one launch whose column
-        // block t is global block J0 + t P (cstride), checksum rows appended as its second segment
+        // the owned block columns J in [jlo, jhi) are J0, J0 + Pc, ...: one launch whose column
+        // block t is global block J0 + t Pc (cstride), checksum rows appended as its second segment;
+        // 2D: only the row blocks I = J0 + rfirst + u Pr (this rank's tiles) are computed
         int64_t J0 = jlo;
-        while (J0 % P != q.r) ++J0;
-        const int64_t nt = (jhi - 1 - J0) / P + 1, t0 = J0 / P;
+        while (J0 % Pc != q.pc) ++J0;
+        const int64_t nt = (jhi - 1 - J0) / Pc + 1, t0 = J0 / Pc;
+        const int64_t rfirst = ((q.pr - J0 % Pr) % Pr + Pr) % Pr;
         double* W0 = W + (J0 - k - 1) * B;
         double* C = q.A + t0 * B * q.lda + J0 * B;
         // this rank's UPDATE_OUT injections in [jlo, jhi), in the launch's local coordinates
         EpiInj ei; ei.n = 0;
         for (const auto& sp : inj)
-            if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && (sp.col / B) % P == q.r && sp.col / B >= jlo &&
-                sp.col / B < jhi) {
+            if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && G.owner(inj_row_block(sp, B), sp.col / B) == q.r &&
+                sp.col / B >= jlo && sp.col / B < jhi) {
                 if (ei.n < kMaxEpiInj) {
                     EpiInjOp& e = ei.op[ei.n];
                     e.seg = sp.target == ABFT_TGT_DATA ? 0 : 1;
                     e.r = sp.target == ABFT_TGT_DATA ? sp.row - J0 * B : sp.row - 2 * J0;
-                    e.c = ((sp.col / B) / P - t0) * B + sp.col % B; e.mask = sp.xor_mask; e.pad = 0;
+                    e.c = ((sp.col / B) / Pc - t0) * B + sp.col % B; e.mask = sp.xor_mask; e.pad = 0;
                 }
                 ei.n++;
             }
@@ -1083,13 +1165,14 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         ColSumOut cso{q.w.cs, q.ncl, q.w.cs_nslab, J0 * B, t0 * B, B, 64, J0 * B};
         const int f = abft ? launch_update_with_chk((N - J0) * B, nt * B, B, W0, ldw, W0, ldw, C, q.lda, 2 * (N - J0),
                                                     W + mB + 2 + 2 * (J0 - k - 1), q.w.chk + t0 * B * q.w.ldc + 2 * J0,
-                                                    q.w.ldc, B, ab, s, all_fused ? &cso : nullptr, 0, P, &ei)
+                                                    q.w.ldc, B, ab, s, all_fused ? &cso : nullptr, 0, Pc, &ei, 2, Pr,
+                                                    rfirst)
                            : launch_update_with_chk((N - J0) * B, nt * B, B, W0, ldw, W0, ldw, C, q.lda, 0, W0, C,
-                                                    q.lda, B, ab, s, nullptr, 0, P);
+                                                    q.lda, B, ab, s, nullptr, 0, Pc, nullptr, 2, Pr, rfirst);
         if (f < 0) {   // shapes the strided launch cannot take (or ABFT off): one launch per block column
             if (ei.n > 0) all_fused = false;   // the hook is applied after the launches
-            for (int64_t J = J0; J < jhi; J += P) {
-                const int64_t t = J / P;
+            for (int64_t J = J0; J < jhi; J += Pc) {
+                const int64_t t = J / Pc;
                 double* Wj = W + (J - k - 1) * B;
                 double* Cj = q.A + t * B * q.lda + J * B;
                 ColSumOut csj{q.w.cs, q.ncl, q.w.cs_nslab, J * B, t * B, B, 64, J * B};
@@ -1097,7 +1180,8 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
                 if (abft)
                     fj = launch_update_with_chk((N - J) * B, B, B, Wj, ldw, Wj, ldw, Cj, q.lda, 2 * (N - J),
                                                 W + mB + 2 + 2 * (J - k - 1), q.w.chk + t * B * q.w.ldc + 2 * J,
-                                                q.w.ldc, B, ab, s, all_fused ? &csj : nullptr);
+                                                q.w.ldc, B, ab, s, all_fused ? &csj : nullptr, 0, 1, nullptr, 2, Pr,
+                                                ((q.pr - J % Pr) % Pr + Pr) % Pr);
                 else
                     fj = launch_gemm((N - J) * B, B, B, Wj, ldw, Wj, ldw, Cj, q.lda, -1.0, 1.0, true, 1, 0, 0, 0, 0, ab, s);
                 if (!(fj & 1)) all_fused = false;
@@ -1113,7 +1197,7 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
             std::vector<abft_inject_spec_t> sub;
             for (const auto& sp : inj)
                 if (sp.k == k && sp.hook == ABFT_HOOK_UPDATE_OUT && sp.col / B >= jlo && sp.col / B < jhi) sub.push_back(sp);
-            if (!sub.empty()) dist_inject(sub, k, ABFT_HOOK_UPDATE_OUT, B, P, q, ldw, mB, s);
+            if (!sub.empty()) dist_inject(sub, k, ABFT_HOOK_UPDATE_OUT, B, G, q, ldw, mB, s);
         }
         const bool gated = ((k + 1) % K == 0) || k == N - 2;
         if (!gated) return;
@@ -1133,19 +1217,19 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     {   // P streams see those injections before the first panel
         cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(PS, e, 0);
     }
-    for (auto& q : R) if (q.r == 0) { const int rcp = panel(q, 0); if (rcp) return rcp; }
+    { const int rcp = panel(0); if (rcp) return rcp; }
     if (N > 1) { int rc2 = bcast(0); if (rc2) return rc2; }
     for (int64_t k = 0; k + 1 < N; ++k) {
         for (int i = 0; i < nlocal; ++i) cudaStreamWaitEvent(s, evB[i], 0);      // panel k usable
-        const int o1 = (int)((k + 1) % P);
-        // (a) block column k+1 on its owner: update, UPDATE_OUT, V5 -> panel k+1 on PS
-        for (auto& q : R) {
-            if (q.r != o1) continue;
-            update(q, k, k + 1, k + 2);
+        const int c1 = (int)((k + 1) % Pc);
+        // (a) block column k+1 on its owners: update, UPDATE_OUT, V5 -> panel k+1 on PS
+        bool mine = false;
+        for (auto& q : R) if (q.pc == c1) { update(q, k, k + 1, k + 2); mine = true; }
+        if (mine) {
             cudaEvent_t ec = new_event(); cudaEventRecord(ec, s); cudaStreamWaitEvent(PS, ec, 0);
-            { const int rcp = panel(q, k + 1); if (rcp) return rcp; }
+            const int rcp = panel(k + 1); if (rcp) return rcp;
         }
-        // (b) the rest of update k on every rank (the owner of k+1 included)
+        // (b) the rest of update k on every rank (the owners of k+1 included)
         for (auto& q : R) update(q, k, k + 2, N);
         for (int i = 0; i < nlocal; ++i) { evUprev[i] = evU[i]; evU[i] = new_event(); cudaEventRecord(evU[i], s); }
         if (push && tp->mark_free(k + 1, s)) return ABFT_ERR_NCCL;   // buffer (k & 1) read for the last time
@@ -1162,12 +1246,14 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
         cudaEvent_t e = new_event(); cudaEventRecord(e, PS); cudaStreamWaitEvent(s, e, 0);
     }
     for (auto& q : R) {
+        if (q.Wt) cudaFreeAsync(q.Wt, s);
+        q.Wt = nullptr;
         if (q.Wb[1] && !push) cudaFreeAsync(q.Wb[1], s);
         q.Wb[1] = nullptr; q.w.W = push ? nullptr : q.Wb[0];   // push mode: the transport owns them
     }
     if (abft) {
         for (auto& q : R) {
-            dist_inject(inj, N, ABFT_HOOK_REST, B, P, q, 1, 0, s);
+            dist_inject(inj, N, ABFT_HOOK_REST, B, G, q, 1, 0, s);
             StageArgs a6 = stage(q, SK_ALL, ABFT_V6, (int)N);
             a6.factored = 1;
             launch_check(a6, s);                                                       // V6
@@ -1272,8 +1358,9 @@ extern "C" int abft_potrf_dist_sim(int64_t n, int64_t nb, int nranks, double* co
     if (!A_locals) return -4;
     if (lda_local < std::max<int64_t>(1, n)) return -5;
     std::vector<DistLocal> L(nranks);
+    const int Pc = (opt && opt->prows > 1 && nranks % opt->prows == 0) ? nranks / opt->prows : nranks;
     for (int r = 0; r < nranks; ++r) {
-        if (!A_locals[r] && (n / nb - r + nranks - 1) / nranks > 0) return -4;
+        if (!A_locals[r] && (n / nb - r % Pc + Pc - 1) / Pc > 0) return -4;
         L[r] = DistLocal{r, A_locals[r], lda_local};
     }
     return run_dist(n, nb, nranks, L.data(), nranks, nullptr, (cudaStream_t)stream, inj, rep, opt);

@@ -72,7 +72,7 @@ __device__ void phase1_reread(const StageArgs& a, int part, int64_t bid) {
     const int64_t c0 = (bid % chunks) * kChkCols;
     int64_t I, J;
     stage_tile(a, t, I, J);
-    const bool mine = (J % a.col_owner_mod == a.col_owner_rank);   // dist: this rank's column
+    const bool mine = tile_mine(a, I, J);   // dist: this rank's tile (CTA-uniform)
     const TileView v = stage_view(a, I, J);
     const int cw = (int)((B - c0) < kChkCols ? (B - c0) : kChkCols);
     __shared__ double s_r1[kChkCols], s_r2[kChkCols], s_r3[kChkCols];
@@ -161,7 +161,7 @@ __device__ void phase1_fused(const StageArgs& a, int part, int64_t bid) {
     const int64_t c = (bid % chunks) * kChkThreads + threadIdx.x;
     int64_t I, J;
     stage_tile(a, t, I, J);
-    if (J % a.col_owner_mod != a.col_owner_rank) return;   // CTA-uniform
+    if (!tile_mine(a, I, J)) return;   // CTA-uniform
     if (threadIdx.x == 0 && c == 0) atomicAdd(&a.st->n_checks, 1ull);
     const bool act = c < B;
     const TileView v = stage_view(a, I, J);

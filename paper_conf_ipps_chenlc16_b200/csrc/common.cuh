@@ -74,7 +74,13 @@ struct StageArgs {
     int32_t nchk, pad3;             // checksum rows per block: 2 or 3 (reading B10)
     double c_tau;
     int32_t col_owner_mod, col_owner_rank;  // dist: local column mapping (1, 0 on one GPU)
-    int32_t flist, pad2;            // flag list used by this stage (one per stream)
+    // dist, 2D block-cyclic (NEXT-3): tile (I, J) belongs to this rank iff J % col_owner_mod ==
+    // col_owner_rank and I % row_owner_mod == row_owner_rank (rows stay global: every rank stores its
+    // block columns full height and maintains only its own tiles); own_invert = 1 selects the tiles
+    // this rank does NOT own (V4R: the received panel tiles)
+    int32_t row_owner_mod, row_owner_rank;
+    int32_t own_invert;
+    int32_t flist;                  // flag list used by this stage (one per stream)
     int64_t j_lo, j_hi;             // SK_TRAIL*: block columns [j_lo, j_hi)
     const double* cs; int64_t cs_ld, cs_nslab, cs_slab_rows;   // SK_TRAIL_OFF: fused partials
     DevState* st;
@@ -135,6 +141,12 @@ __device__ __forceinline__ void stage_tile(const StageArgs& a, int64_t t, int64_
             J = j0 + jj; I = J + rem; return;
         }
     }
+}
+
+// Does this rank check tile (I, J) in this stage (dist ownership; always true on one GPU)?
+__device__ __forceinline__ bool tile_mine(const StageArgs& a, int64_t I, int64_t J) {
+    const bool own = (J % a.col_owner_mod == a.col_owner_rank) && (I % a.row_owner_mod == a.row_owner_rank);
+    return a.own_invert ? !own : own;
 }
 
 // Local column offset of global block column J (1D block-cyclic in dist mode).
@@ -270,12 +282,18 @@ struct DistTransport {
     virtual int post_panel(int64_t panel, cudaStream_t s) { (void)panel; (void)s; return 0; }  // owner: panel stored
     virtual int wait_panel(int root, int64_t panel, cudaStream_t s) { (void)root; (void)panel; (void)s; return 0; }
     virtual int mark_free(int64_t value, cudaStream_t s) { (void)value; (void)s; return 0; }     // this rank's reads done
+    // 2D block-cyclic push mode: the diagonal block's owner stores inv(L_kk) into the receive
+    // buffers of its process column and publishes it (post_li); those ranks wait for it (wait_li)
+    virtual int post_li(int64_t panel, cudaStream_t s) { (void)panel; (void)s; return 0; }
+    virtual int wait_li(int root, int64_t panel, cudaStream_t s) { (void)root; (void)panel; (void)s; return 0; }
 };
 // The owner's write-back of panel k fused with the push to its peers: data rows -> A panel,
-// checksum rows -> chk, the whole W (+ abort slot) -> every peer's receive buffer (util.cu).
+// checksum rows -> chk, the whole W (+ abort slot `slot`) -> every peer's receive buffer (util.cu).
+// 2D block-cyclic (rmod > 1): only the rows of this rank's tiles (data block b with b % rmod ==
+// dphase, checksum block c with c % rmod == cphase, two checksum rows per block) are written.
 int launch_panel_out(const double* W, int64_t ldw, int64_t mB, int64_t ncrows, int64_t B, double* Apanel,
                      int64_t lda, double* chk, int64_t ldc, double* const* peers, int npeer, const int32_t* abort_flag,
-                     cudaStream_t s);
+                     cudaStream_t s, int64_t rmod = 1, int64_t dphase = 0, int64_t cphase = 0, int slot = 0);
 // The 1D block-cyclic driver (abft.cu). ranks: local ranks driven by this call — one with a
 // transport (NCCL, one process per GPU) or all P of them with tp == nullptr (single-process
 // simulation on one device: the broadcast becomes a device-to-device copy).
@@ -295,11 +313,14 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
 // Panel TRSM + its checksum rows in one launch (second row segment); returns 1 if fused.
 int launch_trsm_with_chk(int64_t mB, int64_t B, const double* Ap, int64_t lda, const double* Li, double* W,
                          int64_t ldw, int64_t M2, const double* A2, int64_t lda2, const int32_t* abort_flag,
-                         cudaStream_t s);
+                         cudaStream_t s, int64_t rstride = 1, int64_t rfirst = 0);
+// rstride > 1 (2D block-cyclic): only the data-row blocks rfirst + u * rstride (relative to C's row
+// 0) are computed — this rank's tiles; the checksum segment is computed for every row.
 // Returns a bit mask: 1 = the fused V5 partials were written, 2 = the epilogue applied `inj`
 // (the caller applies the hook itself otherwise); -1 if cstride > 1 and the shapes do not allow it.
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s,
                            abft::ColSumOut* cs, int64_t lda2 = 0, int64_t cstride = 1,
-                           const abft::EpiInj* inj = nullptr, int nchk = 2);
+                           const abft::EpiInj* inj = nullptr, int nchk = 2, int64_t rstride = 1,
+                           int64_t rfirst = 0);

@@ -51,6 +51,11 @@ struct GemmArgs {
     // column-block stride (ws kernel, MASK_LOWER + checksum segment): column block t of C and of
     // the B operand's rows is global block t * cstride (1D block-cyclic local columns; 1 = dense)
     int64_t cstride;
+    // data-row block filter (ws kernel, 2D block-cyclic NEXT-3; rstride = 1: every row): only the
+    // nb-row blocks b = rfirst + u * rstride (relative to row 0 of A and C) are computed, the rest
+    // belong to other ranks. Rows stay global (no remapping of A or C), requires nb % BM == 0 and
+    // M % nb == 0 (the launchers fall back to rstride = 1, computing every row, otherwise)
+    int64_t rstride, rfirst;
     // ws kernel: prefetch into L2 the C tile of tile index t + pf_ahead (0 = off; the launcher
     // sets it to the number of CTAs resident at once)
     int64_t pf_ahead;
@@ -422,13 +427,29 @@ struct WsTile {
     bool seg2;              // checksum-row segment: A2 / C2 / ldc2 / M2, MASK_CHK with tile offsets 0
 };
 
+// Data-segment tile rows the ws kernel enumerates (the owned row blocks only when rstride > 1),
+// and the global tile row of enumerated tile row tmL.
+template <int BM>
+__host__ __device__ __forceinline__ int64_t ws_tm(const GemmArgs& g) {
+    const int64_t TM = (g.M + BM - 1) / BM;
+    if (g.rstride <= 1) return TM;
+    const int64_t nbt = g.nb / BM, NB = g.M / g.nb;
+    return NB > g.rfirst ? ((NB - g.rfirst + g.rstride - 1) / g.rstride) * nbt : 0;
+}
+template <int BM>
+__device__ __forceinline__ int64_t ws_row_of(const GemmArgs& g, int64_t tmL) {
+    if (g.rstride <= 1) return tmL;
+    const int64_t nbt = g.nb / BM;
+    return (g.rfirst + (tmL / nbt) * g.rstride) * nbt + tmL % nbt;
+}
+
 // tile index -> tile; returns false for tiles with nothing to write. Segment-1 tiles are
 // enumerated group by group (kWsGroup tile rows), column-major inside a group, so the CTAs
 // running at the same time share operand tiles in L2; the checksum-row segment follows.
 template <int BM, int BN>
 __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t n1tiles, WsTile& T) {
     constexpr int R = BM / BN;
-    const int64_t TN = g.tiles_n, TM = (g.M + BM - 1) / BM;
+    const int64_t TN = g.tiles_n, TM = ws_tm<BM>(g);
     int64_t tm, tn;
     if (idx >= n1tiles) {   // second segment: checksum rows, rectangular, row-major
         const int64_t e = idx - n1tiles;
@@ -437,10 +458,10 @@ __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t 
         const int64_t qmax = min(g.M2, T.m0 + BM) - 1;
         return chk_block(qmax, g.nchk) >= (T.n0 / g.nb) * g.cstride;
     }
-    if (g.mask == MASK_LOWER && g.cstride > 1) {   // strided columns: grouped rectangle, skip tiles above
+    if (g.mask == MASK_LOWER && (g.cstride > 1 || g.rstride > 1)) {   // strided: grouped rectangle, skip tiles above
         const int64_t q = idx / (kWsGroup * TN), a0 = q * kWsGroup, Gp = ((TM - a0) < kWsGroup ? (TM - a0) : (int64_t)kWsGroup);
         const int64_t e = idx - a0 * TN;
-        tn = e / Gp; tm = a0 + e % Gp;
+        tn = e / Gp; tm = ws_row_of<BM>(g, a0 + e % Gp);
         T.m0 = tm * BM; T.n0 = tn * BN; T.seg2 = false;
         const int64_t rmax = min(g.M, T.m0 + BM) - 1;
         return rmax >= T.n0 + (T.n0 / g.nb) * g.nb * (g.cstride - 1);
@@ -466,7 +487,7 @@ __device__ __forceinline__ bool ws_tile(const GemmArgs& g, int64_t idx, int64_t 
     } else {
         const int64_t q = idx / (kWsGroup * TN), a0 = q * kWsGroup, Gp = ((TM - a0) < kWsGroup ? (TM - a0) : (int64_t)kWsGroup);
         const int64_t e = idx - a0 * TN;
-        tn = e / Gp; tm = a0 + e % Gp;
+        tn = e / Gp; tm = ws_row_of<BM>(g, a0 + e % Gp);
     }
     T.m0 = tm * BM; T.n0 = tn * BN; T.seg2 = false;
     if (g.mask == MASK_CHK) {
@@ -818,9 +839,11 @@ static int run_ws(GemmArgs g, cudaStream_t s, bool update) {
         cudaFuncSetAttribute(k_update_ws<C_, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C_::SMEM);
         attr = true;
     }
-    const int64_t tm = (g.M + C_::BM - 1) / C_::BM, tn = (g.N + C_::BN - 1) / C_::BN;
+    if (g.rstride > 1 && (g.nb % C_::BM != 0 || g.M % g.nb != 0)) { g.rstride = 1; g.rfirst = 0; }   // every row
+    const int64_t tm = ws_tm<C_::BM>(g), tn = (g.N + C_::BN - 1) / C_::BN;
     g.tiles_n = tn;
-    const int64_t n1 = (g.mask == MASK_LOWER && g.cstride <= 1) ? lower_prefix<C_::BM / C_::BN>(tm, tn) : tm * tn;
+    const int64_t n1 = (g.mask == MASK_LOWER && g.cstride <= 1 && g.rstride <= 1) ? lower_prefix<C_::BM / C_::BN>(tm, tn)
+                                                                                  : tm * tn;
     const int64_t ntiles = n1 + (g.M2 > 0 ? ((g.M2 + C_::BM - 1) / C_::BM) * tn : 0);
     if (ntiles <= 0) return 0;
     // tiles per CTA: 1 lets the block scheduler interleave the high-priority look-ahead stream's
@@ -909,6 +932,7 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
     g.q_tile0 = q_tile0; g.c_tile0 = c_tile0; g.tiles_n = 1; g.abort = abort_flag;
     g.cs = cs ? *cs : ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0, 2};
     g.M2 = 0; g.A2 = nullptr; g.C2 = nullptr; g.ldc2 = 1; g.lda2 = 1; g.cstride = 1;
+    g.rstride = 1; g.rfirst = 0;
     g.inj.n = 0;
     g.vecA = aligned16(A) && (lda % 2 == 0);
     g.vecB = aligned16(B) && (ldb % 2 == 0);
@@ -953,7 +977,8 @@ int launch_gemm(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, c
 int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int64_t lda, const double* B,
                            int64_t ldb, double* C, int64_t ldc, int64_t M2, const double* A2, double* C2,
                            int64_t ldc2, int64_t nb, const int32_t* abort_flag, cudaStream_t s, ColSumOut* cs,
-                           int64_t lda2, int64_t cstride, const EpiInj* inj, int nchk) {
+                           int64_t lda2, int64_t cstride, const EpiInj* inj, int nchk, int64_t rstride,
+                           int64_t rfirst) {
     if (lda2 <= 0) lda2 = lda;
     if (cstride < 1) cstride = 1;
     // the data segment's kernel must not depend on the checksum segment (same rounding with two or
@@ -982,6 +1007,7 @@ int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int
     g.cs = ColSumOut{nullptr, 0, 0, 0, 0, 1, 64, 0, 2};
     g.inj.n = 0;
     g.nchk = nchk;
+    g.rstride = rstride > 1 ? rstride : 1; g.rfirst = rstride > 1 ? rfirst : 0;
     int ret = 0;
     bool inj_chk = false;   // a checksum-row target, which a split-off checksum launch cannot apply
     for (int q = 0; inj && q < inj->n && q < kMaxEpiInj; ++q) inj_chk |= inj->op[q].seg == 1;
@@ -1011,7 +1037,7 @@ int launch_update_with_chk(int64_t M, int64_t N, int64_t K, const double* A, int
 // would not fill the GPU (small panels) or the shapes do not allow it.
 int launch_trsm_with_chk(int64_t mB, int64_t B, const double* Ap, int64_t lda, const double* Li, double* W,
                          int64_t ldw, int64_t M2, const double* A2, int64_t lda2, const int32_t* abort_flag,
-                         cudaStream_t s) {
+                         cudaStream_t s, int64_t rstride, int64_t rfirst) {
     const int64_t tiles = ((mB + WsCfg::BM - 1) / WsCfg::BM) * ((B + 63) / 64);
     const bool ok = mB > 0 && M2 > 0 && tiles >= 148 && (mB % 2 == 0) && (M2 % 2 == 0) && (B % WsCfg::BK == 0) &&
                     (B % 2 == 0) && aligned16(Ap) && aligned16(Li) && aligned16(A2) && aligned16(W) && aligned16(W + mB) &&
@@ -1030,6 +1056,7 @@ int launch_trsm_with_chk(int64_t mB, int64_t B, const double* Ap, int64_t lda, c
     g.inj.n = 0;
     g.nchk = 2;   // the TRSM's second segment covers every row (column block 0 only)
     g.M2 = M2; g.A2 = A2; g.C2 = W + mB; g.ldc2 = ldw; g.lda2 = lda2; g.cstride = 1;
+    g.rstride = rstride > 1 ? rstride : 1; g.rfirst = rstride > 1 ? rfirst : 0;   // 2D: this rank's panel rows
     run_ws_any(g, s);
     return 1;
 }

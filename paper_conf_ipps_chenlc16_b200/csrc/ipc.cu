@@ -27,7 +27,8 @@ constexpr size_t kCtlBytes = 256;   // flag words at the head of every arena
 // posted/done: collective sequence numbers; panel: 1 + the last panel this rank pushed into its
 // peers' receive buffers; freed: panels p < freed + 2 may be pushed into this rank's buffers
 // (its update p - 2, the last reader of buffer p & 1, is complete)
-struct Ctl { unsigned long long posted, done, panel, freed; };
+// li: 1 + the last panel whose inv(L_kk) this rank (the diagonal block's owner, 2D) pushed
+struct Ctl { unsigned long long posted, done, panel, freed, li; };
 
 __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
     unsigned long long v;
@@ -46,12 +47,12 @@ __global__ void k_ipc_wait(PeerTable t, int np, int skip, int which, unsigned lo
     for (int r = 0; r < np; ++r) {
         if (r == skip) continue;
         const unsigned long long* w = which == 0 ? &t.ctl[r]->posted : which == 1 ? &t.ctl[r]->done
-                                    : which == 2 ? &t.ctl[r]->panel : &t.ctl[r]->freed;
+                                    : which == 2 ? &t.ctl[r]->panel : which == 3 ? &t.ctl[r]->freed : &t.ctl[r]->li;
         while (ld_acquire_sys(w) < v) __nanosleep(256);
     }
 }
 __device__ __forceinline__ const unsigned long long* ctl_word(const Ctl* c, int which) {
-    return which == 0 ? &c->posted : which == 1 ? &c->done : which == 2 ? &c->panel : &c->freed;
+    return which == 0 ? &c->posted : which == 1 ? &c->done : which == 2 ? &c->panel : which == 3 ? &c->freed : &c->li;
 }
 __global__ void k_ipc_wait_one(const Ctl* c, int which, unsigned long long v) {
     if (threadIdx.x != 0) return;
@@ -104,6 +105,14 @@ struct IpcTransport : DistTransport {
     }
     int wait_panel(int root, int64_t panel, cudaStream_t s) override {
         k_ipc_wait_one<<<1, 32, 0, s>>>(reinterpret_cast<const Ctl*>(peer[root]), 2, (unsigned long long)(panel + 1));
+        return cudaGetLastError() == cudaSuccess ? 0 : 1;
+    }
+    int post_li(int64_t panel, cudaStream_t s) override {
+        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 4, (unsigned long long)(panel + 1));
+        return cudaGetLastError() == cudaSuccess ? 0 : 1;
+    }
+    int wait_li(int root, int64_t panel, cudaStream_t s) override {
+        k_ipc_wait_one<<<1, 32, 0, s>>>(reinterpret_cast<const Ctl*>(peer[root]), 4, (unsigned long long)(panel + 1));
         return cudaGetLastError() == cudaSuccess ? 0 : 1;
     }
     int mark_free(int64_t value, cudaStream_t s) override {

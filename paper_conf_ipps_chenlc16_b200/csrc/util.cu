@@ -53,23 +53,26 @@ __global__ void k_abort_from_slot(const double* slot, DevState* st) {
 
 // Fused write-back + push (NEXT-3): one read of W per element; local stores (A panel / chk) and
 // one peer store per receiving rank (P2P over NVLink when the peer is another GPU). The abort slot
-// after the panel travels with it. Column c of W is blockIdx.y; rows in 16-byte pairs.
-struct PeerList { double* p[15]; int n, pad; };
+// `slot` after the panel travels with it. Column c of W is blockIdx.y; rows in 16-byte pairs.
+// 2D block-cyclic (rmod > 1): only this rank's rows move — data row r (block r / B) iff
+// (r / B) % rmod == dphase, checksum row q = r - mB (block q / 2) iff (q / 2) % rmod == cphase.
+struct PeerList { double* p[16]; int n, pad; };
 __global__ void k_panel_out(const double* W, int64_t ldw, int64_t mB, int64_t rows, int64_t B, double* Ap,
-                            int64_t lda, double* ck, int64_t ldc, PeerList peers, const int32_t* abort_flag) {
+                            int64_t lda, double* ck, int64_t ldc, PeerList peers, int64_t rmod, int64_t dphase,
+                            int64_t cphase, int slot) {
     const int64_t c = blockIdx.y;
     const double* col = W + c * ldw;
     for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 2; r < rows; r += (int64_t)gridDim.x * blockDim.x * 2) {
+        if (rmod > 1 && (r < mB ? (r / B) % rmod != dphase : ((r - mB) / 2) % rmod != cphase)) continue;
         const double2 v = *reinterpret_cast<const double2*>(col + r);   // ldw, mB even: pairs never straddle
         for (int q = 0; q < peers.n; ++q) *reinterpret_cast<double2*>(peers.p[q] + c * ldw + r) = v;
         if (r < mB) { Ap[c * lda + r] = v.x; Ap[c * lda + r + 1] = v.y; }   // mB even
         else { ck[c * ldc + (r - mB)] = v.x; if (r + 1 < rows) ck[c * ldc + (r + 1 - mB)] = v.y; }
     }
-    if (c == 0 && blockIdx.x == 0 && threadIdx.x == 0) {   // abort slot at W[ldw * B]
-        const double slot = W[ldw * B];
-        for (int q = 0; q < peers.n; ++q) peers.p[q][ldw * B] = slot;
+    if (c == 0 && blockIdx.x == 0 && threadIdx.x == 0) {   // abort slot at W[ldw * B + slot]
+        const double v = W[ldw * B + slot];
+        for (int q = 0; q < peers.n; ++q) peers.p[q][ldw * B + slot] = v;
     }
-    (void)abort_flag;
 }
 
 }  // namespace abft
@@ -78,15 +81,16 @@ using namespace abft;
 
 int launch_panel_out(const double* W, int64_t ldw, int64_t mB, int64_t ncrows, int64_t B, double* Apanel,
                      int64_t lda, double* chk, int64_t ldc, double* const* peers, int npeer, const int32_t* abort_flag,
-                     cudaStream_t s) {
+                     cudaStream_t s, int64_t rmod, int64_t dphase, int64_t cphase, int slot) {
+    (void)abort_flag;
     PeerList pl;
     pl.n = 0;
-    for (int q = 0; q < npeer && q < 15; ++q) pl.p[pl.n++] = peers[q];
-    if (npeer > 15) return -1;
+    if (npeer > 16) return -1;
+    for (int q = 0; q < npeer; ++q) pl.p[pl.n++] = peers[q];
     const int64_t rows = mB + ncrows;
     const int64_t bx = std::min<int64_t>(std::max<int64_t>((rows / 2 + 255) / 256, 1), 32);
     k_panel_out<<<dim3((unsigned)bx, (unsigned)B), 256, 0, s>>>(W, ldw, mB, rows, B, Apanel, lda, chk, ldc, pl,
-                                                               abort_flag);
+                                                               rmod < 1 ? 1 : rmod, dphase, cphase, slot);
     abft_count_launch();
     return 0;
 }
