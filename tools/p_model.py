@@ -1,33 +1,45 @@
-"""Model of the P-rank critical path of the 1D block-cyclic distributed factorisation at C4
-(DESIGN.md §5): per iteration k the step takes max(U_k / P, panel_{k+1}) — every rank applies its
-share of update k while the owner of column k+1 runs its panel chain (look-ahead depth 1).
+"""Model of the P-rank critical path of the distributed factorisation at C4: per
+iteration k the step takes max(U_k / P, panel_{k+1}) — every rank applies its share of update k
+while the owners of column k+1 run the panel chain (look-ahead depth 1).
 
-Inputs are the single-GPU measurements quoted in DESIGN.md §5/§7 (C4, n = 32768, nb = 512):
-363 ms of update per factorisation (bulk-copy producer; the LDGSTS producer is `ldg` times
-slower), the TRSM 13.7 ms in total, checks 0.25 ms per panel, write-back at 6 TB/s, broadcast at
-700 GB/s. Usage: python tools/p_model.py
+Inputs are single-GPU measurements at C4 (n = 32768, nb = 512; profiles/r02/bench_r02_final.jsonl):
+366 ms of update per factorisation, the diagonal block 20.2 ms in total (task graph, 0.32 ms per
+block), the TRSM 14.9 ms in total, checks 0.25 ms per panel, write-back at 6 TB/s; links at 700
+GB/s per direction (NVLink 5 usable).
+  1D: the owner of column k solves the whole panel and broadcasts it (NCCL: ~ w / link bandwidth).
+  2D (Pr x Pc grid, peer-memory push): the diagonal block's owner pushes inv(L_kk) (nb^2 doubles) to
+      its process column, each of the Pr column ranks solves 1/Pr of the panel and pushes its rows to
+      the P - 1 other ranks (egress w (P - 1) / Pr per contributor, ingress w per receiver).
+Usage: python tools/p_model.py
 """
 import sys
 
 n, nb = 32768, 512
 N = n // nb
-U_TOTAL, TRSM_TOTAL, CHECKS = 363.0, 13.7, 0.25     # ms
-WB_BW, BC_BW = 6.0e9, 0.7e9                          # bytes per ms
+U_TOTAL, DIAG_TOTAL, TRSM_TOTAL, CHECKS = 366.4, 20.2, 14.9, 0.25   # ms
+WB_BW, LINK = 6.0e9, 0.7e9                                          # bytes per ms
 
 
-def step_ms(P, diag_ms, ldg=1.0):
+def step_ms(P, Pr=1):
     ms = [N - k - 1 for k in range(N)]
     s2, s1 = sum(m * m for m in ms), sum(ms)
+    diag = DIAG_TOTAL / N
     t, bound = 0.0, 0
 
     def panel(k):
         m = ms[k]
         w = (m * nb + 2 * m + 2) * nb * 8
-        return diag_ms + TRSM_TOTAL * m / s1 + CHECKS + w / WB_BW + (w / BC_BW if P > 1 else 0.0)
+        if P == 1:
+            return diag + TRSM_TOTAL * m / s1 + CHECKS + w / WB_BW
+        if Pr == 1:   # owner solves everything, broadcast
+            return diag + TRSM_TOTAL * m / s1 + CHECKS + w / WB_BW + w / LINK
+        li = nb * nb * 8 / LINK
+        push = max(w * (P - 1) / Pr / LINK, w / LINK)
+        return diag + li + TRSM_TOTAL * m / s1 / Pr + CHECKS + w / Pr / WB_BW + push
 
     t += panel(0)
     for k in range(N):
-        u = ldg * U_TOTAL * ms[k] ** 2 / s2 / P
+        u = U_TOTAL * ms[k] ** 2 / s2 / P
         p = panel(k + 1) if k + 1 < N else 0.0
         if p > u:
             bound += 1
@@ -37,19 +49,15 @@ def step_ms(P, diag_ms, ldg=1.0):
 
 def main():
     flops = n ** 3 / 3
+    base1 = step_ms(1)[0]
+    print("| P | grid | modelled step | TFLOP/s | of linear | panel-bound iterations |")
+    print("|---|---|---|---|---|---|")
     rows = []
-    base1 = step_ms(1, 0.89)[0]
-    print("| P | recursive diagonal block (0.89 ms), bulk-copy update | panel-bound | "
-          "task-graph diagonal block (0.25 ms), LDGSTS update (x1.09) | panel-bound |")
-    print("|---|---|---|---|---|")
-    for P in (1, 2, 4, 8):
-        a, ba = step_ms(P, 0.89)
-        b, bb = step_ms(P, 0.25, 1.09)
-        ea = base1 / (P * a)
-        eb = base1 / (P * b)
-        rows.append((P, a, b))
-        print(f"| {P} | {a:.0f} ms ({flops / a / 1e9:.1f} TFLOP/s, {100 * ea:.0f} % of linear) | {ba} / {N} | "
-              f"{b:.0f} ms ({flops / b / 1e9:.1f} TFLOP/s, {100 * eb:.0f} %) | {bb} / {N} |")
+    for P, Pr in ((1, 1), (2, 1), (2, 2), (4, 1), (4, 2), (8, 1), (8, 2), (8, 4)):
+        t, b = step_ms(P, Pr)
+        grid = "1" if P == 1 else (f"1D x{P}" if Pr == 1 else f"2D {Pr}x{P // Pr}")
+        rows.append((P, Pr, t))
+        print(f"| {P} | {grid} | {t:.0f} ms | {flops / t / 1e9:.1f} | {100 * base1 / (P * t):.0f} % | {b} / {N} |")
     return rows
 
 
