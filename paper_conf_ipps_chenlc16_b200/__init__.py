@@ -18,7 +18,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libabft.so")
+# ABFT_LIB_NAME: another in-tree build of the same library (development A/B timing on one box)
+LIB_PATH = os.path.join(_HERE, os.environ.get("ABFT_LIB_NAME", "libabft.so"))
 
 # Codes restated from include/abft.h
 OK, UNCORRECTABLE, NOT_SPD, ERR_CUDA, ERR_NCCL = 0, 1, 2, 3, 4

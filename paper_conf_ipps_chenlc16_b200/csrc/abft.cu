@@ -17,6 +17,8 @@
 #include <algorithm>
 #include <cstdio>
 #include <cstring>
+#include <tuple>
+#include <utility>
 #include <vector>
 
 #include "common.cuh"
@@ -427,6 +429,10 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         prof.end(t_enc, PH_ENCODE, s, 4.0 * el, 8.0 * el);
     }
 
+    // ABFT_WB_EARLY=1: the main stream starts update k+1 as soon as panel k passed V3/V4 and the
+    // write-back of L(:,k) runs behind it (measured: -0.15 ms wait_panel but +1.2 ms of update at
+    // C4 from the concurrent write-back, profiles/r02/ab_wb_early.txt; off by default)
+    static const bool wb_early = [] { const char* e = getenv("ABFT_WB_EARLY"); return e && !strcmp(e, "1"); }();
     // ---- the panel of iteration k, on stream P ----
     auto panel = [&](int64_t k) {
         const int64_t m = N - k - 1, mB = m * B;
@@ -500,12 +506,21 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
                 }
             }
         }
+        // the panel is final once V3/V4 passed: the trailing update reads W, not A's panel, so with
+        // ABFT_WB_EARLY=1 the main stream may start while the write-back of L(:,k) runs behind it
+        cudaEvent_t ready = nullptr;
+        if (wb_early) { ready = new_event(); cudaEventRecord(ready, P); }
         t = prof.begin(P);
-        launch_copy(mB, B, W, ldw, Akk + B, lda, ab, P);                        // L panel
-        if (abft && !(abl & 1)) launch_copy(nc * m + nc, B, W + mB, ldw, w.chk + k * B * w.ldc + nc * k, w.ldc, ab, P);
+        if (abft && !(abl & 1) && mB % 2 == 0)   // L panel + its checksum rows: one pass over W, one launch
+            launch_panel_out(W, ldw, mB, nc * m + nc, B, Akk + B, lda, w.chk + k * B * w.ldc + nc * k, w.ldc, nullptr, 0,
+                             ab, P);
+        else {
+            launch_copy(mB, B, W, ldw, Akk + B, lda, ab, P);                    // L panel
+            if (abft && !(abl & 1)) launch_copy(nc * m + nc, B, W + mB, ldw, w.chk + k * B * w.ldc + nc * k, w.ldc, ab, P);
+        }
         prof.end(t, PH_WB, P, 0, 16.0 * (mBd + (abft ? (double)nc * (md + 1) : 0)) * Bd);
         cudaEvent_t e = new_event(); cudaEventRecord(e, P);
-        return e;
+        return std::make_pair(ready ? ready : e, e);
     };
 
     int64_t slab_rows_used = 64;
@@ -572,7 +587,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         }
     };
 
-    std::vector<cudaEvent_t> pan(N, nullptr);
+    std::vector<cudaEvent_t> pan(N, nullptr), wbk(N, nullptr);   // panel k checked / written back
     if (abft) {   // REST(0) outside block column 0 (column 0 is handled by the panel stream)
         const Loc L0{A, lda, w.chk, w.ldc, Wbuf[0], 1, 0};
         do_inject_if(inj, 0, ABFT_HOOK_REST, B, L0, ab, s, 0, 1, false);
@@ -580,12 +595,12 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     const bool sink = g_sink.host != nullptr && !ps;
     auto sink_col = [&](int64_t k) {   // L(kB:n, block column k) -> host, after panel k's write-back
         if (!sink) return;
-        cudaStreamWaitEvent(g_sink.cs, pan[k], 0);
+        cudaStreamWaitEvent(g_sink.cs, wbk[k], 0);
         cudaMemcpy2DAsync(g_sink.host + k * B * g_sink.ldh + k * B, g_sink.ldh * sizeof(double), A + k * B * lda + k * B,
                           lda * sizeof(double), (size_t)(n - k * B) * sizeof(double), (size_t)B,
                           cudaMemcpyDeviceToHost, g_sink.cs);
     };
-    pan[0] = panel(0);
+    std::tie(pan[0], wbk[0]) = panel(0);
     sink_col(0);
     for (int64_t k = 0; k < N; ++k) {
         {
@@ -606,7 +621,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         }
         cudaEvent_t ec = new_event(); cudaEventRecord(ec, s);
         cudaStreamWaitEvent(P, ec, 0);
-        pan[k + 1] = panel(k + 1);
+        std::tie(pan[k + 1], wbk[k + 1]) = panel(k + 1);
         sink_col(k + 1);
         // (b) the rest of the trailing matrix
         if (m > 1) {
@@ -617,10 +632,13 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
             }
         }
         if (abft) {   // REST(k+1) outside block column k+1 (that one was applied on P)
+            // a target in a finished panel must follow its write-back (which runs behind S on P)
+            if (has_inj(inj, k + 1, ABFT_HOOK_REST)) cudaStreamWaitEvent(s, wbk[k], 0);
             const Loc L1{A, lda, w.chk, w.ldc, Wbuf[(k + 1) & 1], 1, 0};
             do_inject_if(inj, k + 1, ABFT_HOOK_REST, B, L1, ab, s, k + 1, k + 2, false);
         }
     }
+    if (N > 0) cudaStreamWaitEvent(s, wbk[N - 1], 0);   // every write-back (P is in order) before V6 / the end
     if (abft && !(abl & 16)) {
         const Loc L{A, lda, w.chk, w.ldc, w.W, 1, 0};
         do_inject(inj, N, ABFT_HOOK_REST, B, L, ab, s);
@@ -889,8 +907,8 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     // push mode (NEXT-3): a peer-memory transport owns every rank's two receive buffers; the owner's
     // write-back kernel stores the panel straight into them (launch_panel_out)
     const bool push = tp && tp->recv_buf(tp->rank, 0) != nullptr && tp->recv_capacity() >= wbuf &&
-                      tp->nranks <= 16 && getenv("ABFT_DIST_PULL") == nullptr;
-    if (Pr > 1 && tp && !push) return -11;   // 2D needs peer memory (IPC transport) or the one-device harness
+                      tp->nranks <= 16 && nb % 2 == 0 && getenv("ABFT_DIST_PULL") == nullptr;
+    if (Pr > 1 && ((tp && !push) || nb % 2)) return -11;   // the row-filtered push moves 16-byte row pairs   // 2D needs peer memory (IPC transport) or the one-device harness
     for (int i = 0; i < nlocal; ++i) {
         RankState& q = R[i];
         q.r = locals[i].rank; q.pr = q.r / Pc; q.pc = q.r % Pc; q.A = locals[i].A; q.lda = locals[i].lda;
@@ -1075,8 +1093,12 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
                 q.w.W = q.Wb[k & 1];
                 continue;
             }
-            launch_copy(mB, B, q.w.W, ldw, Akk + B, q.lda, ab, PS);
-            if (abft) launch_copy(ncr, B, q.w.W + mB, ldw, ckk + 2 * k, q.w.ldc, ab, PS);
+            if (abft && mB % 2 == 0 && ldw % 2 == 0)
+                launch_panel_out(q.w.W, ldw, mB, ncr, B, Akk + B, q.lda, ckk + 2 * k, q.w.ldc, nullptr, 0, ab, PS);
+            else {
+                launch_copy(mB, B, q.w.W, ldw, Akk + B, q.lda, ab, PS);
+                if (abft) launch_copy(ncr, B, q.w.W + mB, ldw, ckk + 2 * k, q.w.ldc, ab, PS);
+            }
             q.w.W = q.Wb[k & 1];
         }
         return 0;

@@ -27,7 +27,12 @@ __device__ __forceinline__ void note_ratio(DevState* st, double q) {
     q = fmax(q, __shfl_xor_sync(0xffffffffu, q, 4));
     q = fmax(q, __shfl_xor_sync(0xffffffffu, q, 2));
     q = fmax(q, __shfl_xor_sync(0xffffffffu, q, 1));
-    if ((threadIdx.x & 31) == 0 && q > 0.0) atomicMax(&st->max_ratio_bits, (unsigned long long)__double_as_longlong(q));
+    // one atomic per warp at most, and only when it raises the maximum (the common fault-free case
+    // reads the current value and skips the atomic: thousands of warps per launch hit one address)
+    if ((threadIdx.x & 31) == 0 && q > 0.0) {
+        const unsigned long long b = (unsigned long long)__double_as_longlong(q);
+        if (b > __ldcg(&st->max_ratio_bits)) atomicMax(&st->max_ratio_bits, b);
+    }
 }
 
 // Compare a recalculated column with its stored checksums, flag it if |d| > tau or d is
@@ -490,10 +495,11 @@ __global__ void __launch_bounds__(kChkThreads, 4) k_check(StageArgs a0, StageArg
         else phase1_reread(a, p1 ? 1 : 0, bid);
     }
     if (a0.encode) return;   // encode launches resolve nothing (no counter use)
-    __threadfence();
+    // the CTA's flags are ordered before its completion count by the barrier and thread 0's
+    // (cumulative) gpu-scope fence: one fence per CTA, not one per thread
     __syncthreads();
     const int fl = a0.flist;
-    if (threadIdx.x == 0) s_last = atomicAdd(&a0.st->done[fl], 1u) == gridDim.x - 1;
+    if (threadIdx.x == 0) { __threadfence(); s_last = atomicAdd(&a0.st->done[fl], 1u) == gridDim.x - 1; }
     __syncthreads();
     if (!s_last) return;
     __threadfence();

@@ -59,10 +59,12 @@ __global__ void k_abort_from_slot(const double* slot, DevState* st) {
 struct PeerList { double* p[16]; int n, pad; };
 __global__ void k_panel_out(const double* W, int64_t ldw, int64_t mB, int64_t rows, int64_t B, double* Ap,
                             int64_t lda, double* ck, int64_t ldc, PeerList peers, int64_t rmod, int64_t dphase,
-                            int64_t cphase, int slot) {
+                            int64_t cphase, int slot, const int32_t* abort_flag) {
     const int64_t c = blockIdx.y;
     const double* col = W + c * ldw;
-    for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 2; r < rows; r += (int64_t)gridDim.x * blockDim.x * 2) {
+    // after an abort only the abort slot travels (the receivers stop on it)
+    const int64_t rows_live = *(volatile const int32_t*)abort_flag ? 0 : rows;
+    for (int64_t r = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) * 2; r < rows_live; r += (int64_t)gridDim.x * blockDim.x * 2) {
         if (rmod > 1 && (r < mB ? (r / B) % rmod != dphase : ((r - mB) / 2) % rmod != cphase)) continue;
         const double2 v = *reinterpret_cast<const double2*>(col + r);   // ldw, mB even: pairs never straddle
         for (int q = 0; q < peers.n; ++q) *reinterpret_cast<double2*>(peers.p[q] + c * ldw + r) = v;
@@ -82,7 +84,6 @@ using namespace abft;
 int launch_panel_out(const double* W, int64_t ldw, int64_t mB, int64_t ncrows, int64_t B, double* Apanel,
                      int64_t lda, double* chk, int64_t ldc, double* const* peers, int npeer, const int32_t* abort_flag,
                      cudaStream_t s, int64_t rmod, int64_t dphase, int64_t cphase, int slot) {
-    (void)abort_flag;
     PeerList pl;
     pl.n = 0;
     if (npeer > 16) return -1;
@@ -90,7 +91,7 @@ int launch_panel_out(const double* W, int64_t ldw, int64_t mB, int64_t ncrows, i
     const int64_t rows = mB + ncrows;
     const int64_t bx = std::min<int64_t>(std::max<int64_t>((rows / 2 + 255) / 256, 1), 32);
     k_panel_out<<<dim3((unsigned)bx, (unsigned)B), 256, 0, s>>>(W, ldw, mB, rows, B, Apanel, lda, chk, ldc, pl,
-                                                               rmod < 1 ? 1 : rmod, dphase, cphase, slot);
+                                                               rmod < 1 ? 1 : rmod, dphase, cphase, slot, abort_flag);
     abft_count_launch();
     return 0;
 }
