@@ -52,9 +52,13 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=32768)
+    ap.add_argument("--n", "--matrix-n", dest="n", type=int, default=32768)
     ap.add_argument("--nb", type=int, default=512)
     ap.add_argument("--no-extras", action="store_true", help="main metric only (for ncu launch lists)")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "ipc"],
+                    help="N > 1: NCCL panel broadcast, or the peer-memory (CUDA IPC) fused push (NEXT-3)")
+    ap.add_argument("--prows", type=int, default=1,
+                    help="N > 1: process-grid rows of a 2D block-cyclic layout (needs --transport ipc); 1 = 1D")
     return ap.parse_args()
 
 
@@ -199,25 +203,32 @@ def golden_equal(events, P):
     return P.sorted_event_tuples(events) == want
 
 
-def recv_injections(n, nb, world):
-    """RECV hooks for the multi-GPU injected run: rank (k+1) mod P corrupts its received copy of
-    panel k (never the owner k mod P)."""
+def grid_owner(I, J, world, prows):
+    pc = world // prows
+    return (I % prows) * pc + J % pc
+
+
+def recv_injections(n, nb, world, prows=1):
+    """RECV hooks for the multi-GPU injected run: a rank that does not own the target tile of panel
+    k corrupts its received copy (1D: rank (k+1) mod P, never the owner k mod P)."""
     N = n // nb
     out = []
     for k in range(0, N - 1, 5):
-        r = (k + 1) % world
-        out.append(dict(k=k, hook="RECV", target="DATA", row=(k + 1) * nb + (7 * k) % ((N - k - 1) * nb),
-                        col=k * nb + (3 * k) % nb, bit=50, rank=r))
+        row = (k + 1) * nb + (7 * k) % ((N - k - 1) * nb)
+        r = (grid_owner(row // nb, k, world, prows) + 1) % world
+        out.append(dict(k=k, hook="RECV", target="DATA", row=row, col=k * nb + (3 * k) % nb, bit=50, rank=r))
     return out
 
 
-def events_vs_prediction(events, specs, n, nb, P):
+def events_vs_prediction(events, specs, n, nb, P, world=1, prows=1):
     """Every injection must produce exactly the event the verification schedule predicts
     (tests/_predict.py): same (k, check, tile, column, row); kind DATA (or NONFINITE for an
-    overflowing flip, located by the same row) / CHK1 / CHK2."""
+    overflowing flip, located by the same row) / CHK1 / CHK2; the rank that ran the check is the
+    tile's owner (the receiver for V4R)."""
     from tests._predict import predict
     got = sorted(t[:6] + (t[7],) for t in P.sorted_event_tuples(events))
-    want = sorted(p[:6] + (p[7],) for p in (predict(s, n, nb) for s in specs))
+    want = sorted(p[:6] + (p[7] if p[1] == 7 else grid_owner(p[3], p[2], world, prows),)
+                  for p in (predict(s, n, nb) for s in specs))
     kinds_ok = all(int(e["kind"]) in (1, 2, 3, 4) for e in events)
     return got == want and kinds_ok
 
@@ -236,11 +247,20 @@ def main():
     import synthetic as syn
 
     local = int(os.environ.get("LOCAL_RANK", 0))
+    # BENCH_SHARE_DEVICE=1 (code-path check only, not a measurement): every rank on device 0 with
+    # the peer-memory transport and gloo host plumbing (NCCL refuses two ranks on one device)
+    share = os.environ.get("BENCH_SHARE_DEVICE") == "1"
+    if share:
+        local = 0
+        args.transport = "ipc"
     torch.cuda.set_device(local)
     dist = world > 1
     if dist:
         import torch.distributed as tdist
-        tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            tdist.init_process_group("gloo")
+        else:
+            tdist.init_process_group("nccl", device_id=torch.device("cuda", local))
     n, nb = args.n, args.nb
     flops = n ** 3 / 3
     stream = torch.cuda.current_stream()
@@ -248,18 +268,25 @@ def main():
     A0 = torch.empty(n, n, dtype=torch.float64, device="cuda").T
     assert P.abft_gen_spd(n, A0) == 0
     comm = None
+    prows = args.prows if dist else 1
     if dist:
-        # 1D block-cyclic: this rank keeps its block columns (J mod world == rank)
-        idx = torch.cat([torch.arange(J * nb, (J + 1) * nb) for J in P.owned_blocks(n // nb, rank, world)])
+        # block-cyclic: this rank keeps its block columns (J mod Pc == rank mod Pc; 1D: Pc = world),
+        # full height (2D: it maintains only the tiles of its process row)
+        pcols = world // prows
+        idx = torch.cat([torch.arange(J * nb, (J + 1) * nb) for J in P.owned_blocks(n // nb, rank % pcols, pcols)])
         A0 = A0.T[idx.cuda()].contiguous().T          # column-major n x n_local
         torch.cuda.synchronize()
-        nid = P.nccl_id_exchange()
-        st, comm = P.abft_comm_init(world, nid, rank)
-        assert st == 0, "abft_comm_init failed"
+        if args.transport == "ipc":
+            comm = P.ipc_comm(n, nb)
+        else:
+            nid = P.nccl_id_exchange()
+            st, comm = P.abft_comm_init(world, nid, rank)
+            assert st == 0, "abft_comm_init failed"
     A = torch.empty_like(A0.T).T
 
     def factor(opt, inj=None, cap=4096):
         if dist:
+            opt.prows = prows
             return P.abft_potrf_dist(n, nb, A, comm, rank, world, inj=inj, opt=opt, report=True, cap=cap)
         return P.abft_potrf_ex(n, nb, A, inj=inj, opt=opt, report=True, cap=cap)
 
@@ -273,7 +300,7 @@ def main():
         if not dist:
             return x
         import torch.distributed as tdist
-        t = torch.tensor([x], device="cuda")
+        t = torch.tensor([x], device="cpu" if share else "cuda")
         tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
         return t.item()
 
@@ -335,7 +362,9 @@ def main():
         "config": {"workload": wk, "n": n, "nb": nb,
                    "l2": "inputs (8 GiB) larger than L2; restore copy between steps outside the CUDA events",
                    "timing": "median of the K steps (CUDA events on the launching stream), max over ranks",
-                   "parallelism": f"1D block-cyclic x{world}, NCCL panel broadcast" if world > 1 else "single GPU"},
+                   "parallelism": ("single GPU" if world == 1 else
+                                   f"{'1D' if prows == 1 else f'2D {prows}x{world // prows}'} block-cyclic x{world}, "
+                                   f"{'NCCL panel broadcast' if args.transport == 'nccl' else 'peer-memory panel push'}")},
         "gpu_launches": int(launches) * args.steps,
         "roofline": {"bound": "tensor", "kernel": "k_update_ws (warp-specialised DMMA, 128x64 tiles, 2 CTAs/SM) trailing SYRK update + checksum rows",
                      "achieved": round(achieved, 3) if achieved else None,
@@ -384,7 +413,7 @@ def main():
     # every event checked against the schedule's prediction
     specs = syn.mixed_injections(n, nb)
     if dist:
-        specs += recv_injections(n, nb, world)
+        specs += recv_injections(n, nb, world, prows)
     inj = syn.inj_array(specs)
     t_inj, rep_inj = run_steps(P.options(), inj=inj, steps=max(1, min(3, args.steps)), warmup=1, fault_free=False)
     r0 = rep_inj[-1]
@@ -393,7 +422,8 @@ def main():
                         "injections": len(specs), "events": int(r0["n_events"]),
                         "corrected": int(r0["n_data"] + r0["n_nonfinite"] + r0["n_chk1"] + r0["n_chk2"]),
                         "uncorrectable": int(r0["n_uncorrectable"]),
-                        "events_match_schedule_prediction": bool(rank != 0 or events_vs_prediction(r0["events"], specs, n, nb, P)),
+                        "events_match_schedule_prediction": bool(rank != 0 or events_vs_prediction(r0["events"], specs, n, nb, P,
+                                                                                                   world, prows)),
                         "overhead_vs_fault_free_pct": round(100 * (ms_inj - ms) / ms, 3)}
 
     if world == 1:

@@ -908,7 +908,10 @@ int run_dist(int64_t n, int64_t nb, int P, const DistLocal* locals, int nlocal, 
     // write-back kernel stores the panel straight into them (launch_panel_out)
     const bool push = tp && tp->recv_buf(tp->rank, 0) != nullptr && tp->recv_capacity() >= wbuf &&
                       tp->nranks <= 16 && nb % 2 == 0 && getenv("ABFT_DIST_PULL") == nullptr;
-    if (Pr > 1 && ((tp && !push) || nb % 2)) return -11;   // the row-filtered push moves 16-byte row pairs   // 2D needs peer memory (IPC transport) or the one-device harness
+    // 2D needs peer memory (IPC transport) or the one-device harness; the row-filtered push moves
+    // 16-byte row pairs
+    if (Pr > 1 && ((tp && !push) || nb % 2)) return -11;
+    if (tp && tp->begin_call(N, s)) return ABFT_ERR_NCCL;   // fresh flag range for this call (IPC)
     for (int i = 0; i < nlocal; ++i) {
         RankState& q = R[i];
         q.r = locals[i].rank; q.pr = q.r / Pc; q.pc = q.r % Pc; q.A = locals[i].A; q.lda = locals[i].lda;

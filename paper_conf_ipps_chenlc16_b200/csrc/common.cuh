@@ -284,6 +284,10 @@ struct DistTransport {
     virtual int mark_free(int64_t value, cudaStream_t s) { (void)value; (void)s; return 0; }     // this rank's reads done
     // 2D block-cyclic push mode: the diagonal block's owner stores inv(L_kk) into the receive
     // buffers of its process column and publishes it (post_li); those ranks wait for it (wait_li)
+    // start of one factorisation with N block columns: flag-based transports move their flag
+    // values to a fresh range, so that flags left by an earlier call on this comm cannot satisfy
+    // this call's waits
+    virtual int begin_call(int64_t N, cudaStream_t s) { (void)N; (void)s; return 0; }
     virtual int post_li(int64_t panel, cudaStream_t s) { (void)panel; (void)s; return 0; }
     virtual int wait_li(int root, int64_t panel, cudaStream_t s) { (void)root; (void)panel; (void)s; return 0; }
 };

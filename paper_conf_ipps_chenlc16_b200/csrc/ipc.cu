@@ -82,6 +82,9 @@ struct IpcTransport : DistTransport {
     size_t cap = 0;                       // data bytes per arena (= bytes of each receive buffer)
     std::vector<char*> peer;              // mapped arenas (peer[rank] == mine)
     unsigned long long seq = 0;           // collectives issued (same sequence on every rank)
+    // push-mode flag values of the current call are base + (panel index ...): every call moves base
+    // past the previous call's range (same N and call sequence on every rank)
+    unsigned long long base = 0, stride = 0;
     PeerTable table() const {
         PeerTable t;
         memset(&t, 0, sizeof t);
@@ -94,29 +97,37 @@ struct IpcTransport : DistTransport {
     // push mode: receive buffer `slot` of rank r (mapped into this process)
     double* recv_buf(int r, int slot) override { return reinterpret_cast<double*>(peer[r] + kCtlBytes + slot * cap); }
     size_t recv_capacity() const override { return cap / sizeof(double); }
+    int begin_call(int64_t N, cudaStream_t s) override {
+        // the previous call on this comm finished on every rank (its closing collectives need every
+        // rank's updates), so this rank's receive buffers are free: freed = the new base
+        base += stride;
+        stride = (unsigned long long)N + 4;
+        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 3, base);
+        return cudaGetLastError() == cudaSuccess ? 0 : 1;
+    }
     int wait_free(int64_t panel, cudaStream_t s) override {   // every peer finished update panel - 2
         const PeerTable t = table();
-        k_ipc_wait<<<1, 32, 0, s>>>(t, nranks, rank, 3, (unsigned long long)(panel >= 1 ? panel - 1 : 0));
+        k_ipc_wait<<<1, 32, 0, s>>>(t, nranks, rank, 3, base + (unsigned long long)(panel >= 1 ? panel - 1 : 0));
         return cudaGetLastError() == cudaSuccess ? 0 : 1;
     }
     int post_panel(int64_t panel, cudaStream_t s) override {
-        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 2, (unsigned long long)(panel + 1));
+        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 2, base + (unsigned long long)(panel + 1));
         return cudaGetLastError() == cudaSuccess ? 0 : 1;
     }
     int wait_panel(int root, int64_t panel, cudaStream_t s) override {
-        k_ipc_wait_one<<<1, 32, 0, s>>>(reinterpret_cast<const Ctl*>(peer[root]), 2, (unsigned long long)(panel + 1));
+        k_ipc_wait_one<<<1, 32, 0, s>>>(reinterpret_cast<const Ctl*>(peer[root]), 2, base + (unsigned long long)(panel + 1));
         return cudaGetLastError() == cudaSuccess ? 0 : 1;
     }
     int post_li(int64_t panel, cudaStream_t s) override {
-        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 4, (unsigned long long)(panel + 1));
+        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 4, base + (unsigned long long)(panel + 1));
         return cudaGetLastError() == cudaSuccess ? 0 : 1;
     }
     int wait_li(int root, int64_t panel, cudaStream_t s) override {
-        k_ipc_wait_one<<<1, 32, 0, s>>>(reinterpret_cast<const Ctl*>(peer[root]), 4, (unsigned long long)(panel + 1));
+        k_ipc_wait_one<<<1, 32, 0, s>>>(reinterpret_cast<const Ctl*>(peer[root]), 4, base + (unsigned long long)(panel + 1));
         return cudaGetLastError() == cudaSuccess ? 0 : 1;
     }
     int mark_free(int64_t value, cudaStream_t s) override {
-        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 3, (unsigned long long)value);
+        k_ipc_set<<<1, 32, 0, s>>>(my_ctl(), 3, base + (unsigned long long)value);
         return cudaGetLastError() == cudaSuccess ? 0 : 1;
     }
     // publish `bytes` from src into my arena as collective s (after every peer finished s-1)

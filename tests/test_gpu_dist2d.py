@@ -133,16 +133,23 @@ def _worker(rank, world, prows, port, n, nb, specs, q):
     At = P.colmajor(P.block_cyclic_split_2d(A, nb, world, prows)[rank])
     comm = P.ipc_comm(n, nb)
     inj = syn.inj_array(specs) if specs else None
+    A0 = At.clone()
+    # two calls on the same comm (the transport's flags must not leak from one call into the next),
+    # a fault-free one first, then the injected one
+    st0, rep0 = P.abft_potrf_dist(n, nb, At, comm, rank, world, lda=n, opt=P.options(prows=prows))
+    torch.cuda.synchronize()
+    At.copy_(A0)
     st, rep = P.abft_potrf_dist(n, nb, At, comm, rank, world, lda=n, inj=inj, opt=P.options(prows=prows))
     torch.cuda.synchronize()
     L = P.to_numpy_colmajor(At)
     dist.barrier()
     P.abft_comm_destroy(comm)
+    assert st0 == 0 and rep0["n_events"] == 0, (st0, rep0["n_events"])
     q.put((rank, st, P.sorted_event_tuples(rep["events"]), L))
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,prows", [(2, 2), (4, 2)])
+@pytest.mark.parametrize("world,prows", [(2, 1), (2, 2), (4, 2)])
 def test_processes_ipc_2d_match_oracle(P, world, prows):
     import torch.multiprocessing as mp
     n, nb = 1024, 128
