@@ -1767,7 +1767,6 @@ extern "C" int abft_dev_chol_trace(int64_t nb, double* A, int64_t lda, double* L
                                    abft_stream_t stream) {
     const int nt = chol_task_count(nb);
     if (nt <= 0 || cap < 4 * (int64_t)nt) return -1;
-    cudaStream_t s = (cudaStream_t)stream;
     unsigned long long* d = nullptr;
     ABFT_CUDA_TRY(cudaMalloc((void**)&d, sizeof(uint64_t) * 4 * (size_t)nt));
     ABFT_CUDA_TRY(cudaMemset(d, 0, sizeof(uint64_t) * 4 * (size_t)nt));
@@ -1776,7 +1775,6 @@ extern "C" int abft_dev_chol_trace(int64_t nb, double* A, int64_t lda, double* L
     chol_set_trace(nullptr);
     ABFT_CUDA_TRY(cudaMemcpy(trace_host, d, sizeof(uint64_t) * 4 * (size_t)nt, cudaMemcpyDeviceToHost));
     cudaFree(d);
-    (void)s;
     return st == 0 ? nt : -2;
 }
 

@@ -535,8 +535,6 @@ __device__ __forceinline__ void ws_body(const GemmArgs& g, int64_t ntiles, int64
             const int kt_n = (int)(ke / BK);
             const int64_t Ms = T.seg2 ? g.M2 : g.M;
             const double* Ap = T.seg2 ? g.A2 : g.A;
-            double* Cp = T.seg2 ? g.C2 : g.C;
-            const int64_t ldcp = T.seg2 ? g.ldc2 : g.ldc;
             const uint32_t rowsA = (uint32_t)(Ms - m0 < BM ? Ms - m0 : BM), rowsB = (uint32_t)(g.N - n0 < BN ? g.N - n0 : BN);
             const int64_t bn0 = n0 + (g.cstride > 1 ? (n0 / g.nb) * g.nb * (g.cstride - 1) : 0);   // B row of column n0
             for (int kt = 0; kt < kt_n; ++kt, ++it) {
