@@ -211,3 +211,41 @@ def test_fault_free_runs_raise_no_event(P, path, monkeypatch):
         torch.cuda.synchronize()
         assert st == 0 and rep["n_events"] == 0, (path, rep_i, st, P.sorted_event_tuples(rep["events"])[:4])
         assert rep["max_noise_ratio"] <= 2.0 ** -6
+
+
+@pytest.mark.skipif(not __import__("os").environ.get("ABFT_FULL_C4"),
+                    reason="whole-factor C4 parity: ~7 min of oracle time (ABFT_FULL_C4=1; log in profiles/r02/)")
+@pytest.mark.parametrize("case", ["clean", "mixed_injections"])
+def test_c4_whole_factor_vs_oracle(P, case):
+    """C4 (n = 32768, nb = 512, the headline workload) in the bench's launch configuration: the WHOLE
+    factor elementwise against the oracle (1e-11 floor-relative fault-free; the B6 tolerance with
+    corrections), every event identical to the oracle's, the literal max-relative error reported."""
+    import time
+    import torch
+    n, nb = 32768, 512
+    A = syn.spd_matrix(n)
+    specs = syn.mixed_injections(n, nb) if case == "mixed_injections" else []
+    inj = syn.inj_array(specs) if specs else None
+    At = P.colmajor(A)
+    st, rep = P.abft_potrf_ex(n, nb, At, inj=inj, cap=1 << 14)
+    torch.cuda.synchronize()
+    L = P.to_numpy_colmajor(At)
+    del At
+    torch.cuda.empty_cache()
+    t0 = time.time()
+    ref = oracle.potrf(A, nb, inj=inj, cap=1 << 14)
+    t_oracle = time.time() - t0
+    assert st == ref.status == 0
+    assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
+    fr = floor_rel(L, ref.L, A)
+    lit = literal_max_rel(L, ref.L)
+    print(f"C4 {case}: events {len(ref.events)}, floor-rel {fr:.3e}, literal max-rel {lit:.3e}, "
+          f"oracle {t_oracle:.1f} s ({n ** 3 / 3 / t_oracle / 1e9:.1f} GFLOP/s, {oracle.num_threads()} threads)")
+    if not specs:
+        assert fr <= 1e-11, fr
+    else:   # reading B6, the bound of the C3 test: corrected values carry the checksum's noise
+        s = np.sqrt(np.diag(A))
+        tau1_max = 64 * EPS * max(s[I * nb:(I + 1) * nb].sum() for I in range(n // nb)) * s.max()
+        noise = max(rep["max_noise_ratio"], float(ref.counts["max_ratio"]))
+        bound = 1e-11 + 2 * noise * tau1_max / (1e-3 * s.min())
+        assert fr <= bound, (fr, bound)
