@@ -6,6 +6,9 @@
 // bandwidth-bound launch covers every tile of a check stage: one warp per tile column,
 // coalesced column loads and warp-shuffle reductions (the mirrored half of an unfactored
 // diagonal tile is read row-wise, also coalesced).
+#include <algorithm>
+#include <cstdlib>
+
 #include "common.cuh"
 
 namespace abft {
@@ -484,15 +487,20 @@ __device__ void phase2_body(const StageArgs& a0, const StageArgs& a1, int flist)
 // oracle's order. Every CTA reaches the completion counter (also when the run is aborted), and
 // the last one resets it, so the counter is zero again for the next launch on this flag list.
 // min 4 CTAs/SM: phase 1 is the hot part (bandwidth-bound); the rare phase 2 may spill instead
-__global__ void __launch_bounds__(kChkThreads, 4) k_check(StageArgs a0, StageArgs a1, int64_t nblk0) {
+// The grid may be smaller than the work (launch_check caps it, ABFT_CHK_GRID): each CTA then takes
+// work blocks blockIdx.x, + gridDim.x, ... so its fixed costs are paid once for several tiles.
+__global__ void __launch_bounds__(kChkThreads, 4) k_check(StageArgs a0, StageArgs a1, int64_t nblk0, int64_t nblk) {
     __shared__ int s_last;
     const bool aborted = cta_aborted(&a0.st->abort);
     if (!aborted) {
-        const bool p1 = (int64_t)blockIdx.x >= nblk0;
-        const StageArgs& a = p1 ? a1 : a0;
-        const int64_t bid = p1 ? (int64_t)blockIdx.x - nblk0 : (int64_t)blockIdx.x;
-        if (a.kind == SK_TRAIL_OFF) phase1_fused(a, p1 ? 1 : 0, bid);
-        else phase1_reread(a, p1 ? 1 : 0, bid);
+        for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+            const bool p1 = blk >= nblk0;
+            const StageArgs& a = p1 ? a1 : a0;
+            const int64_t bid = p1 ? blk - nblk0 : blk;
+            if (a.kind == SK_TRAIL_OFF) phase1_fused(a, p1 ? 1 : 0, bid);
+            else phase1_reread(a, p1 ? 1 : 0, bid);
+            if (blk + gridDim.x < nblk) __syncthreads();   // shared sums are reused by the next block
+        }
     }
     if (a0.encode) return;   // encode launches resolve nothing (no counter use)
     // the CTA's flags are ordered before its completion count by the barrier and thread 0's
@@ -538,10 +546,17 @@ static int64_t check_blocks(const StageArgs& a) {
     return count * ((a.nb + per - 1) / per);
 }
 
+// grid of a check launch: one CTA per work block, or at most ABFT_CHK_GRID CTAs (0: uncapped)
+static int64_t check_grid(int64_t nblk) {
+    static int64_t cap = -1;
+    if (cap < 0) { const char* e = getenv("ABFT_CHK_GRID"); cap = e ? std::max(0, atoi(e)) : 0; }
+    return cap > 0 && nblk > cap ? cap : nblk;
+}
+
 int launch_check(const StageArgs& a, cudaStream_t s) {
     const int64_t nb0 = check_blocks(a);
     if (nb0 <= 0) return 0;
-    k_check<<<(unsigned)nb0, kChkThreads, 0, s>>>(a, a, nb0);
+    k_check<<<(unsigned)check_grid(nb0), kChkThreads, 0, s>>>(a, a, nb0, nb0);
     abft_count_launch();
     return 0;
 }
@@ -552,7 +567,7 @@ int launch_check(const StageArgs& a, cudaStream_t s) {
 int launch_check2(const StageArgs& a0, const StageArgs& a1, cudaStream_t s) {
     const int64_t nb0 = check_blocks(a0), nb1 = check_blocks(a1);
     if (nb0 + nb1 <= 0) return 0;
-    k_check<<<(unsigned)(nb0 + nb1), kChkThreads, 0, s>>>(a0, a1, nb0);
+    k_check<<<(unsigned)check_grid(nb0 + nb1), kChkThreads, 0, s>>>(a0, a1, nb0, nb0 + nb1);
     abft_count_launch();
     return 0;
 }

@@ -117,6 +117,26 @@ __host__ __device__ __forceinline__ int64_t stage_count(const StageArgs& a) {
     }
 }
 
+// Column-major tile enumeration over block columns J >= j0 where column J holds N - J - d tiles
+// (d = 0: I >= J, d = 1: I > J): the column J and the offset rem inside it of tile t, in closed form
+// (a root of the quadratic prefix count, corrected by at most a step or two) — every CTA of a check
+// launch decodes its tile, and a per-column loop cost up to N iterations per thread.
+__host__ __device__ __forceinline__ int64_t tiles_before(int64_t J, int64_t j0, int64_t N, int64_t d) {
+    return (J - j0) * (N - d) - (J * (J - 1) - j0 * (j0 - 1)) / 2;
+}
+__host__ __device__ __forceinline__ void decode_cols(int64_t t, int64_t j0, int64_t N, int64_t d, int64_t& J,
+                                                     int64_t& rem) {
+    const double a = (double)(N - d) + 0.5;
+    const double C = (double)j0 * (double)(N - d) - 0.5 * (double)j0 * (double)(j0 - 1);
+    const double disc = a * a - 2.0 * ((double)t + C);
+    int64_t j = (int64_t)(a - sqrt(disc > 0.0 ? disc : 0.0));
+    if (j < j0) j = j0;
+    while (j > j0 && tiles_before(j, j0, N, d) > t) --j;
+    while (tiles_before(j + 1, j0, N, d) <= t) ++j;
+    J = j;
+    rem = t - tiles_before(j, j0, N, d);
+}
+
 // t-th tile of the stage, in the oracle's check order (column-major over tiles).
 __device__ __forceinline__ void stage_tile(const StageArgs& a, int64_t t, int64_t& I, int64_t& J) {
     const int64_t N = a.N, k = a.k;
@@ -129,16 +149,14 @@ __device__ __forceinline__ void stage_tile(const StageArgs& a, int64_t t, int64_
         case SK_TRAIL_DIAG: I = J = a.j_lo + t; return;
         case SK_LEFT_L: J = t / a.j_hi; I = k + t % a.j_hi; return;
         case SK_TRAIL_OFF: {   // column-major over (I > J), J in [j_lo, j_hi)
-            int64_t jj = a.j_lo, rem = t;
-            while (rem >= N - jj - 1) { rem -= N - jj - 1; ++jj; }
-            J = jj; I = jj + 1 + rem; return;
+            int64_t rem;
+            decode_cols(t, a.j_lo, N, 1, J, rem);
+            I = J + 1 + rem; return;
         }
-        default: {
-            const int64_t j0 = (a.kind == SK_TRAIL) ? a.j_lo : 0;
-            const int64_t m = N - j0;
-            int64_t jj = 0, rem = t;
-            while (rem >= m - jj) { rem -= m - jj; ++jj; }
-            J = j0 + jj; I = J + rem; return;
+        default: {             // column-major over (I >= J), J from j_lo (SK_TRAIL) or 0
+            int64_t rem;
+            decode_cols(t, (a.kind == SK_TRAIL) ? a.j_lo : 0, N, 0, J, rem);
+            I = J + rem; return;
         }
     }
 }
