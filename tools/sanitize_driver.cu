@@ -40,6 +40,44 @@ int main(int argc, char** argv) {
                (long long)rep.n_checks, cudaGetErrorString(cudaGetLastError()));
         bad |= rc != 0 || rep.n_events != (pass ? 2 : 0);
     }
+    // multi-GPU driver in the one-device harness: 1D (4 ranks) and 2D block-cyclic (2 x 2 grid),
+    // each rank's block columns (J mod Pc == rank mod Pc) full height, fault-free + one RECV error
+    const int64_t N = n / nb;
+    for (int prows = 1; prows <= 2; ++prows) {
+        const int P = 4, Pc = P / prows;
+        abft_gen_spd(n, n, A, n, nullptr);
+        std::vector<double*> loc(P, nullptr);
+        for (int r = 0; r < P; ++r) {
+            const int64_t nbl = (N - r % Pc + Pc - 1) / Pc;
+            if (nbl <= 0) continue;
+            cudaMalloc(&loc[r], 8 * n * nbl * nb);
+            for (int64_t t = 0; t < nbl; ++t)
+                cudaMemcpy(loc[r] + t * nb * n, A + (t * Pc + r % Pc) * nb * n, 8 * n * nb, cudaMemcpyDeviceToDevice);
+        }
+        abft_options_t o{};
+        o.abft_enabled = 1; o.K = 1; o.c_tau = 64.0; o.prows = prows;
+        for (int pass = 0; pass < 2; ++pass) {
+            abft_report_t rep{};
+            rep.cap = 64; rep.events = ev.data();
+            abft_inject_spec_t inj[2] = {};
+            // RECV on a rank that does not own panel tile (2, 1) (owner: (2 mod Pr) * Pc + 1 mod Pc)
+            const int owner = (int)((2 % prows) * Pc + 1 % Pc);
+            inj[0] = {1, ABFT_HOOK_RECV, ABFT_TGT_DATA, 0, 2 * nb + 7, nb + 3, 1ull << 50, (owner + 1) % P, 0};
+            inj[1].k = -1;
+            if (pass == 1) {   // restore the inputs
+                for (int r = 0; r < P; ++r) {
+                    const int64_t nbl = (N - r % Pc + Pc - 1) / Pc;
+                    for (int64_t t = 0; t < nbl; ++t)
+                        cudaMemcpy(loc[r] + t * nb * n, A + (t * Pc + r % Pc) * nb * n, 8 * n * nb, cudaMemcpyDeviceToDevice);
+                }
+            }
+            rc = abft_potrf_dist_sim(n, nb, P, loc.data(), n, nullptr, pass ? inj : nullptr, &rep, &o);
+            printf("dist_sim prows %d pass %d rc=%d events=%lld checks=%lld (%s)\n", prows, pass, rc,
+                   (long long)rep.n_events, (long long)rep.n_checks, cudaGetErrorString(cudaGetLastError()));
+            bad |= rc != 0 || rep.n_events != (pass ? 1 : 0);
+        }
+        for (double* p : loc) if (p) cudaFree(p);
+    }
     printf("%s\n", bad ? "FAIL" : "OK");
     return bad;
 }
