@@ -171,3 +171,18 @@ def test_processes_ipc_2d_match_oracle(P, world, prows):
     assert res[0][2] == ref.event_tuples()
     L = P.block_cyclic_join_2d([r[3] for r in res], nb, n, prows)
     assert floor_rel(L, ref.L, A) <= 1e-11
+
+
+@pytest.mark.parametrize("n,nb,Pn,prows", [(128, 128, 4, 2), (256, 128, 4, 2), (384, 128, 6, 3), (256, 64, 8, 4),
+                                           (512, 128, 4, 1)])
+def test_sim2d_small_grids_more_ranks_than_tiles(P, n, nb, Pn, prows):
+    """Degenerate 2D cases: one block column (no panel to broadcast), fewer block rows / columns
+    than process rows / columns (ranks owning nothing in some iterations), ragged ownership."""
+    A = syn.spd_matrix(n)
+    specs = [dict(k=0, hook="REST", row=n - 1, col=0, bit=50)] if n > nb else []
+    inj = syn.inj_array(specs) if specs else None
+    ref = oracle.potrf(A, nb, inj=inj, nranks=Pn, prows=prows)
+    st, rep, L = run_sim2d(P, A, nb, Pn, prows, inj=inj)
+    assert st == ref.status == 0
+    assert P.sorted_event_tuples(rep["events"]) == ref.event_tuples()
+    assert floor_rel(L, ref.L, A) <= 1e-11
