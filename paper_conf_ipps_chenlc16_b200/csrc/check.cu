@@ -491,8 +491,9 @@ __device__ void phase2_body(const StageArgs& a0, const StageArgs& a1, int flist)
 // work blocks blockIdx.x, + gridDim.x, ... so its fixed costs are paid once for several tiles.
 __global__ void __launch_bounds__(kChkThreads, 4) k_check(StageArgs a0, StageArgs a1, int64_t nblk0, int64_t nblk) {
     __shared__ int s_last;
-    const bool aborted = cta_aborted(&a0.st->abort);
-    if (!aborted) {
+    // no abort test at entry (it would put a dependent global round trip in front of every check on
+    // the panel chain): after an abort phase 1 only reads, and phase 2 resolves nothing
+    {
         for (int64_t blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
             const bool p1 = blk >= nblk0;
             const StageArgs& a = p1 ? a1 : a0;
