@@ -374,15 +374,23 @@ def test_two_errors_in_a_column_redo_matches_oracle(P, mode):
         assert floor_rel(L, ref.L, A) <= 1e-11
 
 
+@pytest.mark.parametrize("pinned", [True, False])
 @pytest.mark.parametrize("n,nb", [(2048, 256), (3072, 512)])
-def test_host_entry_overlapped_writeback(P, n, nb, monkeypatch):
+def test_host_entry_overlapped_writeback(P, n, nb, pinned, monkeypatch):
     """abft_potrf_host copies each finished block column of L to the host while the factorisation
-    continues (fault-free direct path; ABFT_GRAPH=0 forces direct launches at this size): the host
-    result equals the device path bit for bit and the strict upper triangle keeps the input."""
+    continues (fault-free direct path on page-locked memory — a torch pinned tensor's column-major
+    numpy view; ABFT_GRAPH=0 forces direct launches at this size), or takes the plain
+    copy-factor-copy path on pageable memory: either way the host result equals the device path
+    bit for bit and the strict upper triangle keeps the input."""
     import torch
     monkeypatch.setenv("ABFT_GRAPH", "0")
     A = syn.spd_matrix(n)
-    Ah = A.copy(order="F")
+    if pinned:
+        buf = torch.empty((n, n), dtype=torch.float64, pin_memory=True)
+        Ah = buf.T.numpy()                      # F-contiguous view of page-locked memory
+        Ah[:, :] = A
+    else:
+        Ah = A.copy(order="F")
     st, rep = P.abft_potrf_host(n, nb, Ah)
     assert st == 0 and rep["n_events"] == 0
     Ad = P.colmajor(A)
