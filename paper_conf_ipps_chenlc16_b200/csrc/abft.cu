@@ -244,6 +244,7 @@ struct ThreadCache {
     cudaStream_t P = nullptr;
     cudaStream_t P2 = nullptr;   // panel side stream: V2 runs here while P factors the diagonal block
     cudaStream_t C = nullptr;    // copy stream of abft_potrf_host's overlapped write-back
+    cudaStream_t Cin = nullptr;  // copy stream of abft_potrf_host's streamed input
     EventPool sync{cudaEventDisableTiming};
     EventPool timing{cudaEventDefault};
 };
@@ -345,6 +346,16 @@ struct HostSink {
     cudaStream_t cs = nullptr;
 };
 static thread_local HostSink g_sink;
+// abft_potrf_host's input streamed in behind the factorisation's start: the block columns arrive
+// on a copy stream (first every diagonal tile — the threshold scales need the whole diagonal —
+// then each column below its diagonal tile, in order); ev[0] marks the diagonal tiles, ev[1 + k]
+// block column k. The encode of later block columns and update 0 then run in column chunks as
+// their data lands, overlapped with the transfer of the rest.
+struct HostSource {
+    bool active = false;
+    std::vector<cudaEvent_t> ev;
+};
+static thread_local HostSource g_src;
 
 // Buffers owned by a captured graph (graph mode, see run_graph): run_potrf then only enqueues the
 // work (resets, kernels, cross-stream events) and leaves the report to the caller.
@@ -409,6 +420,25 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
     // reads only column 0's checksums), and the rest of the matrix is encoded on S concurrently
     // with panel 0 — before update 0, the first reader of those checksums (reading B9)
     cudaEvent_t t_enc = nullptr;
+    // streamed input (abft_potrf_host): the diagonal tiles and block column 0 before anything reads
+    // them; the other block columns are awaited chunk by chunk (ensure_chunk) before their encode
+    const bool src = g_src.active && !ps && nc == 2 && N >= 2 && (int64_t)g_src.ev.size() >= N + 1;
+    constexpr int64_t kSrcChunk = 8;   // block columns per chunk of the streamed input
+    std::vector<char> chunk_done(src ? (size_t)((N + kSrcChunk - 1) / kSrcChunk) : 0, 0);
+    if (src) { cudaStreamWaitEvent(s, g_src.ev[0], 0); cudaStreamWaitEvent(s, g_src.ev[1], 0); }
+    else if (g_src.active && !ps && (int64_t)g_src.ev.size() >= N + 1) cudaStreamWaitEvent(s, g_src.ev[N], 0);   // all of it
+    auto ensure_chunk = [&](int64_t c) {   // chunk c = block columns [c kSrcChunk, (c + 1) kSrcChunk)
+        if (!src || chunk_done[(size_t)c]) return;
+        const int64_t J0 = std::max<int64_t>(1, c * kSrcChunk), J1 = std::min<int64_t>(N, (c + 1) * kSrcChunk);
+        chunk_done[(size_t)c] = 1;
+        if (J0 >= J1) return;
+        cudaStreamWaitEvent(s, g_src.ev[1 + J1 - 1], 0);   // in-order copies: the chunk's last column
+        if (abft && !(abl & 16)) {
+            StageArgs a = stage_base(w, A, lda, o.c_tau, SK_TRAIL, 0, 0);
+            a.j_lo = J0; a.j_hi = J1; a.encode = 1;
+            launch_check(a, s);
+        }
+    };
     if (abft && !(abl & 16)) {
         t_enc = prof.begin(s);
         launch_scales(n, nb, A, lda, w.scl, s, (int)nc);
@@ -420,7 +450,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         cudaEvent_t e = new_event(); cudaEventRecord(e, s); cudaStreamWaitEvent(P, e, 0);
     }
     if (abft && !(abl & 16)) {
-        if (N > 1) {
+        if (N > 1 && !src) {
             StageArgs a = stage_base(w, A, lda, o.c_tau, SK_TRAIL, 0, 0);
             a.j_lo = 1; a.j_hi = N; a.encode = 1;
             launch_check(a, s);
@@ -614,6 +644,7 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         const Loc L{A, lda, w.chk, w.ldc, Wbuf[k & 1], ldw, mB, (int)nc};
         const bool gated = (((k + 1) % K == 0) || k == N - 2) && mode != ABFT_MODE_OFFLINE;
         // (a) block column k+1 first: update, UPDATE_OUT hook, V5 -> hand it to the panel stream
+        if (k == 0) ensure_chunk(1 / kSrcChunk);
         const int fa = update_cols(k, k + 1, k + 2);
         if (abft) {
             if (!(fa & 2)) do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 1, k + 2, true);
@@ -623,9 +654,19 @@ static int run_potrf(int64_t n, int64_t nb, double* A, int64_t lda, cudaStream_t
         cudaStreamWaitEvent(P, ec, 0);
         std::tie(pan[k + 1], wbk[k + 1]) = panel(k + 1);
         sink_col(k + 1);
-        // (b) the rest of the trailing matrix
+        // (b) the rest of the trailing matrix (streamed input, k = 0: chunk by chunk as it lands)
         if (m > 1) {
-            const int fb = update_cols(k, k + 2, N);
+            int fb;
+            if (src && k == 0) {
+                fb = 1 | 2;
+                for (int64_t c = 2 / kSrcChunk; c * kSrcChunk < N; ++c) {
+                    ensure_chunk(c);
+                    const int64_t J0 = std::max<int64_t>(2, c * kSrcChunk), J1 = std::min<int64_t>(N, (c + 1) * kSrcChunk);
+                    if (J0 < J1) fb &= update_cols(0, J0, J1);
+                }
+            } else {
+                fb = update_cols(k, k + 2, N);
+            }
             if (abft) {
                 if (!(fb & 2)) do_inject_if(inj, k, ABFT_HOOK_UPDATE_OUT, B, L, ab, s, k + 2, N, true);
                 if (gated && !(abl & 2)) v5_cols(k, k + 2, N, (fb & 1) != 0);
@@ -1625,7 +1666,39 @@ extern "C" int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t ld
     const bool overlap = pinned && !has_inj && o.order == ABFT_ORDER_RIGHT &&
                          (o.mode == ABFT_MODE_ENHANCED || !o.abft_enabled) && !graph_mode_enabled(n) &&
                          getenv("ABFT_HOST_OVERLAP") == nullptr;
-    if (overlap) {
+    const int64_t N = n / nb;
+    const bool stream_in = overlap && N >= 2 && (!opt || opt->nchk == 0 || opt->nchk == 2) &&
+                           getenv("ABFT_HOST_STREAM_IN") == nullptr;   // dev knob: set = copy all first
+    if (stream_in) {
+        // only what the factorisation reads goes over PCIe, and it streams in behind the start of
+        // the factorisation on its own copy stream (HostSource): every diagonal tile first (the
+        // threshold scales need the whole diagonal), then each block column below its diagonal
+        // tile, in order, one event each
+        ThreadCache& tc = thread_cache();
+        if (!tc.Cin) ABFT_CUDA_TRY(cudaStreamCreateWithFlags(&tc.Cin, cudaStreamNonBlocking));
+        while ((int64_t)g_src.ev.size() < N + 2) {
+            cudaEvent_t e;
+            ABFT_CUDA_TRY(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+            g_src.ev.push_back(e);
+        }
+        cudaEvent_t alloc = g_src.ev[N + 1];   // dA allocated on s
+        ABFT_CUDA_TRY(cudaEventRecord(alloc, s));
+        ABFT_CUDA_TRY(cudaStreamWaitEvent(tc.Cin, alloc, 0));
+        for (int64_t k = 0; k < N; ++k)
+            ABFT_CUDA_TRY(cudaMemcpy2DAsync(dA + k * nb * n + k * nb, n * sizeof(double), A_host + k * nb * lda + k * nb,
+                                            lda * sizeof(double), (size_t)nb * sizeof(double), (size_t)nb,
+                                            cudaMemcpyHostToDevice, tc.Cin));
+        ABFT_CUDA_TRY(cudaEventRecord(g_src.ev[0], tc.Cin));
+        for (int64_t k = 0; k < N; ++k) {
+            if (k + 1 < N)
+                ABFT_CUDA_TRY(cudaMemcpy2DAsync(dA + k * nb * n + (k + 1) * nb, n * sizeof(double),
+                                                A_host + k * nb * lda + (k + 1) * nb, lda * sizeof(double),
+                                                (size_t)(n - (k + 1) * nb) * sizeof(double), (size_t)nb,
+                                                cudaMemcpyHostToDevice, tc.Cin));
+            ABFT_CUDA_TRY(cudaEventRecord(g_src.ev[1 + k], tc.Cin));
+        }
+        g_src.active = true;
+    } else if (overlap) {
         // only what the factorisation reads goes over PCIe: each block column from its diagonal
         // block down (the strict upper triangle outside the diagonal blocks is never read)
         for (int64_t k = 0; k < n / nb; ++k)
@@ -1650,6 +1723,10 @@ extern "C" int abft_potrf_host(int64_t n, int64_t nb, double* A_host, int64_t ld
         g_sink.host = A_host; g_sink.ldh = lda; g_sink.cs = tc.C;
     }
     rc = abft_potrf_ex(n, nb, dA, n, stream, inj, r, opt);
+    if (stream_in) {   // s has consumed every column unless the call failed early: join the copies anyway
+        g_src.active = false;
+        ABFT_CUDA_TRY(cudaStreamWaitEvent(s, g_src.ev[N], 0));
+    }
     bool recopy = !overlap;
     if (overlap) {
         g_sink = HostSink();
