@@ -278,29 +278,53 @@ __device__ bool leaf_tile(double* Ls, double* Us, double* Zs, LeafSmem& ls, doub
     const int tid = threadIdx.x, r = tid & 63, g = tid >> 6;
     const int lane = tid & 31, warp = tid >> 5, fr = lane >> 2, fc = lane & 3;
     if (dbg) dbg[0] = clock64();
+    __shared__ int s_bad;   // first non-positive pivot + 1 (0: none)
+    if (tid == 0) s_bad = 0;
+    (void)r; (void)g;
     for (int p = 0; p < 8; ++p) {
         const int c0 = 8 * p;
-        for (int j = 0; j < 8; ++j) {
-            const int cj = c0 + j;
-            __syncthreads();
-            const double d = Ls[cj * kTP + cj];
-            if (!(d > 0.0)) {
-                if (tid == 0 && atomicCAS(&st->abort, 0, 1) == 0) { st->status = ABFT_NOT_SPD; st->info = info0 + cj + 1; }
-                return false;
-            }
-            if (r > cj) {
-                const double f = Ls[cj * kTP + r] * __drcp_rn(d);
-                if (g == 0) Us[cj * kTP + r] = f;
+        __syncthreads();
+        // the 8-column panel, by warp 0 alone in registers (lane holds rows lane and lane + 32):
+        // no CTA barrier per column step, the pivot and column j's panel rows by shuffles. Same
+        // operations per element as a shared-memory step (f = a_rj * rcp(d), a_rc -= f a_cj).
+        if (warp == 0) {
+            const bool hi = p >= 4;          // rows c0..c0+7 are the lanes' second row (lane + 32)
+            double a0[8], a1[8];
 #pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                    const int c = c0 + 2 * g + h;
-                    if (c > cj) Ls[c * kTP + r] = fma(-f, Ls[cj * kTP + c], Ls[c * kTP + r]);
+            for (int c = 0; c < 8; ++c) { a0[c] = Ls[(c0 + c) * kTP + lane]; a1[c] = Ls[(c0 + c) * kTP + lane + 32]; }
+            int bad = 0;
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+                const int cj = c0 + j;
+                const double d = __shfl_sync(0xffffffffu, hi ? a1[j] : a0[j], cj & 31);
+                if (!(d > 0.0)) { bad = cj + 1; break; }   // warp-uniform
+                const double rd = __drcp_rn(d);
+                double acj[8];
+#pragma unroll
+                for (int c = 0; c < 8; ++c) acj[c] = __shfl_sync(0xffffffffu, hi ? a1[j] : a0[j], (c0 + c) & 31);
+                if (lane > cj) {
+                    const double f = a0[j] * rd;
+                    Us[cj * kTP + lane] = f;
+#pragma unroll
+                    for (int c = j + 1; c < 8; ++c) a0[c] = fma(-f, acj[c], a0[c]);
                 }
-            } else if (tid == 0) {
-                piv_s[cj] = d;
+                if (lane + 32 > cj) {
+                    const double f = a1[j] * rd;
+                    Us[cj * kTP + lane + 32] = f;
+#pragma unroll
+                    for (int c = j + 1; c < 8; ++c) a1[c] = fma(-f, acj[c], a1[c]);
+                }
+                if (lane == 0) piv_s[cj] = d;
+            }
+#pragma unroll
+            for (int c = 0; c < 8; ++c) { Ls[(c0 + c) * kTP + lane] = a0[c]; Ls[(c0 + c) * kTP + lane + 32] = a1[c]; }
+            if (bad && lane == 0) {
+                s_bad = bad;
+                if (atomicCAS(&st->abort, 0, 1) == 0) { st->status = ABFT_NOT_SPD; st->info = info0 + bad; }
             }
         }
         __syncthreads();
+        if (s_bad) return false;
         const int nt = 7 - p;            // trailing 8 x 8 tiles per side
         for (int e = warp; e < nt * (nt + 1) / 2; e += 8) {
             int tj = 0, rem = e;
